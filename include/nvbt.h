@@ -1,0 +1,163 @@
+/* nvbt — B200-native device-side instrumentation hot path of NVBit (Villa et al., MICRO'19).
+ *
+ * C ABI of libnvbt.so. Citations "P:Lnnn (§x)" are lines of /root/reference/PAPER.md; the event model
+ * every call follows is docs/EVENT_MODEL.md (EM §n).
+ *
+ * Conventions (all entry points):
+ *  - Every function returns int: NVBT_OK (0) or a negative nvbt_status. No C++ exception crosses the
+ *    ABI. nvbt_last_error() returns a thread-local message for the last failing call on this thread.
+ *  - Ownership: ALL device memory and pinned host memory are caller-owned (allocated by PyTorch). The
+ *    library never calls cudaMalloc/cudaHostAlloc. Streams are caller-owned (cudaStream_t as void*).
+ *  - Results are cumulative since nvbt_init / nvbt_reset, like NVBit's __managed__ counters read at
+ *    nvbit_at_term (P:L190-192, P:L254-258 (§6.1)). Read calls synchronise the context's stream, run the
+ *    fold kernel on it and copy into caller host buffers.
+ *  - Device pointers passed to workload/replay calls must be 16-byte aligned device addresses.
+ */
+#ifndef NVBT_H
+#define NVBT_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define NVBT_ABI_VERSION 1
+
+enum nvbt_status {
+  NVBT_OK = 0,
+  NVBT_EINVAL = -1,     /* null pointer, size or flag mismatch */
+  NVBT_ESTATE = -2,     /* feature not enabled at init, or channel not open */
+  NVBT_ENOMEM = -3,     /* workspace or ring too small */
+  NVBT_ECUDA = -4,      /* CUDA runtime error; message carries cudaGetErrorString */
+  NVBT_ETIMEDOUT = -5,  /* channel drain timeout, or a producer gave up on backpressure */
+  NVBT_EVERSION = -6    /* ABI version mismatch */
+};
+
+/* Context flags: what the context collects (EM §2). */
+enum nvbt_flags {
+  NVBT_COUNT = 1,       /* thread/warp issued/executed counts (Listing 1 tool, P:L80-89 (§3)) */
+  NVBT_OPHIST = 2,      /* per-opcode histogram (§6.2 Top-5 tool) */
+  NVBT_BB = 4,          /* per-basic-block entries/instructions (BB rule P:L115-117 (§4)) */
+  NVBT_MEMDIV = 8,      /* unique 32B sectors / 128B lines per warp global LD/ST (Listing 8) */
+  NVBT_PER_WARP = 16,   /* per-warp thread/warp executed counts (n_warps entries) */
+  NVBT_TRACE = 32       /* per-warp address records through the device->host channel */
+};
+
+/* Per-launch tool selection for instrumented workload launches (the compiled-in analogue of
+ * nvbit_insert_call + nvbit_enable_instrumented, P:L123, P:L169 (§4, §5.1)). */
+enum nvbt_tools {
+  NVBT_TOOL_NONE = 0,     /* uninstrumented launch of the same source (slowdown baseline) */
+  NVBT_TOOL_COUNT = 1,    /* a hook at every pc: counts, opcode and BB histograms */
+  NVBT_TOOL_BBCOUNT = 2,  /* hooks only at BB leaders and guarded pcs; per-pc counts derived */
+  NVBT_TOOL_MEMDIV = 4,   /* hooks at global-memory pcs: sector/line divergence */
+  NVBT_TOOL_TRACE = 8     /* hooks at global-memory pcs: one 288 B record per executed event (EM §5) */
+};
+
+enum nvbt_kind { NVBT_K_ALU = 0, NVBT_K_CTRL = 1, NVBT_K_GLD = 2, NVBT_K_GST = 3, NVBT_K_GATOM = 4,
+                 NVBT_K_OTHERMEM = 5 };
+
+/* One row of a program table ("virtual SASS", EM §3) — stands in for NVBit's class Instr. */
+typedef struct {
+  uint16_t opcode;
+  uint8_t kind;       /* enum nvbt_kind */
+  uint8_t width;      /* bytes per lane for memory kinds (1,2,4,8,16), else 0 */
+  uint32_t bb;        /* basic block id */
+  uint8_t is_leader;  /* first pc of its basic block */
+  uint8_t guarded;    /* carries a guard predicate (P may differ from A) */
+  uint16_t pad;
+} nvbt_instr_desc;
+
+typedef struct {
+  uint32_t version;        /* NVBT_ABI_VERSION */
+  int32_t device;          /* CUDA device ordinal the workspace lives on */
+  void* stream;            /* cudaStream_t every call of this context is ordered on */
+  const nvbt_instr_desc* prog;  /* host array [n_pcs], copied at init */
+  uint32_t n_pcs;          /* 1..4096 */
+  uint32_t n_opcodes;      /* 1..256, > every opcode in prog */
+  uint32_t n_bbs;          /* > every bb in prog, <= n_pcs */
+  uint32_t n_warps;        /* global warp ids are < n_warps when NVBT_PER_WARP (else ignored) */
+  uint32_t flags;          /* enum nvbt_flags */
+  void* d_workspace;       /* device memory, >= nvbt_workspace_size bytes, 256-byte aligned */
+  size_t workspace_bytes;
+} nvbt_config;
+
+typedef struct nvbt_ctx_s* nvbt_ctx;
+typedef struct nvbt_chan_s* nvbt_channel;
+
+int nvbt_abi_version(void);
+const char* nvbt_last_error(void);
+
+/* Bytes of device workspace a config needs (only n_pcs, n_opcodes, n_bbs, n_warps, flags are read). */
+int nvbt_workspace_size(const nvbt_config* cfg, size_t* bytes);
+
+/* Validates cfg, uploads the program table into the workspace and zeroes the accumulators (on
+ * cfg->stream). EINVAL on a malformed table or config, ENOMEM if the workspace is too small. */
+int nvbt_init(const nvbt_config* cfg, nvbt_ctx* out);
+int nvbt_reset(nvbt_ctx ctx);            /* zero accumulators and the launch counter (async on stream) */
+int nvbt_fini(nvbt_ctx ctx);             /* frees host-side state only; closes an open channel */
+
+/* The packed int64 accumulator region (device pointer + length in int64 words): per-pc site bins,
+ * BB-mode bins, memory-divergence bins, S/L histograms and per-warp arrays. Sums of disjoint event
+ * sets add elementwise, so a multi-GPU merge is one int64 SUM all-reduce of this region (EM §4). */
+int nvbt_accum_view(nvbt_ctx ctx, void** d_ptr, size_t* n_int64);
+
+/* ---- read calls (EM §2); all synchronise the stream ---- */
+typedef struct { uint64_t thread_issued, thread_exec, warp_issued, warp_exec; } nvbt_counts;
+/* per_warp_thread / per_warp_warp: nullable host arrays [n_warps] (need NVBT_PER_WARP). */
+int nvbt_count(nvbt_ctx ctx, nvbt_counts* out, uint64_t* per_warp_thread, uint64_t* per_warp_warp);
+/* thread_exec / warp_exec: host arrays [n_opcodes]. */
+int nvbt_opcode_hist(nvbt_ctx ctx, uint64_t* thread_exec, uint64_t* warp_exec, uint32_t n_opcodes);
+typedef struct { uint64_t entries_warp, entries_thread, instrs_warp, instrs_thread; } nvbt_bb_stats;
+int nvbt_bb_count(nvbt_ctx ctx, nvbt_bb_stats* out, uint32_t n_bbs);
+typedef struct { uint64_t accesses, sectors, lines; } nvbt_memdiv;       /* per pc: n, ΣS, ΣL */
+typedef struct { nvbt_memdiv sum; uint64_t hist_sectors[33], hist_lines[33]; } nvbt_memdiv_total;
+/* per_pc: nullable host array [n_pcs]. The paper's printed figure is sum.lines/sum.accesses. */
+int nvbt_mem_divergence(nvbt_ctx ctx, nvbt_memdiv* per_pc, uint32_t n_pcs, nvbt_memdiv_total* tot);
+
+/* ---- trace channel (a6; "sent to the CPU for further processing", P:L187 (§6.1)) ----
+ * pinned_ring: caller-owned pinned, device-mapped host memory (cudaHostAlloc / torch pin_memory), at
+ * least 64 + 288 * 2 bytes, 64-byte aligned. Its first 64 bytes hold the consumer index the producers
+ * read for backpressure; the rest is floor((ring_bytes - 64) / 288) record slots. record_bytes must be
+ * 288 (EM §5). One channel per context. */
+int nvbt_channel_open(nvbt_ctx ctx, void* pinned_ring, size_t ring_bytes, uint32_t record_bytes,
+                      nvbt_channel* out);
+/* Called with a batch of n contiguous, fully written records (reserved field zeroed); return 0 to
+ * continue, non-zero to stop draining (nvbt_channel_drain then returns NVBT_ESTATE). */
+typedef int (*nvbt_drain_fn)(const void* records, uint64_t n_records, void* user);
+/* Consumes records in ticket order until the context's stream is idle and every reserved record has
+ * been delivered, or timeout_us elapses (-1 = no limit; NVBT_ETIMEDOUT). Runs on the calling thread,
+ * concurrently with kernels already enqueued. *n_drained (nullable) = records delivered by this call. */
+int nvbt_channel_drain(nvbt_channel ch, nvbt_drain_fn fn, void* user, int64_t timeout_us,
+                       uint64_t* n_drained);
+int nvbt_channel_close(nvbt_channel ch);
+/* Records the producers dropped after waiting ~2 s on a full ring (0 in a healthy run). */
+int nvbt_channel_dropped(nvbt_channel ch, uint64_t* dropped);
+
+/* Built-in drain callbacks. */
+typedef struct { uint64_t n_rec, d1, d2; } nvbt_digest;         /* EM §5 multiset digest */
+int nvbt_drain_digest(const void* records, uint64_t n_records, void* user /* nvbt_digest* */);
+typedef struct { void* dst; uint64_t capacity; uint64_t n; } nvbt_copy_sink;   /* dst: host [capacity*288] */
+int nvbt_drain_copy(const void* records, uint64_t n_records, void* user /* nvbt_copy_sink* */);
+/* Host-side digest of an array of records (for checking copies). */
+int nvbt_digest_records(const void* records, uint64_t n_records, nvbt_digest* out);
+
+/* ---- trace-replay mode (a7; EM §3.5) ---- */
+/* Writes events [first, first+n) of the counter-based generator (seed) as 16 B headers at d_hdr[n]
+ * and, for memory pcs, 32 x u64 addresses at d_addr + 256*i. The context's program must be the
+ * replay program (nvbt_program(NVBT_W_REPLAY, ...)). */
+int nvbt_gen_events(nvbt_ctx ctx, uint64_t seed, uint64_t first, uint64_t n, void* d_hdr, void* d_addr);
+/* Applies EM §2 items 1-4 to n events {u32 pc, warp, A, P} at d_hdr (slot i at d_addr + 256*i is read
+ * only when kind(pc) is a memory kind and A&P != 0). pc >= n_pcs -> the event is ignored and counted
+ * in the error word (nvbt_replay_errors). */
+int nvbt_replay(nvbt_ctx ctx, const void* d_hdr, const void* d_addr, uint64_t n);
+int nvbt_replay_errors(nvbt_ctx ctx, uint64_t* bad_events);
+
+/* Number of kernels this context launched since init (for the bench's gpu_launches claim). */
+int nvbt_launch_count(nvbt_ctx ctx, uint64_t* n);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* NVBT_H */

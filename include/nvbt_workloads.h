@@ -1,0 +1,51 @@
+/* nvbt synthetic workloads with compiled-in injection points (EM = docs/EVENT_MODEL.md §3).
+ *
+ * NVBit injects calls into SASS at run time (P:L123, P:L147-167 (§4, §5.1)); SASS decode and
+ * trampolines are out of scope here, so each workload kernel is written once with a hook at every
+ * injection point of its program table and compiled in several variants: `tools` (enum nvbt_tools)
+ * picks the variant per launch, NVBT_TOOL_NONE being the same source with every hook compiled out
+ * (the slowdown baseline). Conventions as in nvbt.h; all pointers are caller-owned device memory and
+ * every launch is enqueued on the context's stream (asynchronous). Each instrumented launch takes the
+ * next launch id ℓ of the context (EM §5).
+ */
+#ifndef NVBT_WORKLOADS_H
+#define NVBT_WORKLOADS_H
+
+#include "nvbt.h"
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+enum nvbt_workload { NVBT_W_VECTORADD = 1, NVBT_W_SGEMM = 2, NVBT_W_BFS = 3, NVBT_W_STENCIL = 4,
+                     NVBT_W_REPLAY = 5 };
+
+/* Copies a workload's program table (EM §3.1-3.5) into out[cap]; *n_pcs, *n_opcodes, *n_bbs receive
+ * its sizes (any may be null). EINVAL if cap is too small (with *n_pcs still set). Host-only. */
+int nvbt_program(int workload, nvbt_instr_desc* out, uint32_t cap, uint32_t* n_pcs,
+                 uint32_t* n_opcodes, uint32_t* n_bbs);
+
+/* Global warp count of one launch (for sizing PER_WARP contexts). Host-only.
+ * args: VECTORADD {N}; SGEMM {M, N}; BFS {n}; STENCIL {n}. */
+int nvbt_workload_warps(int workload, const int64_t* args, uint32_t n_args, uint64_t* n_warps);
+
+/* C1: c[i] = a[i] + b[i], i < N; CTA 256, grid ceil(N/256) (EM §3.1). ctx may be NULL when tools == 0
+ * (then stream is used); otherwise the context's program must be the vectorAdd program. */
+int nvbt_vectoradd(nvbt_ctx ctx, void* stream, uint32_t tools, const float* a, const float* b, float* c,
+                   int32_t N);
+/* C2: naive row-fastest SGEMM C[M,N] = A[M,K] B[K,N], fp32 row-major, K >= 1 (EM §3.2). */
+int nvbt_sgemm(nvbt_ctx ctx, void* stream, uint32_t tools, const float* A, const float* B, float* C,
+               int32_t M, int32_t N, int32_t K);
+/* C3: one BFS level = kernel 1 (expand) then kernel 2 (update, writes cost = level + 1) (EM §3.3).
+ * mask/visited/updating: u8[n]; cost: i32[n]; over: one i32 (kernel 2 stores 1 into it). The caller
+ * zeroes *over and updating before the call (the host loop of EM §3.3). */
+int nvbt_bfs_level(nvbt_ctx ctx, void* stream, uint32_t tools, const int32_t* rowptr, const int32_t* col,
+                   int32_t n, uint8_t* mask, uint8_t* visited, uint8_t* updating, int32_t* cost,
+                   int32_t* over, int32_t level);
+/* C4: one Jacobi iteration out = stencil(in) on an n x n fp32 grid (EM §3.4). */
+int nvbt_stencil(nvbt_ctx ctx, void* stream, uint32_t tools, const float* in, float* out, int32_t n);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

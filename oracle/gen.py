@@ -12,7 +12,7 @@ M40 = np.uint64((1 << 40) - 1)
 def events(first: int, n: int, prog=None, seed: int = SEED):
     """Events first .. first+n-1 as (pc, warp, A, P, addr[n, 32] uint64 (0 for non-memory pcs))."""
     if prog is None:
-        prog = programs.replay(seed)
+        prog = programs.replay()
     i = np.arange(first, first + n, dtype=np.uint64)
     pc = (R(i, 0, seed) % np.uint64(4096)).astype(np.int64)
     warp = (R(i, 1, seed) % np.uint64(1 << 20)).astype(np.int64)

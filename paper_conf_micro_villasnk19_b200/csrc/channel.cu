@@ -1,0 +1,199 @@
+// Device -> host trace channel (a6): a lock-free multi-producer ring in caller-pinned host memory.
+//
+// "NVBit allows one to ... collect reference addresses, which then can be analyzed directly on the GPU
+// or sent to the CPU for further processing" (P:L187 (§6.1)). The paper gives no mechanism; this one:
+//  * producers (warps, nvbt_dev.cuh emit<>) take a ticket t = atomicAdd(head, 1) in device memory, wait
+//    while t >= tail + cap (tail = consumer index the host publishes in the ring's first 64 bytes, cached
+//    in device memory), write the 288 B record into slot t % cap over PCIe with coalesced stores, then a
+//    system-scope fence and a 16 B store carrying the tag (t / cap) + 1;
+//  * the consumer (nvbt_channel_drain, calling thread) delivers slots in ticket order as soon as their tag
+//    matches, zeroes the tag field (EM §5 "reserved = 0"), calls the user callback on contiguous batches
+//    and publishes tail.
+#include <chrono>
+#include <cstring>
+#include <immintrin.h>
+
+#include "nvbt_internal.h"
+
+struct nvbt_chan_s {
+  nvbt_ctx ctx = nullptr;
+  unsigned char* host = nullptr;      // ring base (host view)
+  unsigned char* dev = nullptr;       // ring base (device view)
+  unsigned char* slots = nullptr;     // host view of slot 0
+  uint64_t cap = 0;
+  uint64_t consumed = 0;
+  bool open = false;
+};
+
+namespace nvbt {
+
+static constexpr size_t HDR = 64;
+
+void channel_state(nvbt_chan_s* ch, DevState* st) {
+  st->ring = ch->dev + HDR;
+  st->tail = reinterpret_cast<const unsigned long long*>(ch->dev);
+  st->cap = ch->cap;
+}
+bool channel_open(nvbt_chan_s* ch) { return ch && ch->open; }
+
+// EM §5 digest constants and mix64 (splitmix64 output function).
+static inline uint64_t mix64(uint64_t z) {
+  z += 0x9E3779B97F4A7C15ull;
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  return z ^ (z >> 31);
+}
+struct DigestConsts {
+  uint64_t c1[36], c2[36];
+  DigestConsts() {
+    for (int j = 0; j < 36; ++j) { c1[j] = mix64(0x1000 + j) | 1; c2[j] = mix64(0x2000 + j) | 1; }
+  }
+};
+static const DigestConsts kDig;
+
+static void digest_range(const unsigned char* rec, uint64_t n, uint64_t* d1, uint64_t* d2) {
+  uint64_t s1 = 0, s2 = 0;
+  for (uint64_t r = 0; r < n; ++r) {
+    uint64_t x[36];
+    std::memcpy(x, rec + r * RECORD_BYTES, RECORD_BYTES);
+    uint64_t h1 = 0, h2 = 0;
+    for (int j = 0; j < 36; ++j) { h1 += x[j] * kDig.c1[j]; h2 += x[j] * kDig.c2[j]; }
+    s1 += mix64(h1);
+    s2 += mix64(h2);
+  }
+  *d1 += s1;
+  *d2 += s2;
+}
+
+}  // namespace nvbt
+
+using namespace nvbt;
+
+extern "C" {
+
+int nvbt_channel_open(nvbt_ctx c, void* ring, size_t bytes, uint32_t record_bytes, nvbt_channel* out) {
+  if (!c || !ring || !out) return set_error(NVBT_EINVAL, "null argument");
+  if (!(c->flags & NVBT_TRACE)) return set_error(NVBT_ESTATE, "NVBT_TRACE not enabled at init");
+  if (c->chan) return set_error(NVBT_ESTATE, "channel already open on this context");
+  if (record_bytes != RECORD_BYTES) return set_error(NVBT_EINVAL, "record_bytes %u != 288", record_bytes);
+  if (reinterpret_cast<uintptr_t>(ring) % 64) return set_error(NVBT_EINVAL, "ring not 64-byte aligned");
+  if (bytes < HDR + 2 * RECORD_BYTES) return set_error(NVBT_ENOMEM, "ring of %zu bytes holds < 2 records", bytes);
+  NVBT_CUDA(cudaSetDevice(c->device));
+  cudaPointerAttributes pa{};
+  NVBT_CUDA(cudaPointerGetAttributes(&pa, ring));
+  if (pa.type != cudaMemoryTypeHost || pa.devicePointer == nullptr)
+    return set_error(NVBT_EINVAL, "ring is not pinned, device-mapped host memory");
+  auto* ch = new (std::nothrow) nvbt_chan_s();
+  if (!ch) return set_error(NVBT_ENOMEM, "host allocation failed");
+  ch->ctx = c;
+  ch->host = static_cast<unsigned char*>(ring);
+  ch->dev = static_cast<unsigned char*>(pa.devicePointer);
+  ch->slots = ch->host + HDR;
+  ch->cap = (bytes - HDR) / RECORD_BYTES;
+  std::memset(ch->host, 0, HDR + ch->cap * RECORD_BYTES);
+  cudaError_t e = cudaMemsetAsync(c->ctl + CTL_HEAD, 0, 3 * 8, c->stream);  // head, tail_cache, dropped
+  if (e == cudaSuccess) e = cudaStreamSynchronize(c->stream);
+  if (e != cudaSuccess) { delete ch; return set_error(NVBT_ECUDA, "channel reset: %s", cudaGetErrorString(e)); }
+  ch->open = true;
+  c->chan = ch;
+  *out = ch;
+  return NVBT_OK;
+}
+
+int nvbt_channel_close(nvbt_channel ch) {
+  if (!ch) return set_error(NVBT_EINVAL, "channel is null");
+  if (ch->ctx && ch->ctx->chan == ch) ch->ctx->chan = nullptr;
+  delete ch;
+  return NVBT_OK;
+}
+
+int nvbt_channel_dropped(nvbt_channel ch, uint64_t* dropped) {
+  if (!ch || !dropped) return set_error(NVBT_EINVAL, "null argument");
+  nvbt_ctx c = ch->ctx;
+  NVBT_CUDA(cudaMemcpyAsync(dropped, c->ctl + CTL_DROPPED, 8, cudaMemcpyDeviceToHost, c->stream));
+  NVBT_CUDA(cudaStreamSynchronize(c->stream));
+  return NVBT_OK;
+}
+
+int nvbt_channel_drain(nvbt_channel ch, nvbt_drain_fn fn, void* user, int64_t timeout_us, uint64_t* n_drained) {
+  if (!ch || !fn) return set_error(NVBT_EINVAL, "null argument");
+  if (!ch->open) return set_error(NVBT_ESTATE, "channel not open");
+  nvbt_ctx c = ch->ctx;
+  NVBT_CUDA(cudaSetDevice(c->device));
+  const auto t0 = std::chrono::steady_clock::now();
+  const uint64_t kBatch = 1u << 16;
+  volatile uint64_t* tail = reinterpret_cast<volatile uint64_t*>(ch->host);
+  uint64_t delivered = 0;
+  int rc = NVBT_OK;
+  for (;;) {
+    const uint64_t slot = ch->consumed % ch->cap;
+    const uint32_t lap = static_cast<uint32_t>(ch->consumed / ch->cap) + 1u;
+    const uint64_t lim = std::min<uint64_t>(ch->cap - slot, kBatch);
+    uint64_t n = 0;
+    while (n < lim) {
+      volatile const uint32_t* tag = reinterpret_cast<volatile const uint32_t*>(ch->slots + (slot + n) * RECORD_BYTES + 28);
+      if (*tag != lap) break;
+      ++n;
+    }
+    if (n) {
+      std::atomic_thread_fence(std::memory_order_acquire);
+      unsigned char* base = ch->slots + slot * RECORD_BYTES;
+      for (uint64_t r = 0; r < n; ++r) std::memset(base + r * RECORD_BYTES + 28, 0, 4);
+      const int urc = fn(base, n, user);
+      ch->consumed += n;
+      delivered += n;
+      std::atomic_thread_fence(std::memory_order_release);
+      *tail = ch->consumed;
+      if (urc) { rc = set_error(NVBT_ESTATE, "drain callback returned %d", urc); break; }
+      continue;
+    }
+    const cudaError_t q = cudaStreamQuery(c->stream);
+    if (q == cudaSuccess) {
+      uint64_t ctl[3];
+      NVBT_CUDA(cudaMemcpyAsync(ctl, c->ctl + CTL_HEAD, sizeof ctl, cudaMemcpyDeviceToHost, c->stream));
+      NVBT_CUDA(cudaStreamSynchronize(c->stream));
+      if (ch->consumed >= ctl[0]) break;  // every ticket handed out has been delivered
+      if (ctl[2] != 0) {
+        rc = set_error(NVBT_ETIMEDOUT, "%llu records dropped by producers (ring full, no consumer)",
+                       (unsigned long long)ctl[2]);
+        break;
+      }
+    } else if (q != cudaErrorNotReady) {
+      rc = set_error(NVBT_ECUDA, "stream error: %s", cudaGetErrorString(q));
+      break;
+    }
+    if (timeout_us >= 0) {
+      const auto us = std::chrono::duration_cast<std::chrono::microseconds>(std::chrono::steady_clock::now() - t0).count();
+      if (us > timeout_us) { rc = set_error(NVBT_ETIMEDOUT, "drain timed out after %lld us", (long long)us); break; }
+    }
+    for (int i = 0; i < 64; ++i) _mm_pause();
+  }
+  if (n_drained) *n_drained = delivered;
+  return rc;
+}
+
+int nvbt_drain_digest(const void* records, uint64_t n, void* user) {
+  auto* d = static_cast<nvbt_digest*>(user);
+  if (!d) return 1;
+  digest_range(static_cast<const unsigned char*>(records), n, &d->d1, &d->d2);
+  d->n_rec += n;
+  return 0;
+}
+
+int nvbt_drain_copy(const void* records, uint64_t n, void* user) {
+  auto* s = static_cast<nvbt_copy_sink*>(user);
+  if (!s || s->n + n > s->capacity) return 1;
+  std::memcpy(static_cast<unsigned char*>(s->dst) + s->n * RECORD_BYTES, records, n * RECORD_BYTES);
+  s->n += n;
+  return 0;
+}
+
+int nvbt_digest_records(const void* records, uint64_t n, nvbt_digest* out) {
+  if (!out || (!records && n)) return set_error(NVBT_EINVAL, "null argument");
+  out->n_rec = n;
+  out->d1 = out->d2 = 0;
+  digest_range(static_cast<const unsigned char*>(records), n, &out->d1, &out->d2);
+  return NVBT_OK;
+}
+
+}  // extern "C"

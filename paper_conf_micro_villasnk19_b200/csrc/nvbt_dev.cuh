@@ -1,0 +1,313 @@
+// nvbt device hook library (L0): the compiled-in analogue of NVBit's injected device functions.
+//
+// NVBit injects a call before an instruction and passes it the guard predicate, register values and
+// immediates (nvbit_insert_call / nvbit_add_call_arg, P:L123 (§4), P:L243-246 (§6.1)); "every active
+// thread enters, then leaves, the instrumentation function" (P:L307 (§7)) after a per-thread register
+// save. Here the hook is inlined at the injection point and works at warp level:
+//   * event formation (a1): A = ballot(in_flow), P = ballot(in_flow && pred), E = A & P — the
+//     "predicate matching before jumping" the paper proposes; one vote per mask.
+//   * counting (a2-a4): per-site warp-uniform counters live in REGISTERS for the whole warp (indices are
+//     compile-time pcs), i.e. the "warp-level reductions" and "radix-tree of counters, one per thread
+//     block" of P:L89: registers -> CTA shared-memory bins -> one global 64-bit atomic per non-zero bin
+//     per CTA (a8). Opcode/BB histograms are folded from per-pc bins at read time (fold kernel), which
+//     is the same integer sum regrouped (EM §2 items 2-3).
+//   * memory divergence (a5): S and L by __match_any_sync on addr>>5 / addr>>7 and a ballot of group
+//     leaders (Listing 8, readings R-2..R-8): exact integer distinct counts instead of the
+//     listing's float 1/cnt sum (R-5).
+//   * trace (a6): one 288 B record per executed global-memory event, written by the warp straight into
+//     the pinned host ring (coalesced 8 B/lane stores), committed with a tag after a system fence.
+// Precondition ("converged-hook discipline"): every hook is called by all 32 lanes of the warp
+// (lanes that have exited or are on another path pass in_flow = false).
+#pragma once
+#include <cstdint>
+#include "nvbt.h"
+
+namespace nvbt {
+
+constexpr unsigned FULL = 0xffffffffu;
+constexpr uint32_t TOOL_COUNT = NVBT_TOOL_COUNT, TOOL_BB = NVBT_TOOL_BBCOUNT, TOOL_MEM = NVBT_TOOL_MEMDIV,
+                   TOOL_TRACE = NVBT_TOOL_TRACE;
+constexpr int RECORD_BYTES = 288;
+constexpr int SITE_WORDS = 7;  // per-pc shared bins: tA, dT, wI, dW, mN, mS, mL
+
+// POD handed by value to every instrumented kernel (kernel parameter space).
+struct DevState {
+  unsigned long long* site;        // [n_pcs][4] u64: t_issued, t_exec, w_issued, w_exec
+  unsigned long long* mem;         // [n_pcs][3] u64: n, ΣS, ΣL
+  unsigned long long* hist;        // [2][33] u64: hS, hL
+  unsigned long long* pw;          // [2][n_warps] u64 or nullptr
+  unsigned char* ring;             // record slots (device view of pinned host memory) or nullptr
+  unsigned long long* head;        // tickets handed out (device memory)
+  const unsigned long long* tail;  // records consumed by the host (device view of pinned memory)
+  unsigned long long* tail_cache;  // last tail a producer saw (device memory)
+  unsigned long long* dropped;     // records given up on (device memory)
+  unsigned long long cap;          // ring slots
+  unsigned launch;
+  unsigned n_warps;
+};
+
+__device__ __forceinline__ unsigned lane_id() { unsigned l; asm("mov.u32 %0, %%laneid;" : "=r"(l)); return l; }
+__device__ __forceinline__ unsigned lanemask_lt() { unsigned m; asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m)); return m; }
+__device__ __forceinline__ unsigned long long globaltimer() {
+  unsigned long long t; asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t)); return t;
+}
+
+__host__ __device__ constexpr bool is_mem_kind(int k) { return k == NVBT_K_GLD || k == NVBT_K_GST || k == NVBT_K_GATOM; }
+
+template <class Prog> __host__ __device__ constexpr int leader_of(int pc) {
+  int p = pc;
+  while (p > 0 && !Prog::t[p].is_leader) --p;
+  return p;
+}
+template <class Prog> __host__ __device__ constexpr int bb_len(int lead) {
+  int n = 1;
+  while (lead + n < Prog::N && !Prog::t[lead + n].is_leader) ++n;
+  return n;
+}
+
+// Number of distinct keys among the lanes of E (lanes outside E may pass any key): a lane of E is its
+// group's leader when no lower lane of E has its key.
+__device__ __forceinline__ unsigned distinct(unsigned long long key, unsigned E, unsigned lanebit, unsigned lmlt) {
+  const unsigned grp = __match_any_sync(FULL, key);
+  return __popc(__ballot_sync(FULL, (E & lanebit) != 0u && (grp & E & lmlt) == 0u));
+}
+__device__ __forceinline__ unsigned umin(unsigned a, unsigned b) { return a < b ? a : b; }
+// h += (v == ref) as a predicated add.
+__device__ __forceinline__ void inc_if_eq(unsigned& h, unsigned v, unsigned ref) {
+  asm("{\n\t.reg .pred p;\n\tsetp.eq.u32 p, %1, %2;\n\t@p add.u32 %0, %0, 1;\n\t}" : "+r"(h) : "r"(v), "r"(ref));
+}
+
+// Ring reservation with backpressure. Returns false if the host never freed a slot
+// within ~2 s (or another producer already gave up): the record is dropped and counted.
+__device__ __forceinline__ bool wait_slot(const DevState& st, unsigned long long t) {
+  const unsigned long long tc = *(volatile const unsigned long long*)st.tail_cache;
+  if (t < tc + st.cap) return true;
+  if (*(volatile const unsigned long long*)st.dropped != 0) return false;
+  const unsigned long long t0 = globaltimer();
+  for (;;) {
+    const unsigned long long tl = *(volatile const unsigned long long*)st.tail;
+    if (t < tl + st.cap) { atomicMax(st.tail_cache, tl); return true; }
+    if (globaltimer() - t0 > 2000000000ull || *(volatile const unsigned long long*)st.dropped != 0) return false;
+    __nanosleep(500);
+  }
+}
+
+template <uint32_t T, class Prog>
+struct Hooks {
+  static constexpr int NPC = Prog::N;
+  static constexpr bool kOn = T != 0;
+  static constexpr bool kCount = (T & (TOOL_COUNT | TOOL_BB)) != 0;
+  static constexpr bool kBB = (T & TOOL_BB) != 0;
+  static constexpr int kSmemWords = kOn ? NPC * SITE_WORDS + 66 : 1;
+  static_assert(!((T & TOOL_COUNT) && (T & TOOL_BB)), "COUNT and BBCOUNT are exclusive");
+
+  const DevState& st;
+  unsigned* sb;
+  unsigned tA[NPC], dT[NPC], wI[NPC], dW[NPC], mN[NPC], mS[NPC], mL[NPC];
+  unsigned hS, hL;            // lane-distributed: lane l counts events with S (L) == l + 1
+  unsigned pwT, pwW;          // this warp's executed thread / warp instructions (PER_WARP)
+  unsigned seq;               // records emitted by this warp in this launch
+  unsigned lane, lane1, lanebit, lmlt, gwarp;
+
+  __device__ __forceinline__ Hooks(const DevState& s, unsigned* smem) : st(s), sb(smem) {
+    zero_range<0, NPC - 1>();
+    hS = hL = pwT = pwW = seq = 0;
+    lane = lane_id();
+    lane1 = lane + 1u;
+    lanebit = 1u << lane;
+    lmlt = lanemask_lt();
+    const unsigned tid = threadIdx.x + threadIdx.y * blockDim.x;
+    gwarp = (blockIdx.x + blockIdx.y * gridDim.x) * ((blockDim.x * blockDim.y) >> 5) + (tid >> 5);
+    if constexpr (kOn) {
+      for (int i = tid; i < kSmemWords; i += blockDim.x * blockDim.y) sb[i] = 0;
+      __syncthreads();
+    }
+  }
+
+  // Active mask of the current basic-block instance: A = lanes with in_flow (EM §1). A is the same for
+  // every pc of a basic block ("each thread will execute without change in control flow", P:L116 (§4)),
+  // so kernels take one ballot per block instance and hand it to that block's hooks.
+  struct Act { unsigned A; };
+  __device__ __forceinline__ Act active(bool in_flow) const {
+    if constexpr (kOn) return Act{__ballot_sync(FULL, in_flow)};
+    else return Act{0u};
+  }
+
+  // Injection point `PC` of the block whose active mask is `m`: pred = the lane's guard predicate
+  // (only read for guarded pcs; false for lanes outside A), addr = effective address (memory pcs).
+  template <int PC>
+  __device__ __forceinline__ void at(Act m, bool pred = true, unsigned long long addr = 0) {
+    constexpr nvbt_instr_desc d = Prog::t[PC];
+    constexpr bool mem = is_mem_kind(d.kind);
+    constexpr bool cnt = (T & TOOL_COUNT) || ((T & TOOL_BB) && (d.is_leader || d.guarded));
+    constexpr bool div = mem && (T & TOOL_MEM);
+    constexpr bool trc = mem && (T & TOOL_TRACE);
+    if constexpr (cnt || div || trc) {
+      const unsigned A = m.A;
+      const unsigned P = d.guarded ? (__ballot_sync(FULL, pred) & A) : A;
+      const unsigned E = P;
+      if constexpr (cnt) {
+        const unsigned pa = __popc(A), wa = umin(pa, 1u);
+        tA[PC] += pa;
+        wI[PC] += wa;
+        if constexpr (d.guarded) {
+          const unsigned pe = __popc(E);
+          dT[PC] += pa - pe;
+          dW[PC] += wa - umin(pe, 1u);
+        }
+      }
+      if constexpr (div || trc) {
+        if (E != 0u) {
+          if constexpr (div) {
+            const unsigned S = distinct(addr >> 5, E, lanebit, lmlt);
+            const unsigned L = distinct(addr >> 7, E, lanebit, lmlt);
+            mN[PC] += 1u; mS[PC] += S; mL[PC] += L;
+            inc_if_eq(hS, S, lane1);
+            inc_if_eq(hL, L, lane1);
+          }
+          if constexpr (trc) emit<PC>(A, P, (E & lanebit) != 0u, addr);
+        }
+      }
+    }
+  }
+
+  template <int PC>
+  __device__ __forceinline__ void emit(unsigned A, unsigned P, bool act, unsigned long long addr) {
+    constexpr nvbt_instr_desc d = Prog::t[PC];
+    unsigned long long t = 0;
+    int ok = 1;
+    if (lane == 0) { t = atomicAdd(st.head, 1ull); ok = wait_slot(st, t); }
+    t = __shfl_sync(FULL, t, 0);
+    ok = __shfl_sync(FULL, ok, 0);
+    if (!ok) {
+      if (lane == 0) atomicAdd(st.dropped, 1ull);
+    } else {
+      const unsigned long long lap = t / st.cap;
+      unsigned char* rec = st.ring + (t - lap * st.cap) * RECORD_BYTES;
+      reinterpret_cast<unsigned long long*>(rec + 32)[lane] = act ? addr : 0ull;
+      if (lane == 0)
+        *reinterpret_cast<uint4*>(rec) = make_uint4(st.launch, gwarp, seq, (unsigned)PC);
+      __syncwarp();
+      if (lane == 0) {
+        __threadfence_system();
+        const unsigned w2 = (unsigned)d.opcode | ((unsigned)d.width << 16) | ((unsigned)d.kind << 24);
+        asm volatile("st.volatile.global.v4.u32 [%0], {%1, %2, %3, %4};" ::"l"(rec + 16), "r"(A), "r"(P), "r"(w2),
+                     "r"((unsigned)lap + 1u)
+                     : "memory");
+      }
+    }
+    ++seq;
+  }
+
+  // executed-instruction totals of pc range [LO, HI] (for PER_WARP), BB-derived where needed
+  template <int PC>
+  __device__ __forceinline__ void texe(unsigned& t, unsigned& w) const {
+    constexpr nvbt_instr_desc d = Prog::t[PC];
+    if constexpr ((T & TOOL_COUNT) || d.is_leader || d.guarded) {
+      t += tA[PC] - dT[PC];
+      w += wI[PC] - dW[PC];
+    } else if constexpr (kBB) {
+      constexpr int L = leader_of<Prog>(PC);
+      t += tA[L];
+      w += wI[L];
+    }
+  }
+
+  // Moves the register counters of pcs [LO, HI] into the CTA's shared bins (lane-parallel: lane l takes
+  // pc LO + 32r + l) and zeroes them, freeing their registers. In BB mode [LO, HI] must be whole blocks.
+  template <int LO, int HI>
+  __device__ __forceinline__ void retire() {
+    if constexpr (kOn) {
+      static_assert(LO >= 0 && HI < NPC && LO <= HI, "bad range");
+      static_assert(!kBB || (Prog::t[LO].is_leader && (HI + 1 == NPC || Prog::t[HI + 1].is_leader)),
+                    "BB mode retires whole blocks");
+      if constexpr (kCount) {
+        unsigned t = 0, w = 0;
+        retire_sum<LO, HI>(t, w);
+        pwT += t; pwW += w;
+      }
+      retire_round<LO, HI, LO>();
+      zero_range<LO, HI>();
+    }
+  }
+
+  template <int LO, int HI, int BASE>
+  __device__ __forceinline__ void retire_round() {
+    if constexpr (BASE <= HI) {
+      unsigned v[SITE_WORDS] = {0, 0, 0, 0, 0, 0, 0};
+      select_lane<BASE, (HI < BASE + 31 ? HI : BASE + 31), BASE>(v);
+      if (BASE + (int)lane <= HI) {
+        const int pc = BASE + (int)lane;
+#pragma unroll
+        for (int k = 0; k < SITE_WORDS; ++k)
+          if (v[k]) atomicAdd(&sb[pc * SITE_WORDS + k], v[k]);
+      }
+      retire_round<LO, HI, BASE + 32>();
+    }
+  }
+
+  template <int PC, int END, int BASE>
+  __device__ __forceinline__ void select_lane(unsigned (&v)[SITE_WORDS]) const {
+    if constexpr (PC <= END) {
+      const bool me = lane == (unsigned)(PC - BASE);
+      v[0] = me ? tA[PC] : v[0]; v[1] = me ? dT[PC] : v[1]; v[2] = me ? wI[PC] : v[2]; v[3] = me ? dW[PC] : v[3];
+      v[4] = me ? mN[PC] : v[4]; v[5] = me ? mS[PC] : v[5]; v[6] = me ? mL[PC] : v[6];
+      select_lane<PC + 1, END, BASE>(v);
+    }
+  }
+
+  template <int LO, int HI>
+  __device__ __forceinline__ void zero_range() {
+    if constexpr (LO <= HI) {
+      tA[LO] = dT[LO] = wI[LO] = dW[LO] = mN[LO] = mS[LO] = mL[LO] = 0;
+      zero_range<LO + 1, HI>();
+    }
+  }
+
+  template <int LO, int HI>
+  __device__ __forceinline__ void retire_sum(unsigned& t, unsigned& w) const {
+    if constexpr (LO <= HI) {
+      texe<LO>(t, w);
+      retire_sum<LO + 1, HI>(t, w);
+    }
+  }
+
+  // CTA epilogue (nvbt_cta_flush): registers -> shared bins -> one global atomic per non-zero bin.
+  // Must be reached by every thread of the CTA.
+  __device__ __forceinline__ void finish() {
+    if constexpr (kOn) {
+      retire<0, NPC - 1>();
+      if (hS) atomicAdd(&sb[NPC * SITE_WORDS + 1 + lane], hS);
+      if (hL) atomicAdd(&sb[NPC * SITE_WORDS + 34 + lane], hL);
+      if constexpr (kCount) {
+        if (st.pw != nullptr && lane == 0 && gwarp < st.n_warps) {
+          atomicAdd(st.pw + gwarp, (unsigned long long)pwT);
+          atomicAdd(st.pw + st.n_warps + gwarp, (unsigned long long)pwW);
+        }
+      }
+      __syncthreads();
+      const int tid = threadIdx.x + threadIdx.y * blockDim.x;
+      const int nt = blockDim.x * blockDim.y;
+      for (int pc = tid; pc < NPC; pc += nt) {
+        const unsigned* b = sb + pc * SITE_WORDS;
+        if (b[0] | b[2]) {
+          unsigned long long* s = st.site + 4 * pc;
+          atomicAdd(s + 0, (unsigned long long)b[0]);
+          if (b[0] - b[1]) atomicAdd(s + 1, (unsigned long long)(b[0] - b[1]));
+          atomicAdd(s + 2, (unsigned long long)b[2]);
+          if (b[2] - b[3]) atomicAdd(s + 3, (unsigned long long)(b[2] - b[3]));
+        }
+        if (b[4]) {
+          unsigned long long* m = st.mem + 3 * pc;
+          atomicAdd(m + 0, (unsigned long long)b[4]);
+          atomicAdd(m + 1, (unsigned long long)b[5]);
+          atomicAdd(m + 2, (unsigned long long)b[6]);
+        }
+      }
+      for (int i = tid; i < 66; i += nt)
+        if (sb[NPC * SITE_WORDS + i]) atomicAdd(st.hist + i, (unsigned long long)sb[NPC * SITE_WORDS + i]);
+    }
+  }
+};
+
+}  // namespace nvbt

@@ -1,0 +1,315 @@
+// Trace-replay mode (a7) and its counter-based event generator (EM §3.5), plus nvbt_program().
+//
+// Replay applies EM §2 items 1-4 to an HBM-resident stream of 16 B event headers and 256 B address
+// slots. It is HBM-bound: the algorithmic bytes are 16 per header plus 256 per executed memory event
+// (the only slots that must be read). Layout of the work:
+//   * persistent grid (2 CTAs x 512 threads per SM), each warp strides over 32-event tiles; lane l owns
+//     header tile*32+l (one 16 B non-coherent load per lane = 512 B coalesced per warp);
+//   * per-pc counters are privatised per CTA in shared memory (u32; t_issued, w_issued and the two
+//     "predicated-off" deltas that only exist when E != A) and folded into the global u64 bins once per
+//     CTA at the end (a8);
+//   * executed memory events of the tile (ballot) are processed by the whole warp: the 256 B slot is
+//     read by 32 lanes (8 B each, coalesced), S/L come from two __match_any_sync + leader ballots, the
+//     S/L histograms live in lane-distributed registers (lane l counts S == l + 1).
+#include <cstring>
+
+#include "nvbt_internal.h"
+#include "nvbt_workloads.h"
+#include "programs.cuh"
+
+namespace nvbt {
+
+// ---------------------------------------------------------------- generator (EM §3.5)
+constexpr unsigned long long kSeed = 0x4E5642544E564254ull;
+constexpr unsigned long long kFStep = 0xD1B54A32D192ED03ull;
+
+__host__ __device__ __forceinline__ unsigned long long mix64(unsigned long long z) {
+  z += 0x9E3779B97F4A7C15ull;
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  return z ^ (z >> 31);
+}
+__host__ __device__ __forceinline__ unsigned long long Kf(unsigned long long seed, unsigned long long f) {
+  return mix64(seed ^ (f * kFStep));
+}
+
+struct GenConsts {
+  unsigned long long k[9];  // K(0..8); K(64 + lane) is computed per lane
+  unsigned long long seed;
+};
+
+__global__ void __launch_bounds__(256) k_gen(GenConsts G, unsigned long long first, unsigned long long n,
+                                             const uint8_t* __restrict__ kind, const nvbt_instr_desc* __restrict__ prog,
+                                             uint4* __restrict__ hdr, unsigned long long* __restrict__ addr) {
+  const unsigned lane = lane_id();
+  const unsigned long long klane = Kf(G.seed, 64 + lane);
+  const unsigned long long warps = (unsigned long long)gridDim.x * (blockDim.x >> 5);
+  for (unsigned long long tile = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; tile * 32 < n; tile += warps) {
+    const unsigned long long li = tile * 32 + lane;
+    const bool valid = li < n;
+    const unsigned long long i = first + li;
+    const unsigned pc = (unsigned)(mix64(G.k[0] ^ i) & 4095ull);
+    const unsigned warp = (unsigned)(mix64(G.k[1] ^ i) & ((1ull << 20) - 1));
+    unsigned A = (mix64(G.k[2] ^ i) % 4 != 0) ? 0xffffffffu : (unsigned)mix64(G.k[3] ^ i);
+    if (A == 0) A = 1;
+    const unsigned P = (mix64(G.k[4] ^ i) % 8 < 6) ? 0xffffffffu : (unsigned)mix64(G.k[5] ^ i);
+    if (valid) hdr[li] = make_uint4(pc, warp, A, P);
+    const bool mem = valid && is_mem_kind(kind[pc]);
+    unsigned pat = 0;
+    unsigned long long base = 0, s = 0;
+    if (mem) {
+      pat = (unsigned)(mix64(G.k[6] ^ i) % 6);
+      base = (mix64(G.k[7] ^ i) & ((1ull << 40) - 1)) & ~127ull;
+      s = mix64(G.k[8] ^ i);
+    }
+    unsigned mm = __ballot_sync(FULL, mem);
+    while (mm) {
+      const int src = __ffs(mm) - 1;
+      mm &= mm - 1;
+      const unsigned long long is = __shfl_sync(FULL, i, src);
+      const unsigned ps = __shfl_sync(FULL, pc, src);
+      const unsigned pt = __shfl_sync(FULL, pat, src);
+      const unsigned long long b = __shfl_sync(FULL, base, src);
+      const unsigned long long ss = __shfl_sync(FULL, s, src);
+      const unsigned long long wd = prog[ps].width;
+      const unsigned long long r = mix64(klane ^ is);
+      unsigned long long a;
+      switch (pt) {
+        case 0: a = b + lane * wd; break;
+        case 1: a = b + lane * (wd << (ss % 10)); break;
+        case 2: a = b; break;
+        case 3: a = b + (r % (4096 / wd)) * wd; break;
+        case 4: a = (r & ((1ull << 40) - 1)) & ~(wd - 1); break;
+        default: a = b + (lane ^ (unsigned)(ss & 31)) * wd; break;
+      }
+      addr[(tile * 32 + src) * 32 + lane] = a;
+    }
+  }
+}
+
+// ---------------------------------------------------------------- replay
+constexpr int RP_THREADS = 512;
+constexpr int RP_BATCH = 4;  // memory events whose slots are loaded before processing
+
+__device__ __forceinline__ uint4 ld_nc_v4(const uint4* p) {
+  uint4 r;
+  asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ unsigned long long ld_nc_u64(const unsigned long long* p) {
+  unsigned long long r;
+  asm volatile("ld.global.nc.L1::no_allocate.u64 %0, [%1];" : "=l"(r) : "l"(p));
+  return r;
+}
+
+__global__ void __launch_bounds__(RP_THREADS, 2)
+k_replay(const uint4* __restrict__ hdr, const unsigned long long* __restrict__ addr, unsigned long long n, unsigned P,
+         const uint8_t* __restrict__ kind, DevState st, unsigned long long* err) {
+  extern __shared__ unsigned sm[];
+  unsigned* sA = sm;            // t_issued
+  unsigned* sW = sm + P;        // w_issued
+  unsigned* sDT = sm + 2 * P;   // popc(A & ~E)
+  unsigned* sDW = sm + 3 * P;   // [A != 0 && E == 0]
+  unsigned* sS = sm + 4 * P;
+  unsigned* sL = sm + 5 * P;
+  unsigned* sH = sm + 6 * P;    // hS[33], hL[33]
+  uint8_t* sK = reinterpret_cast<uint8_t*>(sm + 6 * P + 66);
+  for (unsigned i = threadIdx.x; i < 6 * P + 66; i += blockDim.x) sm[i] = 0;
+  for (unsigned i = threadIdx.x; i < P; i += blockDim.x) sK[i] = is_mem_kind(kind[i]);
+  __syncthreads();
+
+  const unsigned lane = lane_id(), lmlt = lanemask_lt(), lanebit = 1u << lane;
+  unsigned hS = 0, hL = 0;
+  unsigned bad = 0;
+  const unsigned long long warps = (unsigned long long)gridDim.x * (blockDim.x >> 5);
+  unsigned long long tile = (blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x) >> 5;
+  uint4 h = make_uint4(0, 0, 0, 0);
+  if (tile * 32 + lane < n) h = ld_nc_v4(hdr + tile * 32 + lane);
+  for (; tile * 32 < n; tile += warps) {
+    const bool valid = tile * 32 + lane < n;
+    const unsigned pc = h.x, A = h.z, E = h.z & h.w, warp = h.y;
+    // prefetch the next tile's header
+    const unsigned long long nt = tile + warps;
+    uint4 hn = make_uint4(0, 0, 0, 0);
+    if (nt * 32 + lane < n) hn = ld_nc_v4(hdr + nt * 32 + lane);
+    const bool ok = valid && pc < P && A != 0u;
+    bad += valid && pc >= P;
+    if (ok) {
+      atomicAdd(&sA[pc], (unsigned)__popc(A));
+      atomicAdd(&sW[pc], 1u);
+      if (E != A) {
+        atomicAdd(&sDT[pc], (unsigned)__popc(A ^ E));
+        if (E == 0u) atomicAdd(&sDW[pc], 1u);
+      }
+      if (st.pw != nullptr && warp < st.n_warps) {
+        atomicAdd(st.pw + warp, (unsigned long long)__popc(E));
+        if (E) atomicAdd(st.pw + st.n_warps + warp, 1ull);
+      }
+    }
+    unsigned mm = __ballot_sync(FULL, ok && E != 0u && sK[ok ? pc : 0]);
+    while (mm) {
+      int src[RP_BATCH];
+      unsigned long long a[RP_BATCH];
+#pragma unroll
+      for (int b = 0; b < RP_BATCH; ++b) {
+        src[b] = mm ? __ffs(mm) - 1 : -1;
+        if (mm) mm &= mm - 1;
+        if (src[b] >= 0) a[b] = ld_nc_u64(addr + (tile * 32 + src[b]) * 32 + lane);
+      }
+#pragma unroll
+      for (int b = 0; b < RP_BATCH; ++b) {
+        if (src[b] < 0) break;
+        const unsigned es = __shfl_sync(FULL, E, src[b]);
+        const unsigned ps = __shfl_sync(FULL, pc, src[b]);
+        const unsigned S = distinct(a[b] >> 5, es, lanebit, lmlt);
+        const unsigned L = distinct(a[b] >> 7, es, lanebit, lmlt);
+        if (lane == 0) { atomicAdd(&sS[ps], S); atomicAdd(&sL[ps], L); }
+        inc_if_eq(hS, S, lane + 1u);
+        inc_if_eq(hL, L, lane + 1u);
+      }
+    }
+    h = hn;
+  }
+  if (hS) atomicAdd(&sH[1 + lane], hS);
+  if (hL) atomicAdd(&sH[34 + lane], hL);
+  bad = __reduce_add_sync(FULL, bad);
+  if (lane == 0 && bad) atomicAdd(err, (unsigned long long)bad);
+  __syncthreads();
+  for (unsigned pc = threadIdx.x; pc < P; pc += blockDim.x) {
+    const unsigned a = sA[pc], w = sW[pc];
+    if (w) {
+      unsigned long long* s = st.site + 4 * pc;
+      atomicAdd(s + 0, (unsigned long long)a);
+      atomicAdd(s + 1, (unsigned long long)(a - sDT[pc]));
+      atomicAdd(s + 2, (unsigned long long)w);
+      atomicAdd(s + 3, (unsigned long long)(w - sDW[pc]));
+      if (sK[pc] && w != sDW[pc]) {
+        unsigned long long* m = st.mem + 3 * pc;
+        atomicAdd(m + 0, (unsigned long long)(w - sDW[pc]));
+        atomicAdd(m + 1, (unsigned long long)sS[pc]);
+        atomicAdd(m + 2, (unsigned long long)sL[pc]);
+      }
+    }
+  }
+  for (unsigned i = threadIdx.x; i < 66; i += blockDim.x)
+    if (sH[i]) atomicAdd(st.hist + i, (unsigned long long)sH[i]);
+}
+
+static int g_sms = 0;
+static int sm_count(int dev) {
+  if (g_sms == 0) cudaDeviceGetAttribute(&g_sms, cudaDevAttrMultiProcessorCount, dev);
+  return g_sms > 0 ? g_sms : 148;
+}
+
+static size_t replay_smem(unsigned P) { return (6ull * P + 66) * 4 + P + 16; }
+
+}  // namespace nvbt
+
+using namespace nvbt;
+
+extern "C" {
+
+int nvbt_program(int w, nvbt_instr_desc* out, uint32_t cap, uint32_t* n_pcs, uint32_t* n_ops, uint32_t* n_bbs) {
+  const nvbt_instr_desc* t = nullptr;
+  uint32_t n = 0, o = kWorkloadOpcodes, b = 0;
+  static nvbt_instr_desc replay_prog[4096];
+  static bool replay_built = false;
+  switch (w) {
+    case NVBT_W_VECTORADD: t = ProgVectorAdd::t; n = ProgVectorAdd::N; break;
+    case NVBT_W_SGEMM: t = ProgSgemm::t; n = ProgSgemm::N; break;
+    case NVBT_W_BFS: t = ProgBfs::t; n = ProgBfs::N; break;
+    case NVBT_W_STENCIL: t = ProgStencil::t; n = ProgStencil::N; break;
+    case NVBT_W_REPLAY:
+      if (!replay_built) {  // EM §3.5, always from the constant SEED
+        const unsigned long long k100 = Kf(kSeed, 100);
+        for (uint32_t pc = 0; pc < 4096; ++pc) {
+          const unsigned long long h = mix64(k100 ^ pc);
+          nvbt_instr_desc d{};
+          d.bb = pc >> 3;
+          d.is_leader = (pc & 7) == 0;
+          d.guarded = 1;
+          if (h % 4 == 0) {
+            d.kind = ((h >> 8) & 1) ? NVBT_K_GST : NVBT_K_GLD;
+            d.width = (uint8_t)(4u << ((h >> 16) % 3));
+            d.opcode = d.kind == NVBT_K_GLD ? 0 : 1;
+          } else {
+            d.kind = (pc & 7) == 7 ? NVBT_K_CTRL : NVBT_K_ALU;
+            d.width = 0;
+            d.opcode = (uint16_t)(2 + (h >> 24) % 62);
+          }
+          replay_prog[pc] = d;
+        }
+        replay_built = true;
+      }
+      t = replay_prog; n = 4096; o = 64;
+      break;
+    default: return set_error(NVBT_EINVAL, "unknown workload %d", w);
+  }
+  for (uint32_t i = 0; i < n; ++i) b = t[i].bb + 1 > b ? t[i].bb + 1 : b;
+  if (n_pcs) *n_pcs = n;
+  if (n_ops) *n_ops = o;
+  if (n_bbs) *n_bbs = b;
+  if (out) {
+    if (cap < n) return set_error(NVBT_EINVAL, "program has %u pcs, cap %u", n, cap);
+    std::memcpy(out, t, sizeof(nvbt_instr_desc) * n);
+  }
+  return NVBT_OK;
+}
+
+int nvbt_gen_events(nvbt_ctx c, uint64_t seed, uint64_t first, uint64_t n, void* d_hdr, void* d_addr) {
+  if (!c || !d_hdr || !d_addr) return set_error(NVBT_EINVAL, "null argument");
+  if ((reinterpret_cast<uintptr_t>(d_hdr) | reinterpret_cast<uintptr_t>(d_addr)) % 16)
+    return set_error(NVBT_EINVAL, "stream buffers must be 16-byte aligned");
+  nvbt_instr_desc prog[4096];
+  uint32_t np = 0;
+  int rc = nvbt_program(NVBT_W_REPLAY, prog, 4096, &np, nullptr, nullptr);
+  if (rc) return rc;
+  rc = check_program(c, prog, (int)np, "replay");
+  if (rc) return rc;
+  if (n == 0) return NVBT_OK;
+  NVBT_CUDA(cudaSetDevice(c->device));
+  GenConsts G;
+  G.seed = seed;
+  for (int f = 0; f < 9; ++f) G.k[f] = Kf(seed, f);
+  const unsigned long long tiles = (n + 31) / 32;
+  const int blocks = (int)std::min<unsigned long long>((tiles + 7) / 8, (unsigned long long)sm_count(c->device) * 8);
+  k_gen<<<blocks, 256, 0, c->stream>>>(G, first, n, c->d_kind, c->d_prog, static_cast<uint4*>(d_hdr),
+                                       static_cast<unsigned long long*>(d_addr));
+  NVBT_CUDA(cudaGetLastError());
+  c->launches++;
+  return NVBT_OK;
+}
+
+int nvbt_replay(nvbt_ctx c, const void* d_hdr, const void* d_addr, uint64_t n) {
+  if (!c || !d_hdr || !d_addr) return set_error(NVBT_EINVAL, "null argument");
+  if ((reinterpret_cast<uintptr_t>(d_hdr) | reinterpret_cast<uintptr_t>(d_addr)) % 16)
+    return set_error(NVBT_EINVAL, "stream buffers must be 16-byte aligned");
+  if (!(c->flags & (NVBT_COUNT | NVBT_OPHIST | NVBT_BB))) return set_error(NVBT_ESTATE, "replay needs NVBT_COUNT");
+  DevState st;
+  int rc = make_state(c, NVBT_TOOL_COUNT | ((c->flags & NVBT_MEMDIV) ? NVBT_TOOL_MEMDIV : 0), &st);
+  if (rc) return rc;
+  if (n == 0) return NVBT_OK;
+  NVBT_CUDA(cudaSetDevice(c->device));
+  const size_t smem = replay_smem(c->n_pcs);
+  static bool attr_set = false;
+  if (!attr_set) {
+    NVBT_CUDA(cudaFuncSetAttribute(k_replay, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)replay_smem(4096)));
+    attr_set = true;
+  }
+  const unsigned long long kMaxPerLaunch = 1ull << 30;  // keeps every CTA's u32 bins far from overflow
+  const int sms = sm_count(c->device);
+  for (uint64_t off = 0; off < n; off += kMaxPerLaunch) {
+    const uint64_t m = std::min<uint64_t>(kMaxPerLaunch, n - off);
+    const unsigned long long tiles = (m + 31) / 32;
+    const int blocks = (int)std::min<unsigned long long>((tiles + 15) / 16, (unsigned long long)sms * 2);
+    k_replay<<<blocks, RP_THREADS, smem, c->stream>>>(static_cast<const uint4*>(d_hdr) + off,
+                                                      static_cast<const unsigned long long*>(d_addr) + off * 32, m,
+                                                      c->n_pcs, c->d_kind, st, c->ctl + CTL_REPLAY_ERR);
+    NVBT_CUDA(cudaGetLastError());
+    c->launches++;
+  }
+  return NVBT_OK;
+}
+
+}  // extern "C"

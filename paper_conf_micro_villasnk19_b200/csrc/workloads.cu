@@ -1,0 +1,324 @@
+// Synthetic workloads with compiled-in injection points (C1-C4; EM §3.1-3.4) and their launchers.
+//
+// Each kernel is written once, in the "converged-hook discipline": lanes never return early; a lane
+// that "exits" or is on the other side of a branch keeps running with in_flow = false, so every hook is
+// reached by all 32 lanes and A/P are exact ballots (EM §1, reading R-15). Loops whose trip count
+// varies per lane run warp-uniformly to the warp's maximum (SIMT-stack / IPDOM semantics). The
+// template parameter T selects the instrumentation variant; T = 0 is the uninstrumented baseline.
+#include <type_traits>
+
+#include "nvbt_internal.h"
+#include "nvbt_workloads.h"
+#include "programs.cuh"
+
+namespace nvbt {
+
+template <class Prog> struct ProgTraits;
+
+// ---------------------------------------------------------------- C1 vectorAdd (§3.1)
+template <uint32_t T>
+__global__ void __launch_bounds__(256) k_vectoradd(const float* __restrict__ a, const float* __restrict__ b,
+                                                   float* __restrict__ c, int N, DevState st) {
+  __shared__ unsigned sb[Hooks<T, ProgVectorAdd>::kSmemWords];
+  Hooks<T, ProgVectorAdd> h(st, sb);
+  const auto m0 = h.active(true);              // BB0: every lane
+  const int tid = threadIdx.x;                 h.template at<0>(m0);
+  const int cta = blockIdx.x;                  h.template at<1>(m0);
+  const int i = cta * 256 + tid;               h.template at<2>(m0);
+  const bool p0 = i >= N;                      h.template at<3>(m0);
+                                               h.template at<4>(m0, p0);  // @P0 EXIT
+  const bool live = !p0;
+  const auto m1 = h.active(live);              // BB1: lanes that did not exit
+  const float* pa = a + i;                     h.template at<5>(m1);
+  const float* pb = b + i;                     h.template at<6>(m1);
+  float x = 0.f, y = 0.f;
+  if (live) x = *pa;                           h.template at<7>(m1, true, (unsigned long long)pa);
+  if (live) y = *pb;                           h.template at<8>(m1, true, (unsigned long long)pb);
+  float* pc = c + i;                           h.template at<9>(m1);
+  const float z = __fadd_rn(x, y);             h.template at<10>(m1);
+  if (live) *pc = z;                           h.template at<11>(m1, true, (unsigned long long)pc);
+                                               h.template at<12>(m1);
+  h.finish();
+}
+
+// ---------------------------------------------------------------- C2 naive SGEMM (§3.2)
+template <uint32_t T>
+__global__ void __launch_bounds__(256) k_sgemm(const float* __restrict__ A, const float* __restrict__ B,
+                                               float* __restrict__ C, int M, int N, int K, DevState st) {
+  __shared__ unsigned sb[Hooks<T, ProgSgemm>::kSmemWords];
+  Hooks<T, ProgSgemm> h(st, sb);
+  const auto m0 = h.active(true);
+  const int tx = threadIdx.x;                  h.template at<0>(m0);
+  const int ty = threadIdx.y;                  h.template at<1>(m0);
+  const int bx = blockIdx.x;                   h.template at<2>(m0);
+  const int by = blockIdx.y;                   h.template at<3>(m0);
+  const int row = bx * 32 + tx;                h.template at<4>(m0);
+  const int col = by * 8 + ty;                 h.template at<5>(m0);
+  const bool p0 = row >= M || col >= N;        h.template at<6>(m0);
+                                               h.template at<7>(m0, p0);  // @P0 EXIT
+  const bool live = !p0;
+  // BB1, every BB2 instance and BB3 have the same active mask (the lanes that did not exit): K is
+  // warp-uniform, so the loop runs K times for every live lane.
+  const auto m1 = h.active(live);
+  float acc = 0.f;                             h.template at<8>(m1);
+                                               h.template at<9>(m1);
+  h.template retire<0, 9>();
+  if (__any_sync(FULL, live)) {
+    const float* pa = A + (size_t)row * K;
+    const float* pb = B + col;
+    for (int k = 0; k < K; ++k) {
+      float x = 0.f, y = 0.f;
+      if (live) x = pa[k];                     h.template at<10>(m1, true, (unsigned long long)(pa + k));
+      if (live) y = pb[(size_t)k * N];         h.template at<11>(m1, true, (unsigned long long)(pb + (size_t)k * N));
+      acc = fmaf(x, y, acc);                   h.template at<12>(m1);
+                                               h.template at<13>(m1);
+                                               h.template at<14>(m1);
+                                               h.template at<15>(m1, k + 1 < K);  // @P1 BRA
+    }
+  }
+  float* pc = C + (size_t)row * N + col;
+  if (live) *pc = acc;                         h.template at<16>(m1, true, (unsigned long long)pc);
+                                               h.template at<17>(m1);
+  h.finish();
+}
+
+// ---------------------------------------------------------------- C3 BFS (§3.3)
+template <uint32_t T>
+__global__ void __launch_bounds__(256) k_bfs_expand(const int* __restrict__ rowptr, const int* __restrict__ colidx,
+                                                    int n, unsigned char* mask, const unsigned char* __restrict__ visited,
+                                                    unsigned char* updating, DevState st) {
+  __shared__ unsigned sb[Hooks<T, ProgBfs>::kSmemWords];
+  Hooks<T, ProgBfs> h(st, sb);
+  const auto m0 = h.active(true);
+  const int tid = threadIdx.x;                 h.template at<0>(m0);
+  const int cta = blockIdx.x;                  h.template at<1>(m0);
+  const int t = cta * 256 + tid;               h.template at<2>(m0);
+  const bool p0 = t >= n;                      h.template at<3>(m0);
+                                               h.template at<4>(m0, p0);  // @P0 EXIT
+  const bool live = !p0;
+  const auto m1 = h.active(live);              // BB1 (and BB6 after reconvergence)
+  unsigned char mk = 0;
+  if (live) mk = mask[t];                      h.template at<5>(m1, true, (unsigned long long)(mask + t));
+  const bool p1 = mk != 0;                     h.template at<6>(m1);
+                                               h.template at<7>(m1, !p1);  // @!P1 BRA exit
+  const bool front = live && p1;
+  h.template retire<0, 7>();
+  const auto m2 = h.active(front);             // BB2: frontier lanes
+  int start = 0, end = 0;
+  if (front) mask[t] = 0;                      h.template at<8>(m2, true, (unsigned long long)(mask + t));
+  if (front) start = rowptr[t];                h.template at<9>(m2, true, (unsigned long long)(rowptr + t));
+  if (front) end = rowptr[t + 1];              h.template at<10>(m2, true, (unsigned long long)(rowptr + t + 1));
+  const bool p2 = start >= end;                h.template at<11>(m2);
+                                               h.template at<12>(m2, p2);  // @P2 BRA exit
+  h.template retire<8, 12>();
+  bool in_loop = front && !p2;
+  int e = start;
+  while (__any_sync(FULL, in_loop)) {          // warp-uniform edge loop; instance k has e = start + k
+    const auto m3 = h.active(in_loop);         // BB3 and BB5 of this instance
+    int nb = 0;
+    if (in_loop) nb = colidx[e];               h.template at<13>(m3, true, (unsigned long long)(colidx + e));
+    unsigned char v = 0;
+    if (in_loop) v = visited[nb];              h.template at<14>(m3, true, (unsigned long long)(visited + nb));
+    const bool p3 = v != 0;                    h.template at<15>(m3);
+                                               h.template at<16>(m3, p3);  // @P3 BRA
+    const bool unv = in_loop && !p3;
+    const auto m4 = h.active(unv);             // BB4: unvisited neighbour
+    if (unv) updating[nb] = 1;                 h.template at<17>(m4, true, (unsigned long long)(updating + nb));
+    const int e1 = e + 1;                      h.template at<18>(m3);
+    const bool p4 = e1 < end;                  h.template at<19>(m3);
+                                               h.template at<20>(m3, p4);  // @P4 BRA loop
+    if (in_loop) e = e1;
+    in_loop = in_loop && p4;
+  }
+                                               h.template at<21>(m1);
+  h.finish();
+}
+
+template <uint32_t T>
+__global__ void __launch_bounds__(256) k_bfs_update(int n, unsigned char* mask, unsigned char* visited,
+                                                    unsigned char* updating, int* cost, int* over, int level,
+                                                    DevState st) {
+  __shared__ unsigned sb[Hooks<T, ProgBfs>::kSmemWords];
+  Hooks<T, ProgBfs> h(st, sb);
+  const auto m0 = h.active(true);
+  const int tid = threadIdx.x;                 h.template at<22>(m0);
+  const int cta = blockIdx.x;                  h.template at<23>(m0);
+  const int t = cta * 256 + tid;               h.template at<24>(m0);
+  const bool p0 = t >= n;                      h.template at<25>(m0);
+                                               h.template at<26>(m0, p0);
+  const bool live = !p0;
+  const auto m1 = h.active(live);              // BB8 (and BB10)
+  unsigned char u = 0;
+  if (live) u = updating[t];                   h.template at<27>(m1, true, (unsigned long long)(updating + t));
+  const bool p1 = u != 0;                      h.template at<28>(m1);
+                                               h.template at<29>(m1, !p1);
+  const bool up = live && p1;
+  const auto m2 = h.active(up);                // BB9
+  if (up) mask[t] = 1;                         h.template at<30>(m2, true, (unsigned long long)(mask + t));
+  if (up) visited[t] = 1;                      h.template at<31>(m2, true, (unsigned long long)(visited + t));
+  if (up) cost[t] = level + 1;                 h.template at<32>(m2, true, (unsigned long long)(cost + t));
+  if (up) updating[t] = 0;                     h.template at<33>(m2, true, (unsigned long long)(updating + t));
+  if (up) *over = 1;                           h.template at<34>(m2, true, (unsigned long long)over);
+                                               h.template at<35>(m1);
+  h.finish();
+}
+
+// ---------------------------------------------------------------- C4 5-point stencil (§3.4)
+template <uint32_t T>
+__global__ void __launch_bounds__(256) k_stencil(const float* __restrict__ in, float* __restrict__ out, int n,
+                                                 DevState st) {
+  __shared__ unsigned sb[Hooks<T, ProgStencil>::kSmemWords];
+  Hooks<T, ProgStencil> h(st, sb);
+  const auto m0 = h.active(true);
+  const int tx = threadIdx.x;                  h.template at<0>(m0);
+  const int ty = threadIdx.y;                  h.template at<1>(m0);
+  const int bx = blockIdx.x;                   h.template at<2>(m0);
+  const int by = blockIdx.y;                   h.template at<3>(m0);
+  const int j = bx * 32 + tx;                  h.template at<4>(m0);
+  const int i = by * 8 + ty;                   h.template at<5>(m0);
+  const bool p0 = i >= n || j >= n;            h.template at<6>(m0);
+                                               h.template at<7>(m0, p0);
+  const bool live = !p0;
+  const auto m1 = h.active(live);              // BB1 (boundaries are predicated, not branched)
+  const bool p1 = live && i > 0 && i < n - 1 && j > 0 && j < n - 1;
+                                               h.template at<8>(m1);
+  const size_t o = (size_t)i * n + j;
+  float c = 0.f, u = 0.f, d = 0.f, l = 0.f, r = 0.f;
+  if (live) c = in[o];                         h.template at<9>(m1, true, (unsigned long long)(in + o));
+  if (p1) u = in[o - n];                       h.template at<10>(m1, p1, (unsigned long long)(in + o - n));
+  if (p1) d = in[o + n];                       h.template at<11>(m1, p1, (unsigned long long)(in + o + n));
+  if (p1) l = in[o - 1];                       h.template at<12>(m1, p1, (unsigned long long)(in + o - 1));
+  if (p1) r = in[o + 1];                       h.template at<13>(m1, p1, (unsigned long long)(in + o + 1));
+  float s = __fadd_rn(u, d);                   h.template at<14>(m1, p1);
+  s = __fadd_rn(s, l);                         h.template at<15>(m1, p1);
+  s = __fadd_rn(s, r);                         h.template at<16>(m1, p1);
+  s = __fmul_rn(0.25f, s);                     h.template at<17>(m1, p1);
+  const float v = p1 ? s : c;                  h.template at<18>(m1);
+  if (live) out[o] = v;                        h.template at<19>(m1, true, (unsigned long long)(out + o));
+                                               h.template at<20>(m1);
+  h.finish();
+}
+
+// ---------------------------------------------------------------- dispatch over tool variants
+template <class F>
+static int dispatch(uint32_t tools, F&& f) {
+#define NVBT_CASE(v) case v: f(std::integral_constant<uint32_t, v>{}); return NVBT_OK;
+  switch (tools) {
+    NVBT_CASE(0) NVBT_CASE(1) NVBT_CASE(2) NVBT_CASE(4) NVBT_CASE(5) NVBT_CASE(6) NVBT_CASE(8) NVBT_CASE(9)
+    NVBT_CASE(10) NVBT_CASE(12) NVBT_CASE(13) NVBT_CASE(14)
+    default: return set_error(NVBT_EINVAL, "unsupported tools combination 0x%x", tools);
+  }
+#undef NVBT_CASE
+}
+
+struct LaunchCtx {
+  cudaStream_t stream = nullptr;
+  DevState st{};
+};
+
+template <class Prog>
+static int prepare(nvbt_ctx ctx, void* stream, uint32_t tools, const char* name, LaunchCtx* lc) {
+  if (tools != 0) {
+    if (!ctx) return set_error(NVBT_EINVAL, "instrumented launch needs a context");
+    int rc = check_program(ctx, Prog::t, Prog::N, name);
+    if (rc) return rc;
+    rc = make_state(ctx, tools, &lc->st);
+    if (rc) return rc;
+    lc->stream = ctx->stream;
+    NVBT_CUDA(cudaSetDevice(ctx->device));
+  } else {
+    lc->stream = ctx ? ctx->stream : static_cast<cudaStream_t>(stream);
+  }
+  return NVBT_OK;
+}
+
+static int done(nvbt_ctx ctx, int n_kernels) {
+  NVBT_CUDA(cudaGetLastError());
+  if (ctx) ctx->launches += n_kernels;
+  return NVBT_OK;
+}
+
+}  // namespace nvbt
+
+using namespace nvbt;
+
+extern "C" {
+
+int nvbt_program(int w, nvbt_instr_desc* out, uint32_t cap, uint32_t* n_pcs, uint32_t* n_ops, uint32_t* n_bbs);
+
+int nvbt_workload_warps(int w, const int64_t* a, uint32_t na, uint64_t* n) {
+  if (!a || !n) return set_error(NVBT_EINVAL, "null argument");
+  switch (w) {
+    case NVBT_W_VECTORADD: case NVBT_W_BFS:
+      if (na < 1 || a[0] < 0) break;
+      *n = (uint64_t)((a[0] + 255) / 256) * 8; return NVBT_OK;
+    case NVBT_W_SGEMM:
+      if (na < 2 || a[0] < 0 || a[1] < 0) break;
+      *n = (uint64_t)((a[0] + 31) / 32) * (uint64_t)((a[1] + 7) / 8) * 8; return NVBT_OK;
+    case NVBT_W_STENCIL:
+      if (na < 1 || a[0] < 0) break;
+      *n = (uint64_t)((a[0] + 31) / 32) * (uint64_t)((a[0] + 7) / 8) * 8; return NVBT_OK;
+    default: break;
+  }
+  return set_error(NVBT_EINVAL, "bad workload %d or arguments", w);
+}
+
+int nvbt_vectoradd(nvbt_ctx ctx, void* stream, uint32_t tools, const float* a, const float* b, float* c, int32_t N) {
+  if (!a || !b || !c || N < 0) return set_error(NVBT_EINVAL, "bad vectorAdd arguments");
+  LaunchCtx lc;
+  int rc = prepare<ProgVectorAdd>(ctx, stream, tools, "vectorAdd", &lc);
+  if (rc) return rc;
+  if (N == 0) return NVBT_OK;
+  const dim3 grid((N + 255) / 256);
+  rc = dispatch(tools, [&](auto tag) { k_vectoradd<decltype(tag)::value><<<grid, 256, 0, lc.stream>>>(a, b, c, N, lc.st); });
+  return rc ? rc : done(ctx, 1);
+}
+
+int nvbt_sgemm(nvbt_ctx ctx, void* stream, uint32_t tools, const float* A, const float* B, float* C, int32_t M,
+               int32_t N, int32_t K) {
+  if (!A || !B || !C || M < 0 || N < 0 || K < 1) return set_error(NVBT_EINVAL, "bad SGEMM arguments");
+  if ((M + 31) / 32 > 0x7fffffff || (N + 7) / 8 > 65535) return set_error(NVBT_EINVAL, "SGEMM grid too large");
+  LaunchCtx lc;
+  int rc = prepare<ProgSgemm>(ctx, stream, tools, "SGEMM", &lc);
+  if (rc) return rc;
+  if (M == 0 || N == 0) return NVBT_OK;
+  const dim3 grid((M + 31) / 32, (N + 7) / 8), block(32, 8);
+  rc = dispatch(tools, [&](auto tag) { k_sgemm<decltype(tag)::value><<<grid, block, 0, lc.stream>>>(A, B, C, M, N, K, lc.st); });
+  return rc ? rc : done(ctx, 1);
+}
+
+int nvbt_bfs_level(nvbt_ctx ctx, void* stream, uint32_t tools, const int32_t* rowptr, const int32_t* col, int32_t n,
+                   uint8_t* mask, uint8_t* visited, uint8_t* updating, int32_t* cost, int32_t* over, int32_t level) {
+  if (!rowptr || !col || !mask || !visited || !updating || !cost || !over || n < 0)
+    return set_error(NVBT_EINVAL, "bad BFS arguments");
+  LaunchCtx lc;
+  int rc = prepare<ProgBfs>(ctx, stream, tools, "BFS", &lc);
+  if (rc) return rc;
+  if (n == 0) return NVBT_OK;
+  const dim3 grid((n + 255) / 256);
+  DevState st2 = lc.st;
+  if (tools != 0) {  // kernel 2 is a launch of its own (next launch id)
+    rc = make_state(ctx, tools, &st2);
+    if (rc) return rc;
+  }
+  rc = dispatch(tools, [&](auto tag) {
+    constexpr uint32_t TT = decltype(tag)::value;
+    k_bfs_expand<TT><<<grid, 256, 0, lc.stream>>>(rowptr, col, n, mask, visited, updating, lc.st);
+    k_bfs_update<TT><<<grid, 256, 0, lc.stream>>>(n, mask, visited, updating, cost, over, level, st2);
+  });
+  return rc ? rc : done(ctx, 2);
+}
+
+int nvbt_stencil(nvbt_ctx ctx, void* stream, uint32_t tools, const float* in, float* out, int32_t n) {
+  if (!in || !out || n < 0) return set_error(NVBT_EINVAL, "bad stencil arguments");
+  if ((n + 7) / 8 > 65535) return set_error(NVBT_EINVAL, "stencil grid too large");
+  LaunchCtx lc;
+  int rc = prepare<ProgStencil>(ctx, stream, tools, "stencil", &lc);
+  if (rc) return rc;
+  if (n == 0) return NVBT_OK;
+  const dim3 grid((n + 31) / 32, (n + 7) / 8), block(32, 8);
+  rc = dispatch(tools, [&](auto tag) { k_stencil<decltype(tag)::value><<<grid, block, 0, lc.stream>>>(in, out, n, lc.st); });
+  return rc ? rc : done(ctx, 1);
+}
+
+}  // extern "C"

@@ -1,0 +1,83 @@
+"""Host-side drivers of the synthetic workloads and the multi-GPU merge.
+
+Everything here is orchestration: it enqueues library kernels on the context's stream and moves a few
+scalars (the BFS `over` flag). No event arithmetic happens in Python.
+"""
+from __future__ import annotations
+
+from . import nvbt as nb
+
+
+def shard_range(n: int, rank: int, world: int):
+    """Contiguous [lo, hi) share of n units for `rank` of `world` (event ranges for C5)."""
+    lo = n * rank // world
+    hi = n * (rank + 1) // world
+    return lo, hi
+
+
+def bfs_buffers(n, device):
+    import torch
+    return {
+        "mask": torch.zeros(n, dtype=torch.uint8, device=device),
+        "visited": torch.zeros(n, dtype=torch.uint8, device=device),
+        "updating": torch.zeros(n, dtype=torch.uint8, device=device),
+        "cost": torch.full((n,), -1, dtype=torch.int32, device=device),
+        "over": torch.zeros(1, dtype=torch.int32, device=device),
+    }
+
+
+def run_bfs(ctx, tools, rowptr, col, src, bufs=None, stream=None, max_levels=1 << 20):
+    """Level-synchronous BFS of EM §3.3 from `src` (rowptr/col: int32 CUDA tensors).
+
+    Returns (cost tensor, levels, over_host_list)."""
+    import torch
+    n = rowptr.numel() - 1
+    b = bfs_buffers(n, rowptr.device) if bufs is None else bufs
+    b["mask"].zero_(); b["visited"].zero_(); b["updating"].zero_(); b["cost"].fill_(-1)
+    b["mask"][src] = 1
+    b["visited"][src] = 1
+    b["cost"][src] = 0
+    over_h = torch.zeros(1, dtype=torch.int32, pin_memory=True)
+    level = 0
+    while level < max_levels:
+        b["over"].zero_()
+        b["updating"].zero_()
+        nb.nvbt_bfs_level(ctx, tools, rowptr, col, n, b["mask"], b["visited"], b["updating"], b["cost"],
+                          b["over"], level, stream=stream)
+        over_h.copy_(b["over"], non_blocking=True)
+        torch.cuda.current_stream().synchronize() if ctx is None else _sync(ctx)
+        level += 1
+        if int(over_h[0]) == 0:
+            break
+    return b["cost"], level
+
+
+def _sync(ctx):
+    import torch
+    s = ctx.stream if ctx.stream is not None else torch.cuda.current_stream(ctx.device)
+    s.synchronize()
+
+
+def run_stencil(ctx, tools, buf0, buf1, n, iters, stream=None):
+    """Iteration it reads buffer it % 2 and writes (it + 1) % 2 (EM §3.4). Returns the final buffer."""
+    bufs = (buf0, buf1)
+    for it in range(iters):
+        nb.nvbt_stencil(ctx, tools, bufs[it % 2], bufs[(it + 1) % 2], n, stream=stream)
+    return bufs[iters % 2]
+
+
+def replay_range(ctx, seed, first, n, hdr, addr, chunk=None):
+    """Generate-then-replay events [first, first + n) in chunks that fit the given stream buffers."""
+    cap = hdr.numel() // 16 if chunk is None else chunk
+    done = 0
+    while done < n:
+        m = min(cap, n - done)
+        nb.nvbt_gen_events(ctx, seed, first + done, m, hdr, addr)
+        nb.nvbt_replay(ctx, hdr, addr, m)
+        done += m
+
+
+def merge(ctx, group=None):
+    """a8: one int64 SUM all-reduce of the packed accumulator region (NCCL over NVLink on GPUs)."""
+    import torch.distributed as dist
+    dist.all_reduce(nb.nvbt_accum_view(ctx), op=dist.ReduceOp.SUM, group=group)

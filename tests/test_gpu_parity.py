@@ -1,0 +1,255 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle, bit-exact.
+
+Every input is seeded; addresses in events are the real device addresses, which the oracle models
+receive as inputs. Sizes span several CTAs and ragged tails; full-size cases check closed forms, the
+oracle on sampled warps and invariants."""
+import numpy as np
+import pytest
+
+from oracle import events as ev, programs, gen, trace
+from oracle.models import vectoradd as m_va, sgemm as m_sg, stencil as m_st, bfs as m_bfs
+from synth import uniform_f32, rmat_csr, bfs_source
+
+from .gpu_util import read_all, assert_same, gpu_invariants
+
+pytestmark = pytest.mark.gpu
+
+COUNT_KEYS = ["counts", "H_t", "H_w", "Ent_w", "Ent_t", "Ins_w", "Ins_t"]
+MEM_KEYS = ["mem_n", "mem_S", "mem_L", "hS", "hL"]
+
+
+def cuda(x):
+    import torch
+    return torch.from_numpy(np.ascontiguousarray(x)).cuda()
+
+
+# ---------------------------------------------------------------- C1 vectorAdd
+@pytest.mark.parametrize("N", [65536, 65500, 1000, 31, 257])
+@pytest.mark.parametrize("count_tool", ["COUNT", "BBCOUNT"])
+def test_vectoradd_parity(nvbt, N, count_tool):
+    import torch
+    nb = nvbt.nvbt
+    tools = getattr(nb, "TOOL_" + count_tool) | nb.TOOL_MEMDIV
+    nw = nb.nvbt_workload_warps(nb.W_VECTORADD, N)
+    ctx = nb.nvbt_init(nb.W_VECTORADD, nb.COUNT | nb.OPHIST | nb.BB | nb.MEMDIV | nb.PER_WARP, n_warps=nw)
+    a, b = cuda(uniform_f32(N, 1)), cuda(uniform_f32(N, 2))
+    c = torch.empty_like(a)
+    nb.nvbt_vectoradd(ctx, tools, a, b, c, N)
+    g = read_all(nb, ctx, per_warp=True)
+    acc = ev.Accumulator(programs.vectoradd(), n_warps=nw)
+    m_va.run(acc, N, a.data_ptr(), b.data_ptr(), c.data_ptr())
+    assert_same(g, acc.result(), COUNT_KEYS + MEM_KEYS + ["PW_T", "PW_W"], f"vectorAdd N={N} {count_tool}")
+    assert torch.equal(c, a + b)
+    gpu_invariants(g)
+
+
+def test_vectoradd_plain_and_cumulative(nvbt):
+    """Uninstrumented launches count nothing; instrumented results accumulate until reset."""
+    import torch
+    nb = nvbt.nvbt
+    N = 4096
+    ctx = nb.nvbt_init(nb.W_VECTORADD, nb.COUNT)
+    a, b = cuda(uniform_f32(N, 1)), cuda(uniform_f32(N, 2))
+    c = torch.empty_like(a)
+    nb.nvbt_vectoradd(ctx, nb.TOOL_NONE, a, b, c, N)
+    assert (nb.nvbt_count(ctx) == 0).all()
+    nb.nvbt_vectoradd(ctx, nb.TOOL_COUNT, a, b, c, N)
+    one = nb.nvbt_count(ctx).copy()
+    nb.nvbt_vectoradd(ctx, nb.TOOL_COUNT, a, b, c, N)
+    assert (nb.nvbt_count(ctx) == 2 * one).all()
+    nb.nvbt_reset(ctx)
+    assert (nb.nvbt_count(ctx) == 0).all()
+    with pytest.raises(nb.NvbtError):            # MEMDIV not enabled at init
+        nb.nvbt_vectoradd(ctx, nb.TOOL_MEMDIV, a, b, c, N)
+    with pytest.raises(nb.NvbtError):            # wrong program for this context
+        nb.nvbt_sgemm(ctx, nb.TOOL_COUNT, a, b, c, 32, 8, 1)
+
+
+# ---------------------------------------------------------------- C2 SGEMM
+@pytest.mark.parametrize("M,N,K", [(64, 32, 48), (100, 20, 5), (33, 9, 1), (96, 64, 130)])
+@pytest.mark.parametrize("tools", ["COUNT|MEMDIV", "BBCOUNT|MEMDIV", "MEMDIV"])
+def test_sgemm_parity(nvbt, M, N, K, tools):
+    import torch
+    nb = nvbt.nvbt
+    t = 0
+    for x in tools.split("|"):
+        t |= getattr(nb, "TOOL_" + x)
+    nw = nb.nvbt_workload_warps(nb.W_SGEMM, M, N)
+    ctx = nb.nvbt_init(nb.W_SGEMM, nb.COUNT | nb.OPHIST | nb.BB | nb.MEMDIV | nb.PER_WARP, n_warps=nw)
+    A = cuda(uniform_f32((M, K), 3, -1, 1))
+    B = cuda(uniform_f32((K, N), 4, -1, 1))
+    Cm = torch.empty(M, N, device="cuda")
+    nb.nvbt_sgemm(ctx, t, A, B, Cm, M, N, K)
+    g = read_all(nb, ctx, per_warp=True)
+    acc = ev.Accumulator(programs.sgemm(), n_warps=nw)
+    m_sg.run(acc, M, N, K, A.data_ptr(), B.data_ptr(), Cm.data_ptr())
+    ref = acc.result()
+    keys = MEM_KEYS + (COUNT_KEYS + ["PW_T", "PW_W"] if "COUNT" in tools else [])
+    assert_same(g, ref, keys, f"SGEMM {M}x{N}x{K} {tools}")
+    torch.testing.assert_close(Cm, A @ B, rtol=1e-4, atol=1e-4)
+
+
+@pytest.mark.slow
+def test_sgemm_full_size(nvbt):
+    """C2 at 1024^3 in the bench's launch configuration: closed forms (I-3) and sampled warps."""
+    import torch
+    nb = nvbt.nvbt
+    M = N = K = 1024
+    nw = nb.nvbt_workload_warps(nb.W_SGEMM, M, N)
+    ctx = nb.nvbt_init(nb.W_SGEMM, nb.COUNT | nb.MEMDIV | nb.PER_WARP, n_warps=nw)
+    A = cuda(uniform_f32((M, K), 3, -1, 1))
+    B = cuda(uniform_f32((K, N), 4, -1, 1))
+    Cm = torch.empty(M, N, device="cuda")
+    nb.nvbt_sgemm(ctx, nb.TOOL_COUNT | nb.TOOL_MEMDIV, A, B, Cm, M, N, K)
+    g = read_all(nb, ctx, per_warp=True)
+    W = nw
+    w_iss = W * (12 + 6 * K)
+    assert g["counts"].tolist() == [32 * w_iss, 32 * (w_iss - 2 * W), w_iss, w_iss - 2 * W]
+    assert g["mem_n"].sum() == 67_141_632
+    assert g["mem_S"].sum() == g["mem_L"].sum() == 1_108_344_832
+    rng = np.random.default_rng(0)
+    sample = np.sort(rng.choice(W, size=6, replace=False))
+    acc = ev.Accumulator(programs.sgemm(), n_warps=W)
+    m_sg.run(acc, M, N, K, A.data_ptr(), B.data_ptr(), Cm.data_ptr(), warps=sample)
+    r = acc.result()
+    assert (g["PW_T"][sample] == r["PW_T"][sample]).all() and (g["PW_W"][sample] == r["PW_W"][sample]).all()
+    gpu_invariants(g)
+
+
+# ---------------------------------------------------------------- C3 BFS
+@pytest.mark.parametrize("scale,tools", [(12, "BBCOUNT"), (12, "COUNT|MEMDIV"), (10, "BBCOUNT|MEMDIV")])
+def test_bfs_parity(nvbt, scale, tools):
+    nb, dr = nvbt.nvbt, nvbt.drivers
+    t = 0
+    for x in tools.split("|"):
+        t |= getattr(nb, "TOOL_" + x)
+    rowptr, col = rmat_csr(scale, 16, seed=3)
+    n = len(rowptr) - 1
+    src = bfs_source(rowptr)
+    nw = nb.nvbt_workload_warps(nb.W_BFS, n)
+    ctx = nb.nvbt_init(nb.W_BFS, nb.COUNT | nb.BB | nb.MEMDIV | nb.PER_WARP, n_warps=nw)
+    rp, cl = cuda(rowptr), cuda(col)
+    bufs = dr.bfs_buffers(n, "cuda")
+    cost, levels = dr.run_bfs(ctx, t, rp, cl, src, bufs)
+    g = read_all(nb, ctx, per_warp=True)
+    acc = ev.Accumulator(programs.bfs(), n_warps=nw)
+    ptr = m_bfs.Ptrs(bufs["mask"].data_ptr(), bufs["visited"].data_ptr(), bufs["updating"].data_ptr(),
+                     bufs["cost"].data_ptr(), bufs["over"].data_ptr(), rp.data_ptr(), cl.data_ptr())
+    ocost, olevels, _ = m_bfs.run(acc, rowptr, col, src, ptr)
+    assert levels == olevels
+    assert (cost.cpu().numpy() == ocost).all()
+    ref = acc.result()
+    keys = (COUNT_KEYS + ["PW_T", "PW_W"]) + (MEM_KEYS if "MEMDIV" in tools else [])
+    assert_same(g, ref, keys, f"BFS scale {scale} {tools}")
+
+
+# ---------------------------------------------------------------- C4 stencil + trace channel
+def _stencil_case(nvbt, n, iters, ring_records, tools_names=("TRACE", "MEMDIV", "COUNT")):
+    import torch
+    nb, dr = nvbt.nvbt, nvbt.drivers
+    t = 0
+    for x in tools_names:
+        t |= getattr(nb, "TOOL_" + x)
+    ctx = nb.nvbt_init(nb.W_STENCIL, nb.COUNT | nb.MEMDIV | nb.TRACE)
+    x0 = cuda(uniform_f32((n, n), 4))
+    buf0, buf1 = x0.clone(), torch.zeros_like(x0)
+    ring = torch.empty(64 + 288 * ring_records, dtype=torch.uint8, pin_memory=True)
+    ch = nb.nvbt_channel_open(ctx, ring)
+    dr.run_stencil(ctx, t, buf0, buf1, n, iters)
+    acc = ev.Accumulator(programs.stencil(), trace=True, keep_records=True)
+    m_st.run_iterations(acc, n, buf0.data_ptr(), buf1.data_ptr(), iters)
+    exp = acc.record_array()
+    dst = np.zeros((len(exp) + 16, 288), dtype=np.uint8)
+    got_n = nb.nvbt_channel_drain_copy(ch, dst, timeout_us=60_000_000)
+    assert nb.nvbt_channel_dropped(ch) == 0
+    got = dst[:got_n]
+    assert got_n == len(exp)
+    assert (trace.sort_records(got) == trace.sort_records(exp)).all()
+    out = buf0 if iters % 2 == 0 else buf1
+    ref_grid = m_st.jacobi_reference(x0.cpu().numpy(), iters)
+    assert np.array_equal(out.cpu().numpy(), ref_grid)
+    return ctx, acc, got
+
+
+@pytest.mark.parametrize("n,iters", [(96, 3), (100, 2), (64, 1)])
+def test_stencil_trace_parity(nvbt, n, iters):
+    nb = nvbt.nvbt
+    ctx, acc, got = _stencil_case(nvbt, n, iters, ring_records=1 << 16)
+    g = read_all(nb, ctx)
+    assert_same(g, acc.result(), COUNT_KEYS + MEM_KEYS, f"stencil n={n}")
+    assert nb.nvbt_digest_records(got) == (acc.digest.n, acc.digest.d1, acc.digest.d2)
+
+
+def test_channel_tiny_ring_backpressure(nvbt):
+    """A 5-slot ring forces wrap-around and producer backpressure; nothing lost or duplicated."""
+    _stencil_case(nvbt, 64, 2, ring_records=5, tools_names=("TRACE",))
+
+
+def test_channel_digest_drain(nvbt):
+    import torch
+    nb, dr = nvbt.nvbt, nvbt.drivers
+    n, iters = 128, 2
+    ctx = nb.nvbt_init(nb.W_STENCIL, nb.TRACE)
+    x0 = cuda(uniform_f32((n, n), 4))
+    buf0, buf1 = x0.clone(), torch.zeros_like(x0)
+    ring = torch.empty(64 + 288 * 1000, dtype=torch.uint8, pin_memory=True)
+    ch = nb.nvbt_channel_open(ctx, ring)
+    dr.run_stencil(ctx, nb.TOOL_TRACE, buf0, buf1, n, iters)
+    d = nb.nvbt_channel_drain_digest(ch, timeout_us=60_000_000)
+    acc = ev.Accumulator(programs.stencil(), trace=True)
+    m_st.run_iterations(acc, n, buf0.data_ptr(), buf1.data_ptr(), iters)
+    assert (d.n_rec, d.d1, d.d2) == (acc.digest.n, acc.digest.d1, acc.digest.d2)
+
+
+# ---------------------------------------------------------------- C5 generator + replay
+def test_generator_bytes_match_oracle(nvbt):
+    import torch
+    nb = nvbt.nvbt
+    ctx = nb.nvbt_init(nb.W_REPLAY, nb.COUNT)
+    for first, n in [(0, 1 << 16), (10**10 - 4099, 4099)]:
+        hdr = torch.zeros(n * 16, dtype=torch.uint8, device="cuda")
+        addr = torch.zeros(n * 256, dtype=torch.uint8, device="cuda")
+        nb.nvbt_gen_events(ctx, gen.SEED, first, n, hdr, addr)
+        pc, warp, A, P, oaddr = gen.events(first, n)
+        h = hdr.cpu().numpy().view("<u4").reshape(n, 4)
+        assert (h[:, 0] == pc).all() and (h[:, 1] == warp).all() and (h[:, 2] == A).all() and (h[:, 3] == P).all()
+        ga = addr.cpu().numpy().view("<u8").reshape(n, 32)
+        assert (ga == oaddr).all()   # non-memory slots are not written by either side (zeros here)
+
+
+@pytest.mark.parametrize("first,n", [(0, 1 << 18), (123456789, 100_003)])
+def test_replay_parity(nvbt, first, n):
+    import torch
+    nb, dr = nvbt.nvbt, nvbt.drivers
+    ctx = nb.nvbt_init(nb.W_REPLAY, nb.COUNT | nb.OPHIST | nb.BB | nb.MEMDIV | nb.PER_WARP, n_warps=1 << 20)
+    chunk = 1 << 16
+    hdr = torch.empty(chunk * 16, dtype=torch.uint8, device="cuda")
+    addr = torch.empty(chunk * 256, dtype=torch.uint8, device="cuda")
+    dr.replay_range(ctx, gen.SEED, first, n, hdr, addr)
+    g = read_all(nb, ctx, per_warp=True)
+    acc = ev.Accumulator(programs.replay(), n_warps=1 << 20)
+    gen.replay(acc, first, n)
+    assert_same(g, acc.result(), COUNT_KEYS + MEM_KEYS + ["PW_T", "PW_W"], f"replay [{first}, +{n})")
+    assert nb.nvbt_replay_errors(ctx) == 0
+
+
+def test_replay_merge_equals_single(nvbt):
+    """a8: two partitions merged by summing the packed accumulator region equal one run (I-6)."""
+    import torch
+    nb, dr = nvbt.nvbt, nvbt.drivers
+    n = 200_000
+    hdr = torch.empty((1 << 16) * 16, dtype=torch.uint8, device="cuda")
+    addr = torch.empty((1 << 16) * 256, dtype=torch.uint8, device="cuda")
+    whole = nb.nvbt_init(nb.W_REPLAY, nb.COUNT | nb.MEMDIV)
+    dr.replay_range(whole, gen.SEED, 0, n, hdr, addr)
+    parts = []
+    for r in range(3):
+        lo, hi = dr.shard_range(n, r, 3)
+        c = nb.nvbt_init(nb.W_REPLAY, nb.COUNT | nb.MEMDIV)
+        dr.replay_range(c, gen.SEED, lo, hi - lo, hdr, addr)
+        parts.append(c)
+    v0 = nb.nvbt_accum_view(parts[0])
+    v0 += nb.nvbt_accum_view(parts[1]) + nb.nvbt_accum_view(parts[2])
+    torch.cuda.synchronize()
+    assert torch.equal(nb.nvbt_accum_view(parts[0]), nb.nvbt_accum_view(whole))
+    assert_same(read_all(nb, parts[0]), read_all(nb, whole), what="merged replay")
