@@ -1,0 +1,432 @@
+#!/usr/bin/env python
+"""nvbt benchmark: instrumented warp-instruction events/s and slowdown vs the uninstrumented kernel.
+
+Default workload (BASELINE.json configs[1]): C2 — naive row-fastest SGEMM 1024^3 with the full tool set
+compiled in (counts, opcode/BB histograms, per-instruction memory divergence), one step = one
+instrumented launch (+ the int64 all-reduce merge of the accumulators when N > 1). Other workloads
+(`--workload c1|c3|c4|c5`) are for profiling; the driver's bench line is C2.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload c2] [--impl ours|reference]
+
+Multi-GPU (weak scaling): torchrun, one rank per GPU, every rank runs its own instance; the time of
+the job is the max over ranks. Timing: CUDA events on the context's stream around each step, L2
+flushed (256 MiB write) between steps, clocks sampled with nvidia-smi during the timed region.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+PEAKS_FALLBACK = {"hbm_gbs": 6650.0, "sm_max_mhz": 1965.0}
+N_SM = 148
+METRIC = "instrumented warp-instr events/sec and slowdown vs uninstrumented"
+
+
+def load_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            p = json.load(f)
+        return p, "measured"
+    except Exception:
+        return PEAKS_FALLBACK, "fallback"
+
+
+# --------------------------------------------------------------------------- clocks
+class ClockSampler:
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index):
+        self.gpu = gpu_index
+        self.rows = []
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits", "-lms", "100",
+                 "-i", str(self.gpu)], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.thr = threading.Thread(target=self._read, daemon=True)
+            self.thr.start()
+        except FileNotFoundError:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def __exit__(self, *a):
+        if self.proc:
+            time.sleep(0.25)
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=2)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        sm = [float(r[1]) for r in self.rows if len(r) > 2 and r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in self.rows if len(r) > 2 and r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[k] for r in self.rows for k in range(4) if len(r) > 5 + k and r[5 + k] == "Active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.rows)}
+
+
+# --------------------------------------------------------------------------- distributed
+def dist_setup(args):
+    import torch
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "ours":
+        torch.cuda.set_device(local)
+    if world > 1:
+        import torch.distributed as dist
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        backend = "nccl" if args.impl == "ours" else "gloo"
+        kw = {"device_id": torch.device("cuda", local)} if backend == "nccl" else {}
+        dist.init_process_group(backend, **kw)
+    return rank, world, local
+
+
+def barrier(world):
+    if world > 1:
+        import torch.distributed as dist
+        dist.barrier()
+
+
+def max_over_ranks(x, world, device=None):
+    if world == 1:
+        return x
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([x], dtype=torch.float64, device=device)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+def sum_over_ranks(x, world, device=None):
+    if world == 1:
+        return x
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([x], dtype=torch.float64, device=device)
+    dist.all_reduce(t, op=dist.ReduceOp.SUM)
+    return float(t.item())
+
+
+# --------------------------------------------------------------------------- C2 SGEMM
+class SgemmBench:
+    name = "c2"
+    M = N = K = 1024
+    desc = "C2 naive row-fastest SGEMM 1024^3 (fp32), tools COUNT|MEMDIV (counts, opcode+BB histograms, divergence)"
+
+    def __init__(self, torch, nb, dr, world):
+        self.torch, self.nb, self.dr, self.world = torch, nb, dr, world
+        from synth import uniform_f32
+        M, N, K = self.M, self.N, self.K
+        self.nw = nb.nvbt_workload_warps(nb.W_SGEMM, M, N)
+        self.ctx = nb.nvbt_init(nb.W_SGEMM, nb.COUNT | nb.OPHIST | nb.BB | nb.MEMDIV)
+        self.tools = nb.TOOL_COUNT | nb.TOOL_MEMDIV
+        self.hA = torch.from_numpy(uniform_f32((M, K), 3, -1, 1)).pin_memory()
+        self.hB = torch.from_numpy(uniform_f32((K, N), 4, -1, 1)).pin_memory()
+        self.A, self.B = self.hA.cuda(), self.hB.cuda()
+        self.C = torch.empty(M, N, device="cuda")
+        # events per launch (EM §3.2): every warp runs 12 + 6K warp-level instructions
+        self.events = self.nw * (12 + 6 * K)
+        self.kernels_per_step = 1
+
+    def plain(self):
+        self.nb.nvbt_sgemm(self.ctx, self.nb.TOOL_NONE, self.A, self.B, self.C, self.M, self.N, self.K)
+
+    def instr(self):
+        self.nb.nvbt_sgemm(self.ctx, self.tools, self.A, self.B, self.C, self.M, self.N, self.K)
+
+    def e2e_step(self, out_host):
+        """Through the public API with host buffers: H2D inputs, instrumented launch, read results."""
+        nb = self.nb
+        self.A.copy_(self.hA, non_blocking=True)
+        self.B.copy_(self.hB, non_blocking=True)
+        nb.nvbt_sgemm(self.ctx, self.tools, self.A, self.B, self.C, self.M, self.N, self.K)
+        out_host["counts"] = nb.nvbt_count(self.ctx)
+        out_host["memdiv"] = nb.nvbt_mem_divergence(self.ctx)
+        out_host["ophist"] = nb.nvbt_opcode_hist(self.ctx)
+        return self.hA.numel() * 4 + self.hB.numel() * 4, 8 * (4 + 3 * 18 + 3 + 66 + 2 * 16)
+
+    def roofline(self, t_kernel_s, peaks):
+        """Issue roofline ("alu"): algorithmic warp-instructions per launch ÷ launch time vs
+        148 SMs x 4 schedulers x 1 warp-instr/clk at the max SM clock."""
+        K, W = self.K, self.nw
+        per_warp = (12 + 6 * K) * (1 + HOOK_OPS["count"]) + (K + 1) * HOOK_OPS["guard"] + \
+            (2 * K + 1) * HOOK_OPS["mem"]
+        ops = W * per_warp
+        peak = N_SM * 4 * peaks.get("sm_max_mhz", 1965.0) * 1e6
+        ach = ops / t_kernel_s
+        return {"bound": "alu", "achieved": ach / 1e9, "peak": peak / 1e9, "unit": "Gwarp-inst/s",
+                "frac": ach / peak, "traffic": None, "algorithmic_warp_inst_per_launch": ops}
+
+    def oracle_sample(self, budget_s):
+        """The oracle on a bounded sample of the same workload: whole warps, full K."""
+        from oracle import events as ev, programs
+        from oracle.models import sgemm as m_sg
+        acc = ev.Accumulator(programs.sgemm())
+        rng = np.random.default_rng(1)
+        warps = np.sort(rng.choice(self.nw, size=64, replace=False))
+        t0 = time.perf_counter()
+        done = 0
+        while True:
+            m_sg.run(acc, self.M, self.N, self.K, self.A.data_ptr(), self.B.data_ptr(), self.C.data_ptr(),
+                     warps=warps)
+            done += len(warps) * (12 + 6 * self.K)
+            if time.perf_counter() - t0 > budget_s:
+                break
+        dt = time.perf_counter() - t0
+        return done / dt, f"{done} warp events: SGEMM 1024^3 oracle model on 64 sampled warps x full K"
+
+
+# hook instruction costs per event used for the issue roofline (minimal SASS per hook)
+HOOK_OPS = {"count": 4, "guard": 6, "mem": 21}
+
+
+# --------------------------------------------------------------------------- C5 replay
+class ReplayBench:
+    name = "c5"
+    desc = "C5 trace replay of 10^10 generated events (counts, histograms, divergence), 2^27-event chunks"
+
+    def __init__(self, torch, nb, dr, world, rank, n_total=10**10, chunk=1 << 27):
+        self.torch, self.nb, self.dr = torch, nb, dr
+        self.lo, self.hi = dr.shard_range(n_total, rank, world)
+        self.n = self.hi - self.lo
+        self.chunk = chunk
+        self.ctx = nb.nvbt_init(nb.W_REPLAY, nb.COUNT | nb.OPHIST | nb.BB | nb.MEMDIV)
+        self.hdr = torch.empty(chunk * 16, dtype=torch.uint8, device="cuda")
+        self.addr = torch.empty(chunk * 256, dtype=torch.uint8, device="cuda")
+        self.events = self.n
+        self.kernels_per_step = -(-self.n // chunk)
+
+    def run(self, stream_events):
+        """One step: generate (untimed) and replay (timed with events) every chunk."""
+        torch, nb = self.torch, self.nb
+        t = 0.0
+        off = 0
+        while off < self.n:
+            m = min(self.chunk, self.n - off)
+            nb.nvbt_gen_events(self.ctx, 0x4E5642544E564254, self.lo + off, m, self.hdr, self.addr)
+            e0, e1 = stream_events
+            e0.record()
+            nb.nvbt_replay(self.ctx, self.hdr, self.addr, m)
+            e1.record()
+            e1.synchronize()
+            t += e0.elapsed_time(e1) / 1e3
+            off += m
+        return t
+
+
+# --------------------------------------------------------------------------- main
+def run_ours(args):
+    import torch
+    rank, world, local = dist_setup(args)
+    import paper_conf_micro_villasnk19_b200 as pkg
+    nb, dr = pkg.nvbt, pkg.drivers
+    peaks, peaks_src = load_peaks()
+    dev = torch.device("cuda", local)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+
+    if args.workload == "c5":
+        return run_replay(args, torch, nb, dr, rank, world, local, peaks, peaks_src)
+
+    wl = SgemmBench(torch, nb, dr, world)
+    launches0 = nb.nvbt_launch_count(wl.ctx)
+
+    def timed(fn, n, merge=False):
+        ts = []
+        for _ in range(n):
+            flush.zero_()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            fn()
+            if merge and world > 1:
+                dr.merge(wl.ctx)
+            e1.record()
+            e1.synchronize()
+            ts.append(e0.elapsed_time(e1) / 1e3)
+        return ts
+
+    # warm-up (untimed), plain baseline
+    timed(wl.instr, args.warmup)
+    timed(wl.plain, max(args.warmup, 3))
+    t_plain = timed(wl.plain, args.steps)
+    nb.nvbt_reset(wl.ctx)
+    barrier(world)
+    torch.cuda.synchronize()
+    l0 = nb.nvbt_launch_count(wl.ctx)
+    with ClockSampler(local) as clk:
+        barrier(world)
+        torch.cuda.synchronize()
+        t_instr = timed(wl.instr, args.steps, merge=True)
+        torch.cuda.synchronize()
+        barrier(world)
+    gpu_launches = nb.nvbt_launch_count(wl.ctx) - l0
+    # result check of the timed steps: exactly K x the per-launch closed form (I-3)
+    cnt = nb.nvbt_count(wl.ctx)
+    expect = wl.events * args.steps * (world if world > 1 else 1)
+    ok = int(cnt[2]) == expect
+    tot_instr = max_over_ranks(sum(t_instr), world, dev)
+    tot_plain = max_over_ranks(sum(t_plain), world, dev)
+    events_all = wl.events * args.steps * world
+    value = events_all / tot_instr
+    slowdown = tot_instr / tot_plain
+    t_kernel = statistics.median(t_instr)
+    # e2e through the public API with host buffers
+    out = {}
+    for _ in range(2):
+        wl.e2e_step(out)
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    e2e_steps = max(3, min(args.steps, 10))
+    for _ in range(e2e_steps):
+        h2d, d2h = wl.e2e_step(out)
+    torch.cuda.synchronize()
+    e2e_t = max_over_ranks(time.perf_counter() - t0, world, dev)
+    e2e_value = wl.events * e2e_steps * world / e2e_t
+    line = {
+        "metric": METRIC, "value": value, "unit": "events/s", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": 1e3 * tot_instr / args.steps, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+        "config": {"workload": wl.desc, "M": wl.M, "N": wl.N, "K": wl.K, "warp_events_per_launch": wl.events,
+                   "tools": "COUNT|MEMDIV", "l2": "flushed between steps (256 MiB write)",
+                   "parallelism": f"replicas x{world} + int64 all-reduce merge per step" if world > 1 else "1 GPU"},
+        "slowdown": slowdown, "plain_ms_per_launch": 1e3 * statistics.median(t_plain),
+        "instr_ms_per_launch": 1e3 * t_kernel, "counts_check": "ok" if ok else f"mismatch {int(cnt[2])} != {expect}",
+        "roofline": wl.roofline(t_kernel, peaks),
+        "e2e": {"value": e2e_value, "unit": "events/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h},
+        "gpu_launches": int(gpu_launches), "clocks": clk.summary(), "peaks_source": peaks_src,
+    }
+    line["roofline"]["peak_source"] = f"148 SMs x 4 issue/clk x sm_max_mhz ({peaks_src})"
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        rate, sample = wl.oracle_sample(args.cpu_budget)
+        line["cpu_baseline"] = {"value": rate, "unit": "events/s", "cores": 1, "kind": "oracle", "sample": sample}
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        import torch.distributed as dist
+        dist.destroy_process_group()
+
+
+def run_replay(args, torch, nb, dr, rank, world, local, peaks, peaks_src):
+    dev = torch.device("cuda", local)
+    wl = ReplayBench(torch, nb, dr, world, rank, n_total=args.replay_events)
+    evs = (torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+    # warm-up on one chunk
+    for _ in range(args.warmup):
+        nb.nvbt_gen_events(wl.ctx, 0x4E5642544E564254, 0, min(wl.chunk, wl.n), wl.hdr, wl.addr)
+        nb.nvbt_replay(wl.ctx, wl.hdr, wl.addr, min(wl.chunk, wl.n))
+    nb.nvbt_reset(wl.ctx)
+    torch.cuda.synchronize()
+    barrier(world)
+    l0 = nb.nvbt_launch_count(wl.ctx)
+    with ClockSampler(local) as clk:
+        ts = [wl.run(evs) for _ in range(args.steps)]
+        if world > 1:
+            dr.merge(wl.ctx)
+        torch.cuda.synchronize()
+        barrier(world)
+    launches = nb.nvbt_launch_count(wl.ctx) - l0
+    per, tot, hs, hl = nb.nvbt_mem_divergence(wl.ctx)
+    cnt = nb.nvbt_count(wl.ctx)
+    t_total = max_over_ranks(sum(ts), world, dev)
+    n_all = wl.n * world if world > 1 else wl.n
+    value = args.steps * sum_over_ranks(wl.n, world, dev) / t_total
+    # algorithmic bytes: 16 B per header + 256 B per executed memory event (slots that must be read)
+    mem_exec = int(tot[0]) // max(1, world if world > 1 else 1)
+    bytes_rank = 16 * wl.n + 256 * (mem_exec // args.steps)
+    ach = bytes_rank * args.steps / (sum(ts))
+    line = {
+        "metric": "replayed warp-instr events/sec", "value": value, "unit": "events/s", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * t_total / args.steps,
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+        "config": {"workload": wl.desc, "events": args.replay_events, "chunk": wl.chunk,
+                   "l2": "inputs (36.5 GB per chunk) larger than L2"},
+        "roofline": {"bound": "hbm", "achieved": ach / 1e9, "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                     "frac": ach / 1e9 / peaks["hbm_gbs"], "traffic": None, "peak_source": peaks_src},
+        "gpu_launches": int(launches), "clocks": clk.summary(),
+        "check": {"W_issued": int(cnt[2]), "expected": args.steps * n_all},
+    }
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+
+
+def run_reference(args):
+    """Reference arm = the CPU oracle (this tier has no runnable reference)."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    from oracle import events as ev, programs
+    from oracle.models import sgemm as m_sg
+    M = N = K = 1024
+    nw = (M // 32) * (N // 8) * 8
+    events_per_launch = nw * (12 + 6 * K)
+    base = 1 << 32
+    rng = np.random.default_rng(1)
+    warps = np.sort(rng.choice(nw, size=16, replace=False))
+    per_step_events = len(warps) * (12 + 6 * K)
+    for _ in range(args.warmup):
+        acc = ev.Accumulator(programs.sgemm())
+        m_sg.run(acc, M, N, K, base, base + (8 << 20), base + (16 << 20), warps=warps[:2])
+    ts = []
+    for _ in range(args.steps):
+        acc = ev.Accumulator(programs.sgemm())
+        t0 = time.perf_counter()
+        m_sg.run(acc, M, N, K, base, base + (8 << 20), base + (16 << 20), warps=warps)
+        ts.append(time.perf_counter() - t0)
+    value = per_step_events * args.steps / sum(ts)
+    sample = (f"{per_step_events} warp events per step: 16 sampled warps (full K) of C2 SGEMM 1024^3 "
+              f"({events_per_launch} events per launch)")
+    line = {
+        "metric": METRIC, "value": value, "unit": "events/s", "n_gpus": int(os.environ.get("WORLD_SIZE", "1")),
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * sum(ts) / args.steps,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
+        "config": {"workload": SgemmBench.desc, "M": M, "N": N, "K": K}, "impl": "reference",
+        "cpu_baseline": {"value": value, "unit": "events/s", "cores": 1, "kind": "oracle", "sample": sample},
+        "e2e": {"value": value, "unit": "events/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--workload", choices=["c2", "c5"], default="c2")
+    ap.add_argument("--replay-events", type=int, default=10**10)
+    ap.add_argument("--cpu-budget", type=float, default=15.0)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

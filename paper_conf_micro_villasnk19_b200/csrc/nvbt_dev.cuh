@@ -65,12 +65,77 @@ template <class Prog> __host__ __device__ constexpr int bb_len(int lead) {
   return n;
 }
 
-// Number of distinct keys among the lanes of E (lanes outside E may pass any key): a lane of E is its
-// group's leader when no lower lane of E has its key.
-__device__ __forceinline__ unsigned distinct(unsigned long long key, unsigned E, unsigned lanebit, unsigned lmlt) {
+// Number of distinct keys among the lanes of E with __match_any_sync (kept for comparison; MATCH's
+// cost grows with the number of distinct keys, so the hot path uses sectors_lines() below).
+__device__ __forceinline__ unsigned distinct_match(unsigned long long key, unsigned E, unsigned lanebit, unsigned lmlt) {
   const unsigned grp = __match_any_sync(FULL, key);
   return __popc(__ballot_sync(FULL, (E & lanebit) != 0u && (grp & E & lmlt) == 0u));
 }
+
+constexpr int SCRATCH_WORDS = 192;  // per-warp scratch of sectors_lines(): 64 x u64 keys + 64 x u32 masks
+// Initial contents of scratch word i (keys empty = ~0, masks 0).
+__host__ __device__ constexpr unsigned scratch_init_word(int i) { return i < 128 ? 0xffffffffu : 0u; }
+
+// a5 kernel of Listing 8 (readings R-3, R-5, R-6): S = number of distinct 32 B
+// sectors and L = number of distinct 128 B lines touched by the lanes of E (E != 0). Exact integers.
+// Cheapest applicable method first (the warp takes one branch; every test is a vote):
+//  1. sector keys non-decreasing in lane order over E (coalesced, strided, broadcast, stencil
+//     neighbours): count lanes whose key differs from the previous lane of E — line keys are then
+//     sorted too. 1 shuffle (64-bit), 3 votes;
+//  2. every key inside the first lane's 32-sector (1 KB) word: OR-reduce one bit per sector;
+//     S = popc, L = popc of the OR-ed 4-bit groups;
+//  3. otherwise a per-warp open-addressing hash set of LINE keys in shared memory (`scr`: shared
+//     address of SCRATCH_WORDS words in their initial state, restored before returning): each lane of E
+//     inserts its line with a 64-bit CAS (linear probing, 64 slots >= 2 x 32 keys), then ORs its
+//     sector's bit into the slot's 4-bit mask; L = lanes that inserted, S = sum of mask popcounts.
+__device__ __forceinline__ void sectors_lines(unsigned long long addr, unsigned E, unsigned lane, unsigned lanebit,
+                                              unsigned lmlt, unsigned scr, unsigned& S, unsigned& L) {
+  const bool act = (E & lanebit) != 0u;
+  const unsigned long long sk = addr >> 5;
+  const unsigned below = E & lmlt;
+  const int src = below ? 31 - __clz(below) : (int)lane;
+  const unsigned long long prev = __shfl_sync(FULL, sk, src);
+  if (__all_sync(FULL, !act || below == 0u || prev <= sk)) {
+    const bool first = below == 0u;
+    S = __popc(__ballot_sync(FULL, act && (first || sk != prev)));
+    L = __popc(__ballot_sync(FULL, act && (first || (sk >> 2) != (prev >> 2))));
+    return;
+  }
+  const unsigned long long sk0 = __shfl_sync(FULL, sk, __ffs(E) - 1);
+  if (__all_sync(FULL, !act || (sk >> 5) == (sk0 >> 5))) {
+    const unsigned word = __reduce_or_sync(FULL, act ? 1u << (unsigned)(sk & 31) : 0u);
+    const unsigned g = word | (word >> 1) | (word >> 2) | (word >> 3);
+    S = __popc(word);
+    L = __popc(g & 0x11111111u);
+    return;
+  }
+  const unsigned long long line = sk >> 2;
+  unsigned slot = (((unsigned)line ^ (unsigned)(line >> 32)) * 0x9E3779B1u) >> 26;
+  bool pending = act, inserted = false;
+  while (__any_sync(FULL, pending)) {
+    if (pending) {
+      unsigned long long old;
+      asm volatile("atom.shared.cas.b64 %0, [%1], %2, %3;" : "=l"(old) : "r"(scr + 8u * slot), "l"(~0ull), "l"(line)
+                   : "memory");
+      if (old == ~0ull || old == line) {
+        pending = false;
+        inserted = old == ~0ull;
+      } else {
+        slot = (slot + 1u) & 63u;
+      }
+    }
+  }
+  if (act) asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(scr + 512u + 4u * slot), "r"(1u << (unsigned)(sk & 3)) : "memory");
+  L = __popc(__ballot_sync(FULL, inserted));
+  __syncwarp();
+  unsigned m0, m1;
+  asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(m0), "=r"(m1) : "r"(scr + 512u + 8u * lane) : "memory");
+  asm volatile("st.shared.v2.u32 [%0], {%1, %1};" ::"r"(scr + 512u + 8u * lane), "r"(0u) : "memory");
+  asm volatile("st.shared.v4.u32 [%0], {%1, %1, %1, %1};" ::"r"(scr + 16u * lane), "r"(0xffffffffu) : "memory");
+  S = __reduce_add_sync(FULL, __popc(m0) + __popc(m1));
+  __syncwarp();
+}
+
 __device__ __forceinline__ unsigned umin(unsigned a, unsigned b) { return a < b ? a : b; }
 // h += (v == ref) as a predicated add.
 __device__ __forceinline__ void inc_if_eq(unsigned& h, unsigned v, unsigned ref) {
@@ -98,7 +163,9 @@ struct Hooks {
   static constexpr bool kOn = T != 0;
   static constexpr bool kCount = (T & (TOOL_COUNT | TOOL_BB)) != 0;
   static constexpr bool kBB = (T & TOOL_BB) != 0;
-  static constexpr int kSmemWords = kOn ? NPC * SITE_WORDS + 66 : 1;
+  static constexpr int kMaxWarps = 8;  // workload CTAs have 256 threads
+  static constexpr int kScratchWord0 = (NPC * SITE_WORDS + 66 + 3) & ~3;  // 16-byte aligned
+  static constexpr int kSmemWords = kOn ? kScratchWord0 + SCRATCH_WORDS * kMaxWarps : 1;
   static_assert(!((T & TOOL_COUNT) && (T & TOOL_BB)), "COUNT and BBCOUNT are exclusive");
 
   const DevState& st;
@@ -107,7 +174,7 @@ struct Hooks {
   unsigned hS, hL;            // lane-distributed: lane l counts events with S (L) == l + 1
   unsigned pwT, pwW;          // this warp's executed thread / warp instructions (PER_WARP)
   unsigned seq;               // records emitted by this warp in this launch
-  unsigned lane, lane1, lanebit, lmlt, gwarp;
+  unsigned lane, lane1, lanebit, lmlt, gwarp, scr;
 
   __device__ __forceinline__ Hooks(const DevState& s, unsigned* smem) : st(s), sb(smem) {
     zero_range<0, NPC - 1>();
@@ -118,8 +185,10 @@ struct Hooks {
     lmlt = lanemask_lt();
     const unsigned tid = threadIdx.x + threadIdx.y * blockDim.x;
     gwarp = (blockIdx.x + blockIdx.y * gridDim.x) * ((blockDim.x * blockDim.y) >> 5) + (tid >> 5);
+    scr = (unsigned)__cvta_generic_to_shared(sb + kScratchWord0 + SCRATCH_WORDS * ((tid >> 5) & (kMaxWarps - 1)));
     if constexpr (kOn) {
-      for (int i = tid; i < kSmemWords; i += blockDim.x * blockDim.y) sb[i] = 0;
+      for (int i = tid; i < kSmemWords; i += blockDim.x * blockDim.y)
+        sb[i] = i < kScratchWord0 ? 0u : scratch_init_word((i - kScratchWord0) % SCRATCH_WORDS);
       __syncthreads();
     }
   }
@@ -159,8 +228,8 @@ struct Hooks {
       if constexpr (div || trc) {
         if (E != 0u) {
           if constexpr (div) {
-            const unsigned S = distinct(addr >> 5, E, lanebit, lmlt);
-            const unsigned L = distinct(addr >> 7, E, lanebit, lmlt);
+            unsigned S, L;
+            sectors_lines(addr, E, lane, lanebit, lmlt, scr, S, L);
             mN[PC] += 1u; mS[PC] += S; mL[PC] += L;
             inc_if_eq(hS, S, lane1);
             inc_if_eq(hL, L, lane1);

@@ -11,6 +11,7 @@
 //   * executed memory events of the tile (ballot) are processed by the whole warp: the 256 B slot is
 //     read by 32 lanes (8 B each, coalesced), S/L come from two __match_any_sync + leader ballots, the
 //     S/L histograms live in lane-distributed registers (lane l counts S == l + 1).
+#include <cstdlib>
 #include <cstring>
 
 #include "nvbt_internal.h"
@@ -89,8 +90,11 @@ __global__ void __launch_bounds__(256) k_gen(GenConsts G, unsigned long long fir
 
 // ---------------------------------------------------------------- replay
 constexpr int RP_THREADS = 512;
-constexpr int RP_BATCH = 4;  // memory events whose slots are loaded before processing
+constexpr int RP_BATCH = 8;  // memory events whose slots are loaded before processing
 
+__device__ __forceinline__ void red_shared_add(unsigned saddr, unsigned v) {
+  asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(saddr), "r"(v) : "memory");
+}
 __device__ __forceinline__ uint4 ld_nc_v4(const uint4* p) {
   uint4 r;
   asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
@@ -103,10 +107,25 @@ __device__ __forceinline__ unsigned long long ld_nc_u64(const unsigned long long
   return r;
 }
 
-__global__ void __launch_bounds__(RP_THREADS, 2)
+// Replay kernel variants (same results, different staging of the address slots):
+//   V = 0: 8 slot loads per batch into registers, batch processing unrolled (large code);
+//   V = 1: 8 slot loads per batch into registers, rolled processing loop (register select);
+//   V = 2: slots staged into shared memory with cp.async (8 B per lane), rolled processing loop.
+template <int V> struct ReplayCfg;
+template <> struct ReplayCfg<0> { static constexpr int THREADS = 512, MINB = 2; };
+template <> struct ReplayCfg<1> { static constexpr int THREADS = 512, MINB = 2; };
+template <> struct ReplayCfg<2> { static constexpr int THREADS = 1024, MINB = 1; };
+
+__device__ __forceinline__ void cp_async8(unsigned saddr, const void* g) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(saddr), "l"(g) : "memory");
+}
+
+template <int V>
+__global__ void __launch_bounds__(ReplayCfg<V>::THREADS, ReplayCfg<V>::MINB)
 k_replay(const uint4* __restrict__ hdr, const unsigned long long* __restrict__ addr, unsigned long long n, unsigned P,
          const uint8_t* __restrict__ kind, DevState st, unsigned long long* err) {
-  extern __shared__ unsigned sm[];
+  constexpr int NW = ReplayCfg<V>::THREADS / 32;
+  extern __shared__ __align__(16) unsigned sm[];
   unsigned* sA = sm;            // t_issued
   unsigned* sW = sm + P;        // w_issued
   unsigned* sDT = sm + 2 * P;   // popc(A & ~E)
@@ -114,18 +133,38 @@ k_replay(const uint4* __restrict__ hdr, const unsigned long long* __restrict__ a
   unsigned* sS = sm + 4 * P;
   unsigned* sL = sm + 5 * P;
   unsigned* sH = sm + 6 * P;    // hS[33], hL[33]
-  uint8_t* sK = reinterpret_cast<uint8_t*>(sm + 6 * P + 66);
+  unsigned* sScr = sm + ((6 * P + 66 + 3) & ~3u);   // per-warp scratch of sectors_lines() (16 B aligned)
+  unsigned long long* sStage = reinterpret_cast<unsigned long long*>(sScr + SCRATCH_WORDS * NW);  // V2: [NW][8][32]
+  uint8_t* sK = reinterpret_cast<uint8_t*>(sScr + SCRATCH_WORDS * NW + (V == 2 ? 2 * NW * RP_BATCH * 32 : 0));
   for (unsigned i = threadIdx.x; i < 6 * P + 66; i += blockDim.x) sm[i] = 0;
+  for (unsigned i = threadIdx.x; i < SCRATCH_WORDS * NW; i += blockDim.x) sScr[i] = scratch_init_word(i % SCRATCH_WORDS);
   for (unsigned i = threadIdx.x; i < P; i += blockDim.x) sK[i] = is_mem_kind(kind[i]);
   __syncthreads();
 
   const unsigned lane = lane_id(), lmlt = lanemask_lt(), lanebit = 1u << lane;
+  const unsigned s_base = (unsigned)__cvta_generic_to_shared(sm);
+  const unsigned s_scr = (unsigned)__cvta_generic_to_shared(sScr + SCRATCH_WORDS * (threadIdx.x >> 5));
+  const unsigned s_stage = (unsigned)__cvta_generic_to_shared(sStage + (threadIdx.x >> 5) * RP_BATCH * 32 + lane);
   unsigned hS = 0, hL = 0;
   unsigned bad = 0;
   const unsigned long long warps = (unsigned long long)gridDim.x * (blockDim.x >> 5);
   unsigned long long tile = (blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x) >> 5;
   uint4 h = make_uint4(0, 0, 0, 0);
   if (tile * 32 + lane < n) h = ld_nc_v4(hdr + tile * 32 + lane);
+
+  auto process = [&](unsigned long long a, int src, unsigned E) {
+    const unsigned es = __shfl_sync(FULL, E, src);
+    const unsigned ps = __shfl_sync(FULL, h.x, src);
+    unsigned S, L;
+    sectors_lines(a, es, lane, lanebit, lmlt, s_scr, S, L);
+    if (lane == 0) {
+      red_shared_add(s_base + 4u * (4 * P + ps), S);   // sS[ps]
+      red_shared_add(s_base + 4u * (5 * P + ps), L);   // sL[ps]
+    }
+    inc_if_eq(hS, S, lane + 1u);
+    inc_if_eq(hL, L, lane + 1u);
+  };
+
   for (; tile * 32 < n; tile += warps) {
     const bool valid = tile * 32 + lane < n;
     const unsigned pc = h.x, A = h.z, E = h.z & h.w, warp = h.y;
@@ -136,11 +175,12 @@ k_replay(const uint4* __restrict__ hdr, const unsigned long long* __restrict__ a
     const bool ok = valid && pc < P && A != 0u;
     bad += valid && pc >= P;
     if (ok) {
-      atomicAdd(&sA[pc], (unsigned)__popc(A));
-      atomicAdd(&sW[pc], 1u);
+      const unsigned a4 = s_base + 4u * pc;
+      red_shared_add(a4, (unsigned)__popc(A));          // sA[pc]
+      red_shared_add(a4 + 4u * P, 1u);                  // sW[pc]
       if (E != A) {
-        atomicAdd(&sDT[pc], (unsigned)__popc(A ^ E));
-        if (E == 0u) atomicAdd(&sDW[pc], 1u);
+        red_shared_add(a4 + 8u * P, (unsigned)__popc(A ^ E));   // sDT[pc]
+        if (E == 0u) red_shared_add(a4 + 12u * P, 1u);          // sDW[pc]
       }
       if (st.pw != nullptr && warp < st.n_warps) {
         atomicAdd(st.pw + warp, (unsigned long long)__popc(E));
@@ -148,25 +188,67 @@ k_replay(const uint4* __restrict__ hdr, const unsigned long long* __restrict__ a
       }
     }
     unsigned mm = __ballot_sync(FULL, ok && E != 0u && sK[ok ? pc : 0]);
+    const unsigned long long* tbase = addr + tile * 32 * 32 + lane;
     while (mm) {
-      int src[RP_BATCH];
-      unsigned long long a[RP_BATCH];
+      if constexpr (V == 0) {
+        int src[RP_BATCH];
+        unsigned long long a[RP_BATCH];
 #pragma unroll
-      for (int b = 0; b < RP_BATCH; ++b) {
-        src[b] = mm ? __ffs(mm) - 1 : -1;
-        if (mm) mm &= mm - 1;
-        if (src[b] >= 0) a[b] = ld_nc_u64(addr + (tile * 32 + src[b]) * 32 + lane);
-      }
+        for (int b = 0; b < RP_BATCH; ++b) {
+          src[b] = mm ? __ffs(mm) - 1 : -1;
+          if (mm) mm &= mm - 1;
+          if (src[b] >= 0) a[b] = ld_nc_u64(tbase + src[b] * 32);
+        }
 #pragma unroll
-      for (int b = 0; b < RP_BATCH; ++b) {
-        if (src[b] < 0) break;
-        const unsigned es = __shfl_sync(FULL, E, src[b]);
-        const unsigned ps = __shfl_sync(FULL, pc, src[b]);
-        const unsigned S = distinct(a[b] >> 5, es, lanebit, lmlt);
-        const unsigned L = distinct(a[b] >> 7, es, lanebit, lmlt);
-        if (lane == 0) { atomicAdd(&sS[ps], S); atomicAdd(&sL[ps], L); }
-        inc_if_eq(hS, S, lane + 1u);
-        inc_if_eq(hL, L, lane + 1u);
+        for (int b = 0; b < RP_BATCH; ++b) {
+          if (src[b] < 0) break;
+          process(a[b], src[b], E);
+        }
+      } else if constexpr (V == 1) {
+        unsigned long long a[RP_BATCH];
+        const unsigned batch = mm;
+        int nb = 0;
+#pragma unroll
+        for (int b = 0; b < RP_BATCH; ++b) {
+          if (mm) {
+            a[b] = ld_nc_u64(tbase + (__ffs(mm) - 1) * 32);
+            mm &= mm - 1;
+            ++nb;
+          }
+        }
+        unsigned rest = batch;
+#pragma unroll 1
+        for (int b = 0; b < nb; ++b) {
+          const int src = __ffs(rest) - 1;
+          rest &= rest - 1;
+          unsigned long long x = a[0];
+#pragma unroll
+          for (int k = 1; k < RP_BATCH; ++k) x = (b == k) ? a[k] : x;
+          process(x, src, E);
+        }
+      } else {
+        const unsigned batch = mm;
+        int nb = 0;
+#pragma unroll
+        for (int b = 0; b < RP_BATCH; ++b) {
+          if (mm) {
+            cp_async8(s_stage + 8u * 32u * b, tbase + (__ffs(mm) - 1) * 32);
+            mm &= mm - 1;
+            ++nb;
+          }
+        }
+        asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
+        __syncwarp();
+        unsigned rest = batch;
+#pragma unroll 1
+        for (int b = 0; b < nb; ++b) {
+          const int src = __ffs(rest) - 1;
+          rest &= rest - 1;
+          unsigned long long x;
+          asm volatile("ld.shared.u64 %0, [%1];" : "=l"(x) : "r"(s_stage + 8u * 32u * b) : "memory");
+          process(x, src, E);
+        }
+        __syncwarp();
       }
     }
     h = hn;
@@ -202,7 +284,12 @@ static int sm_count(int dev) {
   return g_sms > 0 ? g_sms : 148;
 }
 
-static size_t replay_smem(unsigned P) { return (6ull * P + 66) * 4 + P + 16; }
+template <int V>
+static size_t replay_smem(unsigned P) {
+  constexpr int NW = ReplayCfg<V>::THREADS / 32;
+  return (((6ull * P + 66 + 3) & ~3ull) + SCRATCH_WORDS * NW + (V == 2 ? 2ull * NW * RP_BATCH * 32 : 0)) * 4 + P + 16;
+}
+static int g_replay_variant = -1;
 
 }  // namespace nvbt
 
@@ -281,6 +368,35 @@ int nvbt_gen_events(nvbt_ctx c, uint64_t seed, uint64_t first, uint64_t n, void*
   return NVBT_OK;
 }
 
+}  // extern "C"
+
+template <int V>
+static int launch_replay(nvbt_ctx c, const void* d_hdr, const void* d_addr, uint64_t n, const DevState& st) {
+  const size_t smem = replay_smem<V>(c->n_pcs);
+  static bool attr_set = false;
+  if (!attr_set) {
+    NVBT_CUDA(cudaFuncSetAttribute(k_replay<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)replay_smem<V>(4096)));
+    attr_set = true;
+  }
+  const unsigned long long kMaxPerLaunch = 1ull << 30;  // keeps every CTA's u32 bins far from overflow
+  const int sms = sm_count(c->device);
+  const int per_sm = ReplayCfg<V>::MINB;
+  for (uint64_t off = 0; off < n; off += kMaxPerLaunch) {
+    const uint64_t m = std::min<uint64_t>(kMaxPerLaunch, n - off);
+    const unsigned long long tiles = (m + 31) / 32;
+    const int wpc = ReplayCfg<V>::THREADS / 32;
+    const int blocks = (int)std::min<unsigned long long>((tiles + 2 * wpc - 1) / (2 * wpc), (unsigned long long)sms * per_sm);
+    k_replay<V><<<blocks, ReplayCfg<V>::THREADS, smem, c->stream>>>(
+        static_cast<const uint4*>(d_hdr) + off, static_cast<const unsigned long long*>(d_addr) + off * 32, m,
+        c->n_pcs, c->d_kind, st, c->ctl + CTL_REPLAY_ERR);
+    NVBT_CUDA(cudaGetLastError());
+    c->launches++;
+  }
+  return NVBT_OK;
+}
+
+extern "C" {
+
 int nvbt_replay(nvbt_ctx c, const void* d_hdr, const void* d_addr, uint64_t n) {
   if (!c || !d_hdr || !d_addr) return set_error(NVBT_EINVAL, "null argument");
   if ((reinterpret_cast<uintptr_t>(d_hdr) | reinterpret_cast<uintptr_t>(d_addr)) % 16)
@@ -291,25 +407,15 @@ int nvbt_replay(nvbt_ctx c, const void* d_hdr, const void* d_addr, uint64_t n) {
   if (rc) return rc;
   if (n == 0) return NVBT_OK;
   NVBT_CUDA(cudaSetDevice(c->device));
-  const size_t smem = replay_smem(c->n_pcs);
-  static bool attr_set = false;
-  if (!attr_set) {
-    NVBT_CUDA(cudaFuncSetAttribute(k_replay, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)replay_smem(4096)));
-    attr_set = true;
+  if (g_replay_variant < 0) {
+    const char* e = getenv("NVBT_REPLAY_VARIANT");
+    g_replay_variant = e ? atoi(e) : 1;
   }
-  const unsigned long long kMaxPerLaunch = 1ull << 30;  // keeps every CTA's u32 bins far from overflow
-  const int sms = sm_count(c->device);
-  for (uint64_t off = 0; off < n; off += kMaxPerLaunch) {
-    const uint64_t m = std::min<uint64_t>(kMaxPerLaunch, n - off);
-    const unsigned long long tiles = (m + 31) / 32;
-    const int blocks = (int)std::min<unsigned long long>((tiles + 15) / 16, (unsigned long long)sms * 2);
-    k_replay<<<blocks, RP_THREADS, smem, c->stream>>>(static_cast<const uint4*>(d_hdr) + off,
-                                                      static_cast<const unsigned long long*>(d_addr) + off * 32, m,
-                                                      c->n_pcs, c->d_kind, st, c->ctl + CTL_REPLAY_ERR);
-    NVBT_CUDA(cudaGetLastError());
-    c->launches++;
+  switch (g_replay_variant) {
+    case 0: return launch_replay<0>(c, d_hdr, d_addr, n, st);
+    case 2: return launch_replay<2>(c, d_hdr, d_addr, n, st);
+    default: return launch_replay<1>(c, d_hdr, d_addr, n, st);
   }
-  return NVBT_OK;
 }
 
 }  // extern "C"

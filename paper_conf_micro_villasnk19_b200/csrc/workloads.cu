@@ -19,7 +19,7 @@ template <class Prog> struct ProgTraits;
 template <uint32_t T>
 __global__ void __launch_bounds__(256) k_vectoradd(const float* __restrict__ a, const float* __restrict__ b,
                                                    float* __restrict__ c, int N, DevState st) {
-  __shared__ unsigned sb[Hooks<T, ProgVectorAdd>::kSmemWords];
+  __shared__ __align__(16) unsigned sb[Hooks<T, ProgVectorAdd>::kSmemWords];
   Hooks<T, ProgVectorAdd> h(st, sb);
   const auto m0 = h.active(true);              // BB0: every lane
   const int tid = threadIdx.x;                 h.template at<0>(m0);
@@ -45,7 +45,7 @@ __global__ void __launch_bounds__(256) k_vectoradd(const float* __restrict__ a, 
 template <uint32_t T>
 __global__ void __launch_bounds__(256) k_sgemm(const float* __restrict__ A, const float* __restrict__ B,
                                                float* __restrict__ C, int M, int N, int K, DevState st) {
-  __shared__ unsigned sb[Hooks<T, ProgSgemm>::kSmemWords];
+  __shared__ __align__(16) unsigned sb[Hooks<T, ProgSgemm>::kSmemWords];
   Hooks<T, ProgSgemm> h(st, sb);
   const auto m0 = h.active(true);
   const int tx = threadIdx.x;                  h.template at<0>(m0);
@@ -87,7 +87,7 @@ template <uint32_t T>
 __global__ void __launch_bounds__(256) k_bfs_expand(const int* __restrict__ rowptr, const int* __restrict__ colidx,
                                                     int n, unsigned char* mask, const unsigned char* __restrict__ visited,
                                                     unsigned char* updating, DevState st) {
-  __shared__ unsigned sb[Hooks<T, ProgBfs>::kSmemWords];
+  __shared__ __align__(16) unsigned sb[Hooks<T, ProgBfs>::kSmemWords];
   Hooks<T, ProgBfs> h(st, sb);
   const auto m0 = h.active(true);
   const int tid = threadIdx.x;                 h.template at<0>(m0);
@@ -138,7 +138,7 @@ template <uint32_t T>
 __global__ void __launch_bounds__(256) k_bfs_update(int n, unsigned char* mask, unsigned char* visited,
                                                     unsigned char* updating, int* cost, int* over, int level,
                                                     DevState st) {
-  __shared__ unsigned sb[Hooks<T, ProgBfs>::kSmemWords];
+  __shared__ __align__(16) unsigned sb[Hooks<T, ProgBfs>::kSmemWords];
   Hooks<T, ProgBfs> h(st, sb);
   const auto m0 = h.active(true);
   const int tid = threadIdx.x;                 h.template at<22>(m0);
@@ -167,7 +167,7 @@ __global__ void __launch_bounds__(256) k_bfs_update(int n, unsigned char* mask, 
 template <uint32_t T>
 __global__ void __launch_bounds__(256) k_stencil(const float* __restrict__ in, float* __restrict__ out, int n,
                                                  DevState st) {
-  __shared__ unsigned sb[Hooks<T, ProgStencil>::kSmemWords];
+  __shared__ __align__(16) unsigned sb[Hooks<T, ProgStencil>::kSmemWords];
   Hooks<T, ProgStencil> h(st, sb);
   const auto m0 = h.active(true);
   const int tx = threadIdx.x;                  h.template at<0>(m0);

@@ -253,3 +253,49 @@ def test_replay_merge_equals_single(nvbt):
     torch.cuda.synchronize()
     assert torch.equal(nb.nvbt_accum_view(parts[0]), nb.nvbt_accum_view(whole))
     assert_same(read_all(nb, parts[0]), read_all(nb, whole), what="merged replay")
+
+
+def _adversarial_stream(n, seed):
+    """Handcrafted replay events stressing every sectors_lines() path: monotone runs, 32 KB bitmap window
+    edges (incl. keys below the first lane), 32-bit relative sort, 64-bit sort, partial and sparse masks,
+    duplicate sectors, line-boundary straddles, widths 1..16."""
+    rng = np.random.default_rng(seed)
+    prog = programs.replay()
+    mem_pcs = np.nonzero(programs.is_mem(prog))[0]
+    pc = rng.choice(mem_pcs, size=n)
+    warp = rng.integers(0, 1 << 20, size=n)
+    A = rng.integers(1, 1 << 32, size=n, dtype=np.uint64).astype(np.uint32)
+    A[: n // 2] = 0xFFFFFFFF
+    P = np.where(rng.random(n) < 0.5, np.uint32(0xFFFFFFFF),
+                 rng.integers(0, 1 << 32, size=n, dtype=np.uint64).astype(np.uint32))
+    lane = np.arange(32, dtype=np.int64)[None, :]
+    base = (rng.integers(1 << 20, 1 << 40, size=(n, 1)) & ~127).astype(np.int64)
+    kind = rng.integers(0, 8, size=(n, 1))
+    span = rng.choice([32, 1024 * 32 - 1, 1024 * 32, 1024 * 32 + 32, 1 << 20, 1 << 38], size=(n, 1))
+    r = rng.integers(0, 1 << 62, size=(n, 32)) % span - span // 2       # symmetric around base
+    stride = rng.choice([0, 1, 4, 31, 32, 33, 128, 4096], size=(n, 1))
+    addr = np.select([kind == 0, kind == 1, kind == 2, kind == 3],
+                     [base + lane * stride,                               # monotone
+                      base - lane * stride,                               # decreasing
+                      base + (r // 4) * 4,                                # window / wide random
+                      base + (lane % 3) * 32 + 124],                      # duplicates straddling lines
+                     base + r)
+    addr = np.clip(addr, 0, (1 << 62) - 1).astype(np.uint64)
+    return pc.astype(np.int64), warp.astype(np.int64), A, P, addr
+
+
+@pytest.mark.parametrize("seed", [1, 2])
+def test_replay_adversarial_addresses(nvbt, seed):
+    import torch
+    nb = nvbt.nvbt
+    n = 40_000
+    pc, warp, A, P, addr = _adversarial_stream(n, seed)
+    hdr = gen.header_bytes(pc, warp, A, P)
+    ctx = nb.nvbt_init(nb.W_REPLAY, nb.COUNT | nb.MEMDIV)
+    d_hdr = cuda(hdr.view(np.uint8).reshape(-1))
+    d_addr = cuda(addr.view(np.uint8).reshape(-1))
+    nb.nvbt_replay(ctx, d_hdr, d_addr, n)
+    g = read_all(nb, ctx)
+    acc = ev.Accumulator(programs.replay())
+    acc.add(0, warp, pc, A, P, addr)
+    assert_same(g, acc.result(), COUNT_KEYS + MEM_KEYS, f"adversarial replay seed {seed}")
