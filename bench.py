@@ -135,7 +135,7 @@ def sum_over_ranks(x, world, device=None):
 class SgemmBench:
     name = "c2"
     M = N = K = 1024
-    desc = "C2 naive row-fastest SGEMM 1024^3 (fp32), tools COUNT|MEMDIV (counts, opcode+BB histograms, divergence)"
+    desc = "C2 naive row-fastest SGEMM 1024^3 (fp32), tools BBCOUNT|MEMDIV (counts, opcode+BB histograms via BB-entry hooks, divergence)"
 
     def __init__(self, torch, nb, dr, world):
         self.torch, self.nb, self.dr, self.world = torch, nb, dr, world
@@ -143,7 +143,7 @@ class SgemmBench:
         M, N, K = self.M, self.N, self.K
         self.nw = nb.nvbt_workload_warps(nb.W_SGEMM, M, N)
         self.ctx = nb.nvbt_init(nb.W_SGEMM, nb.COUNT | nb.OPHIST | nb.BB | nb.MEMDIV)
-        self.tools = nb.TOOL_COUNT | nb.TOOL_MEMDIV
+        self.tools = nb.TOOL_BBCOUNT | nb.TOOL_MEMDIV
         self.hA = torch.from_numpy(uniform_f32((M, K), 3, -1, 1)).pin_memory()
         self.hB = torch.from_numpy(uniform_f32((K, N), 4, -1, 1)).pin_memory()
         self.A, self.B = self.hA.cuda(), self.hB.cuda()
@@ -173,7 +173,9 @@ class SgemmBench:
         """Issue roofline ("alu"): algorithmic warp-instructions per launch ÷ launch time vs
         148 SMs x 4 schedulers x 1 warp-instr/clk at the max SM clock."""
         K, W = self.K, self.nw
-        per_warp = (12 + 6 * K) * (1 + HOOK_OPS["count"]) + (K + 1) * HOOK_OPS["guard"] + \
+        # app instructions (one per warp-level event) + BB-entry hooks at the 3 + K leaders + guard
+        # hooks at pc7 and K x pc15 + divergence hooks at the 2K + 1 global LD/ST events
+        per_warp = (12 + 6 * K) + (K + 3) * HOOK_OPS["count"] + (K + 1) * HOOK_OPS["guard"] + \
             (2 * K + 1) * HOOK_OPS["mem"]
         ops = W * per_warp
         peak = N_SM * 4 * peaks.get("sm_max_mhz", 1965.0) * 1e6
@@ -201,7 +203,7 @@ class SgemmBench:
 
 
 # hook instruction costs per event used for the issue roofline (minimal SASS per hook)
-HOOK_OPS = {"count": 4, "guard": 6, "mem": 21}
+HOOK_OPS = {"count": 4, "guard": 6, "mem": 23}
 
 
 # --------------------------------------------------------------------------- C5 replay
@@ -310,7 +312,7 @@ def run_ours(args):
         "warmup": args.warmup, "ms_per_step": 1e3 * tot_instr / args.steps, "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
         "config": {"workload": wl.desc, "M": wl.M, "N": wl.N, "K": wl.K, "warp_events_per_launch": wl.events,
-                   "tools": "COUNT|MEMDIV", "l2": "flushed between steps (256 MiB write)",
+                   "tools": "BBCOUNT|MEMDIV", "l2": "flushed between steps (256 MiB write)",
                    "parallelism": f"replicas x{world} + int64 all-reduce merge per step" if world > 1 else "1 GPU"},
         "slowdown": slowdown, "plain_ms_per_launch": 1e3 * statistics.median(t_plain),
         "instr_ms_per_launch": 1e3 * t_kernel, "counts_check": "ok" if ok else f"mismatch {int(cnt[2])} != {expect}",

@@ -76,38 +76,22 @@ constexpr int SCRATCH_WORDS = 192;  // per-warp scratch of sectors_lines(): 64 x
 // Initial contents of scratch word i (keys empty = ~0, masks 0).
 __host__ __device__ constexpr unsigned scratch_init_word(int i) { return i < 128 ? 0xffffffffu : 0u; }
 
-// a5 kernel of Listing 8 (P:L189-213, P:L263; readings R-3, R-5, R-6): S = number of distinct 32 B
-// sectors and L = number of distinct 128 B lines touched by the lanes of E (E != 0). Exact integers.
-// Cheapest applicable method first (the warp takes one branch; every test is a vote):
-//  1. sector keys non-decreasing in lane order over E (coalesced, strided, broadcast, stencil
-//     neighbours): count lanes whose key differs from the previous lane of E — line keys are then
-//     sorted too. 1 shuffle (64-bit), 3 votes;
-//  2. every key inside the first lane's 32-sector (1 KB) word: OR-reduce one bit per sector;
-//     S = popc, L = popc of the OR-ed 4-bit groups;
-//  3. otherwise a per-warp open-addressing hash set of LINE keys in shared memory (`scr`: shared
-//     address of SCRATCH_WORDS words in their initial state, restored before returning): each lane of E
-//     inserts its line with a 64-bit CAS (linear probing, 64 slots >= 2 x 32 keys), then ORs its
-//     sector's bit into the slot's 4-bit mask; L = lanes that inserted, S = sum of mask popcounts.
-__device__ __forceinline__ void sectors_lines(unsigned long long addr, unsigned E, unsigned lane, unsigned lanebit,
-                                              unsigned lmlt, unsigned scr, unsigned& S, unsigned& L) {
+// Slow paths of sectors_lines() (addresses not non-decreasing in lane order):
+//  * every sector in the first lane's 32-sector (1 KB) word: OR-reduce one bit per sector;
+//    S = popc, L = popc of the OR-ed 4-bit groups;
+//  * otherwise a per-warp open-addressing hash set of LINE keys in shared memory (`scr`: shared address
+//    of SCRATCH_WORDS words in their initial state, restored before returning): each lane of E inserts
+//    its line with a 64-bit CAS (linear probing, 64 slots >= 2 x 32 keys), then ORs its sector's bit
+//    into the slot's 4-bit mask; L = lanes that inserted, S = sum of mask popcounts.
+__device__ __forceinline__ uint2 sectors_lines_unsorted(unsigned long long addr, unsigned E, unsigned lane,
+                                                        unsigned lanebit, unsigned scr) {
   const bool act = (E & lanebit) != 0u;
   const unsigned long long sk = addr >> 5;
-  const unsigned below = E & lmlt;
-  const int src = below ? 31 - __clz(below) : (int)lane;
-  const unsigned long long prev = __shfl_sync(FULL, sk, src);
-  if (__all_sync(FULL, !act || below == 0u || prev <= sk)) {
-    const bool first = below == 0u;
-    S = __popc(__ballot_sync(FULL, act && (first || sk != prev)));
-    L = __popc(__ballot_sync(FULL, act && (first || (sk >> 2) != (prev >> 2))));
-    return;
-  }
   const unsigned long long sk0 = __shfl_sync(FULL, sk, __ffs(E) - 1);
   if (__all_sync(FULL, !act || (sk >> 5) == (sk0 >> 5))) {
     const unsigned word = __reduce_or_sync(FULL, act ? 1u << (unsigned)(sk & 31) : 0u);
     const unsigned g = word | (word >> 1) | (word >> 2) | (word >> 3);
-    S = __popc(word);
-    L = __popc(g & 0x11111111u);
-    return;
+    return make_uint2(__popc(word), __popc(g & 0x11111111u));
   }
   const unsigned long long line = sk >> 2;
   unsigned slot = (((unsigned)line ^ (unsigned)(line >> 32)) * 0x9E3779B1u) >> 26;
@@ -126,14 +110,48 @@ __device__ __forceinline__ void sectors_lines(unsigned long long addr, unsigned 
     }
   }
   if (act) asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(scr + 512u + 4u * slot), "r"(1u << (unsigned)(sk & 3)) : "memory");
-  L = __popc(__ballot_sync(FULL, inserted));
+  const unsigned L = __popc(__ballot_sync(FULL, inserted));
   __syncwarp();
   unsigned m0, m1;
   asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(m0), "=r"(m1) : "r"(scr + 512u + 8u * lane) : "memory");
   asm volatile("st.shared.v2.u32 [%0], {%1, %1};" ::"r"(scr + 512u + 8u * lane), "r"(0u) : "memory");
   asm volatile("st.shared.v4.u32 [%0], {%1, %1, %1, %1};" ::"r"(scr + 16u * lane), "r"(0xffffffffu) : "memory");
-  S = __reduce_add_sync(FULL, __popc(m0) + __popc(m1));
+  const unsigned S = __reduce_add_sync(FULL, __popc(m0) + __popc(m1));
   __syncwarp();
+  return make_uint2(S, L);
+}
+static __device__ __noinline__ uint2 sectors_lines_unsorted_call(unsigned long long addr, unsigned E, unsigned lane,
+                                                                 unsigned lanebit, unsigned scr) {
+  return sectors_lines_unsorted(addr, E, lane, lanebit, scr);
+}
+
+// a5 kernel of Listing 8 (P:L189-213, P:L263; readings R-3, R-5, R-6): S = number of distinct 32 B
+// sectors and L = number of distinct 128 B lines touched by the lanes of E (E != 0). Exact integers.
+// Fast path (coalesced, strided, broadcast, stencil neighbours ...): when the addresses of the lanes of
+// E are non-decreasing in lane order, so are their sectors and lines, and each distinct value starts
+// where a lane's sector (line) differs from the previous lane of E — compared as (a ^ prev) >> 5 (7)
+// on 32-bit halves: 2 shuffles, 3 votes, ~18 instructions. Other orders take the slow paths above
+// (inlined when kInlineSlow, else an out-of-line call to keep the hooks' registers and code small).
+template <bool kInlineSlow = false>
+__device__ __forceinline__ void sectors_lines(unsigned long long addr, unsigned E, unsigned lane, unsigned lanebit,
+                                              unsigned lmlt, unsigned scr, unsigned& S, unsigned& L) {
+  const bool act = (E & lanebit) != 0u;
+  const unsigned below = E & lmlt;
+  const bool first = below == 0u;
+  const int src = 31 - __clz(below);               // previous lane of E (lane 31 when none: unused)
+  const unsigned a_lo = (unsigned)addr, a_hi = (unsigned)(addr >> 32);
+  const unsigned p_lo = __shfl_sync(FULL, a_lo, src), p_hi = __shfl_sync(FULL, a_hi, src);
+  const bool ge = a_hi > p_hi || (a_hi == p_hi && a_lo >= p_lo);
+  if (__all_sync(FULL, !act || first || ge)) {
+    const unsigned x_lo = a_lo ^ p_lo, x_hi = a_hi ^ p_hi;
+    S = __popc(__ballot_sync(FULL, act && (first || ((x_lo & ~31u) | x_hi) != 0u)));
+    L = __popc(__ballot_sync(FULL, act && (first || ((x_lo & ~127u) | x_hi) != 0u)));
+    return;
+  }
+  const uint2 r = kInlineSlow ? sectors_lines_unsorted(addr, E, lane, lanebit, scr)
+                              : sectors_lines_unsorted_call(addr, E, lane, lanebit, scr);
+  S = r.x;
+  L = r.y;
 }
 
 __device__ __forceinline__ unsigned umin(unsigned a, unsigned b) { return a < b ? a : b; }

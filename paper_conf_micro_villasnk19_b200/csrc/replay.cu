@@ -95,6 +95,10 @@ constexpr int RP_BATCH = 8;  // memory events whose slots are loaded before proc
 __device__ __forceinline__ void red_shared_add(unsigned saddr, unsigned v) {
   asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(saddr), "r"(v) : "memory");
 }
+__device__ __forceinline__ void red_shared_add_if(bool p, unsigned saddr, unsigned v) {
+  asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q red.shared.add.u32 [%0], %1;\n\t}"
+               ::"r"(saddr), "r"(v), "r"((unsigned)p) : "memory");
+}
 __device__ __forceinline__ uint4 ld_nc_v4(const uint4* p) {
   uint4 r;
   asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
@@ -120,7 +124,7 @@ __device__ __forceinline__ void cp_async8(unsigned saddr, const void* g) {
   asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(saddr), "l"(g) : "memory");
 }
 
-template <int V>
+template <int V, bool PW>
 __global__ void __launch_bounds__(ReplayCfg<V>::THREADS, ReplayCfg<V>::MINB)
 k_replay(const uint4* __restrict__ hdr, const unsigned long long* __restrict__ addr, unsigned long long n, unsigned P,
          const uint8_t* __restrict__ kind, DevState st, unsigned long long* err) {
@@ -156,11 +160,9 @@ k_replay(const uint4* __restrict__ hdr, const unsigned long long* __restrict__ a
     const unsigned es = __shfl_sync(FULL, E, src);
     const unsigned ps = __shfl_sync(FULL, h.x, src);
     unsigned S, L;
-    sectors_lines(a, es, lane, lanebit, lmlt, s_scr, S, L);
-    if (lane == 0) {
-      red_shared_add(s_base + 4u * (4 * P + ps), S);   // sS[ps]
-      red_shared_add(s_base + 4u * (5 * P + ps), L);   // sL[ps]
-    }
+    sectors_lines<true>(a, es, lane, lanebit, lmlt, s_scr, S, L);
+    red_shared_add_if(lane == 0, s_base + 4u * (4 * P + ps), S);   // sS[ps]
+    red_shared_add_if(lane == 0, s_base + 4u * (5 * P + ps), L);   // sL[ps]
     inc_if_eq(hS, S, lane + 1u);
     inc_if_eq(hL, L, lane + 1u);
   };
@@ -174,17 +176,18 @@ k_replay(const uint4* __restrict__ hdr, const unsigned long long* __restrict__ a
     if (nt * 32 + lane < n) hn = ld_nc_v4(hdr + nt * 32 + lane);
     const bool ok = valid && pc < P && A != 0u;
     bad += valid && pc >= P;
-    if (ok) {
-      const unsigned a4 = s_base + 4u * pc;
-      red_shared_add(a4, (unsigned)__popc(A));          // sA[pc]
-      red_shared_add(a4 + 4u * P, 1u);                  // sW[pc]
-      if (E != A) {
-        red_shared_add(a4 + 8u * P, (unsigned)__popc(A ^ E));   // sDT[pc]
-        if (E == 0u) red_shared_add(a4 + 12u * P, 1u);          // sDW[pc]
-      }
-      if (st.pw != nullptr && warp < st.n_warps) {
-        atomicAdd(st.pw + warp, (unsigned long long)__popc(E));
-        if (E) atomicAdd(st.pw + st.n_warps + warp, 1ull);
+    {  // branch-free: predicated shared reductions (E = A & P, so popc(A) - popc(E) = popc(A & ~E))
+      const unsigned a4 = s_base + 4u * (ok ? pc : 0u);
+      const unsigned pa = __popc(A), pe = __popc(E);
+      red_shared_add_if(ok, a4, pa);                         // sA[pc]
+      red_shared_add_if(ok, a4 + 4u * P, 1u);                // sW[pc]
+      red_shared_add_if(ok && pa != pe, a4 + 8u * P, pa - pe);   // sDT[pc]
+      red_shared_add_if(ok && E == 0u, a4 + 12u * P, 1u);    // sDW[pc]
+      if constexpr (PW) {
+        if (ok && warp < st.n_warps) {
+          atomicAdd(st.pw + warp, (unsigned long long)pe);
+          if (E) atomicAdd(st.pw + st.n_warps + warp, 1ull);
+        }
       }
     }
     unsigned mm = __ballot_sync(FULL, ok && E != 0u && sK[ok ? pc : 0]);
@@ -375,7 +378,8 @@ static int launch_replay(nvbt_ctx c, const void* d_hdr, const void* d_addr, uint
   const size_t smem = replay_smem<V>(c->n_pcs);
   static bool attr_set = false;
   if (!attr_set) {
-    NVBT_CUDA(cudaFuncSetAttribute(k_replay<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)replay_smem<V>(4096)));
+    NVBT_CUDA(cudaFuncSetAttribute(k_replay<V, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)replay_smem<V>(4096)));
+    NVBT_CUDA(cudaFuncSetAttribute(k_replay<V, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)replay_smem<V>(4096)));
     attr_set = true;
   }
   const unsigned long long kMaxPerLaunch = 1ull << 30;  // keeps every CTA's u32 bins far from overflow
@@ -386,7 +390,8 @@ static int launch_replay(nvbt_ctx c, const void* d_hdr, const void* d_addr, uint
     const unsigned long long tiles = (m + 31) / 32;
     const int wpc = ReplayCfg<V>::THREADS / 32;
     const int blocks = (int)std::min<unsigned long long>((tiles + 2 * wpc - 1) / (2 * wpc), (unsigned long long)sms * per_sm);
-    k_replay<V><<<blocks, ReplayCfg<V>::THREADS, smem, c->stream>>>(
+    auto kern = st.pw != nullptr ? k_replay<V, true> : k_replay<V, false>;
+    kern<<<blocks, ReplayCfg<V>::THREADS, smem, c->stream>>>(
         static_cast<const uint4*>(d_hdr) + off, static_cast<const unsigned long long*>(d_addr) + off * 32, m,
         c->n_pcs, c->d_kind, st, c->ctl + CTL_REPLAY_ERR);
     NVBT_CUDA(cudaGetLastError());

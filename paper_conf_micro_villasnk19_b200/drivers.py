@@ -5,7 +5,11 @@ scalars (the BFS `over` flag). No event arithmetic happens in Python.
 """
 from __future__ import annotations
 
-from . import nvbt as nb
+
+
+def _nb():
+    from . import nvbt
+    return nvbt
 
 
 def shard_range(n: int, rank: int, world: int):
@@ -42,7 +46,7 @@ def run_bfs(ctx, tools, rowptr, col, src, bufs=None, stream=None, max_levels=1 <
     while level < max_levels:
         b["over"].zero_()
         b["updating"].zero_()
-        nb.nvbt_bfs_level(ctx, tools, rowptr, col, n, b["mask"], b["visited"], b["updating"], b["cost"],
+        _nb().nvbt_bfs_level(ctx, tools, rowptr, col, n, b["mask"], b["visited"], b["updating"], b["cost"],
                           b["over"], level, stream=stream)
         over_h.copy_(b["over"], non_blocking=True)
         torch.cuda.current_stream().synchronize() if ctx is None else _sync(ctx)
@@ -62,7 +66,7 @@ def run_stencil(ctx, tools, buf0, buf1, n, iters, stream=None):
     """Iteration it reads buffer it % 2 and writes (it + 1) % 2 (EM §3.4). Returns the final buffer."""
     bufs = (buf0, buf1)
     for it in range(iters):
-        nb.nvbt_stencil(ctx, tools, bufs[it % 2], bufs[(it + 1) % 2], n, stream=stream)
+        _nb().nvbt_stencil(ctx, tools, bufs[it % 2], bufs[(it + 1) % 2], n, stream=stream)
     return bufs[iters % 2]
 
 
@@ -72,12 +76,22 @@ def replay_range(ctx, seed, first, n, hdr, addr, chunk=None):
     done = 0
     while done < n:
         m = min(cap, n - done)
-        nb.nvbt_gen_events(ctx, seed, first + done, m, hdr, addr)
-        nb.nvbt_replay(ctx, hdr, addr, m)
+        _nb().nvbt_gen_events(ctx, seed, first + done, m, hdr, addr)
+        _nb().nvbt_replay(ctx, hdr, addr, m)
         done += m
 
 
-def merge(ctx, group=None):
-    """a8: one int64 SUM all-reduce of the packed accumulator region (NCCL over NVLink on GPUs)."""
+def merge_tensor(t, group=None):
+    """Element-wise int64 SUM all-reduce of a packed accumulator tensor (any backend)."""
+    import torch
     import torch.distributed as dist
-    dist.all_reduce(nb.nvbt_accum_view(ctx), op=dist.ReduceOp.SUM, group=group)
+    if t.dtype != torch.int64:
+        raise TypeError("accumulators are int64")
+    dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)
+    return t
+
+
+def merge(ctx, group=None):
+    """a8: one int64 SUM all-reduce of the packed accumulator region (NCCL over NVLink on GPUs).
+    Sums of disjoint event sets add (EM §4), so every rank then holds the whole job's result."""
+    return merge_tensor(_nb().nvbt_accum_view(ctx), group)

@@ -38,7 +38,7 @@ __global__ void k_div(int pat, int iters, unsigned* out) {
     const unsigned E = 0xffffffffu;
     unsigned S, L;
     if (MODE == 0) {
-      sectors_lines(a, E, lane, lanebit, lmlt, bm, S, L);
+      sectors_lines<true>(a, E, lane, lanebit, lmlt, bm, S, L);
     } else {
       S = distinct_match(a >> 5, E, lanebit, lmlt);
       L = distinct_match(a >> 7, E, lanebit, lmlt);

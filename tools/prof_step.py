@@ -14,13 +14,13 @@ nb, dr = pkg.nvbt, pkg.drivers
 which = sys.argv[1] if len(sys.argv) > 1 else "all"
 if which in ("all", "c2"):
     M = N = K = 1024
-    ctx = nb.nvbt_init(nb.W_SGEMM, nb.COUNT | nb.MEMDIV)
+    ctx = nb.nvbt_init(nb.W_SGEMM, nb.COUNT | nb.BB | nb.MEMDIV)
     A = torch.from_numpy(uniform_f32((M, K), 3, -1, 1)).cuda()
     B = torch.from_numpy(uniform_f32((K, N), 4, -1, 1)).cuda()
     C = torch.empty(M, N, device="cuda")
     nb.nvbt_sgemm(ctx, nb.TOOL_NONE, A, B, C, M, N, K)
     nb.nvbt_sgemm(ctx, nb.TOOL_COUNT | nb.TOOL_MEMDIV, A, B, C, M, N, K)
-    nb.nvbt_sgemm(ctx, nb.TOOL_MEMDIV, A, B, C, M, N, K)
+    nb.nvbt_sgemm(ctx, nb.TOOL_BBCOUNT | nb.TOOL_MEMDIV, A, B, C, M, N, K)
     nb.nvbt_count(ctx)
 if which in ("all", "c5"):
     n = 1 << 26
