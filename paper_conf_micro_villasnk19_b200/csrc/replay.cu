@@ -281,6 +281,234 @@ k_replay(const uint4* __restrict__ hdr, const unsigned long long* __restrict__ a
     if (sH[i]) atomicAdd(st.hist + i, (unsigned long long)sH[i]);
 }
 
+// ---------------------------------------------------------------- replay, lane-per-event variant (V = 3)
+// Each warp takes 128 consecutive events per round (4 header tiles). Headers are counted as in the
+// other variants; the executed memory events of the round are compacted into a per-warp list, their
+// 256 B address slots gathered with coalesced 8 B/lane loads into a shared-memory stage (one 272 B row
+// per event), and then every LANE analyses one event on its own, reading its row with 16 B shared loads:
+// one pass over the 32 addresses counts sector/line boundaries (valid if the addresses are
+// non-decreasing) and sets bits in a per-lane 512-sector window bitmap (valid if they span < 16 KB);
+// events that are neither (wide random patterns) fall back to the warp-cooperative sectors_lines().
+// Per event this costs ~1/32 of the warp-cooperative instruction count for the common paths.
+constexpr int L3_NW = 8;                     // warps per CTA (1 CTA per SM)
+constexpr int L3_ROW = 68;                   // words per stage row (272 B: conflict-free 16 B lane reads)
+constexpr int L3_BMS = 17;                   // words per lane bitmap row (16 used; odd stride)
+constexpr int L3_WARP_WORDS = 3 * 128 + 32 * L3_ROW + 32 * L3_BMS + SCRATCH_WORDS;
+
+__device__ __forceinline__ void lds_v4(unsigned a, uint4& v) {
+  asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a));
+}
+__device__ __forceinline__ unsigned lds_u32(unsigned a) {
+  unsigned v;
+  asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a));
+  return v;
+}
+__device__ __forceinline__ void sts_u32(unsigned a, unsigned v) {
+  asm volatile("st.shared.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ void sts_u64(unsigned a, unsigned long long v) {
+  asm volatile("st.shared.u64 [%0], %1;" ::"r"(a), "l"(v) : "memory");
+}
+
+template <bool PW>
+__global__ void __launch_bounds__(32 * L3_NW, 1)
+k_replay_lane(const uint4* __restrict__ hdr, const unsigned long long* __restrict__ addr, unsigned long long n,
+              unsigned P, const uint8_t* __restrict__ kind, DevState st, unsigned long long* err) {
+  extern __shared__ __align__(16) unsigned sm[];
+  const unsigned P4 = (6 * P + 66 + 3) & ~3u;
+  unsigned* sH = sm + 6 * P;
+  unsigned* sWarp = sm + P4 + (threadIdx.x >> 5) * L3_WARP_WORDS;
+  uint8_t* sK = reinterpret_cast<uint8_t*>(sm + P4 + L3_NW * L3_WARP_WORDS);
+  for (unsigned i = threadIdx.x; i < P4; i += blockDim.x) sm[i] = 0;
+  for (unsigned i = threadIdx.x; i < L3_NW * L3_WARP_WORDS; i += blockDim.x) {
+    const unsigned o = i % L3_WARP_WORDS;
+    const unsigned s0 = 3 * 128 + 32 * L3_ROW + 32 * L3_BMS;
+    sm[P4 + i] = o >= s0 ? scratch_init_word(o - s0) : 0u;
+  }
+  for (unsigned i = threadIdx.x; i < P; i += blockDim.x) sK[i] = is_mem_kind(kind[i]);
+  __syncthreads();
+
+  const unsigned lane = lane_id(), lmlt = lanemask_lt(), lanebit = 1u << lane;
+  const unsigned s_base = (unsigned)__cvta_generic_to_shared(sm);
+  const unsigned s_list = (unsigned)__cvta_generic_to_shared(sWarp);            // [128][3]: idx, E, pc
+  const unsigned s_stage = s_list + 4u * 3u * 128u;                              // [32][L3_ROW]
+  const unsigned s_bm = s_stage + 4u * 32u * L3_ROW;                             // [32][L3_BMS]
+  const unsigned s_scr = s_bm + 4u * 32u * L3_BMS;                               // hash scratch
+  const unsigned my_row = s_stage + 4u * L3_ROW * lane;
+  const unsigned my_bm = s_bm + 4u * L3_BMS * lane;
+  unsigned bad = 0;
+  const unsigned long long warps = (unsigned long long)gridDim.x * L3_NW;
+  unsigned long long round = (blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x) >> 5;
+  uint4 h[4];
+#pragma unroll
+  for (int t = 0; t < 4; ++t) {
+    const unsigned long long i = round * 128 + t * 32 + lane;
+    h[t] = i < n ? ld_nc_v4(hdr + i) : make_uint4(0, 0, 0, 0);
+  }
+  for (; round * 128 < n; round += warps) {
+    // ---- headers: counts (predicated shared reductions) and the compacted memory-event list
+    unsigned c = 0;
+#pragma unroll
+    for (int t = 0; t < 4; ++t) {
+      const unsigned long long i = round * 128 + t * 32 + lane;
+      const bool valid = i < n;
+      const unsigned pc = h[t].x, A = h[t].z, E = h[t].z & h[t].w;
+      const bool ok = valid && pc < P && A != 0u;
+      bad += valid && pc >= P;
+      const unsigned a4 = s_base + 4u * (ok ? pc : 0u);
+      const unsigned pa = __popc(A), pe = __popc(E);
+      red_shared_add_if(ok, a4, pa);
+      red_shared_add_if(ok, a4 + 4u * P, 1u);
+      red_shared_add_if(ok && pa != pe, a4 + 8u * P, pa - pe);
+      red_shared_add_if(ok && E == 0u, a4 + 12u * P, 1u);
+      if constexpr (PW) {
+        const unsigned warp = h[t].y;
+        if (ok && warp < st.n_warps) {
+          atomicAdd(st.pw + warp, (unsigned long long)pe);
+          if (E) atomicAdd(st.pw + st.n_warps + warp, 1ull);
+        }
+      }
+      const bool mem = ok && E != 0u && sK[ok ? pc : 0];
+      const unsigned m = __ballot_sync(FULL, mem);
+      if (mem) {
+        const unsigned e = s_list + 12u * (c + __popc(m & lmlt));
+        sts_u32(e, (unsigned)(i - round * 128));   // event offset within the round
+        sts_u32(e + 4, E);
+        sts_u32(e + 8, pc);
+      }
+      c += __popc(m);
+    }
+    // prefetch the next round's headers
+    const unsigned long long nr = round + warps;
+#pragma unroll
+    for (int t = 0; t < 4; ++t) {
+      const unsigned long long i = nr * 128 + t * 32 + lane;
+      h[t] = i < n ? ld_nc_v4(hdr + i) : make_uint4(0, 0, 0, 0);
+    }
+    __syncwarp();
+    const unsigned long long* rbase = addr + round * 128 * 32 + lane;
+    for (unsigned r0 = 0; r0 < c; r0 += 32) {
+      const unsigned nrows = min(32u, c - r0);
+      // ---- gather: row s <- slot of list[r0 + s], lane l loads address l (256 B coalesced per row)
+      for (unsigned s = 0; s < nrows; s += 8) {
+        unsigned long long v[8];
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+          const unsigned row = min(s + k, nrows - 1);
+          const unsigned off = lds_u32(s_list + 12u * (r0 + row));
+          v[k] = ld_nc_u64(rbase + off * 32ull);
+        }
+#pragma unroll
+        for (int k = 0; k < 8; ++k)
+          if (s + k < nrows) sts_u64(s_stage + 4u * L3_ROW * (s + k) + 8u * lane, v[k]);
+      }
+      __syncwarp();
+      // ---- per-lane analysis of row `lane`
+      const bool have = lane < nrows;
+      const unsigned E = have ? lds_u32(s_list + 12u * (r0 + lane) + 4) : 0u;
+      const unsigned pc = have ? lds_u32(s_list + 12u * (r0 + lane) + 8) : 0u;
+      unsigned S = 0, L = 0;
+      bool hard = false;
+      if (have) {
+        const int f = __ffs(E) - 1;
+        const unsigned f_lo = lds_u32(my_row + 8u * f), f_hi = lds_u32(my_row + 8u * f + 4);
+        const unsigned wbase = ((f_lo >> 5) & ~31u) - 256u;     // 512-sector window, 32-sector aligned
+        unsigned prev = f_lo;
+        bool viol = false, hi_bad = false, out = false;
+        unsigned bs = 0, bl = 0;
+#pragma unroll
+        for (int q = 0; q < 16; ++q) {
+          uint4 v;
+          lds_v4(my_row + 16u * q, v);
+#pragma unroll
+          for (int u = 0; u < 2; ++u) {
+            const int l = 2 * q + u;
+            const bool act = (E >> l) & 1u;
+            const unsigned lo = act ? (u ? v.z : v.x) : prev;
+            const unsigned hi = act ? (u ? v.w : v.y) : f_hi;
+            hi_bad |= hi != f_hi;
+            viol |= lo < prev;
+            const unsigned x = lo ^ prev;
+            bs += (x & ~31u) != 0u;
+            bl += (x & ~127u) != 0u;
+            prev = lo;
+            const unsigned w = (lo >> 5) - wbase;
+            const bool in = w < 512u;
+            out |= !in;
+            if (in) asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(my_bm + 4u * (w >> 5)), "r"(1u << (w & 31u)) : "memory");
+          }
+        }
+        if (!hi_bad && !viol) {
+          S = bs + 1u;
+          L = bl + 1u;
+        } else if (!hi_bad && !out) {
+#pragma unroll
+          for (int k = 0; k < 16; ++k) {
+            const unsigned word = lds_u32(my_bm + 4u * k);
+            const unsigned g = word | (word >> 1) | (word >> 2) | (word >> 3);
+            S += __popc(word);
+            L += __popc(g & 0x11111111u);
+          }
+        } else {
+          hard = true;
+        }
+#pragma unroll
+        for (int k = 0; k < 16; ++k) sts_u32(my_bm + 4u * k, 0u);
+      }
+      // ---- hard rows: warp-cooperative exact path
+      unsigned hm = __ballot_sync(FULL, hard);
+      while (hm) {
+        const int src = __ffs(hm) - 1;
+        hm &= hm - 1;
+        const unsigned es = __shfl_sync(FULL, E, src);
+        unsigned long long a;
+        asm volatile("ld.shared.u64 %0, [%1];" : "=l"(a) : "r"(s_stage + 4u * L3_ROW * src + 8u * lane));
+        unsigned s2, l2;
+        sectors_lines<true>(a, es, lane, lanebit, lmlt, s_scr, s2, l2);
+        if (lane == (unsigned)src) { S = s2; L = l2; }
+      }
+      if (have) {
+        red_shared_add(s_base + 4u * (4 * P + pc), S);
+        red_shared_add(s_base + 4u * (5 * P + pc), L);
+        red_shared_add(s_base + 4u * (6 * P + S), 1u);        // hS[S]
+        red_shared_add(s_base + 4u * (6 * P + 33 + L), 1u);   // hL[L]
+      }
+      __syncwarp();
+    }
+  }
+  bad = __reduce_add_sync(FULL, bad);
+  if (lane == 0 && bad) atomicAdd(err, (unsigned long long)bad);
+  __syncthreads();
+  const unsigned* sA = sm;
+  const unsigned* sW = sm + P;
+  const unsigned* sDT = sm + 2 * P;
+  const unsigned* sDW = sm + 3 * P;
+  const unsigned* sS = sm + 4 * P;
+  const unsigned* sL = sm + 5 * P;
+  for (unsigned pc = threadIdx.x; pc < P; pc += blockDim.x) {
+    const unsigned a = sA[pc], w = sW[pc];
+    if (w) {
+      unsigned long long* s = st.site + 4 * pc;
+      atomicAdd(s + 0, (unsigned long long)a);
+      atomicAdd(s + 1, (unsigned long long)(a - sDT[pc]));
+      atomicAdd(s + 2, (unsigned long long)w);
+      atomicAdd(s + 3, (unsigned long long)(w - sDW[pc]));
+      if (sK[pc] && w != sDW[pc]) {
+        unsigned long long* m = st.mem + 3 * pc;
+        atomicAdd(m + 0, (unsigned long long)(w - sDW[pc]));
+        atomicAdd(m + 1, (unsigned long long)sS[pc]);
+        atomicAdd(m + 2, (unsigned long long)sL[pc]);
+      }
+    }
+  }
+  for (unsigned i = threadIdx.x; i < 66; i += blockDim.x)
+    if (sH[i]) atomicAdd(st.hist + i, (unsigned long long)sH[i]);
+}
+
+static size_t replay_lane_smem(unsigned P) {
+  return (((6ull * P + 66 + 3) & ~3ull) + (size_t)L3_NW * L3_WARP_WORDS) * 4 + P + 16;
+}
+
 static int g_sms = 0;
 static int sm_count(int dev) {
   if (g_sms == 0) cudaDeviceGetAttribute(&g_sms, cudaDevAttrMultiProcessorCount, dev);
@@ -400,6 +628,30 @@ static int launch_replay(nvbt_ctx c, const void* d_hdr, const void* d_addr, uint
   return NVBT_OK;
 }
 
+static int launch_replay_lane(nvbt_ctx c, const void* d_hdr, const void* d_addr, uint64_t n, const DevState& st) {
+  const size_t smem = replay_lane_smem(c->n_pcs);
+  static bool attr_set = false;
+  if (!attr_set) {
+    NVBT_CUDA(cudaFuncSetAttribute(k_replay_lane<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)replay_lane_smem(4096)));
+    NVBT_CUDA(cudaFuncSetAttribute(k_replay_lane<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)replay_lane_smem(4096)));
+    attr_set = true;
+  }
+  const unsigned long long kMaxPerLaunch = 1ull << 30;
+  const int sms = sm_count(c->device);
+  for (uint64_t off = 0; off < n; off += kMaxPerLaunch) {
+    const uint64_t m = std::min<uint64_t>(kMaxPerLaunch, n - off);
+    const unsigned long long rounds = (m + 127) / 128;
+    const int blocks = (int)std::min<unsigned long long>((rounds + L3_NW - 1) / L3_NW, (unsigned long long)sms);
+    auto kern = st.pw != nullptr ? k_replay_lane<true> : k_replay_lane<false>;
+    kern<<<blocks, 32 * L3_NW, smem, c->stream>>>(static_cast<const uint4*>(d_hdr) + off,
+                                                  static_cast<const unsigned long long*>(d_addr) + off * 32, m,
+                                                  c->n_pcs, c->d_kind, st, c->ctl + CTL_REPLAY_ERR);
+    NVBT_CUDA(cudaGetLastError());
+    c->launches++;
+  }
+  return NVBT_OK;
+}
+
 extern "C" {
 
 int nvbt_replay(nvbt_ctx c, const void* d_hdr, const void* d_addr, uint64_t n) {
@@ -414,11 +666,12 @@ int nvbt_replay(nvbt_ctx c, const void* d_hdr, const void* d_addr, uint64_t n) {
   NVBT_CUDA(cudaSetDevice(c->device));
   if (g_replay_variant < 0) {
     const char* e = getenv("NVBT_REPLAY_VARIANT");
-    g_replay_variant = e ? atoi(e) : 1;
+    g_replay_variant = e ? atoi(e) : 0;
   }
   switch (g_replay_variant) {
     case 0: return launch_replay<0>(c, d_hdr, d_addr, n, st);
     case 2: return launch_replay<2>(c, d_hdr, d_addr, n, st);
+    case 3: return launch_replay_lane(c, d_hdr, d_addr, n, st);
     default: return launch_replay<1>(c, d_hdr, d_addr, n, st);
   }
 }
