@@ -252,6 +252,11 @@ def run_ours(args):
 
     if args.workload == "c5":
         return run_replay(args, torch, nb, dr, rank, world, local, peaks, peaks_src)
+    if args.workload in ("c1", "c3", "c4"):
+        line = {"c1": run_c1, "c3": run_c3, "c4": run_c4}[args.workload](args, torch, nb, dr, local)
+        if rank == 0:
+            print(json.dumps(line), flush=True)
+        return
 
     wl = SgemmBench(torch, nb, dr, world)
     launches0 = nb.nvbt_launch_count(wl.ctx)
@@ -374,6 +379,123 @@ def run_replay(args, torch, nb, dr, rank, world, local, peaks, peaks_src):
         print(json.dumps(line), flush=True)
 
 
+
+# --------------------------------------------------------------------------- C1 / C3 / C4 (profiling lines)
+def _timed_events(torch, fn, n):
+    ts = []
+    for _ in range(n):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        fn()
+        e1.record()
+        e1.synchronize()
+        ts.append(e0.elapsed_time(e1) / 1e3)
+    return ts
+
+
+def run_c1(args, torch, nb, dr, local):
+    """C1: vectorAdd N = 65536, tools COUNT (instruction count + opcode histogram); a step is one launch."""
+    from synth import uniform_f32
+    N = 65536
+    ctx = nb.nvbt_init(nb.W_VECTORADD, nb.COUNT | nb.OPHIST)
+    a = torch.from_numpy(uniform_f32(N, 1)).cuda()
+    b = torch.from_numpy(uniform_f32(N, 2)).cuda()
+    c = torch.empty_like(a)
+    reps = 200   # launches per timed sample (a launch is a few microseconds)
+    f_plain = lambda: [nb.nvbt_vectoradd(ctx, nb.TOOL_NONE, a, b, c, N) for _ in range(reps)]
+    f_instr = lambda: [nb.nvbt_vectoradd(ctx, nb.TOOL_COUNT, a, b, c, N) for _ in range(reps)]
+    _timed_events(torch, f_instr, args.warmup)
+    _timed_events(torch, f_plain, args.warmup)
+    tp = _timed_events(torch, f_plain, args.steps)
+    nb.nvbt_reset(ctx)
+    with ClockSampler(local) as clk:
+        ti = _timed_events(torch, f_instr, args.steps)
+    cnt = nb.nvbt_count(ctx)
+    ev = int(cnt[2]) // (args.steps * reps)
+    t_i, t_p = sum(ti) / (args.steps * reps), sum(tp) / (args.steps * reps)
+    return {"metric": METRIC, "value": ev / t_i, "unit": "events/s", "n_gpus": 1, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": 1e3 * t_i, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+            "config": {"workload": "C1 vectorAdd N=65536, tools COUNT", "launches_per_sample": reps,
+                       "warp_events_per_launch": ev},
+            "slowdown": t_i / t_p, "plain_us_per_launch": 1e6 * t_p, "instr_us_per_launch": 1e6 * t_i,
+            "bound": "launch latency (26,624 warp events per launch)", "clocks": clk.summary()}
+
+
+def run_c3(args, torch, nb, dr, local):
+    """C3: BFS on an R-MAT scale-20 graph with BB-entry counting; a step is one whole BFS."""
+    from synth import rmat_csr, bfs_source
+    rowptr, col = rmat_csr(args.bfs_scale, 16, seed=3)
+    n = len(rowptr) - 1
+    src = bfs_source(rowptr)
+    rp, cl = torch.from_numpy(rowptr).cuda(), torch.from_numpy(col).cuda()
+    ctx = nb.nvbt_init(nb.W_BFS, nb.COUNT | nb.BB)
+    bufs = dr.bfs_buffers(n, "cuda")
+    f_plain = lambda: dr.run_bfs(ctx, nb.TOOL_NONE, rp, cl, src, bufs)
+    f_instr = lambda: dr.run_bfs(ctx, nb.TOOL_BBCOUNT, rp, cl, src, bufs)
+    for _ in range(args.warmup):
+        f_plain(); f_instr()
+    tp = _timed_events(torch, f_plain, args.steps)
+    nb.nvbt_reset(ctx)
+    with ClockSampler(local) as clk:
+        ti = _timed_events(torch, f_instr, args.steps)
+    cnt = nb.nvbt_count(ctx)
+    ev = int(cnt[2]) // args.steps
+    _, levels = f_plain()
+    return {"metric": METRIC, "value": ev * args.steps / sum(ti), "unit": "events/s", "n_gpus": 1,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * sum(ti) / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+            "config": {"workload": f"C3 BFS R-MAT scale {args.bfs_scale} ef16, tools BBCOUNT",
+                       "vertices": n, "directed_edges": int(len(col)), "levels": levels,
+                       "warp_events_per_bfs": ev},
+            "slowdown": sum(ti) / sum(tp), "plain_ms_per_bfs": 1e3 * sum(tp) / args.steps,
+            "bound": "latency of the hub warp's serial edge loop", "clocks": clk.summary()}
+
+
+def run_c4(args, torch, nb, dr, local):
+    """C4: 8192^2 5-point stencil x 100 iterations, every global LD/ST traced through the channel and
+    drained to pinned host memory (digest callback on all host cores); a step is the whole run."""
+    from synth import uniform_f32
+    n, iters = args.stencil_n, args.stencil_iters
+    ctx = nb.nvbt_init(nb.W_STENCIL, nb.COUNT | nb.TRACE)
+    x0 = torch.from_numpy(uniform_f32((n, n), 4)).cuda()
+    buf0, buf1 = x0.clone(), torch.empty_like(x0)
+    ring = torch.empty(64 + 288 * args.ring_records, dtype=torch.uint8, pin_memory=True)
+    ch = nb.nvbt_channel_open(ctx, ring)
+    # plain baseline
+    for _ in range(args.warmup):
+        dr.run_stencil(ctx, nb.TOOL_NONE, buf0, buf1, n, iters)
+    tp = _timed_events(torch, lambda: dr.run_stencil(ctx, nb.TOOL_NONE, buf0, buf1, n, iters), args.steps)
+    # traced runs: wall time from first launch to the last record drained
+    res = []
+    with ClockSampler(local) as clk:
+        for _ in range(args.steps):
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            dr.run_stencil(ctx, nb.TOOL_TRACE, buf0, buf1, n, iters)
+            e1.record()
+            d = nb.nvbt_channel_drain_digest(ch, timeout_us=600_000_000)
+            torch.cuda.synchronize()
+            res.append((time.perf_counter() - t0, d.n_rec, e0.elapsed_time(e1) / 1e3))
+    dropped = nb.nvbt_channel_dropped(ch)
+    recs = res[-1][1]
+    t_tr = sum(r[0] for r in res) / len(res)
+    G = n // 32
+    expect = iters * (2 * (n * n // 32) + 4 * (n - 2) * G)
+    return {"metric": "traced warp-level memory events/sec (records drained to host)", "value": recs / t_tr,
+            "unit": "records/s", "n_gpus": 1, "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * t_tr,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+            "config": {"workload": f"C4 stencil {n}^2 x {iters}, tools TRACE", "ring_records": args.ring_records},
+            "records_per_run": recs, "records_expected": expect, "dropped": dropped,
+            "gpu_s_per_run": sum(r[2] for r in res) / len(res),
+            "host_threads": os.environ.get("NVBT_DRAIN_THREADS", str(os.cpu_count())),
+            "GB_per_s_to_host": recs * 288 / t_tr / 1e9, "slowdown": t_tr / (sum(tp) / len(tp)),
+            "plain_ms": 1e3 * sum(tp) / len(tp), "bound": "PCIe D2H (measured 52.7 GB/s SM stores to pinned memory)",
+            "clocks": clk.summary()}
+
+
 def run_reference(args):
     """Reference arm = the CPU oracle (this tier has no runnable reference)."""
     rank = int(os.environ.get("RANK", "0"))
@@ -417,7 +539,11 @@ def main():
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--workload", choices=["c2", "c5"], default="c2")
+    ap.add_argument("--workload", choices=["c1", "c2", "c3", "c4", "c5"], default="c2")
+    ap.add_argument("--bfs-scale", type=int, default=20)
+    ap.add_argument("--stencil-n", type=int, default=8192)
+    ap.add_argument("--stencil-iters", type=int, default=100)
+    ap.add_argument("--ring-records", type=int, default=1 << 22)
     ap.add_argument("--replay-events", type=int, default=10**10)
     ap.add_argument("--cpu-budget", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")

@@ -10,8 +10,13 @@
 //    matches, zeroes the tag field (EM §5 "reserved = 0"), calls the user callback on contiguous batches
 //    and publishes tail.
 #include <chrono>
+#include <condition_variable>
 #include <cstring>
+#include <functional>
 #include <immintrin.h>
+#include <thread>
+
+#include <cstdlib>
 
 #include "nvbt_internal.h"
 
@@ -51,11 +56,12 @@ struct DigestConsts {
 };
 static const DigestConsts kDig;
 
-static void digest_range(const unsigned char* rec, uint64_t n, uint64_t* d1, uint64_t* d2) {
+static void digest_serial(const unsigned char* rec, uint64_t n, uint64_t* d1, uint64_t* d2) {
   uint64_t s1 = 0, s2 = 0;
   for (uint64_t r = 0; r < n; ++r) {
     uint64_t x[36];
     std::memcpy(x, rec + r * RECORD_BYTES, RECORD_BYTES);
+    x[3] &= 0x00000000ffffffffull;  // bytes 28..31: ring tag, delivered as 0 (EM §5 reserved)
     uint64_t h1 = 0, h2 = 0;
     for (int j = 0; j < 36; ++j) { h1 += x[j] * kDig.c1[j]; h2 += x[j] * kDig.c2[j]; }
     s1 += mix64(h1);
@@ -65,9 +71,121 @@ static void digest_range(const unsigned char* rec, uint64_t n, uint64_t* d1, uin
   *d2 += s2;
 }
 
+// Small persistent worker pool for host-side record processing (the drain's digest runs on all host
+// cores: 362 GB of C4 records must be consumed at link speed). parallel_for splits [0, n) into equal
+// contiguous parts, the calling thread takes part 0.
+class Pool {
+ public:
+  static Pool& get() {
+    static Pool p;
+    return p;
+  }
+  unsigned size() const { return (unsigned)workers_.size() + 1; }
+  void parallel_for(uint64_t n, const std::function<void(unsigned, uint64_t, uint64_t)>& fn) {
+    const unsigned T = size();
+    if (T == 1 || n < 4096) { fn(0, 0, n); return; }
+    {
+      std::lock_guard<std::mutex> g(m_);
+      fn_ = &fn; n_ = n; parts_ = T; pending_ = T - 1; ++gen_;
+    }
+    cv_.notify_all();
+    fn(0, 0, n / T);
+    std::unique_lock<std::mutex> lk(m_);
+    done_.wait(lk, [&] { return pending_ == 0; });
+    fn_ = nullptr;
+  }
+  ~Pool() {
+    { std::lock_guard<std::mutex> g(m_); stop_ = true; ++gen_; }
+    cv_.notify_all();
+    for (auto& t : workers_) t.join();
+  }
+
+ private:
+  Pool() {
+    unsigned hw = std::thread::hardware_concurrency();
+    const char* e = getenv("NVBT_DRAIN_THREADS");
+    if (e) hw = (unsigned)atoi(e);
+    if (hw == 0) hw = 1;
+    if (hw > 64) hw = 64;
+    for (unsigned i = 1; i < hw; ++i) workers_.emplace_back([this, i] { run(i); });
+  }
+  void run(unsigned id) {
+    uint64_t seen = 0;
+    for (;;) {
+      const std::function<void(unsigned, uint64_t, uint64_t)>* fn;
+      uint64_t n;
+      unsigned parts;
+      {
+        std::unique_lock<std::mutex> lk(m_);
+        cv_.wait(lk, [&] { return stop_ || gen_ != seen; });
+        if (stop_) return;
+        seen = gen_;
+        fn = fn_; n = n_; parts = parts_;
+      }
+      (*fn)(id, n * id / parts, n * (id + 1) / parts);
+      {
+        std::lock_guard<std::mutex> g(m_);
+        if (--pending_ == 0) done_.notify_one();
+      }
+    }
+  }
+  std::vector<std::thread> workers_;
+  std::mutex m_;
+  std::condition_variable cv_, done_;
+  const std::function<void(unsigned, uint64_t, uint64_t)>* fn_ = nullptr;
+  uint64_t n_ = 0, gen_ = 0;
+  unsigned parts_ = 1, pending_ = 0;
+  bool stop_ = false;
+};
+
+static void digest_range(const unsigned char* rec, uint64_t n, uint64_t* d1, uint64_t* d2) {
+  if (n < 8192) { digest_serial(rec, n, d1, d2); return; }
+  Pool& pool = Pool::get();
+  std::vector<uint64_t> p1(pool.size(), 0), p2(pool.size(), 0);
+  pool.parallel_for(n, [&](unsigned id, uint64_t lo, uint64_t hi) {
+    digest_serial(rec + lo * RECORD_BYTES, hi - lo, &p1[id], &p2[id]);
+  });
+  for (size_t i = 0; i < p1.size(); ++i) { *d1 += p1[i]; *d2 += p2[i]; }
+}
+
+
+// Length of the prefix of slots [0, lim) whose tag equals `lap` (written and committed). Scans a short
+// window serially and, when that is all ready, the rest of the batch in parallel on the pool.
+static inline bool slot_ready(const unsigned char* rec, uint32_t lap) {
+  return *reinterpret_cast<volatile const uint32_t*>(rec + 28) == lap;
+}
+static uint64_t ready_prefix(const unsigned char* base, uint64_t lim, uint32_t lap) {
+  const uint64_t w = std::min<uint64_t>(lim, 2048);
+  uint64_t n = 0;
+  while (n < w && slot_ready(base + n * RECORD_BYTES, lap)) ++n;
+  if (n < w || n == lim) return n;
+  Pool& pool = Pool::get();
+  const uint64_t rest = lim - n;
+  std::vector<uint64_t> first(pool.size(), UINT64_MAX);
+  const unsigned char* b2 = base + n * RECORD_BYTES;
+  pool.parallel_for(rest, [&](unsigned id, uint64_t lo, uint64_t hi) {
+    uint64_t i = lo;
+    while (i < hi && slot_ready(b2 + i * RECORD_BYTES, lap)) ++i;
+    first[id] = i < hi ? i : UINT64_MAX;
+  });
+  uint64_t stop = rest;
+  for (uint64_t f : first) stop = std::min(stop, f);
+  return n + stop;
+}
+static void clear_tags(unsigned char* base, uint64_t n) {
+  Pool::get().parallel_for(n, [&](unsigned, uint64_t lo, uint64_t hi) {
+    for (uint64_t r = lo; r < hi; ++r) std::memset(base + r * RECORD_BYTES + 28, 0, 4);
+  });
+}
+
 }  // namespace nvbt
 
 using namespace nvbt;
+
+extern "C" {
+int nvbt_drain_digest(const void* records, uint64_t n_records, void* user);
+int nvbt_drain_copy(const void* records, uint64_t n_records, void* user);
+}
 
 extern "C" {
 
@@ -121,24 +239,20 @@ int nvbt_channel_drain(nvbt_channel ch, nvbt_drain_fn fn, void* user, int64_t ti
   nvbt_ctx c = ch->ctx;
   NVBT_CUDA(cudaSetDevice(c->device));
   const auto t0 = std::chrono::steady_clock::now();
-  const uint64_t kBatch = 1u << 16;
+  const uint64_t kBatch = 1u << 17;
   volatile uint64_t* tail = reinterpret_cast<volatile uint64_t*>(ch->host);
+  const bool builtin = fn == nvbt_drain_digest || fn == nvbt_drain_copy;
   uint64_t delivered = 0;
   int rc = NVBT_OK;
   for (;;) {
     const uint64_t slot = ch->consumed % ch->cap;
     const uint32_t lap = static_cast<uint32_t>(ch->consumed / ch->cap) + 1u;
     const uint64_t lim = std::min<uint64_t>(ch->cap - slot, kBatch);
-    uint64_t n = 0;
-    while (n < lim) {
-      volatile const uint32_t* tag = reinterpret_cast<volatile const uint32_t*>(ch->slots + (slot + n) * RECORD_BYTES + 28);
-      if (*tag != lap) break;
-      ++n;
-    }
+    const uint64_t n = ready_prefix(ch->slots + slot * RECORD_BYTES, lim, lap);
     if (n) {
       std::atomic_thread_fence(std::memory_order_acquire);
       unsigned char* base = ch->slots + slot * RECORD_BYTES;
-      for (uint64_t r = 0; r < n; ++r) std::memset(base + r * RECORD_BYTES + 28, 0, 4);
+      if (!builtin) clear_tags(base, n);   // built-in callbacks ignore / clear the tag themselves
       const int urc = fn(base, n, user);
       ch->consumed += n;
       delivered += n;
@@ -183,7 +297,12 @@ int nvbt_drain_digest(const void* records, uint64_t n, void* user) {
 int nvbt_drain_copy(const void* records, uint64_t n, void* user) {
   auto* s = static_cast<nvbt_copy_sink*>(user);
   if (!s || s->n + n > s->capacity) return 1;
-  std::memcpy(static_cast<unsigned char*>(s->dst) + s->n * RECORD_BYTES, records, n * RECORD_BYTES);
+  unsigned char* dst = static_cast<unsigned char*>(s->dst) + s->n * RECORD_BYTES;
+  const unsigned char* src = static_cast<const unsigned char*>(records);
+  Pool::get().parallel_for(n, [&](unsigned, uint64_t lo, uint64_t hi) {
+    std::memcpy(dst + lo * RECORD_BYTES, src + lo * RECORD_BYTES, (hi - lo) * RECORD_BYTES);
+    for (uint64_t r = lo; r < hi; ++r) std::memset(dst + r * RECORD_BYTES + 28, 0, 4);
+  });
   s->n += n;
   return 0;
 }

@@ -160,11 +160,14 @@ __device__ __forceinline__ void inc_if_eq(unsigned& h, unsigned v, unsigned ref)
   asm("{\n\t.reg .pred p;\n\tsetp.eq.u32 p, %1, %2;\n\t@p add.u32 %0, %0, 1;\n\t}" : "+r"(h) : "r"(v), "r"(ref));
 }
 
-// Ring reservation with backpressure. Returns false if the host never freed a slot
-// within ~2 s (or another producer already gave up): the record is dropped and counted.
-__device__ __forceinline__ bool wait_slot(const DevState& st, unsigned long long t) {
-  const unsigned long long tc = *(volatile const unsigned long long*)st.tail_cache;
-  if (t < tc + st.cap) return true;
+// Ring backpressure: ticket t may be written once t < tail + cap. has_room() is the
+// cheap check against the device-side cache of the host's consumer index; wait_room() spins on the host
+// index (PCIe reads) and returns false if the host never freed a slot within ~2 s or another producer
+// already gave up (the record is then dropped and counted, never hangs the GPU).
+__device__ __forceinline__ bool has_room(const DevState& st, unsigned long long t) {
+  return t < *(volatile const unsigned long long*)st.tail_cache + st.cap;
+}
+__device__ __forceinline__ bool wait_room(const DevState& st, unsigned long long t) {
   if (*(volatile const unsigned long long*)st.dropped != 0) return false;
   const unsigned long long t0 = globaltimer();
   for (;;) {
@@ -192,6 +195,9 @@ struct Hooks {
   unsigned hS, hL;            // lane-distributed: lane l counts events with S (L) == l + 1
   unsigned pwT, pwW;          // this warp's executed thread / warp instructions (PER_WARP)
   unsigned seq;               // records emitted by this warp in this launch
+  unsigned npend = 0;         // uncommitted records of this warp (warp-uniform)
+  unsigned pend_val = 0;      // lane k: tag value of the k-th uncommitted record
+  unsigned char* pend_tag = nullptr;
   unsigned lane, lane1, lanebit, lmlt, gwarp, scr;
 
   __device__ __forceinline__ Hooks(const DevState& s, unsigned* smem) : st(s), sb(smem) {
@@ -258,32 +264,61 @@ struct Hooks {
     }
   }
 
+  // a6 producer. One record per executed global-memory event: lane 0 takes a ticket; the warp writes
+  // the 32 addresses (8 B per lane, 256 B coalesced) and the header with a zero tag straight into the
+  // pinned host ring. Commits are batched: lane (k % 32) remembers the tag word of the warp's k-th
+  // uncommitted record, and commit() makes every pending payload visible system-wide (one fence per lane
+  // per batch instead of one per record) before the tags are stored. A warp commits before it can block
+  // on a full ring, so reserved-but-uncommitted slots never stall the consumer for ever.
   template <int PC>
   __device__ __forceinline__ void emit(unsigned A, unsigned P, bool act, unsigned long long addr) {
     constexpr nvbt_instr_desc d = Prog::t[PC];
     unsigned long long t = 0;
-    int ok = 1;
-    if (lane == 0) { t = atomicAdd(st.head, 1ull); ok = wait_slot(st, t); }
+    int room = 1;
+    if (lane == 0) {
+      t = atomicAdd(st.head, 1ull);
+      room = has_room(st, t);
+    }
     t = __shfl_sync(FULL, t, 0);
-    ok = __shfl_sync(FULL, ok, 0);
-    if (!ok) {
-      if (lane == 0) atomicAdd(st.dropped, 1ull);
-    } else {
-      const unsigned long long lap = t / st.cap;
-      unsigned char* rec = st.ring + (t - lap * st.cap) * RECORD_BYTES;
-      reinterpret_cast<unsigned long long*>(rec + 32)[lane] = act ? addr : 0ull;
-      if (lane == 0)
-        *reinterpret_cast<uint4*>(rec) = make_uint4(st.launch, gwarp, seq, (unsigned)PC);
-      __syncwarp();
-      if (lane == 0) {
-        __threadfence_system();
-        const unsigned w2 = (unsigned)d.opcode | ((unsigned)d.width << 16) | ((unsigned)d.kind << 24);
-        asm volatile("st.volatile.global.v4.u32 [%0], {%1, %2, %3, %4};" ::"l"(rec + 16), "r"(A), "r"(P), "r"(w2),
-                     "r"((unsigned)lap + 1u)
-                     : "memory");
+    if (!__shfl_sync(FULL, room, 0)) {
+      commit();
+      int ok = 1;
+      if (lane == 0) ok = wait_room(st, t);
+      if (!__shfl_sync(FULL, ok, 0)) {
+        if (lane == 0) atomicAdd(st.dropped, 1ull);
+        ++seq;
+        return;
       }
     }
+    const unsigned long long lap = t / st.cap;
+    unsigned char* rec = st.ring + (t - lap * st.cap) * RECORD_BYTES;
+    // the whole 288 B record in ONE warp store: lane j < 18 writes bytes [16j, 16j + 16) — lanes 0, 1 the
+    // header (tag 0), lane j >= 2 the addresses of lanes 2(j-2), 2(j-2)+1 (gathered with shuffles)
+    const unsigned long long a = act ? addr : 0ull;
+    const unsigned src = 2u * (lane - 2u);
+    const unsigned long long a0 = __shfl_sync(FULL, a, src & 31u), a1 = __shfl_sync(FULL, a, (src + 1u) & 31u);
+    if (lane < 18) {
+      const unsigned w2 = (unsigned)d.opcode | ((unsigned)d.width << 16) | ((unsigned)d.kind << 24);
+      const uint4 v = lane == 0   ? make_uint4(st.launch, gwarp, seq, (unsigned)PC)
+                      : lane == 1 ? make_uint4(A, P, w2, 0u)
+                                  : make_uint4((unsigned)a0, (unsigned)(a0 >> 32), (unsigned)a1, (unsigned)(a1 >> 32));
+      *reinterpret_cast<uint4*>(rec + 16 * lane) = v;
+    }
+    if (lane == npend) {
+      pend_tag = rec + 28;
+      pend_val = (unsigned)lap + 1u;
+    }
     ++seq;
+    if (++npend == 32) commit();
+  }
+
+  __device__ __forceinline__ void commit() {
+    if (npend == 0) return;
+    __threadfence_system();   // this lane's payload stores are performed system-wide ...
+    __syncwarp();             // ... for every lane, before any tag below is written
+    if (lane < npend)
+      asm volatile("st.volatile.global.u32 [%0], %1;" ::"l"(pend_tag), "r"(pend_val) : "memory");
+    npend = 0;
   }
 
   // executed-instruction totals of pc range [LO, HI] (for PER_WARP), BB-derived where needed
@@ -363,6 +398,7 @@ struct Hooks {
   // Must be reached by every thread of the CTA.
   __device__ __forceinline__ void finish() {
     if constexpr (kOn) {
+      if constexpr ((T & TOOL_TRACE) != 0) commit();
       retire<0, NPC - 1>();
       if (hS) atomicAdd(&sb[NPC * SITE_WORDS + 1 + lane], hS);
       if (hL) atomicAdd(&sb[NPC * SITE_WORDS + 34 + lane], hL);
