@@ -76,13 +76,21 @@ constexpr int SCRATCH_WORDS = 192;  // per-warp scratch of sectors_lines(): 64 x
 // Initial contents of scratch word i (keys empty = ~0, masks 0).
 __host__ __device__ constexpr unsigned scratch_init_word(int i) { return i < 128 ? 0xffffffffu : 0u; }
 
-// Slow paths of sectors_lines() (addresses not non-decreasing in lane order):
+// Slow paths of sectors_lines() (addresses not non-decreasing in lane order), cheapest first; `scr` is
+// the warp's shared scratch (SCRATCH_WORDS words in their initial state, restored before returning):
 //  * every sector in the first lane's 32-sector (1 KB) word: OR-reduce one bit per sector;
 //    S = popc, L = popc of the OR-ed 4-bit groups;
-//  * otherwise a per-warp open-addressing hash set of LINE keys in shared memory (`scr`: shared address
-//    of SCRATCH_WORDS words in their initial state, restored before returning): each lane of E inserts
-//    its line with a 64-bit CAS (linear probing, 64 slots >= 2 x 32 keys), then ORs its sector's bit
-//    into the slot's 4-bit mask; L = lanes that inserted, S = sum of mask popcounts.
+//  * every sector within a 1024-sector (32 KB) window: a 32-word shared bitmap, same counts;
+//  * all lines distinct (hashed 4096-bucket occupancy == |E|): S = L = |E|;
+//  * otherwise a per-warp open-addressing hash set of LINE keys: each lane of E inserts its line with a
+//    64-bit CAS (linear probing, 64 slots >= 2 x 32 keys), then ORs its sector's bit into the slot's
+//    4-bit mask; L = lanes that inserted, S = sum of mask popcounts.
+__device__ __forceinline__ unsigned lds_u32_(unsigned a) {
+  unsigned v;
+  asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
+  return v;
+}
+
 __device__ __forceinline__ uint2 sectors_lines_unsorted(unsigned long long addr, unsigned E, unsigned lane,
                                                         unsigned lanebit, unsigned scr) {
   const bool act = (E & lanebit) != 0u;
@@ -93,8 +101,33 @@ __device__ __forceinline__ uint2 sectors_lines_unsorted(unsigned long long addr,
     const unsigned g = word | (word >> 1) | (word >> 2) | (word >> 3);
     return make_uint2(__popc(word), __popc(g & 0x11111111u));
   }
+  // 32 KB window around the first lane's sector: clear one bit per sector in the 32 "key" words (kept
+  // at ~0 between uses, so the same area doubles as the hash table's empty keys)
+  const long long wv = (long long)(sk - (sk0 & ~31ull)) + 512;
+  if (__all_sync(FULL, !act || (wv >= 0 && wv < 1024))) {
+    if (act) asm volatile("red.shared.and.b32 [%0], %1;" ::"r"(scr + 4u * (unsigned)(wv >> 5)), "r"(~(1u << (unsigned)(wv & 31))) : "memory");
+    __syncwarp();
+    const unsigned word = ~lds_u32_(scr + 4u * lane);
+    asm volatile("st.shared.u32 [%0], %1;" ::"r"(scr + 4u * lane), "r"(0xffffffffu) : "memory");
+    __syncwarp();
+    const unsigned g = word | (word >> 1) | (word >> 2) | (word >> 3);
+    return make_uint2(__reduce_add_sync(FULL, __popc(word)), __reduce_add_sync(FULL, __popc(g & 0x11111111u)));
+  }
   const unsigned long long line = sk >> 2;
-  unsigned slot = (((unsigned)line ^ (unsigned)(line >> 32)) * 0x9E3779B1u) >> 26;
+  const unsigned hh = ((unsigned)line ^ (unsigned)(line >> 32)) * 0x9E3779B1u;
+  // all lines distinct? (wide random addresses): 4096-bucket hashed bitmap in the 128 key words. No
+  // bucket shared => all lines and hence all sectors distinct => S = L = |E|; else exact hash set below
+  if (act) asm volatile("red.shared.and.b32 [%0], %1;" ::"r"(scr + 4u * (hh >> 25)), "r"(~(1u << ((hh >> 20) & 31u))) : "memory");
+  __syncwarp();
+  {
+    unsigned w0, w1, w2, w3;
+    asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(w0), "=r"(w1), "=r"(w2), "=r"(w3) : "r"(scr + 16u * lane) : "memory");
+    asm volatile("st.shared.v4.u32 [%0], {%1, %1, %1, %1};" ::"r"(scr + 16u * lane), "r"(0xffffffffu) : "memory");
+    const unsigned used = __reduce_add_sync(FULL, __popc(~w0) + __popc(~w1) + __popc(~w2) + __popc(~w3));
+    __syncwarp();
+    if (used == (unsigned)__popc(E)) return make_uint2(used, used);
+  }
+  unsigned slot = hh >> 26;
   bool pending = act, inserted = false;
   while (__any_sync(FULL, pending)) {
     if (pending) {
@@ -135,17 +168,20 @@ static __device__ __noinline__ uint2 sectors_lines_unsorted_call(unsigned long l
 template <bool kInlineSlow = false>
 __device__ __forceinline__ void sectors_lines(unsigned long long addr, unsigned E, unsigned lane, unsigned lanebit,
                                               unsigned lmlt, unsigned scr, unsigned& S, unsigned& L) {
-  const bool act = (E & lanebit) != 0u;
   const unsigned below = E & lmlt;
-  const bool first = below == 0u;
-  const int src = 31 - __clz(below);               // previous lane of E (lane 31 when none: unused)
+  unsigned src;                                    // previous lane of E (0xffffffff -> lane 31: unused)
+  asm("bfind.u32 %0, %1;" : "=r"(src) : "r"(below));
   const unsigned a_lo = (unsigned)addr, a_hi = (unsigned)(addr >> 32);
-  const unsigned p_lo = __shfl_sync(FULL, a_lo, src), p_hi = __shfl_sync(FULL, a_hi, src);
-  const bool ge = a_hi > p_hi || (a_hi == p_hi && a_lo >= p_lo);
-  if (__all_sync(FULL, !act || first || ge)) {
+  unsigned p_lo = __shfl_sync(FULL, a_lo, src), p_hi = __shfl_sync(FULL, a_hi, src);
+  // lanes outside E and the first lane of E compare with themselves: no boundary, no violation
+  const bool take = (E & lanebit) != 0u && below != 0u;
+  p_lo = take ? p_lo : a_lo;
+  p_hi = take ? p_hi : a_hi;
+  const long long d = (long long)(((unsigned long long)a_hi << 32 | a_lo) - ((unsigned long long)p_hi << 32 | p_lo));
+  if (__all_sync(FULL, d >= 0)) {
     const unsigned x_lo = a_lo ^ p_lo, x_hi = a_hi ^ p_hi;
-    S = __popc(__ballot_sync(FULL, act && (first || ((x_lo & ~31u) | x_hi) != 0u)));
-    L = __popc(__ballot_sync(FULL, act && (first || ((x_lo & ~127u) | x_hi) != 0u)));
+    S = 1u + __popc(__ballot_sync(FULL, ((x_lo & ~31u) | x_hi) != 0u));
+    L = 1u + __popc(__ballot_sync(FULL, ((x_lo & ~127u) | x_hi) != 0u));
     return;
   }
   const uint2 r = kInlineSlow ? sectors_lines_unsorted(addr, E, lane, lanebit, scr)

@@ -509,6 +509,152 @@ static size_t replay_lane_smem(unsigned P) {
   return (((6ull * P + 66 + 3) & ~3ull) + (size_t)L3_NW * L3_WARP_WORDS) * 4 + P + 16;
 }
 
+// ---------------------------------------------------------------- replay, lean warp-cooperative variant (V = 4)
+// One CTA of 32 warps per SM. Per 32-event tile: predicated shared reductions for the counts (no
+// branches), then the tile's executed memory events in batches of 8: cp.async (8 B per lane) stages the
+// 8 address slots into the warp's shared rows, and a rolled loop runs sectors_lines() per event with
+// every shared access through explicit 32-bit shared addresses and predicated reductions (compact code:
+// the I-cache holds the whole loop).
+constexpr int L4_NW = 32;  // warps per CTA (1 CTA per SM)
+constexpr int L4_WARP_WORDS = SCRATCH_WORDS + 4 + 8 * 64;   // scratch + pad + 8 stage rows of 32 x u64
+
+__device__ __forceinline__ unsigned lds_u8(unsigned a) {
+  unsigned v;
+  asm volatile("ld.shared.u8 %0, [%1];" : "=r"(v) : "r"(a));
+  return v;
+}
+
+template <bool PW>
+__global__ void __launch_bounds__(32 * L4_NW, 1)
+k_replay4(const uint4* __restrict__ hdr, const unsigned long long* __restrict__ addr, unsigned long long n,
+          unsigned P, const uint8_t* __restrict__ kind, DevState st, unsigned long long* err) {
+  extern __shared__ __align__(16) unsigned sm[];
+  const unsigned P4 = (6 * P + 66 + 3) & ~3u;
+  unsigned* sWarpAll = sm + P4;
+  uint8_t* sK = reinterpret_cast<uint8_t*>(sm + P4 + L4_NW * L4_WARP_WORDS);
+  for (unsigned i = threadIdx.x; i < P4; i += blockDim.x) sm[i] = 0;
+  for (unsigned i = threadIdx.x; i < L4_NW * L4_WARP_WORDS; i += blockDim.x) {
+    const unsigned o = i % L4_WARP_WORDS;
+    sWarpAll[i] = o < SCRATCH_WORDS ? scratch_init_word(o) : 0u;
+  }
+  for (unsigned i = threadIdx.x; i < P; i += blockDim.x) sK[i] = is_mem_kind(kind[i]);
+  __syncthreads();
+
+  const unsigned lane = lane_id(), lmlt = lanemask_lt(), lanebit = 1u << lane;
+  const unsigned s_base = (unsigned)__cvta_generic_to_shared(sm);
+  const unsigned s_kind = (unsigned)__cvta_generic_to_shared(sK);
+  const unsigned s_scr = (unsigned)__cvta_generic_to_shared(sWarpAll + (threadIdx.x >> 5) * L4_WARP_WORDS);
+  const unsigned s_stage0 = s_scr + 4u * SCRATCH_WORDS + 16u;          // row r at + 256 r
+  const unsigned s_sS = s_base + 16u * P, s_sL = s_base + 20u * P;
+  unsigned hS = 0, hL = 0, bad = 0;
+  const unsigned long long warps = (unsigned long long)gridDim.x * L4_NW;
+  unsigned long long tile = (blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x) >> 5;
+  uint4 h = make_uint4(0, 0, 0, 0);
+  if (tile * 32 + lane < n) h = ld_nc_v4(hdr + tile * 32 + lane);
+  for (; tile * 32 < n; tile += warps) {
+    const bool valid = tile * 32 + lane < n;
+    const unsigned pc = h.x, A = h.z, E = h.z & h.w;
+    const unsigned long long nt = tile + warps;
+    uint4 hn = make_uint4(0, 0, 0, 0);
+    if (nt * 32 + lane < n) hn = ld_nc_v4(hdr + nt * 32 + lane);
+    const bool ok = valid && pc < P && A != 0u;
+    bad += valid && pc >= P;
+    const unsigned pcs = ok ? pc : 0u;
+    const unsigned a4 = s_base + 4u * pcs;
+    const unsigned pa = __popc(A), pe = __popc(E);
+    red_shared_add_if(ok, a4, pa);
+    red_shared_add_if(ok, a4 + 4u * P, 1u);
+    red_shared_add_if(ok && pa != pe, a4 + 8u * P, pa - pe);
+    red_shared_add_if(ok && E == 0u, a4 + 12u * P, 1u);
+    if constexpr (PW) {
+      const unsigned warp = h.y;
+      if (ok && warp < st.n_warps) {
+        atomicAdd(st.pw + warp, (unsigned long long)pe);
+        if (E) atomicAdd(st.pw + st.n_warps + warp, 1ull);
+      }
+    }
+    unsigned mm = __ballot_sync(FULL, ok && E != 0u && lds_u8(s_kind + pcs) != 0u);
+    const unsigned long long* tbase0 = addr + tile * 32 * 32;
+    while (mm) {
+      // stage up to 8 address slots (cp.async, 8 B per lane per slot; 256 B coalesced per slot)
+      const unsigned batch = mm;
+      unsigned nb = 0;
+#pragma unroll
+      for (int b = 0; b < 8; ++b) {
+        if (mm) {
+          const int src = __ffs(mm) - 1;
+          mm &= mm - 1;
+          asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(s_stage0 + 256u * b + 8u * lane),
+                       "l"(tbase0 + src * 32 + lane)
+                       : "memory");
+          ++nb;
+        }
+      }
+      asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
+      __syncwarp();
+      unsigned rest = batch;
+      unsigned myS = 0, myL = 0, mySrc = 0;   // lane b keeps event b's results
+#pragma unroll 1
+      for (unsigned b = 0; b < nb; ++b) {
+        const int src = __ffs(rest) - 1;
+        rest &= rest - 1;
+        unsigned long long a;
+        asm volatile("ld.shared.u64 %0, [%1];" : "=l"(a) : "r"(s_stage0 + 256u * b + 8u * lane) : "memory");
+        const unsigned es = __shfl_sync(FULL, E, src);
+        unsigned S, L;
+        sectors_lines<true>(a, es, lane, lanebit, lmlt, s_scr, S, L);
+        const bool mine = lane == b;
+        myS = mine ? S : myS;
+        myL = mine ? L : myL;
+        mySrc = mine ? (unsigned)src : mySrc;
+      }
+      // the batch's shared updates in one go: lanes 0..nb-1 each own one event
+      const unsigned ps = __shfl_sync(FULL, pcs, mySrc);
+      const bool own = lane < nb;
+      red_shared_add_if(own, s_sS + 4u * ps, myS);
+      red_shared_add_if(own, s_sL + 4u * ps, myL);
+      red_shared_add_if(own, s_base + 4u * (6 * P + myS), 1u);        // hS[S]
+      red_shared_add_if(own, s_base + 4u * (6 * P + 33 + myL), 1u);   // hL[L]
+      __syncwarp();
+    }
+    h = hn;
+  }
+  red_shared_add_if(hS != 0u, s_base + 4u * (6 * P + 1 + lane), hS);
+  red_shared_add_if(hL != 0u, s_base + 4u * (6 * P + 34 + lane), hL);
+  bad = __reduce_add_sync(FULL, bad);
+  if (lane == 0 && bad) atomicAdd(err, (unsigned long long)bad);
+  __syncthreads();
+  const unsigned* sA = sm;
+  const unsigned* sW = sm + P;
+  const unsigned* sDT = sm + 2 * P;
+  const unsigned* sDW = sm + 3 * P;
+  const unsigned* sS = sm + 4 * P;
+  const unsigned* sL = sm + 5 * P;
+  const unsigned* sH = sm + 6 * P;
+  for (unsigned pc = threadIdx.x; pc < P; pc += blockDim.x) {
+    const unsigned a = sA[pc], w = sW[pc];
+    if (w) {
+      unsigned long long* s = st.site + 4 * pc;
+      atomicAdd(s + 0, (unsigned long long)a);
+      atomicAdd(s + 1, (unsigned long long)(a - sDT[pc]));
+      atomicAdd(s + 2, (unsigned long long)w);
+      atomicAdd(s + 3, (unsigned long long)(w - sDW[pc]));
+      if (sK[pc] && w != sDW[pc]) {
+        unsigned long long* m = st.mem + 3 * pc;
+        atomicAdd(m + 0, (unsigned long long)(w - sDW[pc]));
+        atomicAdd(m + 1, (unsigned long long)sS[pc]);
+        atomicAdd(m + 2, (unsigned long long)sL[pc]);
+      }
+    }
+  }
+  for (unsigned i = threadIdx.x; i < 66; i += blockDim.x)
+    if (sH[i]) atomicAdd(st.hist + i, (unsigned long long)sH[i]);
+}
+
+static size_t replay4_smem(unsigned P) {
+  return (((6ull * P + 66 + 3) & ~3ull) + (size_t)L4_NW * L4_WARP_WORDS) * 4 + P + 16;
+}
+
 static int g_sms = 0;
 static int sm_count(int dev) {
   if (g_sms == 0) cudaDeviceGetAttribute(&g_sms, cudaDevAttrMultiProcessorCount, dev);
@@ -652,6 +798,30 @@ static int launch_replay_lane(nvbt_ctx c, const void* d_hdr, const void* d_addr,
   return NVBT_OK;
 }
 
+static int launch_replay4(nvbt_ctx c, const void* d_hdr, const void* d_addr, uint64_t n, const DevState& st) {
+  const size_t smem = replay4_smem(c->n_pcs);
+  static bool attr_set = false;
+  if (!attr_set) {
+    NVBT_CUDA(cudaFuncSetAttribute(k_replay4<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)replay4_smem(4096)));
+    NVBT_CUDA(cudaFuncSetAttribute(k_replay4<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)replay4_smem(4096)));
+    attr_set = true;
+  }
+  const unsigned long long kMaxPerLaunch = 1ull << 30;
+  const int sms = sm_count(c->device);
+  for (uint64_t off = 0; off < n; off += kMaxPerLaunch) {
+    const uint64_t m = std::min<uint64_t>(kMaxPerLaunch, n - off);
+    const unsigned long long tiles = (m + 31) / 32;
+    const int blocks = (int)std::min<unsigned long long>((tiles + 2 * L4_NW - 1) / (2 * L4_NW), (unsigned long long)sms);
+    auto kern = st.pw != nullptr ? k_replay4<true> : k_replay4<false>;
+    kern<<<blocks, 32 * L4_NW, smem, c->stream>>>(static_cast<const uint4*>(d_hdr) + off,
+                                                  static_cast<const unsigned long long*>(d_addr) + off * 32, m,
+                                                  c->n_pcs, c->d_kind, st, c->ctl + CTL_REPLAY_ERR);
+    NVBT_CUDA(cudaGetLastError());
+    c->launches++;
+  }
+  return NVBT_OK;
+}
+
 extern "C" {
 
 int nvbt_replay(nvbt_ctx c, const void* d_hdr, const void* d_addr, uint64_t n) {
@@ -666,12 +836,13 @@ int nvbt_replay(nvbt_ctx c, const void* d_hdr, const void* d_addr, uint64_t n) {
   NVBT_CUDA(cudaSetDevice(c->device));
   if (g_replay_variant < 0) {
     const char* e = getenv("NVBT_REPLAY_VARIANT");
-    g_replay_variant = e ? atoi(e) : 0;
+    g_replay_variant = e ? atoi(e) : 4;
   }
   switch (g_replay_variant) {
     case 0: return launch_replay<0>(c, d_hdr, d_addr, n, st);
     case 2: return launch_replay<2>(c, d_hdr, d_addr, n, st);
     case 3: return launch_replay_lane(c, d_hdr, d_addr, n, st);
+    case 4: return launch_replay4(c, d_hdr, d_addr, n, st);
     default: return launch_replay<1>(c, d_hdr, d_addr, n, st);
   }
 }

@@ -274,11 +274,12 @@ def _adversarial_stream(n, seed):
     span = rng.choice([32, 1024 * 32 - 1, 1024 * 32, 1024 * 32 + 32, 1 << 20, 1 << 38], size=(n, 1))
     r = rng.integers(0, 1 << 62, size=(n, 32)) % span - span // 2       # symmetric around base
     stride = rng.choice([0, 1, 4, 31, 32, 33, 128, 4096], size=(n, 1))
-    addr = np.select([kind == 0, kind == 1, kind == 2, kind == 3],
+    addr = np.select([kind == 0, kind == 1, kind == 2, kind == 3, kind == 4],
                      [base + lane * stride,                               # monotone
                       base - lane * stride,                               # decreasing
                       base + (r // 4) * 4,                                # window / wide random
-                      base + (lane % 3) * 32 + 124],                      # duplicates straddling lines
+                      base + (lane % 3) * 32 + 124,                       # duplicates straddling lines
+                      base + r[:, (lane[0] * 7) % 8]],                    # wide random with repeats
                      base + r)
     addr = np.clip(addr, 0, (1 << 62) - 1).astype(np.uint64)
     return pc.astype(np.int64), warp.astype(np.int64), A, P, addr
