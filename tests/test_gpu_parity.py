@@ -300,3 +300,84 @@ def test_replay_adversarial_addresses(nvbt, seed):
     acc = ev.Accumulator(programs.replay())
     acc.add(0, warp, pc, A, P, addr)
     assert_same(g, acc.result(), COUNT_KEYS + MEM_KEYS, f"adversarial replay seed {seed}")
+
+
+# ---------------------------------------------------------------- degenerate cases
+def test_degenerate_shapes(nvbt):
+    """Empty launches, single-element grids, all-boundary stencils, isolated BFS sources."""
+    import torch
+    nb, dr = nvbt.nvbt, nvbt.drivers
+    # vectorAdd N = 0 launches nothing and counts nothing; N = 1 is a single live lane
+    ctx = nb.nvbt_init(nb.W_VECTORADD, nb.COUNT | nb.MEMDIV)
+    a = cuda(uniform_f32(1, 1))
+    c = torch.empty_like(a)
+    nb.nvbt_vectoradd(ctx, nb.TOOL_COUNT | nb.TOOL_MEMDIV, a, a, c, 0)
+    assert (nb.nvbt_count(ctx) == 0).all()
+    nb.nvbt_vectoradd(ctx, nb.TOOL_COUNT | nb.TOOL_MEMDIV, a, a, c, 1)
+    acc = ev.Accumulator(programs.vectoradd())
+    m_va.run(acc, 1, a.data_ptr(), a.data_ptr(), c.data_ptr())
+    assert_same(read_all(nb, ctx), acc.result(), COUNT_KEYS + MEM_KEYS, "vectorAdd N=1")
+    # SGEMM 1x1x1
+    ctx = nb.nvbt_init(nb.W_SGEMM, nb.COUNT | nb.MEMDIV)
+    A = cuda(np.ones((1, 1), np.float32))
+    Cm = torch.empty(1, 1, device="cuda")
+    nb.nvbt_sgemm(ctx, nb.TOOL_COUNT | nb.TOOL_MEMDIV, A, A, Cm, 1, 1, 1)
+    acc = ev.Accumulator(programs.sgemm())
+    m_sg.run(acc, 1, 1, 1, A.data_ptr(), A.data_ptr(), Cm.data_ptr())
+    assert_same(read_all(nb, ctx), acc.result(), COUNT_KEYS + MEM_KEYS, "SGEMM 1x1x1")
+    # stencil n = 2: every point is a boundary point (P1 false everywhere)
+    ctx = nb.nvbt_init(nb.W_STENCIL, nb.COUNT | nb.MEMDIV)
+    x = cuda(uniform_f32((2, 2), 4))
+    y = torch.zeros_like(x)
+    nb.nvbt_stencil(ctx, nb.TOOL_COUNT | nb.TOOL_MEMDIV, x, y, 2)
+    acc = ev.Accumulator(programs.stencil())
+    m_st.run(acc, 2, x.data_ptr(), y.data_ptr())
+    assert_same(read_all(nb, ctx), acc.result(), COUNT_KEYS + MEM_KEYS, "stencil n=2")
+    assert torch.equal(y, x)
+    # BFS from an isolated vertex: one level, nothing reached
+    rowptr = np.array([0, 0, 1, 2], dtype=np.int32)
+    col = np.array([2, 1], dtype=np.int32)
+    ctx = nb.nvbt_init(nb.W_BFS, nb.COUNT | nb.BB | nb.MEMDIV)
+    rp, cl = cuda(rowptr), cuda(col)
+    bufs = dr.bfs_buffers(3, "cuda")
+    cost, levels = dr.run_bfs(ctx, nb.TOOL_BBCOUNT | nb.TOOL_MEMDIV, rp, cl, 0, bufs)
+    acc = ev.Accumulator(programs.bfs())
+    ptr = m_bfs.Ptrs(bufs["mask"].data_ptr(), bufs["visited"].data_ptr(), bufs["updating"].data_ptr(),
+                     bufs["cost"].data_ptr(), bufs["over"].data_ptr(), rp.data_ptr(), cl.data_ptr())
+    ocost, olevels, _ = m_bfs.run(acc, rowptr, col, 0, ptr)
+    assert levels == olevels == 1 and cost.cpu().tolist() == ocost.tolist() == [0, -1, -1]
+    assert_same(read_all(nb, ctx), acc.result(), COUNT_KEYS + MEM_KEYS, "BFS isolated source")
+    # replay of zero events is a no-op; an out-of-range pc is counted as an error and ignored
+    rctx = nb.nvbt_init(nb.W_REPLAY, nb.COUNT | nb.MEMDIV)
+    h = np.zeros((2, 4), dtype="<u4")
+    h[0] = [5, 1, 0xFFFFFFFF, 0xFFFFFFFF]
+    h[1] = [4096 + 7, 1, 0xFFFFFFFF, 0xFFFFFFFF]
+    d_h = cuda(h.view(np.uint8).reshape(-1))
+    d_a = torch.zeros(2 * 256, dtype=torch.uint8, device="cuda")
+    nb.nvbt_replay(rctx, d_h, d_a, 0)
+    assert (nb.nvbt_count(rctx) == 0).all()
+    nb.nvbt_replay(rctx, d_h, d_a, 2)
+    assert nb.nvbt_replay_errors(rctx) == 1
+    assert nb.nvbt_count(rctx).tolist() == [32, 32, 1, 1]
+
+
+def test_api_errors(nvbt):
+    """Argument validation surfaces as NvbtError with the documented codes."""
+    import torch
+    nb = nvbt.nvbt
+    ctx = nb.nvbt_init(nb.W_SGEMM, nb.COUNT)
+    x = torch.zeros(64, device="cuda")
+    with pytest.raises(nb.NvbtError) as e:
+        nb.nvbt_sgemm(ctx, nb.TOOL_COUNT | nb.TOOL_BBCOUNT, x, x, x, 4, 4, 4)
+    assert e.value.code == nb.EINVAL
+    with pytest.raises(nb.NvbtError) as e:
+        nb.nvbt_sgemm(ctx, nb.TOOL_COUNT, x, x, x, 4, 4, 0)          # K >= 1
+    assert e.value.code == nb.EINVAL
+    with pytest.raises(nb.NvbtError) as e:
+        nb.nvbt_sgemm(ctx, nb.TOOL_TRACE, x, x, x, 4, 4, 4)          # TRACE not enabled
+    assert e.value.code == nb.ESTATE
+    ring = torch.empty(4096, dtype=torch.uint8)                       # not pinned
+    tctx = nb.nvbt_init(nb.W_STENCIL, nb.TRACE)
+    with pytest.raises(nb.NvbtError) as e:
+        nb.nvbt_channel_open(tctx, ring)
+    assert e.value.code == nb.EINVAL
