@@ -33,6 +33,15 @@ N_SM = 148
 METRIC = "instrumented warp-instr events/sec and slowdown vs uninstrumented"
 
 
+def load_traffic(kernel):
+    """DRAM bytes per launch of `kernel` from the committed ncu capture (profiles/r1_traffic.json)."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "r1_traffic.json")) as f:
+            return json.load(f).get(kernel)
+    except Exception:
+        return None
+
+
 def load_peaks():
     try:
         with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
@@ -180,8 +189,11 @@ class SgemmBench:
         ops = W * per_warp
         peak = N_SM * 4 * peaks.get("sm_max_mhz", 1965.0) * 1e6
         ach = ops / t_kernel_s
+        t = load_traffic("k_sgemm<6>")
         return {"bound": "alu", "achieved": ach / 1e9, "peak": peak / 1e9, "unit": "Gwarp-inst/s",
-                "frac": ach / peak, "traffic": None, "algorithmic_warp_inst_per_launch": ops}
+                "frac": ach / peak, "traffic": t["traffic_bytes_per_launch"] if t else None,
+                "traffic_unit": "DRAM bytes per launch (ncu, profiles/r1_traffic.json)",
+                "algorithmic_warp_inst_per_launch": ops}
 
     def oracle_sample(self, budget_s):
         """The oracle on a bounded sample of the same workload: whole warps, full K."""
@@ -371,7 +383,11 @@ def run_replay(args, torch, nb, dr, rank, world, local, peaks, peaks_src):
         "config": {"workload": wl.desc, "events": args.replay_events, "chunk": wl.chunk,
                    "l2": "inputs (36.5 GB per chunk) larger than L2"},
         "roofline": {"bound": "hbm", "achieved": ach / 1e9, "peak": peaks["hbm_gbs"], "unit": "GB/s",
-                     "frac": ach / 1e9 / peaks["hbm_gbs"], "traffic": None, "peak_source": peaks_src},
+                     "frac": ach / 1e9 / peaks["hbm_gbs"], "peak_source": peaks_src,
+                     "algorithmic_bytes_per_launch": bytes_rank * wl.chunk / wl.n,
+                     "traffic": (load_traffic("k_replay4") or {}).get("traffic_bytes_per_launch", 0) / 67108864 * wl.chunk
+                     if load_traffic("k_replay4") else None,
+                     "traffic_unit": "DRAM bytes per 2^27-event launch (ncu at 2^26, scaled; profiles/r1_traffic.json)"},
         "gpu_launches": int(launches), "clocks": clk.summary(),
         "check": {"W_issued": int(cnt[2]), "expected": args.steps * n_all},
     }

@@ -516,7 +516,7 @@ static size_t replay_lane_smem(unsigned P) {
 // every shared access through explicit 32-bit shared addresses and predicated reductions (compact code:
 // the I-cache holds the whole loop).
 constexpr int L4_NW = 32;  // warps per CTA (1 CTA per SM)
-constexpr int L4_WARP_WORDS = SCRATCH_WORDS + 4 + 8 * 64;   // scratch + pad + 8 stage rows of 32 x u64
+constexpr int L4_WARP_WORDS = SCRATCH_WORDS + 4 + 8 * 64 + 32;   // scratch + pad + 8 stage rows + row sources
 
 __device__ __forceinline__ unsigned lds_u8(unsigned a) {
   unsigned v;
@@ -545,6 +545,7 @@ k_replay4(const uint4* __restrict__ hdr, const unsigned long long* __restrict__ 
   const unsigned s_kind = (unsigned)__cvta_generic_to_shared(sK);
   const unsigned s_scr = (unsigned)__cvta_generic_to_shared(sWarpAll + (threadIdx.x >> 5) * L4_WARP_WORDS);
   const unsigned s_stage0 = s_scr + 4u * SCRATCH_WORDS + 16u;          // row r at + 256 r
+  const unsigned s_rowsrc = s_stage0 + 8u * 256u;                       // [32] lane of the r-th event
   const unsigned s_sS = s_base + 16u * P, s_sL = s_base + 20u * P;
   unsigned hS = 0, hL = 0, bad = 0;
   const unsigned long long warps = (unsigned long long)gridDim.x * L4_NW;
@@ -573,31 +574,33 @@ k_replay4(const uint4* __restrict__ hdr, const unsigned long long* __restrict__ 
         if (E) atomicAdd(st.pw + st.n_warps + warp, 1ull);
       }
     }
-    unsigned mm = __ballot_sync(FULL, ok && E != 0u && lds_u8(s_kind + pcs) != 0u);
+    const unsigned mm = __ballot_sync(FULL, ok && E != 0u && lds_u8(s_kind + pcs) != 0u);
     const unsigned long long* tbase0 = addr + tile * 32 * 32;
-    while (mm) {
-      // stage up to 8 address slots (cp.async, 8 B per lane per slot; 256 B coalesced per slot)
-      const unsigned batch = mm;
-      unsigned nb = 0;
+    const unsigned total = __popc(mm);
+    if (total) {
+      // row r of the tile's memory events = the r-th set lane of mm (each owner writes its lane id)
+      if ((mm >> lane) & 1u) sts_u32(s_rowsrc + 4u * __popc(mm & lmlt), lane);
+      __syncwarp();
+    }
+    for (unsigned r0 = 0; r0 < total; r0 += 8) {
+      const unsigned nb = total - r0 < 8u ? total - r0 : 8u;
+      // stage rows r0 .. r0+nb-1: one cp.async.cg of 16 B per lane copies two 256 B rows
 #pragma unroll
-      for (int b = 0; b < 8; ++b) {
-        if (mm) {
-          const int src = __ffs(mm) - 1;
-          mm &= mm - 1;
-          asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(s_stage0 + 256u * b + 8u * lane),
-                       "l"(tbase0 + src * 32 + lane)
+      for (int k = 0; k < 4; ++k) {
+        const unsigned row = 2u * k + (lane >> 4);
+        if (row < nb) {
+          const unsigned src = lds_u32(s_rowsrc + 4u * (r0 + row));
+          asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(s_stage0 + 256u * row + 16u * (lane & 15u)),
+                       "l"(tbase0 + src * 32u + 2u * (lane & 15u))
                        : "memory");
-          ++nb;
         }
       }
       asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
       __syncwarp();
-      unsigned rest = batch;
       unsigned myS = 0, myL = 0, mySrc = 0;   // lane b keeps event b's results
 #pragma unroll 1
       for (unsigned b = 0; b < nb; ++b) {
-        const int src = __ffs(rest) - 1;
-        rest &= rest - 1;
+        const unsigned src = lds_u32(s_rowsrc + 4u * (r0 + b));
         unsigned long long a;
         asm volatile("ld.shared.u64 %0, [%1];" : "=l"(a) : "r"(s_stage0 + 256u * b + 8u * lane) : "memory");
         const unsigned es = __shfl_sync(FULL, E, src);
@@ -606,7 +609,7 @@ k_replay4(const uint4* __restrict__ hdr, const unsigned long long* __restrict__ 
         const bool mine = lane == b;
         myS = mine ? S : myS;
         myL = mine ? L : myL;
-        mySrc = mine ? (unsigned)src : mySrc;
+        mySrc = mine ? src : mySrc;
       }
       // the batch's shared updates in one go: lanes 0..nb-1 each own one event
       const unsigned ps = __shfl_sync(FULL, pcs, mySrc);
