@@ -72,6 +72,9 @@ __device__ __forceinline__ unsigned distinct_match(unsigned long long key, unsig
   return __popc(__ballot_sync(FULL, (E & lanebit) != 0u && (grp & E & lmlt) == 0u));
 }
 
+#ifndef NVBT_AP_FASTPATH
+#define NVBT_AP_FASTPATH 1
+#endif
 constexpr int SCRATCH_WORDS = 192;  // per-warp scratch of sectors_lines(): 64 x u64 keys + 64 x u32 masks
 // Initial contents of scratch word i (keys empty = ~0, masks 0).
 __host__ __device__ constexpr unsigned scratch_init_word(int i) { return i < 128 ? 0xffffffffu : 0u; }
@@ -160,18 +163,36 @@ static __device__ __noinline__ uint2 sectors_lines_unsorted_call(unsigned long l
 
 // a5 kernel of Listing 8 (readings R-3, R-5, R-6): S = number of distinct 32 B
 // sectors and L = number of distinct 128 B lines touched by the lanes of E (E != 0). Exact integers.
-// Fast path (coalesced, strided, broadcast, stencil neighbours ...): when the addresses of the lanes of
+// Fast paths (coalesced, strided, broadcast, stencil neighbours ...): when the addresses of the lanes of
 // E are non-decreasing in lane order, so are their sectors and lines, and each distinct value starts
-// where a lane's sector (line) differs from the previous lane of E — compared as (a ^ prev) >> 5 (7)
-// on 32-bit halves: 2 shuffles, 3 votes, ~18 instructions. Other orders take the slow paths above
-// (inlined when kInlineSlow, else an out-of-line call to keep the hooks' registers and code small).
-template <bool kInlineSlow = false>
+// where a lane's sector (line) differs from the previous lane of E — compared as (a ^ prev) >> 5 (7).
+// kApFirst: for a full warp, first try an arithmetic progression a_l = min + l d detected with warp
+// reductions (no shuffles: the instrumented application kernels are L1-bound, and shuffles share the
+// L1/MIO datapath with their loads); otherwise the previous lane's address comes from 2 shuffles.
+// Other orders take the slow paths above (inlined when kInlineSlow, else an out-of-line call to keep the
+// hooks' registers and code small).
+template <bool kInlineSlow = false, bool kApFirst = true>
 __device__ __forceinline__ void sectors_lines(unsigned long long addr, unsigned E, unsigned lane, unsigned lanebit,
                                               unsigned lmlt, unsigned scr, unsigned& S, unsigned& L) {
+  const unsigned a_lo = (unsigned)addr, a_hi = (unsigned)(addr >> 32);
+#if NVBT_AP_FASTPATH
+  if (kApFirst && E == FULL) {
+    // all 32 lanes, addresses an increasing arithmetic progression in lane order inside one 4 GB
+    // region (coalesced, strided, broadcast): warp reductions instead of shuffles — a_l = min + l d
+    const unsigned hmn = __reduce_min_sync(FULL, a_hi), hmx = __reduce_max_sync(FULL, a_hi);
+    const unsigned mn = __reduce_min_sync(FULL, a_lo), mx = __reduce_max_sync(FULL, a_lo);
+    const unsigned dd = (mx - mn) / 31u;
+    if (hmn == hmx && __all_sync(FULL, a_lo == mn + lane * dd)) {
+      const unsigned x = a_lo ^ (a_lo - dd);         // vs the previous lane's address
+      S = 1u + __popc(__ballot_sync(FULL, lane != 0u && (x & ~31u) != 0u));
+      L = 1u + __popc(__ballot_sync(FULL, lane != 0u && (x & ~127u) != 0u));
+      return;
+    }
+  }
+#endif
   const unsigned below = E & lmlt;
   unsigned src;                                    // previous lane of E (0xffffffff -> lane 31: unused)
   asm("bfind.u32 %0, %1;" : "=r"(src) : "r"(below));
-  const unsigned a_lo = (unsigned)addr, a_hi = (unsigned)(addr >> 32);
   unsigned p_lo = __shfl_sync(FULL, a_lo, src), p_hi = __shfl_sync(FULL, a_hi, src);
   // lanes outside E and the first lane of E compare with themselves: no boundary, no violation
   const bool take = (E & lanebit) != 0u && below != 0u;

@@ -160,7 +160,7 @@ k_replay(const uint4* __restrict__ hdr, const unsigned long long* __restrict__ a
     const unsigned es = __shfl_sync(FULL, E, src);
     const unsigned ps = __shfl_sync(FULL, h.x, src);
     unsigned S, L;
-    sectors_lines<true>(a, es, lane, lanebit, lmlt, s_scr, S, L);
+    sectors_lines<true, false>(a, es, lane, lanebit, lmlt, s_scr, S, L);
     red_shared_add_if(lane == 0, s_base + 4u * (4 * P + ps), S);   // sS[ps]
     red_shared_add_if(lane == 0, s_base + 4u * (5 * P + ps), L);   // sL[ps]
     inc_if_eq(hS, S, lane + 1u);
@@ -605,7 +605,7 @@ k_replay4(const uint4* __restrict__ hdr, const unsigned long long* __restrict__ 
         asm volatile("ld.shared.u64 %0, [%1];" : "=l"(a) : "r"(s_stage0 + 256u * b + 8u * lane) : "memory");
         const unsigned es = __shfl_sync(FULL, E, src);
         unsigned S, L;
-        sectors_lines<true>(a, es, lane, lanebit, lmlt, s_scr, S, L);
+        sectors_lines<true, false>(a, es, lane, lanebit, lmlt, s_scr, S, L);
         const bool mine = lane == b;
         myS = mine ? S : myS;
         myL = mine ? L : myL;
