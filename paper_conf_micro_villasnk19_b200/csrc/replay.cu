@@ -89,7 +89,6 @@ __global__ void __launch_bounds__(256) k_gen(GenConsts G, unsigned long long fir
 }
 
 // ---------------------------------------------------------------- replay
-constexpr int RP_THREADS = 512;
 constexpr int RP_BATCH = 8;  // memory events whose slots are loaded before processing
 
 __device__ __forceinline__ void red_shared_add(unsigned saddr, unsigned v) {
@@ -290,10 +289,9 @@ k_replay(const uint4* __restrict__ hdr, const unsigned long long* __restrict__ a
 // non-decreasing) and sets bits in a per-lane 512-sector window bitmap (valid if they span < 16 KB);
 // events that are neither (wide random patterns) fall back to the warp-cooperative sectors_lines().
 // Per event this costs ~1/32 of the warp-cooperative instruction count for the common paths.
-constexpr int L3_NW = 8;                     // warps per CTA (1 CTA per SM)
+constexpr int L3_NW = 10;                    // warps per CTA (1 CTA per SM)
 constexpr int L3_ROW = 68;                   // words per stage row (272 B: conflict-free 16 B lane reads)
-constexpr int L3_BMS = 17;                   // words per lane bitmap row (16 used; odd stride)
-constexpr int L3_WARP_WORDS = 3 * 128 + 32 * L3_ROW + 32 * L3_BMS + SCRATCH_WORDS;
+constexpr int L3_WARP_WORDS = 3 * 128 + 32 * L3_ROW + SCRATCH_WORDS;
 
 __device__ __forceinline__ void lds_v4(unsigned a, uint4& v) {
   asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a));
@@ -322,7 +320,7 @@ k_replay_lane(const uint4* __restrict__ hdr, const unsigned long long* __restric
   for (unsigned i = threadIdx.x; i < P4; i += blockDim.x) sm[i] = 0;
   for (unsigned i = threadIdx.x; i < L3_NW * L3_WARP_WORDS; i += blockDim.x) {
     const unsigned o = i % L3_WARP_WORDS;
-    const unsigned s0 = 3 * 128 + 32 * L3_ROW + 32 * L3_BMS;
+    const unsigned s0 = 3 * 128 + 32 * L3_ROW;
     sm[P4 + i] = o >= s0 ? scratch_init_word(o - s0) : 0u;
   }
   for (unsigned i = threadIdx.x; i < P; i += blockDim.x) sK[i] = is_mem_kind(kind[i]);
@@ -332,10 +330,8 @@ k_replay_lane(const uint4* __restrict__ hdr, const unsigned long long* __restric
   const unsigned s_base = (unsigned)__cvta_generic_to_shared(sm);
   const unsigned s_list = (unsigned)__cvta_generic_to_shared(sWarp);            // [128][3]: idx, E, pc
   const unsigned s_stage = s_list + 4u * 3u * 128u;                              // [32][L3_ROW]
-  const unsigned s_bm = s_stage + 4u * 32u * L3_ROW;                             // [32][L3_BMS]
-  const unsigned s_scr = s_bm + 4u * 32u * L3_BMS;                               // hash scratch
+  const unsigned s_scr = s_stage + 4u * 32u * L3_ROW;                            // hash scratch
   const unsigned my_row = s_stage + 4u * L3_ROW * lane;
-  const unsigned my_bm = s_bm + 4u * L3_BMS * lane;
   unsigned bad = 0;
   const unsigned long long warps = (unsigned long long)gridDim.x * L3_NW;
   unsigned long long round = (blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x) >> 5;
@@ -412,10 +408,8 @@ k_replay_lane(const uint4* __restrict__ hdr, const unsigned long long* __restric
       if (have) {
         const int f = __ffs(E) - 1;
         const unsigned f_lo = lds_u32(my_row + 8u * f), f_hi = lds_u32(my_row + 8u * f + 4);
-        const unsigned wbase = ((f_lo >> 5) & ~31u) - 256u;     // 512-sector window, 32-sector aligned
-        unsigned prev = f_lo;
-        bool viol = false, hi_bad = false, out = false;
-        unsigned bs = 0, bl = 0;
+        unsigned prev = f_lo, hb = 0, bs = 0, bl = 0;
+        bool viol = false;
 #pragma unroll
         for (int q = 0; q < 16; ++q) {
           uint4 v;
@@ -426,34 +420,20 @@ k_replay_lane(const uint4* __restrict__ hdr, const unsigned long long* __restric
             const bool act = (E >> l) & 1u;
             const unsigned lo = act ? (u ? v.z : v.x) : prev;
             const unsigned hi = act ? (u ? v.w : v.y) : f_hi;
-            hi_bad |= hi != f_hi;
+            hb |= hi ^ f_hi;
             viol |= lo < prev;
             const unsigned x = lo ^ prev;
             bs += (x & ~31u) != 0u;
             bl += (x & ~127u) != 0u;
             prev = lo;
-            const unsigned w = (lo >> 5) - wbase;
-            const bool in = w < 512u;
-            out |= !in;
-            if (in) asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(my_bm + 4u * (w >> 5)), "r"(1u << (w & 31u)) : "memory");
           }
         }
-        if (!hi_bad && !viol) {
+        if (hb == 0u && !viol) {
           S = bs + 1u;
           L = bl + 1u;
-        } else if (!hi_bad && !out) {
-#pragma unroll
-          for (int k = 0; k < 16; ++k) {
-            const unsigned word = lds_u32(my_bm + 4u * k);
-            const unsigned g = word | (word >> 1) | (word >> 2) | (word >> 3);
-            S += __popc(word);
-            L += __popc(g & 0x11111111u);
-          }
         } else {
           hard = true;
         }
-#pragma unroll
-        for (int k = 0; k < 16; ++k) sts_u32(my_bm + 4u * k, 0u);
       }
       // ---- hard rows: warp-cooperative exact path
       unsigned hm = __ballot_sync(FULL, hard);
@@ -464,7 +444,7 @@ k_replay_lane(const uint4* __restrict__ hdr, const unsigned long long* __restric
         unsigned long long a;
         asm volatile("ld.shared.u64 %0, [%1];" : "=l"(a) : "r"(s_stage + 4u * L3_ROW * src + 8u * lane));
         unsigned s2, l2;
-        sectors_lines<true>(a, es, lane, lanebit, lmlt, s_scr, s2, l2);
+        sectors_lines<true, false>(a, es, lane, lanebit, lmlt, s_scr, s2, l2);
         if (lane == (unsigned)src) { S = s2; L = l2; }
       }
       if (have) {
