@@ -264,8 +264,8 @@ def run_ours(args):
 
     if args.workload == "c5":
         return run_replay(args, torch, nb, dr, rank, world, local, peaks, peaks_src)
-    if args.workload in ("c1", "c3", "c4"):
-        line = {"c1": run_c1, "c3": run_c3, "c4": run_c4}[args.workload](args, torch, nb, dr, local)
+    if args.workload in ("c1", "c3", "c4", "f1"):
+        line = {"c1": run_c1, "c3": run_c3, "c4": run_c4, "f1": run_f1}[args.workload](args, torch, nb, dr, local)
         if rank == 0:
             print(json.dumps(line), flush=True)
         return
@@ -512,6 +512,52 @@ def run_c4(args, torch, nb, dr, local):
             "clocks": clk.summary()}
 
 
+def run_f1(args, torch, nb, dr, local):
+    """F1 kernel sampling on C4's stencil (8192^2 x 100, BBCOUNT|MEMDIV): plain vs every launch
+    instrumented vs one instrumented launch per grid shape."""
+    from synth import uniform_f32
+    n, iters = args.stencil_n, args.stencil_iters
+    flags = nb.COUNT | nb.OPHIST | nb.BB | nb.MEMDIV
+    full, samp, scratch = (nb.nvbt_init(nb.W_STENCIL, flags) for _ in range(3))
+    x0 = torch.from_numpy(uniform_f32((n, n), 4)).cuda()
+    b = (x0.clone(), torch.empty_like(x0))
+    tools = nb.TOOL_BBCOUNT | nb.TOOL_MEMDIV
+
+    def run(mode):
+        sampler = dr.KernelSampler(samp, scratch) if mode == "sampled" else None
+        if mode == "sampled":
+            nb.nvbt_reset(samp)
+        for it in range(iters):
+            src, dst = b[it % 2], b[(it + 1) % 2]
+            if mode == "plain":
+                nb.nvbt_stencil(full, nb.TOOL_NONE, src, dst, n)
+            elif mode == "full":
+                nb.nvbt_stencil(full, tools, src, dst, n)
+            else:
+                sampler.launch(("stencil", n), lambda c, t: nb.nvbt_stencil(c, t, src, dst, n), tools)
+        if sampler:
+            sampler.finish()
+
+    res = {}
+    exact = None
+    for mode in ("plain", "full", "sampled"):
+        for _ in range(args.warmup):
+            run(mode)
+        nb.nvbt_reset(full)
+        res[mode] = _timed_events(torch, lambda: run(mode), args.steps)
+        if mode == "full":
+            exact = nb.nvbt_count(full).astype("int64") // args.steps
+    est = nb.nvbt_count(samp).astype("int64")
+    err = float(abs(est[2] - exact[2])) / float(exact[2])
+    tp, tf, ts = (sum(res[m]) / len(res[m]) for m in ("plain", "full", "sampled"))
+    return {"metric": "kernel-sampling slowdown vs uninstrumented (F1)", "value": ts / tp, "unit": "x",
+            "n_gpus": 1, "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * ts,
+            "higher_is_better": False, "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+            "config": {"workload": f"F1 sampling on C4 stencil {n}^2 x {iters}, tools BBCOUNT|MEMDIV"},
+            "full_slowdown": tf / tp, "sampled_slowdown": ts / tp, "warp_issued_rel_error": err,
+            "paper_context": "36.4x full vs 2.3x sampled on TITAN V / SpecAccel (P:L280)"}
+
+
 def run_reference(args):
     """Reference arm = the CPU oracle (this tier has no runnable reference)."""
     rank = int(os.environ.get("RANK", "0"))
@@ -555,7 +601,7 @@ def main():
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--workload", choices=["c1", "c2", "c3", "c4", "c5"], default="c2")
+    ap.add_argument("--workload", choices=["c1", "c2", "c3", "c4", "c5", "f1"], default="c2")
     ap.add_argument("--bfs-scale", type=int, default=20)
     ap.add_argument("--stencil-n", type=int, default=8192)
     ap.add_argument("--stencil-iters", type=int, default=100)

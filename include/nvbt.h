@@ -103,6 +103,12 @@ int nvbt_fini(nvbt_ctx ctx);             /* frees host-side state only; closes a
  * sets add elementwise, so a multi-GPU merge is one int64 SUM all-reduce of this region (EM §4). */
 int nvbt_accum_view(nvbt_ctx ctx, void** d_ptr, size_t* n_int64);
 
+/* accum += factor * src over the whole accumulator region (n_int64 words of nvbt_accum_view); src is a
+ * device copy of another context's region with the same layout. Used by kernel sampling (F1,
+ * P:L274-282 (§6.2)): the counts of the one instrumented launch of a grid shape are extrapolated to all
+ * launches of that shape. Asynchronous on the context's stream. */
+int nvbt_accum_axpy(nvbt_ctx ctx, const void* d_src, size_t n_int64, int64_t factor);
+
 /* ---- read calls (EM §2); all synchronise the stream ---- */
 typedef struct { uint64_t thread_issued, thread_exec, warp_issued, warp_exec; } nvbt_counts;
 /* per_warp_thread / per_warp_warp: nullable host arrays [n_warps] (need NVBT_PER_WARP). */

@@ -1,4 +1,5 @@
 // libnvbt.so core: context lifecycle, workspace layout, the fold kernel and the read calls (nvbt.h).
+#include <algorithm>
 #include <cstring>
 #include <new>
 
@@ -26,7 +27,9 @@ Layout make_layout(uint32_t P, uint32_t O, uint32_t B, uint32_t W, uint32_t flag
   L.bbsite = L.site + 4ull * P;
   L.mem = L.bbsite + 4ull * P;
   L.hist = L.mem + 3ull * P;
-  L.pw = L.hist + 66;
+  L.stripe_words = L.hist + 66;
+  L.stripes = P <= 64 ? 32 : 1;   // small programs (the workloads) run many small CTAs
+  L.pw = L.stripe_words * L.stripes;
   L.accum_words = L.pw + ((flags & NVBT_PER_WARP) ? 2ull * W : 0);
   size_t off = align_up(L.accum_words * 8, 256);
   L.ctl = off;
@@ -55,17 +58,24 @@ Layout make_layout(uint32_t P, uint32_t O, uint32_t B, uint32_t W, uint32_t flag
 // Fold kernel: per-pc bins (per-instruction mode + BB mode derived per EM §2 item 3) -> reported
 // counts, opcode histogram, BB statistics and divergence totals. Integer sums only.
 __global__ void fold_kernel(const nvbt_instr_desc* __restrict__ prog, const uint32_t* __restrict__ leader,
-                            uint32_t P, uint32_t O, uint32_t B, const unsigned long long* __restrict__ site,
-                            const unsigned long long* __restrict__ bbsite, const unsigned long long* __restrict__ mem,
-                            const unsigned long long* __restrict__ hist, unsigned long long* out, Layout L) {
+                            uint32_t P, uint32_t O, uint32_t B, const unsigned long long* __restrict__ accum,
+                            unsigned long long* out, Layout L) {
+  const size_t SW = L.stripe_words;
   for (uint32_t pc = blockIdx.x * blockDim.x + threadIdx.x; pc < P; pc += gridDim.x * blockDim.x) {
     const nvbt_instr_desc d = prog[pc];
-    unsigned long long tI = site[4 * pc], tE = site[4 * pc + 1], wI = site[4 * pc + 2], wE = site[4 * pc + 3];
-    if (d.is_leader || d.guarded) {
-      tI += bbsite[4 * pc]; tE += bbsite[4 * pc + 1]; wI += bbsite[4 * pc + 2]; wE += bbsite[4 * pc + 3];
-    } else {  // same active mask as the block's leader (BB rule), unguarded: E = A
-      const uint32_t l = leader[d.bb];
-      tI += bbsite[4 * l]; tE += bbsite[4 * l]; wI += bbsite[4 * l + 2]; wE += bbsite[4 * l + 2];
+    const uint32_t l = leader[d.bb];
+    unsigned long long tI = 0, tE = 0, wI = 0, wE = 0, n = 0, sS = 0, sL = 0;
+    for (size_t s = 0; s < L.stripes; ++s) {
+      const unsigned long long* site = accum + s * SW + L.site;
+      const unsigned long long* bbsite = accum + s * SW + L.bbsite;
+      const unsigned long long* mem = accum + s * SW + L.mem;
+      tI += site[4 * pc]; tE += site[4 * pc + 1]; wI += site[4 * pc + 2]; wE += site[4 * pc + 3];
+      if (d.is_leader || d.guarded) {
+        tI += bbsite[4 * pc]; tE += bbsite[4 * pc + 1]; wI += bbsite[4 * pc + 2]; wE += bbsite[4 * pc + 3];
+      } else {  // same active mask as the block's leader (BB rule), unguarded: E = A
+        tI += bbsite[4 * l]; tE += bbsite[4 * l]; wI += bbsite[4 * l + 2]; wE += bbsite[4 * l + 2];
+      }
+      n += mem[3 * pc]; sS += mem[3 * pc + 1]; sL += mem[3 * pc + 2];
     }
     if (tI | wI) {
       atomicAdd(out + L.o_counts + 0, tI);
@@ -79,18 +89,21 @@ __global__ void fold_kernel(const nvbt_instr_desc* __restrict__ prog, const uint
       atomicAdd(bb + 2, wE);
       atomicAdd(bb + 3, tE);
     }
-    const unsigned long long n = mem[3 * pc], s = mem[3 * pc + 1], l = mem[3 * pc + 2];
     out[L.o_mem + 3 * pc] = n;
-    out[L.o_mem + 3 * pc + 1] = s;
-    out[L.o_mem + 3 * pc + 2] = l;
+    out[L.o_mem + 3 * pc + 1] = sS;
+    out[L.o_mem + 3 * pc + 2] = sL;
     if (n) {
       atomicAdd(out + L.o_memtot, n);
-      atomicAdd(out + L.o_memtot + 1, s);
-      atomicAdd(out + L.o_memtot + 2, l);
+      atomicAdd(out + L.o_memtot + 1, sS);
+      atomicAdd(out + L.o_memtot + 2, sL);
     }
   }
   const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
-  if (t < 66) out[L.o_hist + t] = hist[t];
+  if (t < 66) {
+    unsigned long long h = 0;
+    for (size_t s = 0; s < L.stripes; ++s) h += accum[s * SW + L.hist + t];
+    out[L.o_hist + t] = h;
+  }
 }
 
 int fold(nvbt_ctx c) {
@@ -98,11 +111,17 @@ int fold(nvbt_ctx c) {
   NVBT_CUDA(cudaMemsetAsync(c->out, 0, c->lay.out_words * 8, c->stream));
   const int threads = 256;
   const int blocks = (int)((c->n_pcs + threads - 1) / threads);
-  fold_kernel<<<blocks, threads, 0, c->stream>>>(c->d_prog, c->d_leader, c->n_pcs, c->n_ops, c->n_bbs, c->site(),
-                                                  c->bbsite(), c->mem(), c->hist(), c->out, c->lay);
+  fold_kernel<<<blocks, threads, 0, c->stream>>>(c->d_prog, c->d_leader, c->n_pcs, c->n_ops, c->n_bbs, c->accum,
+                                                  c->out, c->lay);
   NVBT_CUDA(cudaGetLastError());
   c->launches++;
   return NVBT_OK;
+}
+
+__global__ void axpy_kernel(unsigned long long* __restrict__ y, const unsigned long long* __restrict__ x, size_t n,
+                            unsigned long long a) {
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x)
+    y[i] += a * x[i];
 }
 
 static int read_out(nvbt_ctx c, size_t word, size_t n, void* dst) {
@@ -132,6 +151,8 @@ int make_state(nvbt_ctx c, uint32_t tools, DevState* st) {
   st->hist = c->hist();
   st->pw = c->pw();
   st->n_warps = c->n_warps;
+  st->stripes = (unsigned)c->lay.stripes;
+  st->stripe_words = c->lay.stripe_words;
   st->head = c->ctl + CTL_HEAD;
   st->tail_cache = c->ctl + CTL_TAIL_CACHE;
   st->dropped = c->ctl + CTL_DROPPED;
@@ -255,6 +276,20 @@ int nvbt_accum_view(nvbt_ctx c, void** d_ptr, size_t* n) {
   if (!c || !d_ptr || !n) return set_error(NVBT_EINVAL, "null argument");
   *d_ptr = c->accum;
   *n = c->lay.accum_words;
+  return NVBT_OK;
+}
+
+int nvbt_accum_axpy(nvbt_ctx c, const void* d_src, size_t n, int64_t factor) {
+  if (!c || (!d_src && n)) return set_error(NVBT_EINVAL, "null argument");
+  if (n != c->lay.accum_words) return set_error(NVBT_EINVAL, "n_int64 %zu != accumulator words %zu", n, c->lay.accum_words);
+  if (factor < 0) return set_error(NVBT_EINVAL, "factor must be >= 0");
+  if (n == 0 || factor == 0) return NVBT_OK;
+  NVBT_CUDA(cudaSetDevice(c->device));
+  const int blocks = (int)std::min<size_t>((n + 255) / 256, 1024);
+  axpy_kernel<<<blocks, 256, 0, c->stream>>>(c->accum, static_cast<const unsigned long long*>(d_src), n,
+                                             (unsigned long long)factor);
+  NVBT_CUDA(cudaGetLastError());
+  c->launches++;
   return NVBT_OK;
 }
 

@@ -44,6 +44,8 @@ struct DevState {
   unsigned long long cap;          // ring slots
   unsigned launch;
   unsigned n_warps;
+  unsigned stripes;                // site/mem/hist repeat `stripes` times, stride stripe_words
+  unsigned long long stripe_words;
 };
 
 __device__ __forceinline__ unsigned lane_id() { unsigned l; asm("mov.u32 %0, %%laneid;" : "=r"(l)); return l; }
@@ -242,6 +244,7 @@ struct Hooks {
   static constexpr bool kCount = (T & (TOOL_COUNT | TOOL_BB)) != 0;
   static constexpr bool kBB = (T & TOOL_BB) != 0;
   static constexpr int kMaxWarps = 8;  // workload CTAs have 256 threads
+  static constexpr int kThreads = 32 * kMaxWarps;
   static constexpr int kScratchWord0 = (NPC * SITE_WORDS + 66 + 3) & ~3;  // 16-byte aligned
   static constexpr int kSmemWords = kOn ? kScratchWord0 + SCRATCH_WORDS * kMaxWarps : 1;
   static_assert(!((T & TOOL_COUNT) && (T & TOOL_BB)), "COUNT and BBCOUNT are exclusive");
@@ -255,7 +258,7 @@ struct Hooks {
   unsigned npend = 0;         // uncommitted records of this warp (warp-uniform)
   unsigned pend_val = 0;      // lane k: tag value of the k-th uncommitted record
   unsigned char* pend_tag = nullptr;
-  unsigned lane, lane1, lanebit, lmlt, gwarp, scr;
+  unsigned lane, lane1, lanebit, lmlt, gwarp, scr, sbase;
 
   __device__ __forceinline__ Hooks(const DevState& s, unsigned* smem) : st(s), sb(smem) {
     zero_range<0, NPC - 1>();
@@ -267,9 +270,15 @@ struct Hooks {
     const unsigned tid = threadIdx.x + threadIdx.y * blockDim.x;
     gwarp = (blockIdx.x + blockIdx.y * gridDim.x) * ((blockDim.x * blockDim.y) >> 5) + (tid >> 5);
     scr = (unsigned)__cvta_generic_to_shared(sb + kScratchWord0 + SCRATCH_WORDS * ((tid >> 5) & (kMaxWarps - 1)));
+    sbase = (unsigned)__cvta_generic_to_shared(sb);
     if constexpr (kOn) {
-      for (int i = tid; i < kSmemWords; i += blockDim.x * blockDim.y)
-        sb[i] = i < kScratchWord0 ? 0u : scratch_init_word((i - kScratchWord0) % SCRATCH_WORDS);
+      // (CTAs of exactly kThreads threads; fixed-stride loops avoid a run-time trip-count division)
+      constexpr int kInit = (T & TOOL_MEM) ? kSmemWords : kScratchWord0;   // scratch only for divergence
+#pragma unroll
+      for (int k = 0; k < (kInit + kThreads - 1) / kThreads; ++k) {
+        const int i = (int)tid + k * kThreads;
+        if (i < kInit) sb[i] = i < kScratchWord0 ? 0u : scratch_init_word((i - kScratchWord0) % SCRATCH_WORDS);
+      }
       __syncthreads();
     }
   }
@@ -292,18 +301,44 @@ struct Hooks {
     constexpr bool cnt = (T & TOOL_COUNT) || ((T & TOOL_BB) && (d.is_leader || d.guarded));
     constexpr bool div = mem && (T & TOOL_MEM);
     constexpr bool trc = mem && (T & TOOL_TRACE);
+    constexpr bool reg = PC >= Prog::REG_LO && PC <= Prog::REG_HI;   // loop site: register counters
     if constexpr (cnt || div || trc) {
       const unsigned A = m.A;
       const unsigned P = d.guarded ? (__ballot_sync(FULL, pred) & A) : A;
       const unsigned E = P;
       if constexpr (cnt) {
         const unsigned pa = __popc(A), wa = umin(pa, 1u);
-        tA[PC] += pa;
-        wI[PC] += wa;
-        if constexpr (d.guarded) {
-          const unsigned pe = __popc(E);
-          dT[PC] += pa - pe;
-          dW[PC] += wa - umin(pe, 1u);
+        const unsigned pe = d.guarded ? __popc(E) : pa, we = d.guarded ? umin(pe, 1u) : wa;
+        if constexpr (reg) {
+          tA[PC] += pa;
+          wI[PC] += wa;
+          if constexpr (d.guarded) {
+            dT[PC] += pa - pe;
+            dW[PC] += wa - we;
+          }
+        } else {
+          const unsigned b = sbase + 4u * (PC * SITE_WORDS);
+          red_if(lane == 0u, b, pa);
+          red_if(lane == 0u, b + 8u, wa);
+          if constexpr (d.guarded) {
+            red_if(lane == 0u, b + 4u, pa - pe);
+            red_if(lane == 0u, b + 12u, wa - we);
+          }
+          // this warp's executed totals (PER_WARP); register sites add theirs at retire()
+          if constexpr ((T & TOOL_COUNT) != 0) {
+            pwT += pe;
+            pwW += we;
+          } else {
+            if constexpr (d.is_leader) {
+              constexpr unsigned len = (unsigned)bb_len<Prog>(PC);
+              pwT += len * pa;
+              pwW += len * wa;
+            }
+            if constexpr (d.guarded) {
+              pwT -= pa - pe;
+              pwW -= wa - we;
+            }
+          }
         }
       }
       if constexpr (div || trc) {
@@ -311,7 +346,14 @@ struct Hooks {
           if constexpr (div) {
             unsigned S, L;
             sectors_lines(addr, E, lane, lanebit, lmlt, scr, S, L);
-            mN[PC] += 1u; mS[PC] += S; mL[PC] += L;
+            if constexpr (reg) {
+              mN[PC] += 1u; mS[PC] += S; mL[PC] += L;
+            } else {
+              const unsigned b = sbase + 4u * (PC * SITE_WORDS);
+              red_if(lane == 0u, b + 16u, 1u);
+              red_if(lane == 0u, b + 20u, S);
+              red_if(lane == 0u, b + 24u, L);
+            }
             inc_if_eq(hS, S, lane1);
             inc_if_eq(hL, L, lane1);
           }
@@ -319,6 +361,11 @@ struct Hooks {
         }
       }
     }
+  }
+
+  __device__ __forceinline__ static void red_if(bool p, unsigned saddr, unsigned v) {
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q red.shared.add.u32 [%0], %1;\n\t}"
+                 ::"r"(saddr), "r"(v), "r"((unsigned)p) : "memory");
   }
 
   // a6 producer. One record per executed global-memory event: lane 0 takes a ticket; the warp writes
@@ -396,10 +443,18 @@ struct Hooks {
   // pc LO + 32r + l) and zeroes them, freeing their registers. In BB mode [LO, HI] must be whole blocks.
   template <int LO, int HI>
   __device__ __forceinline__ void retire() {
+    constexpr int RLO = LO > Prog::REG_LO ? LO : Prog::REG_LO;
+    constexpr int RHI = HI < Prog::REG_HI ? HI : Prog::REG_HI;
+    if constexpr (kOn && RLO <= RHI) retire_regs<RLO, RHI>();
+  }
+
+  // register-mode pcs [LO, HI] -> shared bins
+  template <int LO, int HI>
+  __device__ __forceinline__ void retire_regs() {
     if constexpr (kOn) {
       static_assert(LO >= 0 && HI < NPC && LO <= HI, "bad range");
       static_assert(!kBB || (Prog::t[LO].is_leader && (HI + 1 == NPC || Prog::t[HI + 1].is_leader)),
-                    "BB mode retires whole blocks");
+                    "register-mode pc ranges are whole basic blocks");
       if constexpr (kCount) {
         unsigned t = 0, w = 0;
         retire_sum<LO, HI>(t, w);
@@ -467,25 +522,27 @@ struct Hooks {
       }
       __syncthreads();
       const int tid = threadIdx.x + threadIdx.y * blockDim.x;
-      const int nt = blockDim.x * blockDim.y;
+      constexpr int nt = kThreads;
+      // this CTA's stripe of the global bins (spreads same-address atomics over st.stripes copies)
+      const unsigned long long so = (unsigned long long)((blockIdx.x + blockIdx.y * gridDim.x) & (st.stripes - 1u)) * st.stripe_words;
       for (int pc = tid; pc < NPC; pc += nt) {
         const unsigned* b = sb + pc * SITE_WORDS;
         if (b[0] | b[2]) {
-          unsigned long long* s = st.site + 4 * pc;
+          unsigned long long* s = st.site + so + 4 * pc;
           atomicAdd(s + 0, (unsigned long long)b[0]);
           if (b[0] - b[1]) atomicAdd(s + 1, (unsigned long long)(b[0] - b[1]));
           atomicAdd(s + 2, (unsigned long long)b[2]);
           if (b[2] - b[3]) atomicAdd(s + 3, (unsigned long long)(b[2] - b[3]));
         }
         if (b[4]) {
-          unsigned long long* m = st.mem + 3 * pc;
+          unsigned long long* m = st.mem + so + 3 * pc;
           atomicAdd(m + 0, (unsigned long long)b[4]);
           atomicAdd(m + 1, (unsigned long long)b[5]);
           atomicAdd(m + 2, (unsigned long long)b[6]);
         }
       }
       for (int i = tid; i < 66; i += nt)
-        if (sb[NPC * SITE_WORDS + i]) atomicAdd(st.hist + i, (unsigned long long)sb[NPC * SITE_WORDS + i]);
+        if (sb[NPC * SITE_WORDS + i]) atomicAdd(st.hist + so + i, (unsigned long long)sb[NPC * SITE_WORDS + i]);
     }
   }
 };

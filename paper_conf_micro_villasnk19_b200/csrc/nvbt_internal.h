@@ -25,9 +25,12 @@ int set_error(int code, const char* fmt, ...);
   } while (0)
 
 // Workspace layout (bytes from d_workspace). The accumulator region comes first and is one packed
-// int64 array: site[4P] | bbsite[4P] | mem[3P] | hist[66] | pw[2W].
+// int64 array: K stripes of {site[4P] | bbsite[4P] | mem[3P] | hist[66]}, then pw[2W]. A CTA flushes its
+// shared bins into stripe (linear CTA id % K), so kernels with many small CTAs do not serialise on the
+// same global addresses; the fold kernel sums the stripes (integer sums, order-free).
 struct Layout {
   size_t site, bbsite, mem, hist, pw, accum_words;   // word offsets into the accumulator region
+  size_t stripe_words, stripes;                     // site..hist repeat `stripes` times (CTA-striped bins)
   size_t ctl;                                       // byte offsets from here on
   size_t prog, leader, kind, out;
   size_t out_words;

@@ -13,8 +13,11 @@ constexpr uint8_t ALU = NVBT_K_ALU, CTRL = NVBT_K_CTRL, GLD = NVBT_K_GLD, GST = 
 
 #define NVBT_D(o, k, w, b, l, g) nvbt_instr_desc{op::o, k, w, b, l, g, 0}
 
+// REG_LO..REG_HI: pcs inside loops; their hooks accumulate in registers (flushed once per warp). Other
+// hooks run once per warp and add straight into the CTA's shared bins.
 struct ProgVectorAdd {  // §3.1
   static constexpr int N = 13;
+  static constexpr int REG_LO = 1, REG_HI = 0;
   static constexpr nvbt_instr_desc t[N] = {
       NVBT_D(S2R, ALU, 0, 0, 1, 0),       NVBT_D(S2R, ALU, 0, 0, 0, 0),       NVBT_D(IMAD, ALU, 0, 0, 0, 0),
       NVBT_D(ISETP, ALU, 0, 0, 0, 0),     NVBT_D(EXIT, CTRL, 0, 0, 0, 1),     NVBT_D(IMAD_WIDE, ALU, 0, 1, 1, 0),
@@ -25,6 +28,7 @@ struct ProgVectorAdd {  // §3.1
 
 struct ProgSgemm {  // §3.2
   static constexpr int N = 18;
+  static constexpr int REG_LO = 10, REG_HI = 15;
   static constexpr nvbt_instr_desc t[N] = {
       NVBT_D(S2R, ALU, 0, 0, 1, 0),  NVBT_D(S2R, ALU, 0, 0, 0, 0),   NVBT_D(S2R, ALU, 0, 0, 0, 0),
       NVBT_D(S2R, ALU, 0, 0, 0, 0),  NVBT_D(IMAD, ALU, 0, 0, 0, 0),  NVBT_D(IMAD, ALU, 0, 0, 0, 0),
@@ -36,6 +40,7 @@ struct ProgSgemm {  // §3.2
 
 struct ProgBfs {  // §3.3 (kernel 1: pcs 0-21, kernel 2: pcs 22-35)
   static constexpr int N = 36;
+  static constexpr int REG_LO = 13, REG_HI = 20;
   static constexpr nvbt_instr_desc t[N] = {
       NVBT_D(S2R, ALU, 0, 0, 1, 0),   NVBT_D(S2R, ALU, 0, 0, 0, 0),   NVBT_D(IMAD, ALU, 0, 0, 0, 0),
       NVBT_D(ISETP, ALU, 0, 0, 0, 0), NVBT_D(EXIT, CTRL, 0, 0, 0, 1),
@@ -57,6 +62,7 @@ struct ProgBfs {  // §3.3 (kernel 1: pcs 0-21, kernel 2: pcs 22-35)
 
 struct ProgStencil {  // §3.4
   static constexpr int N = 21;
+  static constexpr int REG_LO = 1, REG_HI = 0;
   static constexpr nvbt_instr_desc t[N] = {
       NVBT_D(S2R, ALU, 0, 0, 1, 0),   NVBT_D(S2R, ALU, 0, 0, 0, 0),   NVBT_D(S2R, ALU, 0, 0, 0, 0),
       NVBT_D(S2R, ALU, 0, 0, 0, 0),   NVBT_D(IMAD, ALU, 0, 0, 0, 0),  NVBT_D(IMAD, ALU, 0, 0, 0, 0),

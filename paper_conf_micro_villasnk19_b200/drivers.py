@@ -95,3 +95,36 @@ def merge(ctx, group=None):
     """a8: one int64 SUM all-reduce of the packed accumulator region (NCCL over NVLink on GPUs).
     Sums of disjoint event sets add (EM §4), so every rank then holds the whole job's result."""
     return merge_tensor(_nb().nvbt_accum_view(ctx), group)
+
+
+class KernelSampler:
+    """F1 kernel sampling (P:L274-282 (§6.2)): "we launch the instrumented version only once for each set
+    of unique grid dimension values ... for the remaining ... times we run foo uninstrumented. We then use
+    the information collected during the instrumented kernel execution to approximate the information not
+    collected". The one instrumented launch of a key runs on a scratch context; its accumulator region is
+    kept (device) and, at finish(), added to the target context once per launch of that key
+    (nvbt_accum_axpy). When a kernel's control flow depends only on its grid dimensions the result is
+    exact (P:L282)."""
+
+    def __init__(self, ctx, scratch):
+        self.ctx, self.scratch = ctx, scratch
+        self.launches = {}
+        self.snapshots = {}
+
+    def launch(self, key, launch_fn, tools):
+        """launch_fn(ctx_or_None, tools) enqueues one launch; key identifies its grid shape."""
+        nb = _nb()
+        self.launches[key] = self.launches.get(key, 0) + 1
+        if key in self.snapshots:
+            launch_fn(self.ctx, nb.TOOL_NONE)
+            return False
+        nb.nvbt_reset(self.scratch)
+        launch_fn(self.scratch, tools)
+        self.snapshots[key] = nb.nvbt_accum_view(self.scratch).clone()
+        return True
+
+    def finish(self):
+        nb = _nb()
+        for key, snap in self.snapshots.items():
+            nb.nvbt_accum_axpy(self.ctx, snap, self.launches[key])
+        return dict(self.launches)

@@ -71,6 +71,7 @@ _sigs = {
     "nvbt_reset": ([_P], C.c_int),
     "nvbt_fini": ([_P], C.c_int),
     "nvbt_accum_view": ([_P, C.POINTER(_P), C.POINTER(C.c_size_t)], C.c_int),
+    "nvbt_accum_axpy": ([_P, _P, C.c_size_t, C.c_int64], C.c_int),
     "nvbt_count": ([_P, C.POINTER(Counts), _P, _P], C.c_int),
     "nvbt_opcode_hist": ([_P, _P, _P, C.c_uint32], C.c_int),
     "nvbt_bb_count": ([_P, _P, C.c_uint32], C.c_int),
@@ -226,6 +227,11 @@ def nvbt_accum_view(ctx):
     _check(_lib.nvbt_accum_view(ctx.handle, C.byref(p), C.byref(n)))
     off = p.value - ctx.workspace.data_ptr()
     return ctx.workspace[off:off + 8 * n.value].view(torch.int64)
+
+
+def nvbt_accum_axpy(ctx, src, factor):
+    """accum += factor * src (src: int64 CUDA tensor with the accumulator layout)."""
+    _check(_lib.nvbt_accum_axpy(ctx.handle, C.c_void_p(src.data_ptr()), src.numel(), int(factor)))
 
 
 def nvbt_count(ctx, per_warp=False):

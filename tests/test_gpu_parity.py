@@ -381,3 +381,63 @@ def test_api_errors(nvbt):
     with pytest.raises(nb.NvbtError) as e:
         nb.nvbt_channel_open(tctx, ring)
     assert e.value.code == nb.EINVAL
+
+
+# ---------------------------------------------------------------- F1 kernel sampling
+def test_kernel_sampling_exact_when_control_flow_is_grid_only(nvbt):
+    """"If the control flow of a kernel does not change based on the values computed, but it is
+    only a function of the grid dimensions, the sampling error is 0%" — stencil and vectorAdd qualify."""
+    import torch
+    nb, dr = nvbt.nvbt, nvbt.drivers
+    flags = nb.COUNT | nb.OPHIST | nb.BB | nb.MEMDIV
+    full = nb.nvbt_init(nb.W_STENCIL, flags)
+    samp = nb.nvbt_init(nb.W_STENCIL, flags)
+    scratch = nb.nvbt_init(nb.W_STENCIL, flags)
+    sampler = dr.KernelSampler(samp, scratch)
+    tools = nb.TOOL_BBCOUNT | nb.TOOL_MEMDIV
+    for n, iters in [(96, 5), (64, 3), (96, 2)]:
+        x0 = cuda(uniform_f32((n, n), 4))
+        b0, b1 = x0.clone(), torch.zeros_like(x0)
+        bufs = (b0, b1)
+        for it in range(iters):
+            src, dst = bufs[it % 2], bufs[(it + 1) % 2]
+            nb.nvbt_stencil(full, tools, src, dst, n)
+            sampler.launch(("stencil", n), lambda c, t: nb.nvbt_stencil(c, t, src, dst, n), tools)
+    launches = sampler.finish()
+    assert launches == {("stencil", 96): 7, ("stencil", 64): 3}
+    assert_same(read_all(nb, samp), read_all(nb, full), COUNT_KEYS + MEM_KEYS, "sampled stencil")
+
+
+def test_kernel_sampling_error_on_data_dependent_kernels(nvbt):
+    """BFS levels share grid dimensions but not control flow: sampling extrapolates level 0's counts to
+    every level, so its error is large and reported, not hidden."""
+    nb, dr = nvbt.nvbt, nvbt.drivers
+    rowptr, col = rmat_csr(10, 16, seed=3)
+    n = len(rowptr) - 1
+    src = bfs_source(rowptr)
+    rp, cl = cuda(rowptr), cuda(col)
+    full = nb.nvbt_init(nb.W_BFS, nb.COUNT | nb.BB)
+    dr.run_bfs(full, nb.TOOL_BBCOUNT, rp, cl, src)
+    samp = nb.nvbt_init(nb.W_BFS, nb.COUNT | nb.BB)
+    scratch = nb.nvbt_init(nb.W_BFS, nb.COUNT | nb.BB)
+    sampler = dr.KernelSampler(samp, scratch)
+    bufs = dr.bfs_buffers(n, "cuda")
+    dr.run_bfs(None, 0, rp, cl, src, bufs)                 # plain run to know the level count
+    import torch
+    bufs = dr.bfs_buffers(n, "cuda")
+    bufs["mask"][src] = 1; bufs["visited"][src] = 1; bufs["cost"][src] = 0
+    level = 0
+    while True:
+        bufs["over"].zero_(); bufs["updating"].zero_()
+        sampler.launch(("bfs", n), lambda c, t: nb.nvbt_bfs_level(c, t, rp, cl, n, bufs["mask"], bufs["visited"],
+                                                                  bufs["updating"], bufs["cost"], bufs["over"],
+                                                                  level),
+                       nb.TOOL_BBCOUNT)
+        torch.cuda.synchronize()
+        level += 1
+        if int(bufs["over"].item()) == 0:
+            break
+    sampler.finish()
+    exact, est = nb.nvbt_count(full).astype(np.int64), nb.nvbt_count(samp).astype(np.int64)
+    assert est[2] != exact[2]                               # sampling is not exact here
+    assert exact[2] > 0 and abs(est[2] - exact[2]) / exact[2] < 10.0
