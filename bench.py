@@ -476,8 +476,9 @@ def run_c4(args, torch, nb, dr, local):
     ctx = nb.nvbt_init(nb.W_STENCIL, nb.COUNT | nb.TRACE)
     x0 = torch.from_numpy(uniform_f32((n, n), 4)).cuda()
     buf0, buf1 = x0.clone(), torch.empty_like(x0)
-    ring = torch.empty(64 + 288 * args.ring_records, dtype=torch.uint8, pin_memory=True)
-    ch = nb.nvbt_channel_open(ctx, ring)
+    slot = 176 if args.compact else 288
+    ring = torch.empty(64 + slot * args.ring_records, dtype=torch.uint8, pin_memory=True)
+    ch = nb.nvbt_channel_open(ctx, ring, compact=args.compact)
     # plain baseline
     for _ in range(args.warmup):
         dr.run_stencil(ctx, nb.TOOL_NONE, buf0, buf1, n, iters)
@@ -503,11 +504,12 @@ def run_c4(args, torch, nb, dr, local):
     return {"metric": "traced warp-level memory events/sec (records drained to host)", "value": recs / t_tr,
             "unit": "records/s", "n_gpus": 1, "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * t_tr,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-            "config": {"workload": f"C4 stencil {n}^2 x {iters}, tools TRACE", "ring_records": args.ring_records},
+            "config": {"workload": f"C4 stencil {n}^2 x {iters}, tools TRACE", "ring_slots": args.ring_records,
+                       "transport": "compact 176 B slots (EM 5.1)" if args.compact else "288 B records"},
             "records_per_run": recs, "records_expected": expect, "dropped": dropped,
             "gpu_s_per_run": sum(r[2] for r in res) / len(res),
             "host_threads": os.environ.get("NVBT_DRAIN_THREADS", str(os.cpu_count())),
-            "GB_per_s_to_host": recs * 288 / t_tr / 1e9, "slowdown": t_tr / (sum(tp) / len(tp)),
+            "GB_per_s_to_host": recs * slot / t_tr / 1e9, "record_GB_per_s": recs * 288 / t_tr / 1e9, "slowdown": t_tr / (sum(tp) / len(tp)),
             "plain_ms": 1e3 * sum(tp) / len(tp), "bound": "PCIe D2H (measured 52.7 GB/s SM stores to pinned memory)",
             "clocks": clk.summary()}
 
@@ -606,6 +608,7 @@ def main():
     ap.add_argument("--stencil-n", type=int, default=8192)
     ap.add_argument("--stencil-iters", type=int, default=100)
     ap.add_argument("--ring-records", type=int, default=1 << 22)
+    ap.add_argument("--compact", action="store_true", help="C4: compact 176 B transport slots (F3)")
     ap.add_argument("--replay-events", type=int, default=10**10)
     ap.add_argument("--cpu-budget", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")

@@ -124,9 +124,13 @@ int nvbt_mem_divergence(nvbt_ctx ctx, nvbt_memdiv* per_pc, uint32_t n_pcs, nvbt_
 
 /* ---- trace channel (a6; "sent to the CPU for further processing", P:L187 (§6.1)) ----
  * pinned_ring: caller-owned pinned, device-mapped host memory (cudaHostAlloc / torch pin_memory), at
- * least 64 + 288 * 2 bytes, 64-byte aligned. Its first 64 bytes hold the consumer index the producers
- * read for backpressure; the rest is floor((ring_bytes - 64) / 288) record slots. record_bytes must be
- * 288 (EM §5). One channel per context. */
+ * least 64 + 2 * record_bytes bytes, 64-byte aligned. Its first 64 bytes hold the consumer index the
+ * producers read for backpressure; the rest is floor((ring_bytes - 64) / record_bytes) slots.
+ * record_bytes: NVBT_RECORD_BYTES (288: every slot is an EM §5 record) or NVBT_COMPACT_RECORD_BYTES (176:
+ * base + 32-bit deltas, wide address sets as two slots; EM §5.1, F3). Either way the drain delivers EM §5
+ * records. One channel per context. */
+#define NVBT_RECORD_BYTES 288
+#define NVBT_COMPACT_RECORD_BYTES 176
 int nvbt_channel_open(nvbt_ctx ctx, void* pinned_ring, size_t ring_bytes, uint32_t record_bytes,
                       nvbt_channel* out);
 /* Called with a batch of n contiguous, fully written records (reserved field zeroed); return 0 to
@@ -148,6 +152,9 @@ typedef struct { void* dst; uint64_t capacity; uint64_t n; } nvbt_copy_sink;   /
 int nvbt_drain_copy(const void* records, uint64_t n_records, void* user /* nvbt_copy_sink* */);
 /* Host-side digest of an array of records (for checking copies). */
 int nvbt_digest_records(const void* records, uint64_t n_records, nvbt_digest* out);
+/* Decodes n_slots 176 B transport slots (EM §5.1; tags ignored) into EM §5 records at out (capacity
+ * out_cap records); *n_out = records written. EINVAL on an unpaired wide slot or a too-small out. */
+int nvbt_decode_compact(const void* slots, uint64_t n_slots, void* out, uint64_t out_cap, uint64_t* n_out);
 
 /* ---- trace-replay mode (a7; EM §3.5) ---- */
 /* Writes events [first, first+n) of the counter-based generator (seed) as 16 B headers at d_hdr[n]

@@ -27,17 +27,26 @@ struct nvbt_chan_s {
   unsigned char* slots = nullptr;     // host view of slot 0
   uint64_t cap = 0;
   uint64_t consumed = 0;
+  unsigned slot = 288;                 // bytes per ring slot (288 full, 176 compact)
+  bool force_wide = false;
   bool open = false;
+  bool have_half = false;              // compact: first half of a wide pair seen at the ring end
+  unsigned char half[176];
+  std::vector<unsigned char> scratch;  // compact: decoded records of one batch
 };
 
 namespace nvbt {
 
 static constexpr size_t HDR = 64;
+static constexpr unsigned COMPACT_BYTES = NVBT_COMPACT_RECORD_BYTES;
 
 void channel_state(nvbt_chan_s* ch, DevState* st) {
   st->ring = ch->dev + HDR;
   st->tail = reinterpret_cast<const unsigned long long*>(ch->dev);
   st->cap = ch->cap;
+  st->slot_bytes = ch->slot;
+  // compact = 1; 2 forces the wide form for every record (NVBT_COMPACT_FORCE_WIDE=1, tests only)
+  st->compact = ch->slot == COMPACT_BYTES ? (ch->force_wide ? 2u : 1u) : 0u;
 }
 bool channel_open(nvbt_chan_s* ch) { return ch && ch->open; }
 
@@ -154,24 +163,104 @@ static void digest_range(const unsigned char* rec, uint64_t n, uint64_t* d1, uin
 static inline bool slot_ready(const unsigned char* rec, uint32_t lap) {
   return *reinterpret_cast<volatile const uint32_t*>(rec + 28) == lap;
 }
-static uint64_t ready_prefix(const unsigned char* base, uint64_t lim, uint32_t lap) {
+static uint64_t ready_prefix(const unsigned char* base, uint64_t lim, uint32_t lap, unsigned sb) {
   const uint64_t w = std::min<uint64_t>(lim, 2048);
   uint64_t n = 0;
-  while (n < w && slot_ready(base + n * RECORD_BYTES, lap)) ++n;
+  while (n < w && slot_ready(base + n * sb, lap)) ++n;
   if (n < w || n == lim) return n;
   Pool& pool = Pool::get();
   const uint64_t rest = lim - n;
   std::vector<uint64_t> first(pool.size(), UINT64_MAX);
-  const unsigned char* b2 = base + n * RECORD_BYTES;
+  const unsigned char* b2 = base + n * sb;
   pool.parallel_for(rest, [&](unsigned id, uint64_t lo, uint64_t hi) {
     uint64_t i = lo;
-    while (i < hi && slot_ready(b2 + i * RECORD_BYTES, lap)) ++i;
+    while (i < hi && slot_ready(b2 + i * sb, lap)) ++i;
     first[id] = i < hi ? i : UINT64_MAX;
   });
   uint64_t stop = rest;
   for (uint64_t f : first) stop = std::min(stop, f);
   return n + stop;
 }
+// ---- compact transport (EM §5.1): slot flags in byte 27 (kind | 0x80 compact, 0x40 / 0x20 wide halves)
+static inline unsigned slot_flags(const unsigned char* sl) { return sl[27] & 0xE0u; }
+
+static void decode_compact_slot(const unsigned char* sl, unsigned char* out) {
+  std::memcpy(out, sl, 28);
+  out[27] = sl[27] & 0x1Fu;
+  std::memset(out + 28, 0, 4);
+  uint32_t A, P;
+  std::memcpy(&A, sl + 16, 4);
+  std::memcpy(&P, sl + 20, 4);
+  const uint32_t E = A & P;
+  uint64_t base;
+  std::memcpy(&base, sl + 32, 8);
+  for (int l = 0; l < 32; ++l) {
+    int32_t d;
+    std::memcpy(&d, sl + 48 + 4 * l, 4);
+    const uint64_t a = ((E >> l) & 1u) ? base + (uint64_t)(int64_t)d : 0ull;
+    std::memcpy(out + 32 + 8 * l, &a, 8);
+  }
+}
+static void decode_wide_pair(const unsigned char* s0, const unsigned char* s1, unsigned char* out) {
+  std::memcpy(out, s0, 28);
+  out[27] = s0[27] & 0x1Fu;
+  std::memset(out + 28, 0, 4);
+  std::memcpy(out + 32, s0 + 32, 128);
+  std::memcpy(out + 160, s1 + 32, 128);
+}
+
+// Decodes slots [0, n) into records; a wide-first at the end must not occur (caller keeps pairs whole).
+// Parallel: count records per part, prefix, decode. Returns the record count.
+static uint64_t decode_batch(const unsigned char* sl, uint64_t n, unsigned char* out) {
+  Pool& pool = Pool::get();
+  std::vector<uint64_t> cnt(pool.size() + 1, 0), lo_of(pool.size(), 0), hi_of(pool.size(), 0);
+  auto is_rec = [&](uint64_t i) { return slot_flags(sl + (size_t)i * COMPACT_BYTES) != 0x20u; };
+  pool.parallel_for(n, [&](unsigned id, uint64_t lo, uint64_t hi) {
+    uint64_t c = 0;
+    for (uint64_t i = lo; i < hi; ++i) c += is_rec(i);
+    cnt[id + 1] = c;
+    lo_of[id] = lo;
+    hi_of[id] = hi;
+  });
+  for (size_t k = 1; k < cnt.size(); ++k) cnt[k] += cnt[k - 1];
+  pool.parallel_for(n, [&](unsigned id, uint64_t lo, uint64_t hi) {
+    uint64_t o = cnt[id];
+    for (uint64_t i = lo; i < hi; ++i) {
+      const unsigned char* s0 = sl + (size_t)i * COMPACT_BYTES;
+      const unsigned f = slot_flags(s0);
+      if (f == 0x20u) continue;
+      unsigned char* r = out + (size_t)o * RECORD_BYTES;
+      if (f == 0x40u) decode_wide_pair(s0, s0 + COMPACT_BYTES, r);
+      else decode_compact_slot(s0, r);
+      ++o;
+    }
+  });
+  return cnt.back();
+}
+
+// Digest of the records encoded in slots [0, n) without materialising them (built-in digest callback).
+static uint64_t digest_compact(const unsigned char* sl, uint64_t n, uint64_t* d1, uint64_t* d2) {
+  Pool& pool = Pool::get();
+  std::vector<uint64_t> p1(pool.size(), 0), p2(pool.size(), 0), pc(pool.size(), 0);
+  pool.parallel_for(n, [&](unsigned id, uint64_t lo, uint64_t hi) {
+    alignas(16) unsigned char rec[RECORD_BYTES];
+    uint64_t s1 = 0, s2 = 0, c = 0;
+    for (uint64_t i = lo; i < hi; ++i) {
+      const unsigned char* s0 = sl + (size_t)i * COMPACT_BYTES;
+      const unsigned f = slot_flags(s0);
+      if (f == 0x20u) continue;
+      if (f == 0x40u) decode_wide_pair(s0, s0 + COMPACT_BYTES, rec);
+      else decode_compact_slot(s0, rec);
+      digest_serial(rec, 1, &s1, &s2);
+      ++c;
+    }
+    p1[id] = s1; p2[id] = s2; pc[id] = c;
+  });
+  uint64_t c = 0;
+  for (size_t k = 0; k < p1.size(); ++k) { *d1 += p1[k]; *d2 += p2[k]; c += pc[k]; }
+  return c;
+}
+
 static void clear_tags(unsigned char* base, uint64_t n) {
   Pool::get().parallel_for(n, [&](unsigned, uint64_t lo, uint64_t hi) {
     for (uint64_t r = lo; r < hi; ++r) std::memset(base + r * RECORD_BYTES + 28, 0, 4);
@@ -193,9 +282,10 @@ int nvbt_channel_open(nvbt_ctx c, void* ring, size_t bytes, uint32_t record_byte
   if (!c || !ring || !out) return set_error(NVBT_EINVAL, "null argument");
   if (!(c->flags & NVBT_TRACE)) return set_error(NVBT_ESTATE, "NVBT_TRACE not enabled at init");
   if (c->chan) return set_error(NVBT_ESTATE, "channel already open on this context");
-  if (record_bytes != RECORD_BYTES) return set_error(NVBT_EINVAL, "record_bytes %u != 288", record_bytes);
+  if (record_bytes != RECORD_BYTES && record_bytes != COMPACT_BYTES)
+    return set_error(NVBT_EINVAL, "record_bytes %u is neither 288 nor 176", record_bytes);
   if (reinterpret_cast<uintptr_t>(ring) % 64) return set_error(NVBT_EINVAL, "ring not 64-byte aligned");
-  if (bytes < HDR + 2 * RECORD_BYTES) return set_error(NVBT_ENOMEM, "ring of %zu bytes holds < 2 records", bytes);
+  if (bytes < HDR + 2 * record_bytes) return set_error(NVBT_ENOMEM, "ring of %zu bytes holds < 2 slots", bytes);
   NVBT_CUDA(cudaSetDevice(c->device));
   cudaPointerAttributes pa{};
   NVBT_CUDA(cudaPointerGetAttributes(&pa, ring));
@@ -207,8 +297,10 @@ int nvbt_channel_open(nvbt_ctx c, void* ring, size_t bytes, uint32_t record_byte
   ch->host = static_cast<unsigned char*>(ring);
   ch->dev = static_cast<unsigned char*>(pa.devicePointer);
   ch->slots = ch->host + HDR;
-  ch->cap = (bytes - HDR) / RECORD_BYTES;
-  std::memset(ch->host, 0, HDR + ch->cap * RECORD_BYTES);
+  ch->slot = record_bytes;
+  { const char* e = getenv("NVBT_COMPACT_FORCE_WIDE"); ch->force_wide = e && atoi(e) != 0; }
+  ch->cap = (bytes - HDR) / record_bytes;
+  std::memset(ch->host, 0, HDR + ch->cap * record_bytes);
   cudaError_t e = cudaMemsetAsync(c->ctl + CTL_HEAD, 0, 3 * 8, c->stream);  // head, tail_cache, dropped
   if (e == cudaSuccess) e = cudaStreamSynchronize(c->stream);
   if (e != cudaSuccess) { delete ch; return set_error(NVBT_ECUDA, "channel reset: %s", cudaGetErrorString(e)); }
@@ -248,8 +340,9 @@ int nvbt_channel_drain(nvbt_channel ch, nvbt_drain_fn fn, void* user, int64_t ti
     const uint64_t slot = ch->consumed % ch->cap;
     const uint32_t lap = static_cast<uint32_t>(ch->consumed / ch->cap) + 1u;
     const uint64_t lim = std::min<uint64_t>(ch->cap - slot, kBatch);
-    const uint64_t n = ready_prefix(ch->slots + slot * RECORD_BYTES, lim, lap);
-    if (n) {
+    const unsigned sb = ch->slot;
+    const uint64_t n = ready_prefix(ch->slots + slot * sb, lim, lap, sb);
+    if (n && sb == RECORD_BYTES) {
       std::atomic_thread_fence(std::memory_order_acquire);
       unsigned char* base = ch->slots + slot * RECORD_BYTES;
       if (!builtin) clear_tags(base, n);   // built-in callbacks ignore / clear the tag themselves
@@ -260,6 +353,46 @@ int nvbt_channel_drain(nvbt_channel ch, nvbt_drain_fn fn, void* user, int64_t ti
       *tail = ch->consumed;
       if (urc) { rc = set_error(NVBT_ESTATE, "drain callback returned %d", urc); break; }
       continue;
+    }
+    if (n) {  // compact transport: decode slots into EM §5 records, keep wide pairs together
+      std::atomic_thread_fence(std::memory_order_acquire);
+      const unsigned char* base = ch->slots + slot * sb;
+      if (ch->scratch.size() < (kBatch + 1) * RECORD_BYTES) ch->scratch.resize((kBatch + 1) * RECORD_BYTES);
+      unsigned char* out = ch->scratch.data();
+      uint64_t first = 0, end = n, consume = n, o = 0;
+      if (ch->have_half) {
+        if (slot_flags(base) != 0x20u) { rc = set_error(NVBT_ESTATE, "channel: unpaired wide record"); break; }
+        decode_wide_pair(ch->half, base, out);
+        ch->have_half = false;
+        first = 1;
+        o = 1;
+      }
+      if (end > first && slot_flags(base + (end - 1) * sb) == 0x40u) {
+        if (slot + end == ch->cap) {      // partner is slot 0 of the next lap: stash this half
+          std::memcpy(ch->half, base + (end - 1) * sb, COMPACT_BYTES);
+          ch->have_half = true;
+        } else {
+          --consume;                       // partner not ready yet: take the pair next time
+        }
+        --end;
+      }
+      int urc = 0;
+      if (fn == nvbt_drain_digest && user) {   // fused decode + digest, no staging of records
+        auto* dg = static_cast<nvbt_digest*>(user);
+        if (o) urc = fn(out, o, user);
+        const uint64_t k = digest_compact(base + first * sb, end - first, &dg->d1, &dg->d2);
+        dg->n_rec += k;
+        o += k;
+      } else {
+        o += decode_batch(base + first * sb, end - first, out + o * RECORD_BYTES);
+        urc = o ? fn(out, o, user) : 0;
+      }
+      ch->consumed += consume;
+      delivered += o;
+      std::atomic_thread_fence(std::memory_order_release);
+      *tail = ch->consumed;
+      if (urc) { rc = set_error(NVBT_ESTATE, "drain callback returned %d", urc); break; }
+      if (consume) continue;
     }
     const cudaError_t q = cudaStreamQuery(c->stream);
     if (q == cudaSuccess) {
@@ -305,6 +438,32 @@ int nvbt_drain_copy(const void* records, uint64_t n, void* user) {
   });
   s->n += n;
   return 0;
+}
+
+int nvbt_decode_compact(const void* slots, uint64_t n, void* out, uint64_t cap, uint64_t* n_out) {
+  if ((!slots && n) || (!out && cap) || !n_out) return set_error(NVBT_EINVAL, "null argument");
+  const unsigned char* sl = static_cast<const unsigned char*>(slots);
+  unsigned char* o = static_cast<unsigned char*>(out);
+  uint64_t k = 0;
+  for (uint64_t i = 0; i < n; ++i) {
+    const unsigned char* s0 = sl + i * COMPACT_BYTES;
+    const unsigned f = slot_flags(s0);
+    if (f == 0x20u) return set_error(NVBT_EINVAL, "slot %llu: wide second half without first", (unsigned long long)i);
+    if (k >= cap) return set_error(NVBT_EINVAL, "output capacity %llu too small", (unsigned long long)cap);
+    if (f == 0x40u) {
+      if (i + 1 >= n || slot_flags(s0 + COMPACT_BYTES) != 0x20u)
+        return set_error(NVBT_EINVAL, "slot %llu: wide first half without second", (unsigned long long)i);
+      decode_wide_pair(s0, s0 + COMPACT_BYTES, o + k * RECORD_BYTES);
+      ++i;
+    } else if (f == 0x80u) {
+      decode_compact_slot(s0, o + k * RECORD_BYTES);
+    } else {
+      return set_error(NVBT_EINVAL, "slot %llu: not a compact slot (flags 0x%x)", (unsigned long long)i, f);
+    }
+    ++k;
+  }
+  *n_out = k;
+  return NVBT_OK;
 }
 
 int nvbt_digest_records(const void* records, uint64_t n, nvbt_digest* out) {

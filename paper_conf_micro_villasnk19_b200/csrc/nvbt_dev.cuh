@@ -46,6 +46,8 @@ struct DevState {
   unsigned n_warps;
   unsigned stripes;                // site/mem/hist repeat `stripes` times, stride stripe_words
   unsigned long long stripe_words;
+  unsigned slot_bytes;             // 288, or 176 for compact channels (EM §5.1)
+  unsigned compact;
 };
 
 __device__ __forceinline__ unsigned lane_id() { unsigned l; asm("mov.u32 %0, %%laneid;" : "=r"(l)); return l; }
@@ -369,51 +371,111 @@ struct Hooks {
   }
 
   // a6 producer. One record per executed global-memory event: lane 0 takes a ticket; the warp writes
-  // the 32 addresses (8 B per lane, 256 B coalesced) and the header with a zero tag straight into the
+  // the record with ONE 16 B-per-lane store (header with a zero tag + addresses) straight into the
   // pinned host ring. Commits are batched: lane (k % 32) remembers the tag word of the warp's k-th
-  // uncommitted record, and commit() makes every pending payload visible system-wide (one fence per lane
+  // uncommitted slot, and commit() makes every pending payload visible system-wide (one fence per lane
   // per batch instead of one per record) before the tags are stored. A warp commits before it can block
   // on a full ring, so reserved-but-uncommitted slots never stall the consumer for ever.
-  template <int PC>
-  __device__ __forceinline__ void emit(unsigned A, unsigned P, bool act, unsigned long long addr) {
-    constexpr nvbt_instr_desc d = Prog::t[PC];
-    unsigned long long t = 0;
+  // Compact channels (st.compact, EM §5.1, F3) send base + 32-bit deltas in one 176 B slot, or two slots
+  // of 16 full addresses each when the warp's addresses span more than ±2 GB.
+  __device__ __forceinline__ bool reserve(unsigned k, unsigned long long& t) {
     int room = 1;
     if (lane == 0) {
-      t = atomicAdd(st.head, 1ull);
-      room = has_room(st, t);
+      t = atomicAdd(st.head, (unsigned long long)k);
+      room = has_room(st, t + k - 1);
     }
     t = __shfl_sync(FULL, t, 0);
     if (!__shfl_sync(FULL, room, 0)) {
       commit();
       int ok = 1;
-      if (lane == 0) ok = wait_room(st, t);
+      if (lane == 0) ok = wait_room(st, t + k - 1);
       if (!__shfl_sync(FULL, ok, 0)) {
         if (lane == 0) atomicAdd(st.dropped, 1ull);
-        ++seq;
-        return;
+        return false;
       }
     }
+    return true;
+  }
+
+  __device__ __forceinline__ unsigned char* slot_ptr(unsigned long long t, unsigned& tag) const {
     const unsigned long long lap = t / st.cap;
-    unsigned char* rec = st.ring + (t - lap * st.cap) * RECORD_BYTES;
-    // the whole 288 B record in ONE warp store: lane j < 18 writes bytes [16j, 16j + 16) — lanes 0, 1 the
-    // header (tag 0), lane j >= 2 the addresses of lanes 2(j-2), 2(j-2)+1 (gathered with shuffles)
-    const unsigned long long a = act ? addr : 0ull;
-    const unsigned src = 2u * (lane - 2u);
-    const unsigned long long a0 = __shfl_sync(FULL, a, src & 31u), a1 = __shfl_sync(FULL, a, (src + 1u) & 31u);
-    if (lane < 18) {
-      const unsigned w2 = (unsigned)d.opcode | ((unsigned)d.width << 16) | ((unsigned)d.kind << 24);
-      const uint4 v = lane == 0   ? make_uint4(st.launch, gwarp, seq, (unsigned)PC)
-                      : lane == 1 ? make_uint4(A, P, w2, 0u)
-                                  : make_uint4((unsigned)a0, (unsigned)(a0 >> 32), (unsigned)a1, (unsigned)(a1 >> 32));
-      *reinterpret_cast<uint4*>(rec + 16 * lane) = v;
-    }
+    tag = (unsigned)lap + 1u;
+    return st.ring + (t - lap * st.cap) * st.slot_bytes;
+  }
+
+  __device__ __forceinline__ void add_pending(unsigned char* rec, unsigned tag) {
     if (lane == npend) {
       pend_tag = rec + 28;
-      pend_val = (unsigned)lap + 1u;
+      pend_val = tag;
+    }
+    if (++npend == 32) commit();
+  }
+
+  template <int PC>
+  __device__ __forceinline__ void emit(unsigned A, unsigned P, bool act, unsigned long long addr) {
+    constexpr nvbt_instr_desc d = Prog::t[PC];
+    const unsigned w2 = (unsigned)d.opcode | ((unsigned)d.width << 16) | ((unsigned)d.kind << 24);
+    const unsigned long long a = act ? addr : 0ull;
+    unsigned long long t;
+    unsigned tag;
+    if (!st.compact) {
+      if (reserve(1, t)) {
+        unsigned char* rec = slot_ptr(t, tag);
+        // lane j < 18 writes bytes [16j, 16j + 16): lanes 0, 1 the header (tag 0), lane j >= 2 the
+        // addresses of lanes 2(j-2), 2(j-2)+1
+        const unsigned src = 2u * (lane - 2u);
+        const unsigned long long a0 = __shfl_sync(FULL, a, src & 31u), a1 = __shfl_sync(FULL, a, (src + 1u) & 31u);
+        if (lane < 18) {
+          const uint4 v = lane == 0   ? make_uint4(st.launch, gwarp, seq, (unsigned)PC)
+                          : lane == 1 ? make_uint4(A, P, w2, 0u)
+                                      : make_uint4((unsigned)a0, (unsigned)(a0 >> 32), (unsigned)a1, (unsigned)(a1 >> 32));
+          *reinterpret_cast<uint4*>(rec + 16 * lane) = v;
+        }
+        add_pending(rec, tag);
+      }
+      ++seq;
+      return;
+    }
+    const unsigned E = P;
+    const unsigned long long base = __shfl_sync(FULL, addr, __ffs(E) - 1);
+    const long long dl = (long long)(addr - base);
+    if (st.compact == 1u && __all_sync(FULL, !act || (dl >= -0x80000000ll && dl <= 0x7fffffffll))) {
+      if (reserve(1, t)) {
+        unsigned char* rec = slot_ptr(t, tag);
+        // 11 chunks: header, header (kind | 0x80), base, then 4 deltas per chunk (lanes 4(j-3) .. +3)
+        const unsigned dd = act ? (unsigned)dl : 0u;
+        const unsigned s0 = 4u * (lane - 3u);
+        const unsigned d0 = __shfl_sync(FULL, dd, s0 & 31u), d1 = __shfl_sync(FULL, dd, (s0 + 1u) & 31u);
+        const unsigned d2 = __shfl_sync(FULL, dd, (s0 + 2u) & 31u), d3 = __shfl_sync(FULL, dd, (s0 + 3u) & 31u);
+        if (lane < 11) {
+          const uint4 v = lane == 0   ? make_uint4(st.launch, gwarp, seq, (unsigned)PC)
+                          : lane == 1 ? make_uint4(A, P, w2 | 0x80000000u, 0u)
+                          : lane == 2 ? make_uint4((unsigned)base, (unsigned)(base >> 32), 0u, 0u)
+                                      : make_uint4(d0, d1, d2, d3);
+          *reinterpret_cast<uint4*>(rec + 16 * lane) = v;
+        }
+        add_pending(rec, tag);
+      }
+    } else if (reserve(2, t)) {
+      // wide pair: slot t = lanes 0-15, slot t+1 = lanes 16-31 (full addresses); lanes 0-9 write the
+      // first slot's 10 chunks, lanes 16-25 the second's
+      unsigned tag0, tag1;
+      unsigned char* r0 = slot_ptr(t, tag0);
+      unsigned char* r1 = slot_ptr(t + 1, tag1);
+      const unsigned h = lane >> 4, j = lane & 15u;
+      const unsigned src = 16u * h + 2u * (j - 2u);
+      const unsigned long long a0 = __shfl_sync(FULL, a, src & 31u), a1 = __shfl_sync(FULL, a, (src + 1u) & 31u);
+      if (j < 10) {
+        const unsigned flag = h ? 0x20000000u : 0x40000000u;
+        const uint4 v = j == 0   ? make_uint4(st.launch, gwarp, seq, (unsigned)PC)
+                        : j == 1 ? make_uint4(A, P, w2 | flag, 0u)
+                                 : make_uint4((unsigned)a0, (unsigned)(a0 >> 32), (unsigned)a1, (unsigned)(a1 >> 32));
+        *reinterpret_cast<uint4*>((h ? r1 : r0) + 16 * j) = v;
+      }
+      add_pending(r0, tag0);
+      add_pending(r1, tag1);
     }
     ++seq;
-    if (++npend == 32) commit();
   }
 
   __device__ __forceinline__ void commit() {

@@ -25,6 +25,7 @@ COUNT, OPHIST, BB, MEMDIV, PER_WARP, TRACE = 1, 2, 4, 8, 16, 32
 TOOL_NONE, TOOL_COUNT, TOOL_BBCOUNT, TOOL_MEMDIV, TOOL_TRACE = 0, 1, 2, 4, 8
 W_VECTORADD, W_SGEMM, W_BFS, W_STENCIL, W_REPLAY = 1, 2, 3, 4, 5
 RECORD_BYTES = 288
+COMPACT_RECORD_BYTES = 176
 
 
 class InstrDesc(C.Structure):
@@ -81,6 +82,7 @@ _sigs = {
     "nvbt_channel_close": ([_P], C.c_int),
     "nvbt_channel_dropped": ([_P, C.POINTER(C.c_uint64)], C.c_int),
     "nvbt_digest_records": ([_P, C.c_uint64, C.POINTER(Digest)], C.c_int),
+    "nvbt_decode_compact": ([_P, C.c_uint64, _P, C.c_uint64, C.POINTER(C.c_uint64)], C.c_int),
     "nvbt_gen_events": ([_P, C.c_uint64, C.c_uint64, C.c_uint64, _P, _P], C.c_int),
     "nvbt_replay": ([_P, _P, _P, C.c_uint64], C.c_int),
     "nvbt_replay_errors": ([_P, C.POINTER(C.c_uint64)], C.c_int),
@@ -156,6 +158,16 @@ def nvbt_workspace_size(prog_len, n_opcodes, n_bbs, flags, n_warps=0):
     b = C.c_size_t()
     _check(_lib.nvbt_workspace_size(C.byref(cfg), C.byref(b)))
     return b.value
+
+
+def nvbt_decode_compact(slots_u8):
+    """Decode a numpy uint8 [n, 176] array of compact transport slots into EM §5 records [m, 288]."""
+    sl = np.ascontiguousarray(slots_u8, dtype=np.uint8)
+    out = np.zeros((sl.shape[0], RECORD_BYTES), dtype=np.uint8)
+    k = C.c_uint64()
+    _check(_lib.nvbt_decode_compact(sl.ctypes.data_as(C.c_void_p), sl.shape[0], out.ctypes.data_as(C.c_void_p),
+                                    sl.shape[0], C.byref(k)))
+    return out[:k.value]
 
 
 def nvbt_digest_records(records_u8):
@@ -282,10 +294,12 @@ class Channel:
         self.handle, self.ctx, self.ring = handle, ctx, ring
 
 
-def nvbt_channel_open(ctx, ring):
-    """ring: pinned uint8 torch tensor (torch.empty(..., pin_memory=True))."""
+def nvbt_channel_open(ctx, ring, compact=False):
+    """ring: pinned uint8 torch tensor (torch.empty(..., pin_memory=True)); compact: 176 B transport slots
+    (base + 32-bit deltas, EM §5.1) instead of 288 B records."""
     h = C.c_void_p()
-    _check(_lib.nvbt_channel_open(ctx.handle, C.c_void_p(ring.data_ptr()), ring.numel(), RECORD_BYTES, C.byref(h)))
+    rb = COMPACT_RECORD_BYTES if compact else RECORD_BYTES
+    _check(_lib.nvbt_channel_open(ctx.handle, C.c_void_p(ring.data_ptr()), ring.numel(), rb, C.byref(h)))
     ch = Channel(h, ctx, ring)
     ctx.channel = ch
     return ch

@@ -73,3 +73,50 @@ def test_host_digest_matches_oracle():
     stencil.run(acc, 64, 1 << 32, (1 << 32) + (1 << 24))
     recs = acc.record_array()
     assert nb.nvbt_digest_records(recs) == (acc.digest.n, acc.digest.d1, acc.digest.d2)
+
+
+def _encode_compact(recs, wide_mask):
+    """Test-side encoder of EM §5.1 (written from the spec): record r -> one compact slot, or a wide pair
+    when wide_mask[r]."""
+    import struct
+    out = []
+    for r, rec in enumerate(recs):
+        b = bytes(rec)
+        A, P = struct.unpack_from("<II", b, 16)
+        E = A & P
+        addr = struct.unpack_from("<32Q", b, 32)
+        kind = b[27]
+        if not wide_mask[r]:
+            lanes = [l for l in range(32) if (E >> l) & 1]
+            base = addr[lanes[0]]
+            sl = bytearray(176)
+            sl[0:27] = b[0:27]
+            sl[27] = kind | 0x80
+            struct.pack_into("<Q", sl, 32, base)
+            for l in lanes:
+                struct.pack_into("<i", sl, 48 + 4 * l, addr[l] - base)
+            out.append(sl)
+        else:
+            for h, flag in ((0, 0x40), (1, 0x20)):
+                sl = bytearray(176)
+                sl[0:27] = b[0:27]
+                sl[27] = kind | flag
+                sl[32:160] = b[32 + 128 * h:160 + 128 * h]
+                out.append(sl)
+    return np.frombuffer(b"".join(out), dtype=np.uint8).reshape(-1, 176)
+
+
+def test_compact_decode_matches_records():
+    from paper_conf_micro_villasnk19_b200 import nvbt as nb
+    from oracle import events as ev, programs
+    from oracle.models import stencil
+    acc = ev.Accumulator(programs.stencil(), trace=True, keep_records=True)
+    stencil.run(acc, 64, 1 << 32, (1 << 32) + (1 << 24))
+    recs = acc.record_array()
+    wide = np.random.default_rng(0).random(len(recs)) < 0.3
+    slots = _encode_compact(recs, wide)
+    assert len(slots) == len(recs) + wide.sum()
+    dec = nb.nvbt_decode_compact(slots)
+    assert dec.shape == recs.shape and (dec == recs).all()
+    with pytest.raises(nb.NvbtError):          # an unpaired wide half is rejected
+        nb.nvbt_decode_compact(slots[(slots[:, 27] & 0xE0) == 0x20][:1])

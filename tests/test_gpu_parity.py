@@ -144,7 +144,7 @@ def test_bfs_parity(nvbt, scale, tools):
 
 
 # ---------------------------------------------------------------- C4 stencil + trace channel
-def _stencil_case(nvbt, n, iters, ring_records, tools_names=("TRACE", "MEMDIV", "COUNT")):
+def _stencil_case(nvbt, n, iters, ring_records, tools_names=("TRACE", "MEMDIV", "COUNT"), compact=False):
     import torch
     nb, dr = nvbt.nvbt, nvbt.drivers
     t = 0
@@ -153,8 +153,8 @@ def _stencil_case(nvbt, n, iters, ring_records, tools_names=("TRACE", "MEMDIV", 
     ctx = nb.nvbt_init(nb.W_STENCIL, nb.COUNT | nb.MEMDIV | nb.TRACE)
     x0 = cuda(uniform_f32((n, n), 4))
     buf0, buf1 = x0.clone(), torch.zeros_like(x0)
-    ring = torch.empty(64 + 288 * ring_records, dtype=torch.uint8, pin_memory=True)
-    ch = nb.nvbt_channel_open(ctx, ring)
+    ring = torch.empty(64 + (176 if compact else 288) * ring_records, dtype=torch.uint8, pin_memory=True)
+    ch = nb.nvbt_channel_open(ctx, ring, compact=compact)
     dr.run_stencil(ctx, t, buf0, buf1, n, iters)
     acc = ev.Accumulator(programs.stencil(), trace=True, keep_records=True)
     m_st.run_iterations(acc, n, buf0.data_ptr(), buf1.data_ptr(), iters)
@@ -183,6 +183,14 @@ def test_stencil_trace_parity(nvbt, n, iters):
 def test_channel_tiny_ring_backpressure(nvbt):
     """A 5-slot ring forces wrap-around and producer backpressure; nothing lost or duplicated."""
     _stencil_case(nvbt, 64, 2, ring_records=5, tools_names=("TRACE",))
+
+
+@pytest.mark.parametrize("force_wide,ring", [("0", 1 << 16), ("0", 5), ("1", 1 << 16), ("1", 7), ("1", 6)])
+def test_channel_compact_transport(nvbt, monkeypatch, force_wide, ring):
+    """F3 compact 176 B slots (EM §5.1): decoded records equal the oracle's; the forced wide form (two
+    slots per record) with odd and even tiny rings exercises pairs straddling the ring end."""
+    monkeypatch.setenv("NVBT_COMPACT_FORCE_WIDE", force_wide)
+    _stencil_case(nvbt, 64, 2, ring_records=ring, tools_names=("TRACE", "MEMDIV"), compact=True)
 
 
 def test_channel_digest_drain(nvbt):
