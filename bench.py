@@ -3,7 +3,8 @@
 
 Default workload (BASELINE.json configs[1]): C2 — naive row-fastest SGEMM 1024^3 with the full tool set
 compiled in (counts, opcode/BB histograms, per-instruction memory divergence), one step = one
-instrumented launch (+ the int64 all-reduce merge of the accumulators when N > 1). Other workloads
+instrumented launch; with N > 1 each rank runs its own instance and the counters are merged once by an
+int64 all-reduce after the timed steps. Other workloads
 (`--workload c1|c3|c4|c5`) are for profiling; the driver's bench line is C2.
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--workload c2] [--impl ours|reference]
@@ -103,12 +104,14 @@ def dist_setup(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if os.environ.get("NVBT_BENCH_SAME_GPU"):   # test hook: all ranks on GPU 0 (with a gloo backend)
+        local = 0
     if args.impl == "ours":
         torch.cuda.set_device(local)
     if world > 1:
         import torch.distributed as dist
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
-        backend = "nccl" if args.impl == "ours" else "gloo"
+        backend = os.environ.get("NVBT_BENCH_BACKEND", "nccl" if args.impl == "ours" else "gloo")
         kw = {"device_id": torch.device("cuda", local)} if backend == "nccl" else {}
         dist.init_process_group(backend, **kw)
     return rank, world, local
@@ -273,15 +276,13 @@ def run_ours(args):
     wl = SgemmBench(torch, nb, dr, world)
     launches0 = nb.nvbt_launch_count(wl.ctx)
 
-    def timed(fn, n, merge=False):
+    def timed(fn, n):
         ts = []
         for _ in range(n):
             flush.zero_()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record()
             fn()
-            if merge and world > 1:
-                dr.merge(wl.ctx)
             e1.record()
             e1.synchronize()
             ts.append(e0.elapsed_time(e1) / 1e3)
@@ -298,10 +299,19 @@ def run_ours(args):
     with ClockSampler(local) as clk:
         barrier(world)
         torch.cuda.synchronize()
-        t_instr = timed(wl.instr, args.steps, merge=True)
+        t_instr = timed(wl.instr, args.steps)
         torch.cuda.synchronize()
         barrier(world)
     gpu_launches = nb.nvbt_launch_count(wl.ctx) - l0
+    # a8 merge: the per-GPU accumulators are summed once, by one int64 all-reduce (EM §4)
+    merge_ms = 0.0
+    if world > 1:
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        dr.merge(wl.ctx)
+        e1.record()
+        e1.synchronize()
+        merge_ms = e0.elapsed_time(e1)
     # result check of the timed steps: exactly K x the per-launch closed form (I-3)
     cnt = nb.nvbt_count(wl.ctx)
     expect = wl.events * args.steps * (world if world > 1 else 1)
@@ -330,12 +340,13 @@ def run_ours(args):
         "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
         "config": {"workload": wl.desc, "M": wl.M, "N": wl.N, "K": wl.K, "warp_events_per_launch": wl.events,
                    "tools": "BBCOUNT|MEMDIV", "l2": "flushed between steps (256 MiB write)",
-                   "parallelism": f"replicas x{world} + int64 all-reduce merge per step" if world > 1 else "1 GPU"},
+                   "parallelism": f"replicas x{world}, one int64 all-reduce merge of the counters" if world > 1 else "1 GPU"},
         "slowdown": slowdown, "plain_ms_per_launch": 1e3 * statistics.median(t_plain),
         "instr_ms_per_launch": 1e3 * t_kernel, "counts_check": "ok" if ok else f"mismatch {int(cnt[2])} != {expect}",
         "roofline": wl.roofline(t_kernel, peaks),
         "e2e": {"value": e2e_value, "unit": "events/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h},
         "gpu_launches": int(gpu_launches), "clocks": clk.summary(), "peaks_source": peaks_src,
+        "merge_ms": merge_ms,
     }
     line["roofline"]["peak_source"] = f"148 SMs x 4 issue/clk x sm_max_mhz ({peaks_src})"
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
