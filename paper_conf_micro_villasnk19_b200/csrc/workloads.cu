@@ -43,7 +43,7 @@ __global__ void __launch_bounds__(256) k_vectoradd(const float* __restrict__ a, 
 
 // ---------------------------------------------------------------- C2 naive SGEMM (§3.2)
 template <uint32_t T>
-__global__ void __launch_bounds__(256) k_sgemm(const float* __restrict__ A, const float* __restrict__ B,
+__global__ void __launch_bounds__(256, 6) k_sgemm(const float* __restrict__ A, const float* __restrict__ B,
                                                float* __restrict__ C, int M, int N, int K, DevState st) {
   __shared__ __align__(16) unsigned sb[Hooks<T, ProgSgemm>::kSmemWords];
   Hooks<T, ProgSgemm> h(st, sb);
