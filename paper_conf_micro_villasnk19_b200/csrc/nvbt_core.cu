@@ -57,15 +57,24 @@ Layout make_layout(uint32_t P, uint32_t O, uint32_t B, uint32_t W, uint32_t flag
 // ---------------------------------------------------------------------------------------------------
 // Fold kernel: per-pc bins (per-instruction mode + BB mode derived per EM §2 item 3) -> reported
 // counts, opcode histogram, BB statistics and divergence totals. Integer sums only.
+__device__ __forceinline__ unsigned long long warp_sum_u64(unsigned long long v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+
+// One warp per pc; lane s sums stripes s, s+32, ... of the CTA-striped bins.
 __global__ void fold_kernel(const nvbt_instr_desc* __restrict__ prog, const uint32_t* __restrict__ leader,
                             uint32_t P, uint32_t O, uint32_t B, const unsigned long long* __restrict__ accum,
                             unsigned long long* out, Layout L) {
   const size_t SW = L.stripe_words;
-  for (uint32_t pc = blockIdx.x * blockDim.x + threadIdx.x; pc < P; pc += gridDim.x * blockDim.x) {
+  const unsigned lane = threadIdx.x & 31u;
+  const uint32_t warps = (gridDim.x * blockDim.x) >> 5;
+  for (uint32_t pc = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; pc < P; pc += warps) {
     const nvbt_instr_desc d = prog[pc];
     const uint32_t l = leader[d.bb];
     unsigned long long tI = 0, tE = 0, wI = 0, wE = 0, n = 0, sS = 0, sL = 0;
-    for (size_t s = 0; s < L.stripes; ++s) {
+    for (size_t s = lane; s < L.stripes; s += 32) {
       const unsigned long long* site = accum + s * SW + L.site;
       const unsigned long long* bbsite = accum + s * SW + L.bbsite;
       const unsigned long long* mem = accum + s * SW + L.mem;
@@ -77,25 +86,29 @@ __global__ void fold_kernel(const nvbt_instr_desc* __restrict__ prog, const uint
       }
       n += mem[3 * pc]; sS += mem[3 * pc + 1]; sL += mem[3 * pc + 2];
     }
-    if (tI | wI) {
-      atomicAdd(out + L.o_counts + 0, tI);
-      atomicAdd(out + L.o_counts + 1, tE);
-      atomicAdd(out + L.o_counts + 2, wI);
-      atomicAdd(out + L.o_counts + 3, wE);
-      atomicAdd(out + L.o_ht + d.opcode, tE);
-      atomicAdd(out + L.o_hw + d.opcode, wE);
-      unsigned long long* bb = out + L.o_bb + 4ull * d.bb;
-      if (d.is_leader) { atomicAdd(bb + 0, wI); atomicAdd(bb + 1, tI); }
-      atomicAdd(bb + 2, wE);
-      atomicAdd(bb + 3, tE);
-    }
-    out[L.o_mem + 3 * pc] = n;
-    out[L.o_mem + 3 * pc + 1] = sS;
-    out[L.o_mem + 3 * pc + 2] = sL;
-    if (n) {
-      atomicAdd(out + L.o_memtot, n);
-      atomicAdd(out + L.o_memtot + 1, sS);
-      atomicAdd(out + L.o_memtot + 2, sL);
+    tI = warp_sum_u64(tI); tE = warp_sum_u64(tE); wI = warp_sum_u64(wI); wE = warp_sum_u64(wE);
+    n = warp_sum_u64(n); sS = warp_sum_u64(sS); sL = warp_sum_u64(sL);
+    if (lane == 0) {
+      if (tI | wI) {
+        atomicAdd(out + L.o_counts + 0, tI);
+        atomicAdd(out + L.o_counts + 1, tE);
+        atomicAdd(out + L.o_counts + 2, wI);
+        atomicAdd(out + L.o_counts + 3, wE);
+        atomicAdd(out + L.o_ht + d.opcode, tE);
+        atomicAdd(out + L.o_hw + d.opcode, wE);
+        unsigned long long* bb = out + L.o_bb + 4ull * d.bb;
+        if (d.is_leader) { atomicAdd(bb + 0, wI); atomicAdd(bb + 1, tI); }
+        atomicAdd(bb + 2, wE);
+        atomicAdd(bb + 3, tE);
+      }
+      out[L.o_mem + 3 * pc] = n;
+      out[L.o_mem + 3 * pc + 1] = sS;
+      out[L.o_mem + 3 * pc + 2] = sL;
+      if (n) {
+        atomicAdd(out + L.o_memtot, n);
+        atomicAdd(out + L.o_memtot + 1, sS);
+        atomicAdd(out + L.o_memtot + 2, sL);
+      }
     }
   }
   const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
@@ -110,7 +123,7 @@ int fold(nvbt_ctx c) {
   NVBT_CUDA(cudaSetDevice(c->device));
   NVBT_CUDA(cudaMemsetAsync(c->out, 0, c->lay.out_words * 8, c->stream));
   const int threads = 256;
-  const int blocks = (int)((c->n_pcs + threads - 1) / threads);
+  const int blocks = (int)std::min<uint32_t>((c->n_pcs + 7) / 8, 1184);   // 8 warps (pcs) per block
   fold_kernel<<<blocks, threads, 0, c->stream>>>(c->d_prog, c->d_leader, c->n_pcs, c->n_ops, c->n_bbs, c->accum,
                                                   c->out, c->lay);
   NVBT_CUDA(cudaGetLastError());
