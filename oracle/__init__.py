@@ -20,6 +20,8 @@ Modules and their pins (tests/test_oracle_*.py):
                                            partition invariance
   trace        §5 records + digests        pinned: record field layout by hand-built record,
                                            order independence, single-bit sensitivity
+               footprint (F2)              pinned: Python-set brute force on random records, vectorAdd
+                                           closed form 3*ceil(4N/32) sectors / 3*ceil(4N/128) lines
 Parity unpinned: none of the above; the paper's Figs 5–9 values, the 74–96 % library share
 and WFFT32's 21 vs 150 instructions/warp need the paper's workloads and are not modelled.
 """

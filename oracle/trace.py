@@ -71,3 +71,21 @@ def sort_records(recs_u8):
     r = np.ascontiguousarray(recs_u8).view(RECORD_DTYPE).reshape(-1)
     order = np.lexsort((r["seq"], r["warp"], r["launch"]))
     return np.ascontiguousarray(recs_u8)[order]
+
+
+def footprint(recs_u8, n_launches):
+    """F2 on-GPU consumer (P:L187 (§6.1): records "can be analyzed directly on the GPU"): per launch l,
+    [distinct 32 B sectors, distinct 128 B lines, records] over the addresses of the lanes of E = A & P
+    of every record of launch l — the memory footprint of the launch (reading R-18). Plain definition:
+    numpy.unique of the address >> 5 / >> 7 per launch."""
+    out = np.zeros((n_launches, 3), dtype=np.int64)
+    r = np.ascontiguousarray(recs_u8).view(RECORD_DTYPE).reshape(-1)
+    for l in range(n_launches):
+        rl = r[r["launch"] == l]
+        E = (rl["A"] & rl["P"]).astype(np.uint64)
+        act = ((E[:, None] >> np.arange(32, dtype=np.uint64)[None, :]) & np.uint64(1)) == 1
+        a = rl["addr"][act]
+        out[l, 0] = len(np.unique(a >> np.uint64(5)))
+        out[l, 1] = len(np.unique(a >> np.uint64(7)))
+        out[l, 2] = len(rl)
+    return out

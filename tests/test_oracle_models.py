@@ -237,3 +237,37 @@ def test_digest_order_independent_and_sensitive():
     r = recs.view(trace.RECORD_DTYPE).reshape(-1)
     w0 = r[r["warp"] == 300]
     assert sorted(w0["seq"].tolist()) == list(range(len(w0)))
+
+
+def test_footprint_brute_force():
+    """F2 footprint vs Python sets over random records (two launches, random masks, clustered addresses)."""
+    rng = np.random.default_rng(11)
+    n = 300
+    rec = np.zeros(n, dtype=trace.RECORD_DTYPE)
+    rec["launch"] = rng.integers(0, 3, n)
+    rec["A"] = rng.integers(0, 1 << 32, n, dtype=np.uint64).astype(np.uint32)
+    rec["P"] = rng.integers(0, 1 << 32, n, dtype=np.uint64).astype(np.uint32)
+    rec["addr"] = (0x7f0000000000 + rng.integers(0, 1 << 14, (n, 32))).astype(np.uint64)
+    got = trace.footprint(rec.view(np.uint8).reshape(n, -1), 4)
+    for l in range(4):
+        secs, lines, cnt = set(), set(), 0
+        for r in rec:
+            if int(r["launch"]) != l:
+                continue
+            cnt += 1
+            e = int(r["A"]) & int(r["P"])
+            for lane in range(32):
+                if (e >> lane) & 1:
+                    secs.add(int(r["addr"][lane]) // 32)
+                    lines.add(int(r["addr"][lane]) // 128)
+        assert list(got[l]) == [len(secs), len(lines), cnt]
+
+
+@pytest.mark.parametrize("N", [1, 31, 1000, 4097])
+def test_footprint_vectoradd_closed_form(N):
+    """vectorAdd touches three disjoint 128 B-aligned arrays of 4N bytes: 3*ceil(4N/32) sectors and
+    3*ceil(4N/128) lines in its single launch."""
+    acc = ev.Accumulator(programs.vectoradd(), trace=True, keep_records=True)
+    vectoradd.run(acc, N, 0x100000, 0x200000, 0x300000)
+    fp = trace.footprint(acc.record_array(), 1)
+    assert list(fp[0][:2]) == [3 * -(-4 * N // 32), 3 * -(-4 * N // 128)]
