@@ -267,8 +267,9 @@ def run_ours(args):
 
     if args.workload == "c5":
         return run_replay(args, torch, nb, dr, rank, world, local, peaks, peaks_src)
-    if args.workload in ("c1", "c3", "c4", "f1"):
-        line = {"c1": run_c1, "c3": run_c3, "c4": run_c4, "f1": run_f1}[args.workload](args, torch, nb, dr, local)
+    if args.workload in ("c1", "c3", "c4", "f1", "f2"):
+        line = {"c1": run_c1, "c3": run_c3, "c4": run_c4, "f1": run_f1, "f2": run_f2}[args.workload](
+            args, torch, nb, dr, local)
         if rank == 0:
             print(json.dumps(line), flush=True)
         return
@@ -525,6 +526,71 @@ def run_c4(args, torch, nb, dr, local):
             "clocks": clk.summary()}
 
 
+def run_f2(args, torch, nb, dr, local):
+    """F2: C4's traced stencil (8192^2, --f2-iters iterations) with the trace kept in an HBM ring and
+    analysed on the GPU (per-launch footprint) instead of drained to the host. A step = traced run
+    + consumer kernel; the ring is re-zeroed between steps outside the timed region."""
+    from synth import uniform_f32
+    peaks, peaks_src = load_peaks()
+    n, iters = args.stencil_n, args.f2_iters
+    G = n // 32
+    per_iter = 2 * (n * n // 32) + 4 * (n - 2) * G
+    cap = per_iter * iters
+    ctx = nb.nvbt_init(nb.W_STENCIL, nb.COUNT | nb.TRACE)
+    x0 = torch.from_numpy(uniform_f32((n, n), 4)).cuda()
+    buf0, buf1 = x0.clone(), torch.empty_like(x0)
+    slack = torch.cuda.get_device_properties(0).multi_processor_count * 1024   # last chunk per SM
+    ring = torch.empty(64 + 288 * (cap + slack), dtype=torch.uint8, device="cuda")
+    regions = iters * 2 * (-(-n * n * 4 // (1 << 20)) + 1)          # (launch, 1 MB region) pairs
+    slots = 1 << (2 * regions - 1).bit_length()
+    scratch = torch.empty(513 * slots + 3 * iters + 1, dtype=torch.int64, device="cuda")
+    for _ in range(args.warmup):
+        dr.run_stencil(ctx, nb.TOOL_NONE, buf0, buf1, n, iters)
+    tp = _timed_events(torch, lambda: dr.run_stencil(ctx, nb.TOOL_NONE, buf0, buf1, n, iters), args.steps)
+    res, kern, fp = [], [], None
+    l0 = nb.nvbt_launch_count(ctx)
+    with ClockSampler(local) as clk:
+        for step in range(args.warmup + args.steps):
+            ch = nb.nvbt_channel_open(ctx, ring)
+            nb.nvbt_reset(ctx)                               # launch ids restart at 0
+            torch.cuda.synchronize()
+            e0, e1, e2 = (torch.cuda.Event(enable_timing=True) for _ in range(3))
+            e0.record()
+            dr.run_stencil(ctx, nb.TOOL_TRACE, buf0, buf1, n, iters)
+            e1.record()
+            tk = []
+            fp = nb.nvbt_trace_footprint(ch, iters, table_slots=slots, scratch=scratch, timing=tk)
+            e2.record()
+            e2.synchronize()
+            dropped = nb.nvbt_channel_dropped(ch)
+            nb.nvbt_channel_close(ch)
+            if step >= args.warmup:
+                res.append((e0.elapsed_time(e1) / 1e3, e1.elapsed_time(e2) / 1e3))
+                kern.append(tk[0])
+    launches = nb.nvbt_launch_count(ctx) - l0
+    recs = int(fp[:, 2].sum())
+    t_tr = sum(r[0] for r in res) / len(res)
+    t_fp = sum(r[1] for r in res) / len(res)
+    t_k = sum(kern) / len(kern)
+    ach = recs * 288 / t_k / 1e9
+    exp_s, exp_l = 2 * n * n * 4 // 32, 2 * n * n * 4 // 128    # in + out grids, whole sectors / lines
+    return {"metric": "traced warp-level memory events analysed on GPU per second (F2)",
+            "value": recs / (t_tr + t_fp), "unit": "records/s", "n_gpus": 1, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": 1e3 * (t_tr + t_fp), "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+            "config": {"workload": f"F2 stencil {n}^2 x {iters}, tools TRACE, HBM ring + GPU footprint consumer",
+                       "ring_GB": ring.numel() / 1e9, "table_slots": slots,
+                       "l2": "records (36 GB) larger than L2"},
+            "records_per_run": recs, "records_expected": cap, "dropped": dropped,
+            "trace_ms": 1e3 * t_tr, "consumer_ms": 1e3 * t_fp, "consumer_kernel_ms": 1e3 * t_k,
+            "plain_ms": 1e3 * sum(tp) / len(tp), "slowdown_trace_only": t_tr / (sum(tp) / len(tp)),
+            "footprint_launch0": [int(x) for x in fp[0]], "footprint_expected": [exp_s, exp_l],
+            "roofline": {"bound": "hbm", "achieved": ach, "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                         "frac": ach / peaks["hbm_gbs"], "peak_source": peaks_src, "kernel": "k_footprint",
+                         "algorithmic_bytes_per_launch": recs * 288, "traffic": None},
+            "gpu_launches": int(launches) // (args.warmup + args.steps), "clocks": clk.summary()}
+
+
 def run_f1(args, torch, nb, dr, local):
     """F1 kernel sampling on C4's stencil (8192^2 x 100, BBCOUNT|MEMDIV): plain vs every launch
     instrumented vs one instrumented launch per grid shape."""
@@ -614,7 +680,8 @@ def main():
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--workload", choices=["c1", "c2", "c3", "c4", "c5", "f1"], default="c2")
+    ap.add_argument("--workload", choices=["c1", "c2", "c3", "c4", "c5", "f1", "f2"], default="c2")
+    ap.add_argument("--f2-iters", type=int, default=10, help="F2: stencil iterations kept in the HBM ring")
     ap.add_argument("--bfs-scale", type=int, default=20)
     ap.add_argument("--stencil-n", type=int, default=8192)
     ap.add_argument("--stencil-iters", type=int, default=100)

@@ -142,6 +142,22 @@ typedef int (*nvbt_drain_fn)(const void* records, uint64_t n_records, void* user
 int nvbt_channel_drain(nvbt_channel ch, nvbt_drain_fn fn, void* user, int64_t timeout_us,
                        uint64_t* n_drained);
 int nvbt_channel_close(nvbt_channel ch);
+/* F2, on-GPU consumer ("can be analyzed directly on the GPU", P:L187 (§6.1)). A channel whose ring is
+ * DEVICE memory (288 B records) is filled by the producers without backpressure: each SM takes slots
+ * from its own 1024-slot chunk of the ring (so the last chunk of every SM may stay partly empty: size the
+ * ring for the records + 1024 x SMs slots); records that find no chunk are dropped and counted. The ring
+ * is analysed in place: per launch id first_launch + l, l < n_launches,
+ *   out[3l + 0] = distinct 32 B sectors, out[3l + 1] = distinct 128 B lines over the lanes of E of all
+ *   records of that launch (the launch's footprint, reading R-18), out[3l + 2] = records.
+ * d_scratch: caller device memory of 4104 * table_slots + 8 * (3 * n_launches + 1) bytes, 16 B aligned
+ * (an 8 B key and a 4 KB sector bitmap per slot); table_slots (a power of two) must exceed the number of
+ * distinct (launch, 1 MB address region) pairs, ideally by 2x. n_launches <= 65536. EINVAL if a record's
+ * launch id is outside the range or an address >= 2^48, or the table overflows (never hangs).
+ * kernel_ms (nullable) = device time of the consumer kernels. Synchronises the context's stream.
+ * Channels on pinned host memory return NVBT_ESTATE here; device channels return it from drain. */
+int nvbt_trace_footprint(nvbt_channel ch, void* d_scratch, uint64_t table_slots, uint32_t first_launch,
+                         uint32_t n_launches, uint64_t* out, float* kernel_ms);
+
 /* Records the producers dropped after waiting ~2 s on a full ring (0 in a healthy run). */
 int nvbt_channel_dropped(nvbt_channel ch, uint64_t* dropped);
 

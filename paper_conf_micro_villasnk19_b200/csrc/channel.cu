@@ -29,6 +29,8 @@ struct nvbt_chan_s {
   uint64_t consumed = 0;
   unsigned slot = 288;                 // bytes per ring slot (288 full, 176 compact)
   bool force_wide = false;
+  bool on_device = false;              // F2: ring in device memory, consumed by GPU kernels
+  unsigned rstripes = 0;               // device ring: per-SM chunk stripes (see DevState)
   bool open = false;
   bool have_half = false;              // compact: first half of a wide pair seen at the ring end
   unsigned char half[176];
@@ -47,6 +49,9 @@ void channel_state(nvbt_chan_s* ch, DevState* st) {
   st->slot_bytes = ch->slot;
   // compact = 1; 2 forces the wide form for every record (NVBT_COMPACT_FORCE_WIDE=1, tests only)
   st->compact = ch->slot == COMPACT_BYTES ? (ch->force_wide ? 2u : 1u) : 0u;
+  st->no_wait = ch->on_device ? 1u : 0u;   // nobody frees device-ring slots: drop instead of waiting
+  st->rheads = ch->on_device ? ch->ctx->ctl + CTL_RHEAD : nullptr;
+  st->rstripes = ch->rstripes;
 }
 bool channel_open(nvbt_chan_s* ch) { return ch && ch->open; }
 
@@ -289,24 +294,241 @@ int nvbt_channel_open(nvbt_ctx c, void* ring, size_t bytes, uint32_t record_byte
   NVBT_CUDA(cudaSetDevice(c->device));
   cudaPointerAttributes pa{};
   NVBT_CUDA(cudaPointerGetAttributes(&pa, ring));
-  if (pa.type != cudaMemoryTypeHost || pa.devicePointer == nullptr)
-    return set_error(NVBT_EINVAL, "ring is not pinned, device-mapped host memory");
+  const bool on_device = pa.type == cudaMemoryTypeDevice;
+  if (!on_device && (pa.type != cudaMemoryTypeHost || pa.devicePointer == nullptr))
+    return set_error(NVBT_EINVAL, "ring is neither pinned device-mapped host memory nor device memory");
+  if (on_device && record_bytes != RECORD_BYTES)
+    return set_error(NVBT_EINVAL, "device-memory channels use 288 B records");
   auto* ch = new (std::nothrow) nvbt_chan_s();
   if (!ch) return set_error(NVBT_ENOMEM, "host allocation failed");
   ch->ctx = c;
-  ch->host = static_cast<unsigned char*>(ring);
-  ch->dev = static_cast<unsigned char*>(pa.devicePointer);
-  ch->slots = ch->host + HDR;
+  ch->on_device = on_device;
+  ch->host = on_device ? nullptr : static_cast<unsigned char*>(ring);
+  ch->dev = static_cast<unsigned char*>(on_device ? ring : pa.devicePointer);
+  ch->slots = on_device ? nullptr : ch->host + HDR;
   ch->slot = record_bytes;
   { const char* e = getenv("NVBT_COMPACT_FORCE_WIDE"); ch->force_wide = e && atoi(e) != 0; }
   ch->cap = (bytes - HDR) / record_bytes;
-  std::memset(ch->host, 0, HDR + ch->cap * record_bytes);
-  cudaError_t e = cudaMemsetAsync(c->ctl + CTL_HEAD, 0, 3 * 8, c->stream);  // head, tail_cache, dropped
+  if (on_device) {
+    int sms = 148;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, c->device);
+    ch->rstripes = std::min<unsigned>((unsigned)sms, kMaxRingStripes);
+  }
+  cudaError_t e = cudaSuccess;
+  if (on_device) e = cudaMemsetAsync(ring, 0, HDR + ch->cap * record_bytes, c->stream);
+  else std::memset(ch->host, 0, HDR + ch->cap * record_bytes);
+  if (on_device && e == cudaSuccess) {   // every stripe starts without a chunk; chunk counter 0
+    std::vector<unsigned long long> w(ch->rstripes + 1, ((unsigned long long)kRingNoChunk << 32) | kRingChunk);
+    w.back() = 0;
+    e = cudaMemcpyAsync(c->ctl + CTL_RHEAD, w.data(), w.size() * 8, cudaMemcpyHostToDevice, c->stream);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(c->stream);   // w is a host temporary
+  }
+  if (e == cudaSuccess) e = cudaMemsetAsync(c->ctl + CTL_HEAD, 0, 3 * 8, c->stream);  // head, tail_cache, dropped
   if (e == cudaSuccess) e = cudaStreamSynchronize(c->stream);
   if (e != cudaSuccess) { delete ch; return set_error(NVBT_ECUDA, "channel reset: %s", cudaGetErrorString(e)); }
   ch->open = true;
   c->chan = ch;
   *out = ch;
+  return NVBT_OK;
+}
+
+// ---- F2: on-GPU consumer of a device-memory channel ---------------------------------------------
+// Footprint of the recorded accesses per launch: distinct 32 B sectors and 128 B lines over the lanes of
+// E. The set is a sparse bitmap: an open-addressing table of 1 MB regions keyed (launch, addr >> 20),
+// each owning a 4 KB block of 4 sector bits per line (8192 lines). The blocks cost 1/256 of the address
+// span a launch touches and stay L2-resident, so the kernel streams the records from HBM once.
+namespace nvbt {
+constexpr int kFpBatch = 4;                  // records in flight per warp (memory-level parallelism)
+constexpr unsigned long long kFpEmpty = ~0ull;
+constexpr int kFpRegionShift = 20;           // 1 MB regions
+constexpr unsigned kFpWords = (1u << (kFpRegionShift - 7)) / 8;   // 32-bit words per block (8 lines each)
+
+__device__ __forceinline__ unsigned nib_nonzero(unsigned x) { return (x | x >> 1 | x >> 2 | x >> 3) & 0x11111111u; }
+
+// Table slot of region key k (warp-uniform call: every lane probes the same addresses). Two-entry cache
+// (c0 most recent). Returns false if the table is full.
+__device__ __forceinline__ bool fp_slot(unsigned long long k, unsigned long long* __restrict__ keys,
+                                        unsigned long long mask, unsigned long long (&ck)[2],
+                                        unsigned long long (&cs)[2], unsigned long long& slot) {
+  if (k == ck[0]) { slot = cs[0]; return true; }
+  if (k == ck[1]) {
+    slot = cs[1];
+    ck[1] = ck[0]; cs[1] = cs[0]; ck[0] = k; cs[0] = slot;
+    return true;
+  }
+  unsigned long long h = ((k * 0x9E3779B97F4A7C15ull) >> 24) & mask;
+  for (unsigned long long probes = 0; probes <= mask; ++probes) {   // bounded: a full table is an error
+    // lane 0 reads and claims; the warp follows its view (lanes reading on their own could disagree
+    // while another warp inserts)
+    unsigned long long v = 0;
+    if (lane_id() == 0) {
+      v = *reinterpret_cast<volatile unsigned long long*>(keys + h);
+      if (v == kFpEmpty) v = atomicCAS(keys + h, kFpEmpty, k);
+    }
+    v = __shfl_sync(0xffffffffu, v, 0);
+    if (v == kFpEmpty || v == k) {
+      ck[1] = ck[0]; cs[1] = cs[0]; ck[0] = k; cs[0] = h;
+      slot = h;
+      return true;
+    }
+    h = (h + 1) & mask;
+  }
+  return false;
+}
+
+// One record (warp-uniform control flow): for each distinct (region, word) among the lanes of E, OR
+// the lanes' sector bits into the region's block with one fire-and-forget reduction; distinct counts come
+// from k_fp_count afterwards.
+__device__ __forceinline__ void fp_record(unsigned launch, unsigned E, unsigned long long a, unsigned lane,
+                                          unsigned long long* __restrict__ keys, unsigned* __restrict__ pool,
+                                          unsigned long long mask, unsigned long long* err,
+                                          unsigned long long (&ck)[2], unsigned long long (&cs)[2]) {
+  bool on = (E >> lane) & 1u;
+  if (on && (a >> 48)) { atomicAdd(err, 1ull); on = false; }
+  const unsigned long long rkey = ((unsigned long long)launch << (48 - kFpRegionShift)) | (a >> kFpRegionShift);
+  const unsigned line = (unsigned)(a >> 7) & (8 * kFpWords - 1);
+  const unsigned word = line >> 3;
+  const unsigned bits = 1u << ((line & 7) * 4 + ((unsigned)(a >> 5) & 3));
+  unsigned pend = __ballot_sync(0xffffffffu, on);
+  while (pend) {
+    const unsigned f = __ffs(pend) - 1;
+    const unsigned long long k = __shfl_sync(0xffffffffu, rkey, f);
+    const unsigned wd = __shfl_sync(0xffffffffu, word, f);
+    const bool mine = on && rkey == k && word == wd;
+    const unsigned m = __ballot_sync(0xffffffffu, mine);
+    const unsigned v = __reduce_or_sync(0xffffffffu, mine ? bits : 0u);
+    pend &= ~m;
+    on = on && !mine;
+    unsigned long long slot;
+    if (!fp_slot(k, keys, mask, ck, cs, slot)) { if (lane == f) atomicAdd(err, 1ull); continue; }
+    if (lane == f) atomicOr(pool + slot * kFpWords + wd, v);
+  }
+}
+
+// Distinct counts per launch from the region blocks: sectors = set bits, lines = non-zero nibbles.
+// One warp per table slot; per-CTA shared bins when n_launches is small.
+__global__ void __launch_bounds__(256) k_fp_count(const unsigned long long* __restrict__ keys,
+                                                   const unsigned* __restrict__ pool, unsigned long long slots,
+                                                   unsigned long long* __restrict__ counts, unsigned n_launches) {
+  constexpr unsigned kBins = 1024;
+  __shared__ unsigned long long bins[2 * kBins];
+  const bool shared = n_launches <= kBins;
+  if (shared)
+    for (unsigned i = threadIdx.x; i < 2 * n_launches; i += blockDim.x) bins[i] = 0;
+  __syncthreads();
+  const unsigned lane = lane_id();
+  const unsigned long long warps = (unsigned long long)gridDim.x * (blockDim.x >> 5);
+  for (unsigned long long sl = (blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x) >> 5; sl < slots; sl += warps) {
+    const unsigned long long k = keys[sl];
+    if (k == kFpEmpty) continue;
+    unsigned ns = 0, nl = 0;
+    const uint4* blk = reinterpret_cast<const uint4*>(pool + sl * kFpWords);
+    for (unsigned i = lane; i < kFpWords / 4; i += 32) {
+      const uint4 v = blk[i];
+      ns += __popc(v.x) + __popc(v.y) + __popc(v.z) + __popc(v.w);
+      nl += __popc(nib_nonzero(v.x)) + __popc(nib_nonzero(v.y)) + __popc(nib_nonzero(v.z)) + __popc(nib_nonzero(v.w));
+    }
+    ns = __reduce_add_sync(0xffffffffu, ns);
+    nl = __reduce_add_sync(0xffffffffu, nl);
+    if (lane == 0) {
+      const unsigned l = (unsigned)(k >> (48 - kFpRegionShift));
+      if (shared) { atomicAdd(bins + 2 * l, (unsigned long long)ns); atomicAdd(bins + 2 * l + 1, (unsigned long long)nl); }
+      else { atomicAdd(counts + 3ull * l, (unsigned long long)ns); atomicAdd(counts + 3ull * l + 1, (unsigned long long)nl); }
+    }
+  }
+  if (shared) {
+    __syncthreads();
+    for (unsigned i = threadIdx.x; i < 2 * n_launches; i += blockDim.x)
+      if (bins[i]) atomicAdd(counts + 3ull * (i >> 1) + (i & 1), bins[i]);
+  }
+}
+
+// Committed slots lie in the chunks handed out so far, [0, min(chunks * kRingChunk, cap)); slots never
+// written (the unused tail of each SM's last chunk) have tag 0 and are skipped.
+__global__ void __launch_bounds__(256) k_footprint(const unsigned char* __restrict__ ring,
+                                                    const unsigned long long* __restrict__ chunks,
+                                                    unsigned long long cap,
+                                                    unsigned long long* __restrict__ keys, unsigned* __restrict__ pool,
+                                                    unsigned long long mask, unsigned long long* __restrict__ counts,
+                                                    unsigned first, unsigned n_launches) {
+  const unsigned lane = lane_id();
+  const unsigned long long n_slots = *chunks * kRingChunk < cap ? *chunks * kRingChunk : cap;
+  const unsigned long long warps = (unsigned long long)gridDim.x * (blockDim.x >> 5);
+  const unsigned long long w = (blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x) >> 5;
+  // contiguous chunk per warp: launch ids change rarely, so the per-launch record counts stay in registers
+  const unsigned long long per = (n_slots + warps - 1) / warps;
+  const unsigned long long r0 = w * per, r1 = r0 + per < n_slots ? r0 + per : n_slots;
+  unsigned long long* err = counts + 3ull * n_launches;
+  unsigned cur = 0xFFFFFFFFu;
+  unsigned long long nrec = 0;
+  unsigned long long ck[2] = {kFpEmpty, kFpEmpty}, cs[2] = {0, 0};
+  for (unsigned long long r = r0; r < r1; r += kFpBatch) {
+    uint4 h1[kFpBatch];
+    unsigned lid[kFpBatch];
+    unsigned long long a[kFpBatch];
+#pragma unroll
+    for (int i = 0; i < kFpBatch; ++i) {
+      const unsigned long long ri = r + i < r1 ? r + i : r;   // re-read a valid slot past the end, unused
+      const unsigned char* rec = ring + 64 + ri * RECORD_BYTES;
+      lid[i] = __ldcs(reinterpret_cast<const unsigned*>(rec));                 // launch
+      h1[i] = __ldcs(reinterpret_cast<const uint4*>(rec + 16));                // A P op|w|k tag
+      a[i] = __ldcs(reinterpret_cast<const unsigned long long*>(rec + 32) + lane);
+    }
+#pragma unroll
+    for (int i = 0; i < kFpBatch; ++i) {
+      if (r + i >= r1 || h1[i].w != 1u) continue;            // past the chunk / never written (uniform)
+      const unsigned launch = lid[i] - first;
+      if (launch >= n_launches) { if (lane == 0) atomicAdd(err, 1ull); continue; }
+      if (launch != cur) {                                   // flush the running per-launch record count
+        if (lane == 0 && cur != 0xFFFFFFFFu) atomicAdd(counts + 3ull * cur + 2, nrec);
+        cur = launch; nrec = 0;
+      }
+      nrec += 1;
+      fp_record(launch, h1[i].x & h1[i].y, a[i], lane, keys, pool, mask, err, ck, cs);
+    }
+  }
+  if (lane == 0 && cur != 0xFFFFFFFFu) atomicAdd(counts + 3ull * cur + 2, nrec);
+}
+}  // namespace nvbt
+
+int nvbt_trace_footprint(nvbt_channel ch, void* d_scratch, uint64_t table_slots, uint32_t first_launch,
+                         uint32_t n_launches, uint64_t* out, float* kernel_ms) {
+  if (!ch || !d_scratch || !out || n_launches == 0) return set_error(NVBT_EINVAL, "null argument");
+  if (!ch->on_device) return set_error(NVBT_ESTATE, "footprint needs a device-memory channel");
+  if (table_slots == 0 || (table_slots & (table_slots - 1))) return set_error(NVBT_EINVAL, "table_slots must be a power of two");
+  if (n_launches > (1u << 16)) return set_error(NVBT_EINVAL, "n_launches > 65536");
+  nvbt_ctx c = ch->ctx;
+  NVBT_CUDA(cudaSetDevice(c->device));
+  if (reinterpret_cast<uintptr_t>(d_scratch) % 16) return set_error(NVBT_EINVAL, "d_scratch not 16-byte aligned");
+  // [blocks: 4 KB per slot][keys: 8 B per slot][counts]
+  auto* pool = static_cast<unsigned*>(d_scratch);
+  auto* keys = reinterpret_cast<unsigned long long*>(pool + table_slots * kFpWords);
+  unsigned long long* counts = keys + table_slots;
+  NVBT_CUDA(cudaMemsetAsync(keys, 0xff, table_slots * 8, c->stream));
+  NVBT_CUDA(cudaMemsetAsync(pool, 0, table_slots * kFpWords * 4, c->stream));
+  NVBT_CUDA(cudaMemsetAsync(counts, 0, (3ull * n_launches + 1) * 8, c->stream));
+  int sms = 148;
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, c->device);
+  cudaEvent_t ev[2] = {nullptr, nullptr};
+  if (kernel_ms) { NVBT_CUDA(cudaEventCreate(&ev[0])); NVBT_CUDA(cudaEventCreate(&ev[1])); cudaEventRecord(ev[0], c->stream); }
+  k_footprint<<<sms * 8, 256, 0, c->stream>>>(ch->dev, c->ctl + CTL_RHEAD + ch->rstripes, ch->cap, keys, pool,
+                                              table_slots - 1, counts, first_launch, n_launches);
+  NVBT_CUDA(cudaGetLastError());
+  k_fp_count<<<(unsigned)std::min<unsigned long long>((table_slots + 7) / 8, (unsigned long long)sms * 8), 256, 0,
+               c->stream>>>(keys, pool, table_slots, counts, n_launches);
+  NVBT_CUDA(cudaGetLastError());
+  c->launches += 2;
+  if (kernel_ms) {
+    cudaEventRecord(ev[1], c->stream);
+    cudaEventSynchronize(ev[1]);
+    cudaEventElapsedTime(kernel_ms, ev[0], ev[1]);
+    cudaEventDestroy(ev[0]); cudaEventDestroy(ev[1]);
+  }
+  std::vector<unsigned long long> h(3ull * n_launches + 1);
+  NVBT_CUDA(cudaMemcpyAsync(h.data(), counts, h.size() * 8, cudaMemcpyDeviceToHost, c->stream));
+  NVBT_CUDA(cudaStreamSynchronize(c->stream));
+  if (h.back()) return set_error(NVBT_EINVAL, "%llu records out of range (launch id or address >= 2^48) or table_slots too small", h.back());
+  std::memcpy(out, h.data(), 3ull * n_launches * 8);
   return NVBT_OK;
 }
 
@@ -328,6 +550,7 @@ int nvbt_channel_dropped(nvbt_channel ch, uint64_t* dropped) {
 int nvbt_channel_drain(nvbt_channel ch, nvbt_drain_fn fn, void* user, int64_t timeout_us, uint64_t* n_drained) {
   if (!ch || !fn) return set_error(NVBT_EINVAL, "null argument");
   if (!ch->open) return set_error(NVBT_ESTATE, "channel not open");
+  if (ch->on_device) return set_error(NVBT_ESTATE, "device-memory channel: use the GPU consumers (nvbt_trace_footprint)");
   nvbt_ctx c = ch->ctx;
   NVBT_CUDA(cudaSetDevice(c->device));
   const auto t0 = std::chrono::steady_clock::now();

@@ -48,9 +48,18 @@ struct DevState {
   unsigned long long stripe_words;
   unsigned slot_bytes;             // 288, or 176 for compact channels (EM §5.1)
   unsigned compact;
+  unsigned no_wait;                // device-memory ring (F2): drop when full instead of waiting
+  // device ring (F2): slots are handed out in chunks of kRingChunk. Each SM owns a stripe word
+  // rheads[smid % rstripes] = (chunk << 32 | used) and takes tickets from its current chunk; the warp whose
+  // ticket is exactly kRingChunk opens the stripe's next chunk from the global counter rheads[rstripes].
+  unsigned long long* rheads;
+  unsigned rstripes;
 };
+constexpr unsigned kRingChunk = 1024;
+constexpr unsigned kRingNoChunk = 0xFFFFFFFEu, kRingFull = 0xFFFFFFFFu;
 
 __device__ __forceinline__ unsigned lane_id() { unsigned l; asm("mov.u32 %0, %%laneid;" : "=r"(l)); return l; }
+__device__ __forceinline__ unsigned smid() { unsigned s; asm volatile("mov.u32 %0, %%smid;" : "=r"(s)); return s; }
 __device__ __forceinline__ unsigned lanemask_lt() { unsigned m; asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m)); return m; }
 __device__ __forceinline__ unsigned long long globaltimer() {
   unsigned long long t; asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t)); return t;
@@ -379,6 +388,37 @@ struct Hooks {
   // Compact channels (st.compact, EM §5.1, F3) send base + 32-bit deltas in one 176 B slot, or two slots
   // of 16 full addresses each when the warp's addresses span more than ±2 GB.
   __device__ __forceinline__ bool reserve(unsigned k, unsigned long long& t) {
+    if (st.no_wait) {   // device ring: per-SM chunked tickets, no backpressure, k == 1 (288 B records)
+      unsigned long long tt = 0;
+      int ok = 1;
+      if (lane == 0) {
+        unsigned long long* w = st.rheads + smid() % st.rstripes;
+        const unsigned long long t0 = globaltimer();
+        for (;;) {
+          const unsigned long long v = atomicAdd(w, 1ull);
+          const unsigned ck = (unsigned)(v >> 32), off = (unsigned)v;
+          if (ck == kRingFull) { ok = 0; break; }
+          if (off < kRingChunk) {
+            tt = (unsigned long long)ck * kRingChunk + off;
+            ok = tt < st.cap;
+            break;
+          }
+          if (off == kRingChunk) {   // this warp opens the stripe's next chunk
+            const unsigned long long nc = atomicAdd(st.rheads + st.rstripes, 1ull);
+            if (nc * kRingChunk >= st.cap) { atomicExch(w, (unsigned long long)kRingFull << 32); ok = 0; break; }
+            atomicExch(w, (nc << 32) | 1ull);
+            tt = nc * kRingChunk;
+            break;
+          }
+          // another warp is opening the next chunk: wait until the stripe word moves on
+          while ((unsigned)(*(volatile unsigned long long*)w >> 32) == ck && globaltimer() - t0 < 2000000000ull) {}
+          if (globaltimer() - t0 >= 2000000000ull) { ok = 0; break; }
+        }
+        if (!ok) atomicAdd(st.dropped, 1ull);
+      }
+      t = __shfl_sync(FULL, tt, 0);
+      return __shfl_sync(FULL, ok, 0) != 0;
+    }
     int room = 1;
     if (lane == 0) {
       t = atomicAdd(st.head, (unsigned long long)k);
@@ -388,7 +428,7 @@ struct Hooks {
     if (!__shfl_sync(FULL, room, 0)) {
       commit();
       int ok = 1;
-      if (lane == 0) ok = wait_room(st, t + k - 1);
+      if (lane == 0) ok = st.no_wait ? 0 : wait_room(st, t + k - 1);
       if (!__shfl_sync(FULL, ok, 0)) {
         if (lane == 0) atomicAdd(st.dropped, 1ull);
         return false;
@@ -420,18 +460,20 @@ struct Hooks {
     unsigned tag;
     if (!st.compact) {
       if (reserve(1, t)) {
-        unsigned char* rec = slot_ptr(t, tag);
+        // device ring: every slot is lap 1 and the consumer is a later kernel, so the tag goes out with
+        // the header (no fence, no batched commit)
+        unsigned char* rec = st.no_wait ? st.ring + t * RECORD_BYTES : slot_ptr(t, tag);
         // lane j < 18 writes bytes [16j, 16j + 16): lanes 0, 1 the header (tag 0), lane j >= 2 the
         // addresses of lanes 2(j-2), 2(j-2)+1
         const unsigned src = 2u * (lane - 2u);
         const unsigned long long a0 = __shfl_sync(FULL, a, src & 31u), a1 = __shfl_sync(FULL, a, (src + 1u) & 31u);
         if (lane < 18) {
           const uint4 v = lane == 0   ? make_uint4(st.launch, gwarp, seq, (unsigned)PC)
-                          : lane == 1 ? make_uint4(A, P, w2, 0u)
+                          : lane == 1 ? make_uint4(A, P, w2, st.no_wait)
                                       : make_uint4((unsigned)a0, (unsigned)(a0 >> 32), (unsigned)a1, (unsigned)(a1 >> 32));
           *reinterpret_cast<uint4*>(rec + 16 * lane) = v;
         }
-        add_pending(rec, tag);
+        if (!st.no_wait) add_pending(rec, tag);
       }
       ++seq;
       return;

@@ -83,6 +83,7 @@ _sigs = {
     "nvbt_channel_dropped": ([_P, C.POINTER(C.c_uint64)], C.c_int),
     "nvbt_digest_records": ([_P, C.c_uint64, C.POINTER(Digest)], C.c_int),
     "nvbt_decode_compact": ([_P, C.c_uint64, _P, C.c_uint64, C.POINTER(C.c_uint64)], C.c_int),
+    "nvbt_trace_footprint": ([_P, _P, C.c_uint64, C.c_uint32, C.c_uint32, _P, _P], C.c_int),
     "nvbt_gen_events": ([_P, C.c_uint64, C.c_uint64, C.c_uint64, _P, _P], C.c_int),
     "nvbt_replay": ([_P, _P, _P, C.c_uint64], C.c_int),
     "nvbt_replay_errors": ([_P, C.POINTER(C.c_uint64)], C.c_int),
@@ -295,8 +296,8 @@ class Channel:
 
 
 def nvbt_channel_open(ctx, ring, compact=False):
-    """ring: pinned uint8 torch tensor (torch.empty(..., pin_memory=True)); compact: 176 B transport slots
-    (base + 32-bit deltas, EM §5.1) instead of 288 B records."""
+    """ring: pinned uint8 torch tensor (torch.empty(..., pin_memory=True)), or a CUDA uint8 tensor for an
+    on-GPU channel (F2); compact: 176 B transport slots (base + 32-bit deltas, EM §5.1)."""
     h = C.c_void_p()
     rb = COMPACT_RECORD_BYTES if compact else RECORD_BYTES
     _check(_lib.nvbt_channel_open(ctx.handle, C.c_void_p(ring.data_ptr()), ring.numel(), rb, C.byref(h)))
@@ -310,6 +311,22 @@ def nvbt_channel_close(ch):
         _check(_lib.nvbt_channel_close(ch.handle))
         ch.handle = None
         ch.ctx.channel = None
+
+
+def nvbt_trace_footprint(ch, n_launches, table_slots=1 << 10, scratch=None, timing=None, first_launch=0):
+    """F2: per-launch (distinct sectors, distinct lines, records) of a device-memory channel [n, 3]
+    for launch ids first_launch .. first_launch + n_launches - 1.
+    table_slots: power of two above the distinct (launch, 1 MB region) pairs."""
+    import torch
+    if scratch is None:
+        scratch = torch.empty(513 * table_slots + 3 * n_launches + 1, dtype=torch.int64, device=ch.ctx.device)
+    out = np.zeros((n_launches, 3), dtype=np.uint64)
+    ms = C.c_float(0.0)
+    _check(_lib.nvbt_trace_footprint(ch.handle, C.c_void_p(scratch.data_ptr()), table_slots, first_launch, n_launches,
+                                     out.ctypes.data_as(C.c_void_p), C.byref(ms) if timing is not None else None))
+    if timing is not None:
+        timing.append(ms.value / 1e3)   # consumer kernel device seconds
+    return out
 
 
 def nvbt_channel_dropped(ch):

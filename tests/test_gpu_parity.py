@@ -154,16 +154,19 @@ def _stencil_case(nvbt, n, iters, ring_records, tools_names=("TRACE", "MEMDIV", 
     x0 = cuda(uniform_f32((n, n), 4))
     buf0, buf1 = x0.clone(), torch.zeros_like(x0)
     ring = torch.empty(64 + (176 if compact else 288) * ring_records, dtype=torch.uint8, pin_memory=True)
+    ring.view(torch.int32).fill_(1)            # stale "lap 1" tags everywhere: open must clear them
     ch = nb.nvbt_channel_open(ctx, ring, compact=compact)
     dr.run_stencil(ctx, t, buf0, buf1, n, iters)
     acc = ev.Accumulator(programs.stencil(), trace=True, keep_records=True)
     m_st.run_iterations(acc, n, buf0.data_ptr(), buf1.data_ptr(), iters)
     exp = acc.record_array()
-    dst = np.zeros((len(exp) + 16, 288), dtype=np.uint8)
+    dst = np.zeros((len(exp) + 65536, 288), dtype=np.uint8)
     got_n = nb.nvbt_channel_drain_copy(ch, dst, timeout_us=60_000_000)
     assert nb.nvbt_channel_dropped(ch) == 0
     got = dst[:got_n]
-    assert got_n == len(exp)
+    ids, cnt = np.unique(got.view("<u4")[:, 0], return_counts=True)
+    assert got_n == len(exp), f"launch ids {ids} x {cnt}"
+
     assert (trace.sort_records(got) == trace.sort_records(exp)).all()
     out = buf0 if iters % 2 == 0 else buf1
     ref_grid = m_st.jacobi_reference(x0.cpu().numpy(), iters)
@@ -207,6 +210,94 @@ def test_channel_digest_drain(nvbt):
     acc = ev.Accumulator(programs.stencil(), trace=True)
     m_st.run_iterations(acc, n, buf0.data_ptr(), buf1.data_ptr(), iters)
     assert (d.n_rec, d.d1, d.d2) == (acc.digest.n, acc.digest.d1, acc.digest.d2)
+
+
+# ---------------------------------------------------------------- F2 device-memory channel + GPU consumer
+def _device_ring(nb, ctx, records):
+    import torch
+    ring = torch.empty(64 + 288 * records, dtype=torch.uint8, device="cuda")
+    ring.view(torch.int32).fill_(1)            # stale "committed" tags everywhere: open must clear them
+    return ring, nb.nvbt_channel_open(ctx, ring)
+
+
+def _committed(ring):
+    """Records of a device ring with tag 1 (slots are spread over SM regions), tag word cleared."""
+    r = ring[64:].cpu().numpy().reshape(-1, 288)
+    r = r[r[:, 28:32].copy().view("<u4")[:, 0] == 1].copy()
+    r[:, 28:32] = 0
+    return r
+
+
+@pytest.mark.parametrize("n,iters,slots", [(96, 3, 64), (100, 2, 64), (512, 16, 128)])
+def test_device_channel_footprint_stencil(nvbt, n, iters, slots):
+    """F2: records stay in HBM and the GPU consumer's per-launch footprint equals the oracle's; the
+    records themselves (copied back only for the check) equal the oracle's as a multiset."""
+    import torch
+    nb, dr = nvbt.nvbt, nvbt.drivers
+    ctx = nb.nvbt_init(nb.W_STENCIL, nb.TRACE)
+    x0 = cuda(uniform_f32((n, n), 4))
+    buf0, buf1 = x0.clone(), torch.zeros_like(x0)
+    ring, ch = _device_ring(nb, ctx, 1 << 20)
+    dr.run_stencil(ctx, nb.TOOL_TRACE, buf0, buf1, n, iters)
+    acc = ev.Accumulator(programs.stencil(), trace=True, keep_records=True)
+    m_st.run_iterations(acc, n, buf0.data_ptr(), buf1.data_ptr(), iters)
+    exp = acc.record_array()
+    fp = nb.nvbt_trace_footprint(ch, iters + 1, table_slots=slots)   # 512x16: crowded table
+    assert np.array_equal(fp.astype(np.int64), trace.footprint(exp, iters + 1))
+    assert nb.nvbt_channel_dropped(ch) == 0
+    got = _committed(ring)
+    assert len(got) == len(exp)
+    assert (trace.sort_records(got) == trace.sort_records(exp)).all()
+    with pytest.raises(nb.NvbtError):
+        nb.nvbt_channel_drain_digest(ch, timeout_us=1000)
+
+
+def test_device_channel_overflow_drops(nvbt):
+    """A device ring smaller than the trace keeps what fits and counts the rest as dropped (no
+    backpressure wait: nobody frees slots); every kept record is one of the oracle's and the consumer
+    counts exactly the kept ones. A table too small for the footprint is an error, not a hang."""
+    import torch
+    nb, dr = nvbt.nvbt, nvbt.drivers
+    n, iters, cap = 64, 2, 1000
+    ctx = nb.nvbt_init(nb.W_STENCIL, nb.TRACE)
+    buf0 = cuda(uniform_f32((n, n), 4)); buf1 = torch.zeros_like(buf0)
+    ring, ch = _device_ring(nb, ctx, cap)
+    dr.run_stencil(ctx, nb.TOOL_TRACE, buf0, buf1, n, iters)
+    acc = ev.Accumulator(programs.stencil(), trace=True, keep_records=True)
+    m_st.run_iterations(acc, n, buf0.data_ptr(), buf1.data_ptr(), iters)
+    exp = acc.record_array()
+    fp = nb.nvbt_trace_footprint(ch, iters, table_slots=1 << 6)
+    got = _committed(ring)
+    assert 0 < len(got) <= cap
+    assert int(fp[:, 2].sum()) == len(got)
+    assert nb.nvbt_channel_dropped(ch) == len(exp) - len(got)
+    universe = {r.tobytes() for r in exp}
+    assert all(r.tobytes() in universe for r in got)
+    assert len({r.tobytes() for r in got}) == len(got)
+    with pytest.raises(nb.NvbtError):                      # 1 slot < 2 launches x regions: reported, no hang
+        nb.nvbt_trace_footprint(ch, iters, table_slots=1)
+
+
+def test_device_channel_footprint_bfs(nvbt):
+    """F2 on the irregular workload: BFS (two kernels per level) on an R-MAT graph."""
+    nb, dr = nvbt.nvbt, nvbt.drivers
+    rowptr, col = rmat_csr(10)
+    n = len(rowptr) - 1
+    src = bfs_source(rowptr)
+    ctx = nb.nvbt_init(nb.W_BFS, nb.TRACE)
+    rp, cl = cuda(rowptr), cuda(col)
+    bufs = dr.bfs_buffers(n, "cuda")
+    ring, ch = _device_ring(nb, ctx, 1 << 18)
+    cost, levels = dr.run_bfs(ctx, nb.TOOL_TRACE, rp, cl, src, bufs)
+    acc = ev.Accumulator(programs.bfs(), trace=True, keep_records=True)
+    ptr = m_bfs.Ptrs(bufs["mask"].data_ptr(), bufs["visited"].data_ptr(), bufs["updating"].data_ptr(),
+                     bufs["cost"].data_ptr(), bufs["over"].data_ptr(), rp.data_ptr(), cl.data_ptr())
+    m_bfs.run(acc, rowptr, col, src, ptr)
+    exp = acc.record_array()
+    nl = int(exp.view(trace.RECORD_DTYPE)["launch"].max()) + 1
+    fp = nb.nvbt_trace_footprint(ch, nl, table_slots=1 << 12)
+    assert nb.nvbt_channel_dropped(ch) == 0
+    assert np.array_equal(fp.astype(np.int64), trace.footprint(exp, nl))
 
 
 # ---------------------------------------------------------------- C5 generator + replay
