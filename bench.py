@@ -539,7 +539,7 @@ def run_f2(args, torch, nb, dr, local):
     ctx = nb.nvbt_init(nb.W_STENCIL, nb.COUNT | nb.TRACE)
     x0 = torch.from_numpy(uniform_f32((n, n), 4)).cuda()
     buf0, buf1 = x0.clone(), torch.empty_like(x0)
-    slack = torch.cuda.get_device_properties(0).multi_processor_count * 1024   # last chunk per SM
+    slack = cap // 50 + torch.cuda.get_device_properties(0).multi_processor_count * 4096   # nvbt.h sizing
     ring = torch.empty(64 + 288 * (cap + slack), dtype=torch.uint8, device="cuda")
     regions = iters * 2 * (-(-n * n * 4 // (1 << 20)) + 1)          # (launch, 1 MB region) pairs
     slots = 1 << (2 * regions - 1).bit_length()
@@ -587,7 +587,9 @@ def run_f2(args, torch, nb, dr, local):
             "footprint_launch0": [int(x) for x in fp[0]], "footprint_expected": [exp_s, exp_l],
             "roofline": {"bound": "hbm", "achieved": ach, "peak": peaks["hbm_gbs"], "unit": "GB/s",
                          "frac": ach / peaks["hbm_gbs"], "peak_source": peaks_src, "kernel": "k_footprint",
-                         "algorithmic_bytes_per_launch": recs * 288, "traffic": None},
+                         "algorithmic_bytes_per_launch": recs * 288,
+                         "traffic": (load_traffic("k_footprint") or {}).get("traffic_bytes_per_record", 0) * recs or None,
+                         "traffic_unit": "DRAM bytes per consumer launch (ncu per-record figure at 4096^2 x 4, scaled)"},
             "gpu_launches": int(launches) // (args.warmup + args.steps), "clocks": clk.summary()}
 
 

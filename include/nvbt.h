@@ -144,8 +144,10 @@ int nvbt_channel_drain(nvbt_channel ch, nvbt_drain_fn fn, void* user, int64_t ti
 int nvbt_channel_close(nvbt_channel ch);
 /* F2, on-GPU consumer ("can be analyzed directly on the GPU", P:L187 (§6.1)). A channel whose ring is
  * DEVICE memory (288 B records) is filled by the producers without backpressure: each SM takes slots
- * from its own 1024-slot chunk of the ring (so the last chunk of every SM may stay partly empty: size the
- * ring for the records + 1024 x SMs slots); records that find no chunk are dropped and counted. The ring
+ * from its own 4096-slot chunk of the ring and each warp reserves the slots of the rest of its basic block
+ * at once (x4 in loops), so some slots stay empty (the last chunk of every SM, a few per chunk and per
+ * warp): size the ring for the records x 1.02 + 4096 x SMs slots; records that find no chunk are dropped
+ * and counted. The ring
  * is analysed in place: per launch id first_launch + l, l < n_launches,
  *   out[3l + 0] = distinct 32 B sectors, out[3l + 1] = distinct 128 B lines over the lanes of E of all
  *   records of that launch (the launch's footprint, reading R-18), out[3l + 2] = records.

@@ -338,7 +338,7 @@ int nvbt_channel_open(nvbt_ctx c, void* ring, size_t bytes, uint32_t record_byte
 // each owning a 4 KB block of 4 sector bits per line (8192 lines). The blocks cost 1/256 of the address
 // span a launch touches and stay L2-resident, so the kernel streams the records from HBM once.
 namespace nvbt {
-constexpr int kFpBatch = 4;                  // records in flight per warp (memory-level parallelism)
+constexpr int kFpBatch = 8;                  // record address loads in flight per warp
 constexpr unsigned long long kFpEmpty = ~0ull;
 constexpr int kFpRegionShift = 20;           // 1 MB regions
 constexpr unsigned kFpWords = (1u << (kFpRegionShift - 7)) / 8;   // 32-bit words per block (8 lines each)
@@ -390,6 +390,7 @@ __device__ __forceinline__ void fp_record(unsigned launch, unsigned E, unsigned 
   const unsigned word = line >> 3;
   const unsigned bits = 1u << ((line & 7) * 4 + ((unsigned)(a >> 5) & 3));
   unsigned pend = __ballot_sync(0xffffffffu, on);
+  if (pend == 0) return;
   while (pend) {
     const unsigned f = __ffs(pend) - 1;
     const unsigned long long k = __shfl_sync(0xffffffffu, rkey, f);
@@ -444,7 +445,9 @@ __global__ void __launch_bounds__(256) k_fp_count(const unsigned long long* __re
 }
 
 // Committed slots lie in the chunks handed out so far, [0, min(chunks * kRingChunk, cap)); slots never
-// written (the unused tail of each SM's last chunk) have tag 0 and are skipped.
+// written (the unused tail of each SM's last chunk, slots a warp reserved but did not use) have tag 0 and
+// are skipped. Each warp takes a contiguous range of slots, 32 at a time: lane i reads record i's
+// header, then the warp walks the 32 records (addresses coalesced, kFpBatch loads in flight).
 __global__ void __launch_bounds__(256) k_footprint(const unsigned char* __restrict__ ring,
                                                     const unsigned long long* __restrict__ chunks,
                                                     unsigned long long cap,
@@ -455,36 +458,58 @@ __global__ void __launch_bounds__(256) k_footprint(const unsigned char* __restri
   const unsigned long long n_slots = *chunks * kRingChunk < cap ? *chunks * kRingChunk : cap;
   const unsigned long long warps = (unsigned long long)gridDim.x * (blockDim.x >> 5);
   const unsigned long long w = (blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x) >> 5;
-  // contiguous chunk per warp: launch ids change rarely, so the per-launch record counts stay in registers
   const unsigned long long per = (n_slots + warps - 1) / warps;
   const unsigned long long r0 = w * per, r1 = r0 + per < n_slots ? r0 + per : n_slots;
   unsigned long long* err = counts + 3ull * n_launches;
   unsigned cur = 0xFFFFFFFFu;
   unsigned long long nrec = 0;
   unsigned long long ck[2] = {kFpEmpty, kFpEmpty}, cs[2] = {0, 0};
-  for (unsigned long long r = r0; r < r1; r += kFpBatch) {
-    uint4 h1[kFpBatch];
-    unsigned lid[kFpBatch];
-    unsigned long long a[kFpBatch];
-#pragma unroll
-    for (int i = 0; i < kFpBatch; ++i) {
-      const unsigned long long ri = r + i < r1 ? r + i : r;   // re-read a valid slot past the end, unused
-      const unsigned char* rec = ring + 64 + ri * RECORD_BYTES;
-      lid[i] = __ldcs(reinterpret_cast<const unsigned*>(rec));                 // launch
-      h1[i] = __ldcs(reinterpret_cast<const uint4*>(rec + 16));                // A P op|w|k tag
-      a[i] = __ldcs(reinterpret_cast<const unsigned long long*>(rec + 32) + lane);
+  for (unsigned long long base = r0; base < r1; base += 32) {
+    const unsigned cnt = r1 - base < 32 ? (unsigned)(r1 - base) : 32u;
+    unsigned lid = 0xFFFFFFFFu, E = 0;
+    if (lane < cnt) {
+      const unsigned char* rec = ring + 64 + (base + lane) * RECORD_BYTES;
+      const uint4 h1 = __ldcs(reinterpret_cast<const uint4*>(rec + 16));   // A P op|w|k tag
+      const unsigned l = __ldcs(reinterpret_cast<const unsigned*>(rec)) - first;
+      if (h1.w == 1u) { lid = l; E = h1.x & h1.y; }
     }
-#pragma unroll
-    for (int i = 0; i < kFpBatch; ++i) {
-      if (r + i >= r1 || h1[i].w != 1u) continue;            // past the chunk / never written (uniform)
-      const unsigned launch = lid[i] - first;
-      if (launch >= n_launches) { if (lane == 0) atomicAdd(err, 1ull); continue; }
-      if (launch != cur) {                                   // flush the running per-launch record count
-        if (lane == 0 && cur != 0xFFFFFFFFu) atomicAdd(counts + 3ull * cur + 2, nrec);
-        cur = launch; nrec = 0;
+    const bool ok = lid < n_launches;
+    const unsigned bad = __ballot_sync(0xffffffffu, lid != 0xFFFFFFFFu && !ok);
+    if (bad) { if (lane == 0) atomicAdd(err, (unsigned long long)__popc(bad)); E = ok ? E : 0u; }
+    const unsigned okm = __ballot_sync(0xffffffffu, ok);
+    if (okm) {   // record counts: a warp's range nearly always holds one launch
+      const unsigned l0 = __shfl_sync(0xffffffffu, lid, __ffs(okm) - 1);
+      if (__all_sync(0xffffffffu, !ok || lid == l0)) {
+        if (l0 != cur) {
+          if (lane == 0 && cur != 0xFFFFFFFFu) atomicAdd(counts + 3ull * cur + 2, nrec);
+          cur = l0; nrec = 0;
+        }
+        nrec += __popc(okm);
+      } else {
+        unsigned pend = okm;
+        while (pend) {
+          const unsigned l = __shfl_sync(0xffffffffu, lid, __ffs(pend) - 1);
+          const unsigned m = __ballot_sync(0xffffffffu, ok && lid == l);
+          if (lane == 0) atomicAdd(counts + 3ull * l + 2, (unsigned long long)__popc(m));
+          pend &= ~m;
+        }
       }
-      nrec += 1;
-      fp_record(launch, h1[i].x & h1[i].y, a[i], lane, keys, pool, mask, err, ck, cs);
+    }
+    const unsigned live = __ballot_sync(0xffffffffu, ok && E != 0u);
+    for (unsigned j = 0; j < 32; j += kFpBatch) {
+      if (((live >> j) & ((1u << kFpBatch) - 1u)) == 0u) continue;   // uniform
+      unsigned long long a[kFpBatch];
+#pragma unroll
+      for (int u = 0; u < kFpBatch; ++u) {
+        const unsigned jj = (live >> (j + u)) & 1u ? j + u : __ffs(live) - 1;   // keep loads in range
+        a[u] = __ldcs(reinterpret_cast<const unsigned long long*>(ring + 64 + (base + jj) * RECORD_BYTES + 32) + lane);
+      }
+#pragma unroll
+      for (int u = 0; u < kFpBatch; ++u) {
+        const unsigned Ej = __shfl_sync(0xffffffffu, E, j + u);
+        const unsigned lj = __shfl_sync(0xffffffffu, lid, j + u);
+        if ((live >> (j + u)) & 1u) fp_record(lj, Ej, a[u], lane, keys, pool, mask, err, ck, cs);
+      }
     }
   }
   if (lane == 0 && cur != 0xFFFFFFFFu) atomicAdd(counts + 3ull * cur + 2, nrec);

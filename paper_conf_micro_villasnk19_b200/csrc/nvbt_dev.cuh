@@ -55,7 +55,7 @@ struct DevState {
   unsigned long long* rheads;
   unsigned rstripes;
 };
-constexpr unsigned kRingChunk = 1024;
+constexpr unsigned kRingChunk = 4096;
 constexpr unsigned kRingNoChunk = 0xFFFFFFFEu, kRingFull = 0xFFFFFFFFu;
 
 __device__ __forceinline__ unsigned lane_id() { unsigned l; asm("mov.u32 %0, %%laneid;" : "=r"(l)); return l; }
@@ -75,6 +75,12 @@ template <class Prog> __host__ __device__ constexpr int leader_of(int pc) {
 template <class Prog> __host__ __device__ constexpr int bb_len(int lead) {
   int n = 1;
   while (lead + n < Prog::N && !Prog::t[lead + n].is_leader) ++n;
+  return n;
+}
+// memory pcs in [pc, end of pc's basic block]
+template <class Prog> __host__ __device__ constexpr int mem_left(int pc) {
+  int n = 0;
+  for (int p = pc; p < Prog::N && (p == pc || !Prog::t[p].is_leader); ++p) n += is_mem_kind(Prog::t[p].kind) ? 1 : 0;
   return n;
 }
 
@@ -266,6 +272,8 @@ struct Hooks {
   unsigned hS, hL;            // lane-distributed: lane l counts events with S (L) == l + 1
   unsigned pwT, pwW;          // this warp's executed thread / warp instructions (PER_WARP)
   unsigned seq;               // records emitted by this warp in this launch
+  unsigned long long hslot;   // device ring: next slot this warp holds, `held` slots from there
+  unsigned held;
   unsigned npend = 0;         // uncommitted records of this warp (warp-uniform)
   unsigned pend_val = 0;      // lane k: tag value of the k-th uncommitted record
   unsigned char* pend_tag = nullptr;
@@ -274,6 +282,7 @@ struct Hooks {
   __device__ __forceinline__ Hooks(const DevState& s, unsigned* smem) : st(s), sb(smem) {
     zero_range<0, NPC - 1>();
     hS = hL = pwT = pwW = seq = 0;
+    hslot = 0; held = 0;
     lane = lane_id();
     lane1 = lane + 1u;
     lanebit = 1u << lane;
@@ -387,38 +396,43 @@ struct Hooks {
   // on a full ring, so reserved-but-uncommitted slots never stall the consumer for ever.
   // Compact channels (st.compact, EM §5.1, F3) send base + 32-bit deltas in one 176 B slot, or two slots
   // of 16 full addresses each when the warp's addresses span more than ±2 GB.
-  __device__ __forceinline__ bool reserve(unsigned k, unsigned long long& t) {
-    if (st.no_wait) {   // device ring: per-SM chunked tickets, no backpressure, k == 1 (288 B records)
-      unsigned long long tt = 0;
-      int ok = 1;
-      if (lane == 0) {
-        unsigned long long* w = st.rheads + smid() % st.rstripes;
-        const unsigned long long t0 = globaltimer();
-        for (;;) {
-          const unsigned long long v = atomicAdd(w, 1ull);
-          const unsigned ck = (unsigned)(v >> 32), off = (unsigned)v;
-          if (ck == kRingFull) { ok = 0; break; }
-          if (off < kRingChunk) {
-            tt = (unsigned long long)ck * kRingChunk + off;
-            ok = tt < st.cap;
-            break;
-          }
-          if (off == kRingChunk) {   // this warp opens the stripe's next chunk
-            const unsigned long long nc = atomicAdd(st.rheads + st.rstripes, 1ull);
-            if (nc * kRingChunk >= st.cap) { atomicExch(w, (unsigned long long)kRingFull << 32); ok = 0; break; }
-            atomicExch(w, (nc << 32) | 1ull);
-            tt = nc * kRingChunk;
-            break;
-          }
-          // another warp is opening the next chunk: wait until the stripe word moves on
-          while ((unsigned)(*(volatile unsigned long long*)w >> 32) == ck && globaltimer() - t0 < 2000000000ull) {}
-          if (globaltimer() - t0 >= 2000000000ull) { ok = 0; break; }
+  // Device ring (F2): k contiguous slots from this SM's current chunk; the warp whose range covers the
+  // chunk's end opens the stripe's next chunk. No backpressure: a ring without free chunks drops.
+  __device__ __forceinline__ bool reserve_dev(unsigned k, unsigned long long& t) {
+    unsigned long long tt = 0;
+    int ok = 1;
+    if (lane == 0) {
+      const unsigned sm = smid();
+      unsigned long long* w = st.rheads + (sm < st.rstripes ? sm : sm % st.rstripes);
+      const unsigned long long t0 = globaltimer();
+      for (;;) {
+        const unsigned long long v = atomicAdd(w, (unsigned long long)k);
+        const unsigned ck = (unsigned)(v >> 32), off = (unsigned)v;
+        if (ck == kRingFull) { ok = 0; break; }
+        if (off + k <= kRingChunk) {
+          tt = (unsigned long long)ck * kRingChunk + off;
+          ok = tt + k <= st.cap;
+          break;
         }
-        if (!ok) atomicAdd(st.dropped, 1ull);
+        if (off <= kRingChunk) {   // this warp's range covers the chunk end: open the next chunk
+          const unsigned long long nc = atomicAdd(st.rheads + st.rstripes, 1ull);
+          if (nc * kRingChunk >= st.cap) { atomicExch(w, (unsigned long long)kRingFull << 32); ok = 0; break; }
+          atomicExch(w, (nc << 32) | k);
+          tt = nc * kRingChunk;
+          ok = tt + k <= st.cap;
+          break;
+        }
+        // another warp is opening the next chunk: wait until the stripe word moves on
+        while ((unsigned)(*(volatile unsigned long long*)w >> 32) == ck && globaltimer() - t0 < 2000000000ull) {}
+        if (globaltimer() - t0 >= 2000000000ull) { ok = 0; break; }
       }
-      t = __shfl_sync(FULL, tt, 0);
-      return __shfl_sync(FULL, ok, 0) != 0;
+      if (!ok) atomicAdd(st.dropped, 1ull);
     }
+    t = __shfl_sync(FULL, tt, 0);
+    return __shfl_sync(FULL, ok, 0) != 0;
+  }
+
+  __device__ __forceinline__ bool reserve(unsigned k, unsigned long long& t) {
     int room = 1;
     if (lane == 0) {
       t = atomicAdd(st.head, (unsigned long long)k);
@@ -459,9 +473,22 @@ struct Hooks {
     unsigned long long t;
     unsigned tag;
     if (!st.compact) {
-      if (reserve(1, t)) {
-        // device ring: every slot is lap 1 and the consumer is a later kernel, so the tag goes out with
-        // the header (no fence, no batched commit)
+      bool have;
+      if (st.no_wait) {
+        // device ring: a warp reserves the slots of the rest of its basic block at once (x4 in loops)
+        // and carries unused ones over; every slot is lap 1 and the consumer is a later kernel, so the
+        // tag goes out with the header (no fence, no batched commit)
+        constexpr unsigned K = (unsigned)mem_left<Prog>(PC) * ((PC >= Prog::REG_LO && PC <= Prog::REG_HI) ? 4u : 1u);
+        have = held != 0u || reserve_dev(K, hslot);
+        if (have) {
+          held = held ? held : K;
+          t = hslot++;
+          --held;
+        }
+      } else {
+        have = reserve(1, t);
+      }
+      if (have) {
         unsigned char* rec = st.no_wait ? st.ring + t * RECORD_BYTES : slot_ptr(t, tag);
         // lane j < 18 writes bytes [16j, 16j + 16): lanes 0, 1 the header (tag 0), lane j >= 2 the
         // addresses of lanes 2(j-2), 2(j-2)+1

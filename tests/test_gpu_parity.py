@@ -237,7 +237,7 @@ def test_device_channel_footprint_stencil(nvbt, n, iters, slots):
     ctx = nb.nvbt_init(nb.W_STENCIL, nb.TRACE)
     x0 = cuda(uniform_f32((n, n), 4))
     buf0, buf1 = x0.clone(), torch.zeros_like(x0)
-    ring, ch = _device_ring(nb, ctx, 1 << 20)
+    ring, ch = _device_ring(nb, ctx, 1 << 21)
     dr.run_stencil(ctx, nb.TOOL_TRACE, buf0, buf1, n, iters)
     acc = ev.Accumulator(programs.stencil(), trace=True, keep_records=True)
     m_st.run_iterations(acc, n, buf0.data_ptr(), buf1.data_ptr(), iters)
@@ -287,7 +287,7 @@ def test_device_channel_footprint_bfs(nvbt):
     ctx = nb.nvbt_init(nb.W_BFS, nb.TRACE)
     rp, cl = cuda(rowptr), cuda(col)
     bufs = dr.bfs_buffers(n, "cuda")
-    ring, ch = _device_ring(nb, ctx, 1 << 18)
+    ring, ch = _device_ring(nb, ctx, 1 << 20)
     cost, levels = dr.run_bfs(ctx, nb.TOOL_TRACE, rp, cl, src, bufs)
     acc = ev.Accumulator(programs.bfs(), trace=True, keep_records=True)
     ptr = m_bfs.Ptrs(bufs["mask"].data_ptr(), bufs["visited"].data_ptr(), bufs["updating"].data_ptr(),
