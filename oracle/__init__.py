@@ -16,6 +16,9 @@ Modules and their pins (tests/test_oracle_*.py):
   programs     §3 program tables           pinned: BB rule checks (leaders after CTRL and at targets)
   models.*     §3.1-3.4 CPU workload models pinned: closed forms (I-3) for vectorAdd, SGEMM, stencil;
                                            BFS distances vs scipy.sparse.csgraph (I-4); invariants
+  models.wfft  §3.6 F4 WFFT32 emulation    pinned: DFT vs numpy.fft.fft, single-exponential / constant /
+                                           delta closed forms, Parseval, Hermitian symmetry, inverse
+                                           round trip; per-warp count closed forms, BB identity (I-5)
   gen          §3.5 C5 generator           pinned: mix64 vector, distribution/alignment properties,
                                            partition invariance
   trace        §5 records + digests        pinned: record field layout by hand-built record,
@@ -23,5 +26,5 @@ Modules and their pins (tests/test_oracle_*.py):
                footprint (F2)              pinned: Python-set brute force on random records, vectorAdd
                                            closed form 3*ceil(4N/32) sectors / 3*ceil(4N/128) lines
 Parity unpinned: none of the above; the paper's Figs 5–9 values, the 74–96 % library share
-and WFFT32's 21 vs 150 instructions/warp need the paper's workloads and are not modelled.
+and WFFT32's 21 vs 150 instructions/warp need the paper's kernels; §3.6 models our own pair.
 """

@@ -15,6 +15,9 @@ MEM_KINDS = (GLD, GST, GATOM)
 
 S2R, IMAD, ISETP, EXIT, IMAD_WIDE, LDG, STG, FADD, FFMA, MOV, IADD, BRA, SEL = range(13)
 N_OPCODES_WL = 16
+# §3.6 (F4) opcode ids
+SHFL, FMUL, LOP3, I2F, MUFU_SIN, MUFU_COS, FSEL, BREV, SHF, WFFT32 = range(13, 23)
+N_OPCODES_WFFT = 32
 
 
 def _table(rows, n_opcodes=N_OPCODES_WL):
@@ -90,6 +93,38 @@ def stencil():
         (FADD, ALU, 0, 1, 0, 1), (FADD, ALU, 0, 1, 0, 1), (FADD, ALU, 0, 1, 0, 1), (FFMA, ALU, 0, 1, 0, 1),
         (SEL, ALU, 0, 1, 0, 0), (STG, GST, 4, 1, 0, 0), (EXIT, CTRL, 0, 1, 0, 0),
     ])
+
+
+def wfft_emu():
+    """§3.6 program WFFT_EMU (Listing 10 analogue): 14 pcs, 3 BBs."""
+    return _table([
+        (S2R, ALU, 0, 0, 1, 0), (S2R, ALU, 0, 0, 0, 0), (IMAD, ALU, 0, 0, 0, 0), (ISETP, ALU, 0, 0, 0, 0),
+        (EXIT, CTRL, 0, 0, 0, 1),
+        (IMAD_WIDE, ALU, 0, 1, 1, 0), (LDG, GLD, 8, 1, 0, 0), (WFFT32, ALU, 0, 1, 0, 0),
+        (IMAD_WIDE, ALU, 0, 1, 0, 0), (STG, GST, 8, 1, 0, 0), (IADD, ALU, 0, 1, 0, 0), (ISETP, ALU, 0, 1, 0, 0),
+        (BRA, CTRL, 0, 1, 0, 1, 5),
+        (EXIT, CTRL, 0, 2, 1, 0),
+    ], n_opcodes=N_OPCODES_WFFT)
+
+
+def wfft_sw():
+    """§3.6 program WFFT_SW (the transform written in CUDA): 83 pcs, 4 BBs."""
+    rows = [(S2R, ALU, 0, 0, 1, 0), (S2R, ALU, 0, 0, 0, 0), (IMAD, ALU, 0, 0, 0, 0), (ISETP, ALU, 0, 0, 0, 0),
+            (EXIT, CTRL, 0, 0, 0, 1)]
+    for q in range(4):                                   # twiddle setup, pcs 5-36
+        for o in (LOP3, LOP3, ISETP, I2F, MUFU_SIN, MUFU_COS, FSEL, FSEL):
+            rows.append((o, ALU, 0, 1, 1 if len(rows) == 5 else 0, 0))
+    rows += [(BREV, ALU, 0, 1, 0, 0), (SHF, ALU, 0, 1, 0, 0)]
+    rows += [(IMAD_WIDE, ALU, 0, 2, 1, 0), (LDG, GLD, 8, 2, 0, 0)]   # pcs 39, 40
+    for q in range(4):                                   # stages h = 16, 8, 4, 2: pcs 41-72
+        for o in (SHFL, SHFL, FFMA, FFMA, FMUL, FFMA, FMUL, FFMA):
+            rows.append((o, ALU, 0, 2, 0, 0))
+    for o in (SHFL, SHFL, FFMA, FFMA):                   # stage h = 1: pcs 73-76
+        rows.append((o, ALU, 0, 2, 0, 0))
+    rows += [(IMAD_WIDE, ALU, 0, 2, 0, 0), (STG, GST, 8, 2, 0, 0), (IADD, ALU, 0, 2, 0, 0),
+             (ISETP, ALU, 0, 2, 0, 0), (BRA, CTRL, 0, 2, 0, 1, 39), (EXIT, CTRL, 0, 3, 1, 0)]
+    assert len(rows) == 83
+    return _table(rows, n_opcodes=N_OPCODES_WFFT)
 
 
 def replay():

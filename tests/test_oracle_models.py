@@ -18,7 +18,7 @@ BASE = 1 << 32  # 128-byte aligned buffer bases
 
 
 # ---------------------------------------------------------------- programs: BB rule (R-14)
-@pytest.mark.parametrize("name", ["vectoradd", "sgemm", "bfs", "stencil", "replay"])
+@pytest.mark.parametrize("name", ["vectoradd", "sgemm", "bfs", "stencil", "replay", "wfft_emu", "wfft_sw"])
 def test_bb_rule(name):
     p = getattr(programs, name)()
     n = p["n_pcs"]
