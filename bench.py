@@ -267,8 +267,8 @@ def run_ours(args):
 
     if args.workload == "c5":
         return run_replay(args, torch, nb, dr, rank, world, local, peaks, peaks_src)
-    if args.workload in ("c1", "c3", "c4", "f1", "f2"):
-        line = {"c1": run_c1, "c3": run_c3, "c4": run_c4, "f1": run_f1, "f2": run_f2}[args.workload](
+    if args.workload in ("c1", "c3", "c4", "f1", "f2", "f4"):
+        line = {"c1": run_c1, "c3": run_c3, "c4": run_c4, "f1": run_f1, "f2": run_f2, "f4": run_f4}[args.workload](
             args, torch, nb, dr, local)
         if rank == 0:
             print(json.dumps(line), flush=True)
@@ -639,6 +639,63 @@ def run_f1(args, torch, nb, dr, local):
             "paper_context": "36.4x full vs 2.3x sampled on TITAN V / SpecAccel (P:L280)"}
 
 
+def run_f4(args, torch, nb, dr, local):
+    """F4 instruction emulation (EM §3.6): n_fft warp-wide 32-point FFTs, the kernel using the
+    proxy WFFT32 with the emulation tool vs the same transform written in CUDA, each plain and instrumented.
+    Inputs and outputs (2 x n_fft x 256 B) exceed L2, so no flush is needed between steps."""
+    n_fft, ctas = args.fft_n, args.fft_ctas
+    peaks, peaks_src = load_peaks()
+    g = torch.Generator(device="cuda").manual_seed(9)
+    x = (torch.rand((n_fft, 32, 2), generator=g, device="cuda") * 2 - 1).view(torch.complex64).reshape(n_fft, 32)
+    X = torch.empty_like(x)
+    W = 8 * ctas
+    flags = nb.COUNT | nb.OPHIST | nb.BB | nb.MEMDIV
+    cemu, csw = nb.nvbt_init(nb.W_WFFT_EMU, flags), nb.nvbt_init(nb.W_WFFT_SW, flags)
+    P, S = nb.WFFT_PROXY, nb.WFFT_SOFTWARE
+    modes = {
+        "sw_plain": (csw, S, nb.TOOL_NONE), "emu_only": (cemu, P, nb.TOOL_EMU),
+        "sw_bbcount_memdiv": (csw, S, nb.TOOL_BBCOUNT | nb.TOOL_MEMDIV),
+        "emu_bbcount_memdiv": (cemu, P, nb.TOOL_EMU | nb.TOOL_BBCOUNT | nb.TOOL_MEMDIV),
+        "sw_count": (csw, S, nb.TOOL_COUNT), "emu_count": (cemu, P, nb.TOOL_EMU | nb.TOOL_COUNT),
+    }
+    res, warp_inst = {}, {}
+    for name, (ctx, v, t) in modes.items():
+        f = lambda: nb.nvbt_wfft32(ctx, t, v, x, X, n_fft, ctas)
+        _timed_events(torch, f, args.warmup)
+        nb.nvbt_reset(ctx)
+        if name == "emu_bbcount_memdiv":
+            with ClockSampler(local) as clk:
+                res[name] = _timed_events(torch, f, args.steps)
+        else:
+            res[name] = _timed_events(torch, f, args.steps)
+        if t & (nb.TOOL_COUNT | nb.TOOL_BBCOUNT):
+            warp_inst[name] = int(nb.nvbt_count(ctx)[2]) // args.steps
+    med = {k: statistics.median(v) for k, v in res.items()}
+    head = "emu_bbcount_memdiv"
+    ev_launch = warp_inst[head]
+    t_k = med[head]
+    bytes_launch = 512 * n_fft                       # algorithmic: read x, write X once
+    hbm_peak = float(peaks["hbm_gbs"])
+    body = {k: (warp_inst[k] - W * 2) / n_fft for k in warp_inst}   # per-transform (prologue/exit excluded, approx)
+    return {"metric": METRIC, "value": ev_launch * args.steps / sum(res[head]), "unit": "events/s", "n_gpus": 1,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * sum(res[head]) / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": f"F4 WFFT32 emulation: {n_fft} warp-wide 32-point FFTs, grid {ctas} CTAs, tools "
+                                   "EMU|BBCOUNT|MEMDIV", "n_fft": n_fft, "ctas": ctas,
+                       "l2": "inputs+outputs 2 x n_fft x 256 B > L2, no flush"},
+            "fft_per_s": {k: n_fft / v for k, v in med.items()},
+            "ms_per_launch": {k: 1e3 * v for k, v in med.items()},
+            "slowdown_vs_sw_plain": {k: v / med["sw_plain"] for k, v in med.items()},
+            "warp_instr_per_launch": warp_inst,
+            "warp_instr_per_fft_approx": body,
+            "roofline": {"bound": "hbm", "achieved": bytes_launch / t_k / 1e9, "peak": hbm_peak, "unit": "GB/s",
+                         "frac": bytes_launch / t_k / 1e9 / hbm_peak, "traffic": None,
+                         "algorithmic_bytes_per_launch": bytes_launch},
+            "sw_plain_hbm_frac": bytes_launch / med["sw_plain"] / 1e9 / hbm_peak,
+            "clocks": clk.summary(), "peaks_source": peaks_src,
+            "paper_context": "21 vs 150 instructions per warp with and without WFFT32 (P:L295), parity-unpinned"}
+
+
 def run_reference(args):
     """Reference arm = the CPU oracle (this tier has no runnable reference)."""
     rank = int(os.environ.get("RANK", "0"))
@@ -682,7 +739,9 @@ def main():
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--workload", choices=["c1", "c2", "c3", "c4", "c5", "f1", "f2"], default="c2")
+    ap.add_argument("--workload", choices=["c1", "c2", "c3", "c4", "c5", "f1", "f2", "f4"], default="c2")
+    ap.add_argument("--fft-n", type=int, default=1 << 24, help="F4: transforms per launch")
+    ap.add_argument("--fft-ctas", type=int, default=148 * 8, help="F4: grid (persistent CTAs)")
     ap.add_argument("--f2-iters", type=int, default=10, help="F2: stencil iterations kept in the HBM ring")
     ap.add_argument("--bfs-scale", type=int, default=20)
     ap.add_argument("--stencil-n", type=int, default=8192)

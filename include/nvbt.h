@@ -52,7 +52,9 @@ enum nvbt_tools {
   NVBT_TOOL_COUNT = 1,    /* a hook at every pc: counts, opcode and BB histograms */
   NVBT_TOOL_BBCOUNT = 2,  /* hooks only at BB leaders and guarded pcs; per-pc counts derived */
   NVBT_TOOL_MEMDIV = 4,   /* hooks at global-memory pcs: sector/line divergence */
-  NVBT_TOOL_TRACE = 8     /* hooks at global-memory pcs: one 288 B record per executed event (EM §5) */
+  NVBT_TOOL_TRACE = 8,    /* hooks at global-memory pcs: one 288 B record per executed event (EM §5) */
+  NVBT_TOOL_EMU = 16      /* replace proxy instructions by their emulation function (F4, §6.3 P:L286-295;
+                             only the WFFT32 proxy kernel has one, EM §3.6) */
 };
 
 enum nvbt_kind { NVBT_K_ALU = 0, NVBT_K_CTRL = 1, NVBT_K_GLD = 2, NVBT_K_GST = 3, NVBT_K_GATOM = 4,

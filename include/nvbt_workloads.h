@@ -18,7 +18,7 @@ extern "C" {
 #endif
 
 enum nvbt_workload { NVBT_W_VECTORADD = 1, NVBT_W_SGEMM = 2, NVBT_W_BFS = 3, NVBT_W_STENCIL = 4,
-                     NVBT_W_REPLAY = 5 };
+                     NVBT_W_REPLAY = 5, NVBT_W_WFFT_EMU = 6, NVBT_W_WFFT_SW = 7 };
 
 /* Copies a workload's program table (EM §3.1-3.5) into out[cap]; *n_pcs, *n_opcodes, *n_bbs receive
  * its sizes (any may be null). EINVAL if cap is too small (with *n_pcs still set). Host-only. */
@@ -26,7 +26,7 @@ int nvbt_program(int workload, nvbt_instr_desc* out, uint32_t cap, uint32_t* n_p
                  uint32_t* n_opcodes, uint32_t* n_bbs);
 
 /* Global warp count of one launch (for sizing PER_WARP contexts). Host-only.
- * args: VECTORADD {N}; SGEMM {M, N}; BFS {n}; STENCIL {n}. */
+ * args: VECTORADD {N}; SGEMM {M, N}; BFS {n}; STENCIL {n}; WFFT_EMU / WFFT_SW {n_fft, ctas}. */
 int nvbt_workload_warps(int workload, const int64_t* args, uint32_t n_args, uint64_t* n_warps);
 
 /* C1: c[i] = a[i] + b[i], i < N; CTA 256, grid ceil(N/256) (EM §3.1). ctx may be NULL when tools == 0
@@ -44,6 +44,21 @@ int nvbt_bfs_level(nvbt_ctx ctx, void* stream, uint32_t tools, const int32_t* ro
                    int32_t* over, int32_t level);
 /* C4: one Jacobi iteration out = stencil(in) on an n x n fp32 grid (EM §3.4). */
 int nvbt_stencil(nvbt_ctx ctx, void* stream, uint32_t tools, const float* in, float* out, int32_t n);
+
+/* F4, instruction emulation (§6.3; EM §3.6): n_fft warp-wide 32-point FFTs.
+ * x, X: caller-owned device arrays of n_fft x 32 complex64 (interleaved fp32 re, im; 256 B per transform,
+ * 16 B aligned), x and X must not overlap. CTA 256 threads, grid `ctas` (>= 1; part of the event model:
+ * warp w computes transforms w, w + 8 ctas, ...). variant NVBT_WFFT_PROXY runs program WFFT_EMU (the
+ * kernel using the hypothetical WFFT32 instruction, Listing 10 analogue): with NVBT_TOOL_EMU in `tools`
+ * the instruction is replaced by its emulation function (Listing 9's wfft32emu: lane k receives
+ * X[k] = sum_n x[n] exp(-2 pi i n k / 32)); without it the proxy executes natively as a 64-bit register
+ * move, so X = x. variant NVBT_WFFT_SOFTWARE runs program WFFT_SW (the same transform written in CUDA,
+ * radix-2 DIF over warp shuffles; NVBT_TOOL_EMU is EINVAL there). Both compute bit-identical transforms
+ * in fp32. The other tool bits instrument the launch as for every workload (ctx must hold the matching
+ * program); tools in {0, NVBT_TOOL_EMU} need no context (stream is used). */
+enum nvbt_wfft_variant { NVBT_WFFT_PROXY = 0, NVBT_WFFT_SOFTWARE = 1 };
+int nvbt_wfft32(nvbt_ctx ctx, void* stream, uint32_t tools, int32_t variant, const void* x, void* X,
+                int32_t n_fft, int32_t ctas);
 
 #ifdef __cplusplus
 }

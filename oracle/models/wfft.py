@@ -44,6 +44,8 @@ def transforms_per_warp(n_fft, ctas):
 
 def run(acc, variant, n_fft, ctas, x_ptr, X_ptr, launch=0, warps=None):
     """Events of one launch of program WFFT_EMU (variant EMU) or WFFT_SW (variant SW), §3.6."""
+    if n_fft == 0:                                        # nothing is launched (§3.6)
+        return
     W = n_warps(ctas)
     if warps is None:
         warps = np.arange(W)

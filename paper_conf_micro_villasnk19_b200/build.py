@@ -8,7 +8,7 @@ import sys
 HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
-SOURCES = ["nvbt_core.cu", "channel.cu", "workloads.cu", "replay.cu"]
+SOURCES = ["nvbt_core.cu", "channel.cu", "workloads.cu", "replay.cu", "wfft.cu"]
 OUT = os.path.join(HERE, "libnvbt.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo", "-O3", "-std=c++17",

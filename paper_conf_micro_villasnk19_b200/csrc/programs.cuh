@@ -6,9 +6,12 @@
 
 namespace nvbt {
 namespace op {
-enum : uint16_t { S2R = 0, IMAD, ISETP, EXIT, IMAD_WIDE, LDG, STG, FADD, FFMA, MOV, IADD, BRA, SEL };
+enum : uint16_t { S2R = 0, IMAD, ISETP, EXIT, IMAD_WIDE, LDG, STG, FADD, FFMA, MOV, IADD, BRA, SEL,
+                  // §3.6 (F4)
+                  SHFL, FMUL, LOP3, I2F, MUFU_SIN, MUFU_COS, FSEL, BREV, SHF, WFFT32 };
 }
 constexpr uint32_t kWorkloadOpcodes = 16;
+constexpr uint32_t kWfftOpcodes = 32;
 constexpr uint8_t ALU = NVBT_K_ALU, CTRL = NVBT_K_CTRL, GLD = NVBT_K_GLD, GST = NVBT_K_GST;
 
 #define NVBT_D(o, k, w, b, l, g) nvbt_instr_desc{op::o, k, w, b, l, g, 0}
@@ -73,6 +76,44 @@ struct ProgStencil {  // §3.4
       NVBT_D(FADD, ALU, 0, 1, 0, 1),  NVBT_D(FFMA, ALU, 0, 1, 0, 1),  NVBT_D(SEL, ALU, 0, 1, 0, 0),
       NVBT_D(STG, GST, 4, 1, 0, 0),   NVBT_D(EXIT, CTRL, 0, 1, 0, 0)};
 };
+// §3.6 (F4): the kernel that uses the proxy instruction WFFT32 (Listing 10 analogue)
+struct ProgWfftEmu {
+  static constexpr int N = 14;
+  static constexpr int REG_LO = 5, REG_HI = 12;
+  static constexpr nvbt_instr_desc t[N] = {
+      NVBT_D(S2R, ALU, 0, 0, 1, 0),       NVBT_D(S2R, ALU, 0, 0, 0, 0),  NVBT_D(IMAD, ALU, 0, 0, 0, 0),
+      NVBT_D(ISETP, ALU, 0, 0, 0, 0),     NVBT_D(EXIT, CTRL, 0, 0, 0, 1),
+      NVBT_D(IMAD_WIDE, ALU, 0, 1, 1, 0), NVBT_D(LDG, GLD, 8, 1, 0, 0),  NVBT_D(WFFT32, ALU, 0, 1, 0, 0),
+      NVBT_D(IMAD_WIDE, ALU, 0, 1, 0, 0), NVBT_D(STG, GST, 8, 1, 0, 0),  NVBT_D(IADD, ALU, 0, 1, 0, 0),
+      NVBT_D(ISETP, ALU, 0, 1, 0, 0),     NVBT_D(BRA, CTRL, 0, 1, 0, 1),
+      NVBT_D(EXIT, CTRL, 0, 2, 1, 0)};
+};
+
+// §3.6 (F4): the same transform written in CUDA (radix-2 DIF over shuffles)
+#define NVBT_TW(b, l) NVBT_D(LOP3, ALU, 0, b, l, 0), NVBT_D(LOP3, ALU, 0, b, 0, 0), NVBT_D(ISETP, ALU, 0, b, 0, 0), \
+    NVBT_D(I2F, ALU, 0, b, 0, 0), NVBT_D(MUFU_SIN, ALU, 0, b, 0, 0), NVBT_D(MUFU_COS, ALU, 0, b, 0, 0),            \
+    NVBT_D(FSEL, ALU, 0, b, 0, 0), NVBT_D(FSEL, ALU, 0, b, 0, 0)
+#define NVBT_ST(b) NVBT_D(SHFL, ALU, 0, b, 0, 0), NVBT_D(SHFL, ALU, 0, b, 0, 0), NVBT_D(FFMA, ALU, 0, b, 0, 0), \
+    NVBT_D(FFMA, ALU, 0, b, 0, 0), NVBT_D(FMUL, ALU, 0, b, 0, 0), NVBT_D(FFMA, ALU, 0, b, 0, 0),              \
+    NVBT_D(FMUL, ALU, 0, b, 0, 0), NVBT_D(FFMA, ALU, 0, b, 0, 0)
+struct ProgWfftSw {
+  static constexpr int N = 83;
+  static constexpr int REG_LO = 39, REG_HI = 81;
+  static constexpr nvbt_instr_desc t[N] = {
+      NVBT_D(S2R, ALU, 0, 0, 1, 0), NVBT_D(S2R, ALU, 0, 0, 0, 0), NVBT_D(IMAD, ALU, 0, 0, 0, 0),
+      NVBT_D(ISETP, ALU, 0, 0, 0, 0), NVBT_D(EXIT, CTRL, 0, 0, 0, 1),
+      NVBT_TW(1, 1), NVBT_TW(1, 0), NVBT_TW(1, 0), NVBT_TW(1, 0),
+      NVBT_D(BREV, ALU, 0, 1, 0, 0), NVBT_D(SHF, ALU, 0, 1, 0, 0),
+      NVBT_D(IMAD_WIDE, ALU, 0, 2, 1, 0), NVBT_D(LDG, GLD, 8, 2, 0, 0),
+      NVBT_ST(2), NVBT_ST(2), NVBT_ST(2), NVBT_ST(2),
+      NVBT_D(SHFL, ALU, 0, 2, 0, 0), NVBT_D(SHFL, ALU, 0, 2, 0, 0), NVBT_D(FFMA, ALU, 0, 2, 0, 0),
+      NVBT_D(FFMA, ALU, 0, 2, 0, 0),
+      NVBT_D(IMAD_WIDE, ALU, 0, 2, 0, 0), NVBT_D(STG, GST, 8, 2, 0, 0), NVBT_D(IADD, ALU, 0, 2, 0, 0),
+      NVBT_D(ISETP, ALU, 0, 2, 0, 0), NVBT_D(BRA, CTRL, 0, 2, 0, 1),
+      NVBT_D(EXIT, CTRL, 0, 3, 1, 0)};
+};
+#undef NVBT_TW
+#undef NVBT_ST
 #undef NVBT_D
 
 }  // namespace nvbt

@@ -667,6 +667,8 @@ int nvbt_program(int w, nvbt_instr_desc* out, uint32_t cap, uint32_t* n_pcs, uin
     case NVBT_W_SGEMM: t = ProgSgemm::t; n = ProgSgemm::N; break;
     case NVBT_W_BFS: t = ProgBfs::t; n = ProgBfs::N; break;
     case NVBT_W_STENCIL: t = ProgStencil::t; n = ProgStencil::N; break;
+    case NVBT_W_WFFT_EMU: t = ProgWfftEmu::t; n = ProgWfftEmu::N; o = kWfftOpcodes; break;
+    case NVBT_W_WFFT_SW: t = ProgWfftSw::t; n = ProgWfftSw::N; o = kWfftOpcodes; break;
     case NVBT_W_REPLAY:
       if (!replay_built) {  // EM §3.5, always from the constant SEED
         const unsigned long long k100 = Kf(kSeed, 100);

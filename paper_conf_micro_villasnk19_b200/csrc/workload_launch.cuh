@@ -1,0 +1,48 @@
+// Launch helpers shared by the workload translation units (workloads.cu, wfft.cu).
+#pragma once
+#include <type_traits>
+
+#include "nvbt_internal.h"
+
+namespace nvbt {
+
+// ---------------------------------------------------------------- dispatch over tool variants
+template <class F>
+static inline int dispatch(uint32_t tools, F&& f) {
+#define NVBT_CASE(v) case v: f(std::integral_constant<uint32_t, v>{}); return NVBT_OK;
+  switch (tools) {
+    NVBT_CASE(0) NVBT_CASE(1) NVBT_CASE(2) NVBT_CASE(4) NVBT_CASE(5) NVBT_CASE(6) NVBT_CASE(8) NVBT_CASE(9)
+    NVBT_CASE(10) NVBT_CASE(12) NVBT_CASE(13) NVBT_CASE(14)
+    default: return set_error(NVBT_EINVAL, "unsupported tools combination 0x%x", tools);
+  }
+#undef NVBT_CASE
+}
+
+struct LaunchCtx {
+  cudaStream_t stream = nullptr;
+  DevState st{};
+};
+
+template <class Prog>
+static inline int prepare(nvbt_ctx ctx, void* stream, uint32_t tools, const char* name, LaunchCtx* lc) {
+  if (tools != 0) {
+    if (!ctx) return set_error(NVBT_EINVAL, "instrumented launch needs a context");
+    int rc = check_program(ctx, Prog::t, Prog::N, name);
+    if (rc) return rc;
+    rc = make_state(ctx, tools, &lc->st);
+    if (rc) return rc;
+    lc->stream = ctx->stream;
+    NVBT_CUDA(cudaSetDevice(ctx->device));
+  } else {
+    lc->stream = ctx ? ctx->stream : static_cast<cudaStream_t>(stream);
+  }
+  return NVBT_OK;
+}
+
+static inline int done(nvbt_ctx ctx, int n_kernels) {
+  NVBT_CUDA(cudaGetLastError());
+  if (ctx) ctx->launches += n_kernels;
+  return NVBT_OK;
+}
+
+}  // namespace nvbt

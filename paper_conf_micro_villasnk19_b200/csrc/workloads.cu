@@ -10,6 +10,7 @@
 #include "nvbt_internal.h"
 #include "nvbt_workloads.h"
 #include "programs.cuh"
+#include "workload_launch.cuh"
 
 namespace nvbt {
 
@@ -199,45 +200,6 @@ __global__ void __launch_bounds__(256) k_stencil(const float* __restrict__ in, f
   h.finish();
 }
 
-// ---------------------------------------------------------------- dispatch over tool variants
-template <class F>
-static int dispatch(uint32_t tools, F&& f) {
-#define NVBT_CASE(v) case v: f(std::integral_constant<uint32_t, v>{}); return NVBT_OK;
-  switch (tools) {
-    NVBT_CASE(0) NVBT_CASE(1) NVBT_CASE(2) NVBT_CASE(4) NVBT_CASE(5) NVBT_CASE(6) NVBT_CASE(8) NVBT_CASE(9)
-    NVBT_CASE(10) NVBT_CASE(12) NVBT_CASE(13) NVBT_CASE(14)
-    default: return set_error(NVBT_EINVAL, "unsupported tools combination 0x%x", tools);
-  }
-#undef NVBT_CASE
-}
-
-struct LaunchCtx {
-  cudaStream_t stream = nullptr;
-  DevState st{};
-};
-
-template <class Prog>
-static int prepare(nvbt_ctx ctx, void* stream, uint32_t tools, const char* name, LaunchCtx* lc) {
-  if (tools != 0) {
-    if (!ctx) return set_error(NVBT_EINVAL, "instrumented launch needs a context");
-    int rc = check_program(ctx, Prog::t, Prog::N, name);
-    if (rc) return rc;
-    rc = make_state(ctx, tools, &lc->st);
-    if (rc) return rc;
-    lc->stream = ctx->stream;
-    NVBT_CUDA(cudaSetDevice(ctx->device));
-  } else {
-    lc->stream = ctx ? ctx->stream : static_cast<cudaStream_t>(stream);
-  }
-  return NVBT_OK;
-}
-
-static int done(nvbt_ctx ctx, int n_kernels) {
-  NVBT_CUDA(cudaGetLastError());
-  if (ctx) ctx->launches += n_kernels;
-  return NVBT_OK;
-}
-
 }  // namespace nvbt
 
 using namespace nvbt;
@@ -258,6 +220,9 @@ int nvbt_workload_warps(int w, const int64_t* a, uint32_t na, uint64_t* n) {
     case NVBT_W_STENCIL:
       if (na < 1 || a[0] < 0) break;
       *n = (uint64_t)((a[0] + 31) / 32) * (uint64_t)((a[0] + 7) / 8) * 8; return NVBT_OK;
+    case NVBT_W_WFFT_EMU: case NVBT_W_WFFT_SW:
+      if (na < 2 || a[0] < 0 || a[1] < 1) break;
+      *n = (uint64_t)a[1] * 8; return NVBT_OK;
     default: break;
   }
   return set_error(NVBT_EINVAL, "bad workload %d or arguments", w);

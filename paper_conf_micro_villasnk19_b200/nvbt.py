@@ -22,8 +22,9 @@ _lib = C.CDLL(LIB_PATH)
 ABI_VERSION = 1
 OK, EINVAL, ESTATE, ENOMEM, ECUDA, ETIMEDOUT, EVERSION = 0, -1, -2, -3, -4, -5, -6
 COUNT, OPHIST, BB, MEMDIV, PER_WARP, TRACE = 1, 2, 4, 8, 16, 32
-TOOL_NONE, TOOL_COUNT, TOOL_BBCOUNT, TOOL_MEMDIV, TOOL_TRACE = 0, 1, 2, 4, 8
-W_VECTORADD, W_SGEMM, W_BFS, W_STENCIL, W_REPLAY = 1, 2, 3, 4, 5
+TOOL_NONE, TOOL_COUNT, TOOL_BBCOUNT, TOOL_MEMDIV, TOOL_TRACE, TOOL_EMU = 0, 1, 2, 4, 8, 16
+W_VECTORADD, W_SGEMM, W_BFS, W_STENCIL, W_REPLAY, W_WFFT_EMU, W_WFFT_SW = 1, 2, 3, 4, 5, 6, 7
+WFFT_PROXY, WFFT_SOFTWARE = 0, 1
 RECORD_BYTES = 288
 COMPACT_RECORD_BYTES = 176
 
@@ -95,6 +96,7 @@ _sigs = {
     "nvbt_sgemm": ([_P, _P, C.c_uint32, _P, _P, _P, C.c_int32, C.c_int32, C.c_int32], C.c_int),
     "nvbt_bfs_level": ([_P, _P, C.c_uint32, _P, _P, C.c_int32, _P, _P, _P, _P, _P, C.c_int32], C.c_int),
     "nvbt_stencil": ([_P, _P, C.c_uint32, _P, _P, C.c_int32], C.c_int),
+    "nvbt_wfft32": ([_P, _P, C.c_uint32, C.c_int32, _P, _P, C.c_int32, C.c_int32], C.c_int),
 }
 for _name, (_args, _res) in _sigs.items():
     _f = getattr(_lib, _name)
@@ -404,3 +406,8 @@ def nvbt_bfs_level(ctx, tools, rowptr, col, n, mask, visited, updating, cost, ov
 
 def nvbt_stencil(ctx, tools, inp, out, n, stream=None):
     _check(_lib.nvbt_stencil(_h(ctx), _s(ctx, stream), tools, _ptr(inp), _ptr(out), n))
+
+
+def nvbt_wfft32(ctx, tools, variant, x, X, n_fft, ctas, stream=None):
+    """F4 (EM §3.6): n_fft 32-point FFTs of x (complex64 CUDA tensor [n_fft, 32]) into X."""
+    _check(_lib.nvbt_wfft32(_h(ctx), _s(ctx, stream), tools, variant, _ptr(x), _ptr(X), n_fft, ctas))

@@ -35,7 +35,8 @@ def test_binding_covers_declared_symbols():
     assert nb.nvbt_abi_version() == 1
 
 
-@pytest.mark.parametrize("w,name", [(1, "vectoradd"), (2, "sgemm"), (3, "bfs"), (4, "stencil"), (5, "replay")])
+@pytest.mark.parametrize("w,name", [(1, "vectoradd"), (2, "sgemm"), (3, "bfs"), (4, "stencil"), (5, "replay"),
+                                    (6, "wfft_emu"), (7, "wfft_sw")])
 def test_program_tables_match_oracle_transcription(w, name):
     """Both sides transcribe docs/EVENT_MODEL.md §3 independently; the tables must agree."""
     from paper_conf_micro_villasnk19_b200 import nvbt as nb
