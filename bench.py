@@ -648,22 +648,24 @@ def run_f4(args, torch, nb, dr, local):
     g = torch.Generator(device="cuda").manual_seed(9)
     x = (torch.rand((n_fft, 32, 2), generator=g, device="cuda") * 2 - 1).view(torch.complex64).reshape(n_fft, 32)
     X = torch.empty_like(x)
-    W = 8 * ctas
     flags = nb.COUNT | nb.OPHIST | nb.BB | nb.MEMDIV
     cemu, csw = nb.nvbt_init(nb.W_WFFT_EMU, flags), nb.nvbt_init(nb.W_WFFT_SW, flags)
     P, S = nb.WFFT_PROXY, nb.WFFT_SOFTWARE
     modes = {
+        "proxy_plain": (cemu, P, nb.TOOL_NONE),   # native proxy = register move: a pure copy (memory bound)
         "sw_plain": (csw, S, nb.TOOL_NONE), "emu_only": (cemu, P, nb.TOOL_EMU),
         "sw_bbcount_memdiv": (csw, S, nb.TOOL_BBCOUNT | nb.TOOL_MEMDIV),
         "emu_bbcount_memdiv": (cemu, P, nb.TOOL_EMU | nb.TOOL_BBCOUNT | nb.TOOL_MEMDIV),
         "sw_count": (csw, S, nb.TOOL_COUNT), "emu_count": (cemu, P, nb.TOOL_EMU | nb.TOOL_COUNT),
     }
-    res, warp_inst = {}, {}
+    res, warp_inst, grids = {}, {}, {}
     for name, (ctx, v, t) in modes.items():
-        f = lambda: nb.nvbt_wfft32(ctx, t, v, x, X, n_fft, ctas)
+        g_ctas = ctas if ctas > 0 else nb.nvbt_wfft32_max_ctas(t, v, local)   # one resident wave
+        grids[name] = g_ctas
+        f = lambda: nb.nvbt_wfft32(ctx, t, v, x, X, n_fft, g_ctas)
         _timed_events(torch, f, args.warmup)
         nb.nvbt_reset(ctx)
-        if name == "emu_bbcount_memdiv":
+        if name == "emu_count":
             with ClockSampler(local) as clk:
                 res[name] = _timed_events(torch, f, args.steps)
         else:
@@ -671,17 +673,17 @@ def run_f4(args, torch, nb, dr, local):
         if t & (nb.TOOL_COUNT | nb.TOOL_BBCOUNT):
             warp_inst[name] = int(nb.nvbt_count(ctx)[2]) // args.steps
     med = {k: statistics.median(v) for k, v in res.items()}
-    head = "emu_bbcount_memdiv"
+    head = "emu_count"          # the paper's combination: emulation + the instruction-count tool
     ev_launch = warp_inst[head]
     t_k = med[head]
     bytes_launch = 512 * n_fft                       # algorithmic: read x, write X once
     hbm_peak = float(peaks["hbm_gbs"])
-    body = {k: (warp_inst[k] - W * 2) / n_fft for k in warp_inst}   # per-transform (prologue/exit excluded, approx)
+    body = {k: warp_inst[k] / n_fft for k in warp_inst}   # per transform (incl. the per-warp prologue share)
     return {"metric": METRIC, "value": ev_launch * args.steps / sum(res[head]), "unit": "events/s", "n_gpus": 1,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * sum(res[head]) / args.steps,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-            "config": {"workload": f"F4 WFFT32 emulation: {n_fft} warp-wide 32-point FFTs, grid {ctas} CTAs, tools "
-                                   "EMU|BBCOUNT|MEMDIV", "n_fft": n_fft, "ctas": ctas,
+            "config": {"workload": f"F4 WFFT32 emulation: {n_fft} warp-wide 32-point FFTs, persistent grid "
+                                   "(one resident wave), tools EMU|COUNT", "n_fft": n_fft, "ctas": grids,
                        "l2": "inputs+outputs 2 x n_fft x 256 B > L2, no flush"},
             "fft_per_s": {k: n_fft / v for k, v in med.items()},
             "ms_per_launch": {k: 1e3 * v for k, v in med.items()},
@@ -689,8 +691,10 @@ def run_f4(args, torch, nb, dr, local):
             "warp_instr_per_launch": warp_inst,
             "warp_instr_per_fft_approx": body,
             "roofline": {"bound": "hbm", "achieved": bytes_launch / t_k / 1e9, "peak": hbm_peak, "unit": "GB/s",
-                         "frac": bytes_launch / t_k / 1e9 / hbm_peak, "traffic": None,
-                         "algorithmic_bytes_per_launch": bytes_launch},
+                         "frac": bytes_launch / t_k / 1e9 / hbm_peak,
+                         "traffic": (load_traffic("k_wfft<17,0>") or {}).get("traffic_bytes_per_launch"),
+                         "traffic_unit": "DRAM bytes per launch (ncu, profiles/r1_traffic.json)",
+                         "algorithmic_bytes_per_launch": bytes_launch, "kernel": "k_wfft<EMU|COUNT, proxy>"},
             "sw_plain_hbm_frac": bytes_launch / med["sw_plain"] / 1e9 / hbm_peak,
             "clocks": clk.summary(), "peaks_source": peaks_src,
             "paper_context": "21 vs 150 instructions per warp with and without WFFT32 (P:L295), parity-unpinned"}
@@ -741,7 +745,7 @@ def main():
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--workload", choices=["c1", "c2", "c3", "c4", "c5", "f1", "f2", "f4"], default="c2")
     ap.add_argument("--fft-n", type=int, default=1 << 24, help="F4: transforms per launch")
-    ap.add_argument("--fft-ctas", type=int, default=148 * 8, help="F4: grid (persistent CTAs)")
+    ap.add_argument("--fft-ctas", type=int, default=0, help="F4: grid (0 = one resident wave per kernel)")
     ap.add_argument("--f2-iters", type=int, default=10, help="F2: stencil iterations kept in the HBM ring")
     ap.add_argument("--bfs-scale", type=int, default=20)
     ap.add_argument("--stencil-n", type=int, default=8192)

@@ -59,6 +59,9 @@ int nvbt_stencil(nvbt_ctx ctx, void* stream, uint32_t tools, const float* in, fl
 enum nvbt_wfft_variant { NVBT_WFFT_PROXY = 0, NVBT_WFFT_SOFTWARE = 1 };
 int nvbt_wfft32(nvbt_ctx ctx, void* stream, uint32_t tools, int32_t variant, const void* x, void* X,
                 int32_t n_fft, int32_t ctas);
+/* *ctas = SMs of `device` x resident CTAs per SM of the kernel that (tools, variant) selects: the grid
+ * that keeps every warp of a persistent launch resident (one wave). EINVAL as nvbt_wfft32 for tools. */
+int nvbt_wfft32_max_ctas(uint32_t tools, int32_t variant, int32_t device, int32_t* ctas);
 
 #ifdef __cplusplus
 }

@@ -187,7 +187,8 @@ static __device__ __noinline__ uint2 sectors_lines_unsorted_call(unsigned long l
 // where a lane's sector (line) differs from the previous lane of E — compared as (a ^ prev) >> 5 (7).
 // kApFirst: for a full warp, first try an arithmetic progression a_l = min + l d detected with warp
 // reductions (no shuffles: the instrumented application kernels are L1-bound, and shuffles share the
-// L1/MIO datapath with their loads); otherwise the previous lane's address comes from 2 shuffles.
+// L1/MIO datapath with their loads), whose S and L have a closed form in (min, max, d); otherwise the
+// previous lane's address comes from 2 shuffles.
 // Other orders take the slow paths above (inlined when kInlineSlow, else an out-of-line call to keep the
 // hooks' registers and code small).
 template <bool kInlineSlow = false, bool kApFirst = true>
@@ -202,9 +203,11 @@ __device__ __forceinline__ void sectors_lines(unsigned long long addr, unsigned 
     const unsigned mn = __reduce_min_sync(FULL, a_lo), mx = __reduce_max_sync(FULL, a_lo);
     const unsigned dd = (mx - mn) / 31u;
     if (hmn == hmx && __all_sync(FULL, a_lo == mn + lane * dd)) {
-      const unsigned x = a_lo ^ (a_lo - dd);         // vs the previous lane's address
-      S = 1u + __popc(__ballot_sync(FULL, lane != 0u && (x & ~31u) != 0u));
-      L = 1u + __popc(__ballot_sync(FULL, lane != 0u && (x & ~127u) != 0u));
+      // closed form, warp-uniform arithmetic only: a step d < 32 (< 128) can skip no sector (line), so
+      // the distinct sectors (lines) are every one from mn's to mx's; a step >= 32 (>= 128) puts every
+      // lane in its own sector (line)
+      S = dd >= 32u ? 32u : (mx >> 5) - (mn >> 5) + 1u;
+      L = dd >= 128u ? 32u : (mx >> 7) - (mn >> 7) + 1u;
       return;
     }
   }

@@ -97,6 +97,7 @@ _sigs = {
     "nvbt_bfs_level": ([_P, _P, C.c_uint32, _P, _P, C.c_int32, _P, _P, _P, _P, _P, C.c_int32], C.c_int),
     "nvbt_stencil": ([_P, _P, C.c_uint32, _P, _P, C.c_int32], C.c_int),
     "nvbt_wfft32": ([_P, _P, C.c_uint32, C.c_int32, _P, _P, C.c_int32, C.c_int32], C.c_int),
+    "nvbt_wfft32_max_ctas": ([C.c_uint32, C.c_int32, C.c_int32, C.POINTER(C.c_int32)], C.c_int),
 }
 for _name, (_args, _res) in _sigs.items():
     _f = getattr(_lib, _name)
@@ -411,3 +412,10 @@ def nvbt_stencil(ctx, tools, inp, out, n, stream=None):
 def nvbt_wfft32(ctx, tools, variant, x, X, n_fft, ctas, stream=None):
     """F4 (EM §3.6): n_fft 32-point FFTs of x (complex64 CUDA tensor [n_fft, 32]) into X."""
     _check(_lib.nvbt_wfft32(_h(ctx), _s(ctx, stream), tools, variant, _ptr(x), _ptr(X), n_fft, ctas))
+
+
+def nvbt_wfft32_max_ctas(tools, variant, device=0):
+    """Grid of one resident wave for the kernel (tools, variant) selects."""
+    n = C.c_int32()
+    _check(_lib.nvbt_wfft32_max_ctas(tools, variant, device, C.byref(n)))
+    return n.value

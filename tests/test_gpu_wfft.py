@@ -116,31 +116,37 @@ def test_wfft_special_inputs(nvbt):
 
 
 def test_wfft_bench_config_sampled(nvbt):
-    """The launch configuration bench.py times (n_fft = 2^24, ctas = 148 * 8): closed-form totals, the
-    oracle's events on sampled warps (PER_WARP) and sampled transforms against the DFT."""
+    """The launch configuration bench.py times (n_fft = 2^24, one resident wave of CTAs): closed-form
+    totals, the oracle's events on sampled warps (PER_WARP) and sampled transforms against the DFT."""
     import torch
     nb = nvbt.nvbt
-    n_fft, ctas = 1 << 24, 148 * 8
-    W = 8 * ctas
+    n_fft = 1 << 24
     x, X = inputs(n_fft, seed=7)
-    for v, w, body, pre_i, pre_e in ((nb.WFFT_PROXY, nb.W_WFFT_EMU, 8, 6, 4), (nb.WFFT_SOFTWARE, nb.W_WFFT_SW, 43, 40, 38)):
+    cases = [(v, w, body, pre_i, pre_e, ct | (nb.TOOL_EMU if v == nb.WFFT_PROXY else 0))
+             for v, w, body, pre_i, pre_e in ((nb.WFFT_PROXY, nb.W_WFFT_EMU, 8, 6, 4),
+                                              (nb.WFFT_SOFTWARE, nb.W_WFFT_SW, 43, 40, 38))
+             for ct in (nb.TOOL_COUNT, nb.TOOL_BBCOUNT | nb.TOOL_MEMDIV)]
+    for v, w, body, pre_i, pre_e, t in cases:       # EMU|COUNT is the bench's timed launch
+        ctas = nb.nvbt_wfft32_max_ctas(t, v)
+        assert ctas % 148 == 0
+        W = 8 * ctas
         ctx = nb.nvbt_init(w, nb.COUNT | nb.OPHIST | nb.BB | nb.MEMDIV | nb.PER_WARP, n_warps=W)
-        t = nb.TOOL_BBCOUNT | nb.TOOL_MEMDIV | (nb.TOOL_EMU if v == nb.WFFT_PROXY else 0)
         X.zero_()
         nb.nvbt_wfft32(ctx, t, v, x, X, n_fft, ctas)
         g = read_all(nb, ctx, per_warp=True)
         k = np.array([len(range(i, n_fft, W)) for i in range(W)])
         assert g["counts"][2] == (pre_i + body * k).sum() and g["counts"][3] == (pre_e + body * k).sum()
         assert g["counts"][1] == 32 * g["counts"][3]
-        sample = np.array([0, 1, 7, 8, 4095, W // 2, W - 1])
+        sample = np.array([0, 1, 7, 8, W // 3, W // 2, W - 1])
         acc = ev.Accumulator(programs.wfft_emu() if v == nb.WFFT_PROXY else programs.wfft_sw(), n_warps=W)
         m_wf.run(acc, m_wf.EMU if v == nb.WFFT_PROXY else m_wf.SW, n_fft, ctas, x.data_ptr(), X.data_ptr(),
                  warps=sample)
         r = acc.result()
         assert (g["PW_W"][sample] == r["PW_W"][sample]).all() and (g["PW_T"][sample] == r["PW_T"][sample]).all()
-        mem_pcs = [6, 9] if v == nb.WFFT_PROXY else [40, 78]
-        assert (g["mem_n"][mem_pcs] == n_fft).all() and (g["mem_S"][mem_pcs] == 8 * n_fft).all()
-        assert (g["mem_L"][mem_pcs] == 2 * n_fft).all()
+        if t & nb.TOOL_MEMDIV:
+            mem_pcs = [6, 9] if v == nb.WFFT_PROXY else [40, 78]
+            assert (g["mem_n"][mem_pcs] == n_fft).all() and (g["mem_S"][mem_pcs] == 8 * n_fft).all()
+            assert (g["mem_L"][mem_pcs] == 2 * n_fft).all()
         rows = torch.tensor([0, 1, 12345, n_fft // 2, n_fft - 2, n_fft - 1], device="cuda")
         check_values(x[rows], X[rows])
         gpu_invariants(g)

@@ -30,5 +30,18 @@ if which in ("all", "c5"):
     nb.nvbt_gen_events(rctx, 0x4E5642544E564254, 0, n, hdr, addr)
     nb.nvbt_replay(rctx, hdr, addr, n)
     nb.nvbt_count(rctx)
+if which in ("all", "f4"):
+    n_fft = 1 << 24
+    x = (torch.rand((n_fft, 32, 2), device="cuda") * 2 - 1).view(torch.complex64).reshape(n_fft, 32)
+    X = torch.empty_like(x)
+    ce = nb.nvbt_init(nb.W_WFFT_EMU, nb.COUNT | nb.BB | nb.MEMDIV)
+    cs = nb.nvbt_init(nb.W_WFFT_SW, nb.COUNT | nb.BB | nb.MEMDIV)
+    # bench head (EMU|COUNT) first, then the other bench modes
+    for ctx, v, t in ((ce, nb.WFFT_PROXY, nb.TOOL_EMU | nb.TOOL_COUNT), (ce, nb.WFFT_PROXY, nb.TOOL_NONE),
+                      (cs, nb.WFFT_SOFTWARE, nb.TOOL_NONE), (ce, nb.WFFT_PROXY, nb.TOOL_EMU),
+                      (cs, nb.WFFT_SOFTWARE, nb.TOOL_COUNT),
+                      (ce, nb.WFFT_PROXY, nb.TOOL_EMU | nb.TOOL_BBCOUNT | nb.TOOL_MEMDIV)):
+        nb.nvbt_wfft32(ctx, t, v, x, X, n_fft, nb.nvbt_wfft32_max_ctas(t, v))
+    nb.nvbt_count(ce)
 torch.cuda.synchronize()
 print("done")
