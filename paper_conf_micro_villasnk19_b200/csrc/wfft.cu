@@ -10,9 +10,9 @@
 // Both programs compute the transform the same way (radix-2 decimation in frequency over warp shuffles,
 // one complex element per lane, per-lane twiddles computed once per warp), so the emulated and the
 // software kernel produce bit-identical fp32 results. The kernels are persistent: grid `ctas`, warp w
-// handles transforms w, w + W, ... (W = 8 ctas). Inputs stream through a per-warp TMA ring in shared
-// memory (cp.async.bulk + mbarrier, 16 rows ahead) so each SM keeps enough bytes in flight to stream HBM
-// without spending registers. Hooks are called in program order per loop instance (the virtual program
+// handles transforms w, w + W, ... (W = 8 ctas). Inputs stream through a per-warp ring in shared memory
+// (cp.async, 16 rows ahead) so each SM keeps enough bytes in flight to stream HBM without spending
+// registers. Hooks are called in program order per loop instance (the virtual program
 // of EM §3.6); only the data movement is pipelined.
 #include "nvbt_internal.h"
 #include "nvbt_workloads.h"
@@ -104,26 +104,24 @@ __device__ __forceinline__ float2 wfft32emu(float2 v, const WfftLane& c) {
   return v;
 }
 
-// Per-warp TMA ring: the input row of loop instance k lands in slot k % kRing of the warp's ring (one
-// 256 B cp.async.bulk issued by lane 0, completion counted on the slot's mbarrier), kRing - 1 instances
-// ahead of its use. Bytes in flight per SM no longer cost registers: 8 warps x 16 slots x 256 B = 32 KB
-// per CTA. (A CTA-wide ring of 2 KB stages with one producer warp was measured slower: it couples the
-// warps' progress — 1.72 vs 1.57 ms for the software FFT, 2.18 vs 1.94 ms for EMU|COUNT.)
+// Per-warp copy ring: the input row of loop instance k lands in slot k % kRing of the warp's ring,
+// kRing - 1 instances ahead of its use, through cp.async (16 B per lane, lanes 0-15 copy one 256 B row;
+// one commit group per instance, so `cp.async.wait_group kRing - 1` is exactly "row k has landed").
+// Bytes in flight per SM cost no registers: 8 warps x 16 slots x 256 B = 32 KB per CTA. Measured
+// alternatives: a per-warp ring of 256 B cp.async.bulk copies with one mbarrier per slot (same bytes in
+// flight, ~30 more instructions per transform for the barrier phase and the uniform-operand loop around
+// the bulk copy: EMU|COUNT 1.94 ms), and a CTA-wide ring of 2 KB bulk stages with one producer warp (it
+// couples the warps' progress: 2.18 ms).
 constexpr int kRing = 16;
 struct WfftRing {
   float2 slot[8][kRing][32];
-  unsigned long long bar[8][kRing];
 };
 
-__device__ __forceinline__ void ring_issue(unsigned bar, unsigned dst, const float2* src) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], 256;" ::"r"(bar) : "memory");
-  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], 256, [%2];"
-               ::"r"(dst), "l"(src), "r"(bar) : "memory");
-}
-__device__ __forceinline__ void ring_wait(unsigned bar, unsigned parity) {
-  asm volatile("{\n\t.reg .pred p;\n\tWAIT_%=:\n\t"
-               "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t@!p bra WAIT_%=;\n\t}"
-               ::"r"(bar), "r"(parity) : "memory");
+__device__ __forceinline__ void ring_copy(unsigned lane, unsigned dst_row, const float2* src_row, bool on) {
+  if (on && lane < 16u)
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst_row + 16u * lane), "l"(src_row + 2u * lane)
+                 : "memory");
+  asm volatile("cp.async.commit_group;" ::: "memory");
 }
 
 template <uint32_t T, int V>
@@ -158,23 +156,16 @@ __global__ void __launch_bounds__(256) k_wfft(const float2* __restrict__ x, floa
     const int W = (int)gridDim.x * 8;
     const int kw = (n_fft - f0 + W - 1) / W;          // loop instances of this warp (>= 1)
     const unsigned slot0 = (unsigned)__cvta_generic_to_shared(&ring.slot[wib][0][0]);
-    const unsigned bar0 = (unsigned)__cvta_generic_to_shared(&ring.bar[wib][0]);
-    if (lane == 0) {
-#pragma unroll 1
-      for (int d = 0; d < kRing; ++d)
-        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar0 + 8u * d) : "memory");
-      asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-#pragma unroll 1
-      for (int d = 0; d < kRing && d < kw; ++d)
-        ring_issue(bar0 + 8u * d, slot0 + 256u * d, x + (size_t)(f0 + d * W) * 32);
-    }
-    __syncwarp();
+#pragma unroll
+    for (int d = 0; d < kRing; ++d)
+      ring_copy(lane, slot0 + 256u * d, x + (size_t)(f0 + d * W) * 32, d < kw);
 #pragma unroll 1
     for (int k = 0; k < kw; ++k) {                    // warp-uniform: one loop instance per transform
       const int ff = f0 + k * W;
       const unsigned sl = (unsigned)k & (kRing - 1u);
       const float2* px = x + (size_t)ff * 32 + lane;        h.template at<LO>(m1);
-      ring_wait(bar0 + 8u * sl, ((unsigned)k / kRing) & 1u);
+      asm volatile("cp.async.wait_group %0;" ::"n"(kRing - 1) : "memory");   // row k has landed
+      __syncwarp();
       float2 v;
       asm volatile("ld.shared.v2.f32 {%0, %1}, [%2];" : "=f"(v.x), "=f"(v.y) : "r"(slot0 + 256u * sl + 8u * lane) : "memory");
                                                              h.template at<LO + 1>(m1, true, (unsigned long long)px);
@@ -189,15 +180,15 @@ __global__ void __launch_bounds__(256) k_wfft(const float2* __restrict__ x, floa
       }
       float2* pX = X + (size_t)ff * 32 + col;                h.template at<S>(m1);
       __stcs(pX, v);                                         h.template at<S + 1>(m1, true, (unsigned long long)pX);
-      // every lane's slot read has been consumed (the store used it): refill the slot
+      // every lane's slot read has been consumed (the store used it): refill the slot with row k + kRing
       __syncwarp();
-      if (lane == 0 && k + kRing < kw)
-        ring_issue(bar0 + 8u * sl, slot0 + 256u * sl, x + (size_t)(ff + kRing * W) * 32);
+      ring_copy(lane, slot0 + 256u * sl, x + (size_t)(ff + kRing * W) * 32, k + kRing < kw);
                                                              h.template at<S + 2>(m1);
                                                              h.template at<S + 3>(m1);
                                                              h.template at<S + 4>(m1, k + 1 < kw);  // @P1 BRA
     }
   }
+  asm volatile("cp.async.wait_group 0;" ::: "memory");
   h.template at<EXIT_PC>(m1);
   h.finish();
 }
