@@ -42,8 +42,25 @@ int nvbt_sgemm(nvbt_ctx ctx, void* stream, uint32_t tools, const float* A, const
 int nvbt_bfs_level(nvbt_ctx ctx, void* stream, uint32_t tools, const int32_t* rowptr, const int32_t* col,
                    int32_t n, uint8_t* mask, uint8_t* visited, uint8_t* updating, int32_t* cost,
                    int32_t* over, int32_t level);
+/* C3 kernels 1 (expand) and 2 (update) as separate launches, for a multi-GPU BFS that exchanges
+ * `updating` between them and `visited` / `over` after kernel 2. Same arguments and launch
+ * ids as the two halves of nvbt_bfs_level. */
+int nvbt_bfs_expand(nvbt_ctx ctx, void* stream, uint32_t tools, const int32_t* rowptr, const int32_t* col,
+                    int32_t n, uint8_t* mask, const uint8_t* visited, uint8_t* updating);
+int nvbt_bfs_update(nvbt_ctx ctx, void* stream, uint32_t tools, int32_t n, uint8_t* mask, uint8_t* visited,
+                    uint8_t* updating, int32_t* cost, int32_t* over, int32_t level);
 /* C4: one Jacobi iteration out = stencil(in) on an n x n fp32 grid (EM §3.4). */
 int nvbt_stencil(nvbt_ctx ctx, void* stream, uint32_t tools, const float* in, float* out, int32_t n);
+
+/* Multi-GPU partition ("partitioned ... by kernel and warp range"): every later workload
+ * launch through ctx (C1-C4 and F4; not replay, whose event ranges are explicit) runs only rank's share
+ * of its CTA grid. A grid of gy rows of gx CTAs (2D workloads: SGEMM and stencil, gx = ceil(M/32) resp.
+ * ceil(n/32); 1D workloads: gx = 1, gy = CTAs) gives rank r of `world` the whole CTA rows
+ * [floor(gy r / world), floor(gy (r + 1) / world)). Warp ids, addresses and events are those of the
+ * unpartitioned launch (the kernels use the logical CTA id), so the world ranks' accumulators sum to the
+ * single-GPU result (EM §4) and each rank writes only its share of the outputs. A rank with an empty
+ * share still takes the launch id. Default: rank 0 of 1. EINVAL if world == 0 or rank >= world. */
+int nvbt_set_partition(nvbt_ctx ctx, uint32_t rank, uint32_t world);
 
 /* F4, instruction emulation (§6.3; EM §3.6): n_fft warp-wide 32-point FFTs.
  * x, X: caller-owned device arrays of n_fft x 32 complex64 (interleaved fp32 re, im; 256 B per transform,

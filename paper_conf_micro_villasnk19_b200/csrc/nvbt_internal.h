@@ -63,6 +63,7 @@ struct nvbt_ctx_s {
   uint32_t* d_leader = nullptr;
   uint8_t* d_kind = nullptr;
   uint32_t next_launch = 0;
+  uint32_t part_rank = 0, part_world = 1;   // nvbt_set_partition
   std::atomic<uint64_t> launches{0};
   nvbt_chan_s* chan = nullptr;
   std::mutex mu;

@@ -126,7 +126,7 @@ __device__ __forceinline__ void ring_copy(unsigned lane, unsigned dst_row, const
 
 template <uint32_t T, int V>
 __global__ void __launch_bounds__(256) k_wfft(const float2* __restrict__ x, float2* __restrict__ X, int n_fft,
-                                              DevState st) {
+                                              int ctas, DevState st) {
   constexpr uint32_t TH = T & ~TOOL_EMU;
   constexpr bool kEmu = (T & TOOL_EMU) != 0;
   using Prog = std::conditional_t<V == 0, ProgWfftEmu, ProgWfftSw>;
@@ -139,7 +139,7 @@ __global__ void __launch_bounds__(256) k_wfft(const float2* __restrict__ x, floa
   const unsigned lane = threadIdx.x & 31u, wib = threadIdx.x >> 5;
   const auto m0 = h.active(true);
   const int tid = threadIdx.x;                        h.template at<0>(m0);
-  const int cta = blockIdx.x;                         h.template at<1>(m0);
+  const int cta = st.cta_lo + blockIdx.x;            h.template at<1>(m0);   // logical CTA (partition)
   const int f0 = cta * 8 + (tid >> 5);                h.template at<2>(m0);
   const bool p0 = f0 >= n_fft;                        h.template at<3>(m0);
                                                       h.template at<4>(m0, p0);  // @P0 EXIT (warp-uniform)
@@ -153,7 +153,7 @@ __global__ void __launch_bounds__(256) k_wfft(const float2* __restrict__ x, floa
       NoHooks nh;
       wfft_setup<0>(nh, NoHooks::Act{0u}, lane, c);
     }
-    const int W = (int)gridDim.x * 8;
+    const int W = ctas * 8;
     const int kw = (n_fft - f0 + W - 1) / W;          // loop instances of this warp (>= 1)
     const unsigned slot0 = (unsigned)__cvta_generic_to_shared(&ring.slot[wib][0][0]);
 #pragma unroll
@@ -242,10 +242,12 @@ extern "C" int nvbt_wfft32(nvbt_ctx ctx, void* stream, uint32_t tools, int32_t v
                                       : prepare<ProgWfftSw>(ctx, stream, instr, "WFFT_SW", &lc);
   if (rc) return rc;
   if (ctx && instr == 0) lc.stream = ctx->stream;
-  if (n_fft == 0) return NVBT_OK;                     // nothing launched (EM §3.6)
+  rc = partition(ctx, 1, (unsigned long long)ctas, &lc);
+  if (rc) return rc;
+  if (n_fft == 0 || lc.n_ctas == 0) return NVBT_OK;   // nothing launched (EM §3.6)
   rc = dispatch_wfft(tools, variant, [&](auto tag, auto var) {
-    k_wfft<decltype(tag)::value, decltype(var)::value><<<ctas, 256, 0, lc.stream>>>(
-        static_cast<const float2*>(x), static_cast<float2*>(X), n_fft, lc.st);
+    k_wfft<decltype(tag)::value, decltype(var)::value><<<lc.n_ctas, 256, 0, lc.stream>>>(
+        static_cast<const float2*>(x), static_cast<float2*>(X), n_fft, ctas, lc.st);
   });
   return rc ? rc : done(ctx, 1);
 }

@@ -24,7 +24,7 @@ __global__ void __launch_bounds__(256) k_vectoradd(const float* __restrict__ a, 
   Hooks<T, ProgVectorAdd> h(st, sb);
   const auto m0 = h.active(true);              // BB0: every lane
   const int tid = threadIdx.x;                 h.template at<0>(m0);
-  const int cta = blockIdx.x;                  h.template at<1>(m0);
+  const int cta = st.cta_lo + blockIdx.x;     h.template at<1>(m0);
   const int i = cta * 256 + tid;               h.template at<2>(m0);
   const bool p0 = i >= N;                      h.template at<3>(m0);
                                                h.template at<4>(m0, p0);  // @P0 EXIT
@@ -51,8 +51,9 @@ __global__ void __launch_bounds__(256, 6) k_sgemm(const float* __restrict__ A, c
   const auto m0 = h.active(true);
   const int tx = threadIdx.x;                  h.template at<0>(m0);
   const int ty = threadIdx.y;                  h.template at<1>(m0);
-  const int bx = blockIdx.x;                   h.template at<2>(m0);
-  const int by = blockIdx.y;                   h.template at<3>(m0);
+  const unsigned lin = st.cta_lo + blockIdx.x;  // logical CTA (partitioned 1D launch)
+  const int bx = lin % st.grid_x;              h.template at<2>(m0);
+  const int by = lin / st.grid_x;              h.template at<3>(m0);
   const int row = bx * 32 + tx;                h.template at<4>(m0);
   const int col = by * 8 + ty;                 h.template at<5>(m0);
   const bool p0 = row >= M || col >= N;        h.template at<6>(m0);
@@ -92,7 +93,7 @@ __global__ void __launch_bounds__(256) k_bfs_expand(const int* __restrict__ rowp
   Hooks<T, ProgBfs> h(st, sb);
   const auto m0 = h.active(true);
   const int tid = threadIdx.x;                 h.template at<0>(m0);
-  const int cta = blockIdx.x;                  h.template at<1>(m0);
+  const int cta = st.cta_lo + blockIdx.x;     h.template at<1>(m0);
   const int t = cta * 256 + tid;               h.template at<2>(m0);
   const bool p0 = t >= n;                      h.template at<3>(m0);
                                                h.template at<4>(m0, p0);  // @P0 EXIT
@@ -143,7 +144,7 @@ __global__ void __launch_bounds__(256) k_bfs_update(int n, unsigned char* mask, 
   Hooks<T, ProgBfs> h(st, sb);
   const auto m0 = h.active(true);
   const int tid = threadIdx.x;                 h.template at<22>(m0);
-  const int cta = blockIdx.x;                  h.template at<23>(m0);
+  const int cta = st.cta_lo + blockIdx.x;     h.template at<23>(m0);
   const int t = cta * 256 + tid;               h.template at<24>(m0);
   const bool p0 = t >= n;                      h.template at<25>(m0);
                                                h.template at<26>(m0, p0);
@@ -173,8 +174,9 @@ __global__ void __launch_bounds__(256) k_stencil(const float* __restrict__ in, f
   const auto m0 = h.active(true);
   const int tx = threadIdx.x;                  h.template at<0>(m0);
   const int ty = threadIdx.y;                  h.template at<1>(m0);
-  const int bx = blockIdx.x;                   h.template at<2>(m0);
-  const int by = blockIdx.y;                   h.template at<3>(m0);
+  const unsigned lin = st.cta_lo + blockIdx.x;  // logical CTA (partitioned 1D launch)
+  const int bx = lin % st.grid_x;              h.template at<2>(m0);
+  const int by = lin / st.grid_x;              h.template at<3>(m0);
   const int j = bx * 32 + tx;                  h.template at<4>(m0);
   const int i = by * 8 + ty;                   h.template at<5>(m0);
   const bool p0 = i >= n || j >= n;            h.template at<6>(m0);
@@ -232,58 +234,87 @@ int nvbt_vectoradd(nvbt_ctx ctx, void* stream, uint32_t tools, const float* a, c
   if (!a || !b || !c || N < 0) return set_error(NVBT_EINVAL, "bad vectorAdd arguments");
   LaunchCtx lc;
   int rc = prepare<ProgVectorAdd>(ctx, stream, tools, "vectorAdd", &lc);
+  if (!rc) rc = partition(ctx, 1, (N + 255) / 256, &lc);
   if (rc) return rc;
-  if (N == 0) return NVBT_OK;
-  const dim3 grid((N + 255) / 256);
-  rc = dispatch(tools, [&](auto tag) { k_vectoradd<decltype(tag)::value><<<grid, 256, 0, lc.stream>>>(a, b, c, N, lc.st); });
+  if (lc.n_ctas == 0) return NVBT_OK;
+  rc = dispatch(tools, [&](auto tag) { k_vectoradd<decltype(tag)::value><<<lc.n_ctas, 256, 0, lc.stream>>>(a, b, c, N, lc.st); });
   return rc ? rc : done(ctx, 1);
 }
 
 int nvbt_sgemm(nvbt_ctx ctx, void* stream, uint32_t tools, const float* A, const float* B, float* C, int32_t M,
                int32_t N, int32_t K) {
   if (!A || !B || !C || M < 0 || N < 0 || K < 1) return set_error(NVBT_EINVAL, "bad SGEMM arguments");
-  if ((M + 31) / 32 > 0x7fffffff || (N + 7) / 8 > 65535) return set_error(NVBT_EINVAL, "SGEMM grid too large");
   LaunchCtx lc;
   int rc = prepare<ProgSgemm>(ctx, stream, tools, "SGEMM", &lc);
+  if (!rc) rc = partition(ctx, (M + 31) / 32, (N + 7) / 8, &lc);
   if (rc) return rc;
-  if (M == 0 || N == 0) return NVBT_OK;
-  const dim3 grid((M + 31) / 32, (N + 7) / 8), block(32, 8);
-  rc = dispatch(tools, [&](auto tag) { k_sgemm<decltype(tag)::value><<<grid, block, 0, lc.stream>>>(A, B, C, M, N, K, lc.st); });
+  if (lc.n_ctas == 0) return NVBT_OK;
+  const dim3 block(32, 8);
+  rc = dispatch(tools, [&](auto tag) { k_sgemm<decltype(tag)::value><<<lc.n_ctas, block, 0, lc.stream>>>(A, B, C, M, N, K, lc.st); });
   return rc ? rc : done(ctx, 1);
+}
+
+// C3 kernels 1 and 2 as separate launches (a multi-GPU BFS exchanges `updating` between them).
+static int bfs_launch(nvbt_ctx ctx, void* stream, uint32_t tools, int which, const int32_t* rowptr, const int32_t* col,
+                      int32_t n, uint8_t* mask, uint8_t* visited, uint8_t* updating, int32_t* cost, int32_t* over,
+                      int32_t level) {
+  if (!mask || !visited || !updating || n < 0 || (which != 2 && (!rowptr || !col)) || (which != 1 && (!cost || !over)))
+    return set_error(NVBT_EINVAL, "bad BFS arguments");
+  LaunchCtx l1, l2;
+  int rc = NVBT_OK;
+  if (which & 1) {
+    rc = prepare<ProgBfs>(ctx, stream, tools, "BFS", &l1);
+    if (!rc) rc = partition(ctx, 1, (n + 255) / 256, &l1);
+  }
+  if (!rc && (which & 2)) {   // kernel 2 is a launch of its own (next launch id)
+    rc = prepare<ProgBfs>(ctx, stream, tools, "BFS", &l2);
+    if (!rc) rc = partition(ctx, 1, (n + 255) / 256, &l2);
+  }
+  if (rc) return rc;
+  const unsigned nc = (which & 1) ? l1.n_ctas : l2.n_ctas;
+  if (nc == 0) return NVBT_OK;
+  rc = dispatch(tools, [&](auto tag) {
+    constexpr uint32_t TT = decltype(tag)::value;
+    if (which & 1) k_bfs_expand<TT><<<l1.n_ctas, 256, 0, l1.stream>>>(rowptr, col, n, mask, visited, updating, l1.st);
+    if (which & 2) k_bfs_update<TT><<<l2.n_ctas, 256, 0, l2.stream>>>(n, mask, visited, updating, cost, over, level, l2.st);
+  });
+  return rc ? rc : done(ctx, which == 3 ? 2 : 1);
 }
 
 int nvbt_bfs_level(nvbt_ctx ctx, void* stream, uint32_t tools, const int32_t* rowptr, const int32_t* col, int32_t n,
                    uint8_t* mask, uint8_t* visited, uint8_t* updating, int32_t* cost, int32_t* over, int32_t level) {
-  if (!rowptr || !col || !mask || !visited || !updating || !cost || !over || n < 0)
-    return set_error(NVBT_EINVAL, "bad BFS arguments");
-  LaunchCtx lc;
-  int rc = prepare<ProgBfs>(ctx, stream, tools, "BFS", &lc);
-  if (rc) return rc;
-  if (n == 0) return NVBT_OK;
-  const dim3 grid((n + 255) / 256);
-  DevState st2 = lc.st;
-  if (tools != 0) {  // kernel 2 is a launch of its own (next launch id)
-    rc = make_state(ctx, tools, &st2);
-    if (rc) return rc;
-  }
-  rc = dispatch(tools, [&](auto tag) {
-    constexpr uint32_t TT = decltype(tag)::value;
-    k_bfs_expand<TT><<<grid, 256, 0, lc.stream>>>(rowptr, col, n, mask, visited, updating, lc.st);
-    k_bfs_update<TT><<<grid, 256, 0, lc.stream>>>(n, mask, visited, updating, cost, over, level, st2);
-  });
-  return rc ? rc : done(ctx, 2);
+  if (!rowptr || !col || !cost || !over) return set_error(NVBT_EINVAL, "bad BFS arguments");
+  return bfs_launch(ctx, stream, tools, 3, rowptr, col, n, mask, visited, updating, cost, over, level);
+}
+
+int nvbt_bfs_expand(nvbt_ctx ctx, void* stream, uint32_t tools, const int32_t* rowptr, const int32_t* col, int32_t n,
+                    uint8_t* mask, const uint8_t* visited, uint8_t* updating) {
+  return bfs_launch(ctx, stream, tools, 1, rowptr, col, n, mask, const_cast<uint8_t*>(visited), updating, nullptr,
+                    nullptr, 0);
+}
+
+int nvbt_bfs_update(nvbt_ctx ctx, void* stream, uint32_t tools, int32_t n, uint8_t* mask, uint8_t* visited,
+                    uint8_t* updating, int32_t* cost, int32_t* over, int32_t level) {
+  return bfs_launch(ctx, stream, tools, 2, nullptr, nullptr, n, mask, visited, updating, cost, over, level);
 }
 
 int nvbt_stencil(nvbt_ctx ctx, void* stream, uint32_t tools, const float* in, float* out, int32_t n) {
   if (!in || !out || n < 0) return set_error(NVBT_EINVAL, "bad stencil arguments");
-  if ((n + 7) / 8 > 65535) return set_error(NVBT_EINVAL, "stencil grid too large");
   LaunchCtx lc;
   int rc = prepare<ProgStencil>(ctx, stream, tools, "stencil", &lc);
+  if (!rc) rc = partition(ctx, (n + 31) / 32, (n + 7) / 8, &lc);
   if (rc) return rc;
-  if (n == 0) return NVBT_OK;
-  const dim3 grid((n + 31) / 32, (n + 7) / 8), block(32, 8);
-  rc = dispatch(tools, [&](auto tag) { k_stencil<decltype(tag)::value><<<grid, block, 0, lc.stream>>>(in, out, n, lc.st); });
+  if (lc.n_ctas == 0) return NVBT_OK;
+  const dim3 block(32, 8);
+  rc = dispatch(tools, [&](auto tag) { k_stencil<decltype(tag)::value><<<lc.n_ctas, block, 0, lc.stream>>>(in, out, n, lc.st); });
   return rc ? rc : done(ctx, 1);
+}
+
+int nvbt_set_partition(nvbt_ctx ctx, uint32_t rank, uint32_t world) {
+  if (!ctx || world == 0 || rank >= world) return set_error(NVBT_EINVAL, "bad partition rank %u of %u", rank, world);
+  ctx->part_rank = rank;
+  ctx->part_world = world;
+  return NVBT_OK;
 }
 
 }  // extern "C"

@@ -70,6 +70,103 @@ def run_stencil(ctx, tools, buf0, buf1, n, iters, stream=None):
     return bufs[iters % 2]
 
 
+# ------------------------------------------------------------------ multi-GPU partitioned workloads
+def cta_rows(gy: int, rank: int, world: int):
+    """CTA rows [y0, y1) of a gy-row CTA grid that rank runs (the rule nvbt_set_partition documents)."""
+    return gy * rank // world, gy * (rank + 1) // world
+
+
+def run_bfs_dist(ctx, tools, rowptr, col, src, bufs=None, group=None, max_levels=1 << 20):
+    """C3 over `world` ranks: ctx is partitioned (nvbt_set_partition), so each rank runs
+    both BFS kernels on its own vertex range; the graph is replicated. Per level: every rank clears
+    `updating`, runs kernel 1 (it marks any neighbour, owned or not), MAX-all-reduces `updating`, runs
+    kernel 2 on its own vertices, then MAX-all-reduces `visited` and `over`. At the end `cost` (−1 outside
+    a rank's own vertices) is MAX-all-reduced. Every instrumented warp runs on exactly one rank, so the
+    ranks' accumulators sum to the single-GPU result (merge()). Returns (cost, levels)."""
+    import torch
+    import torch.distributed as dist
+    nb = _nb()
+    n = rowptr.numel() - 1
+    b = bfs_buffers(n, rowptr.device) if bufs is None else bufs
+    b["mask"].zero_(); b["visited"].zero_(); b["updating"].zero_(); b["cost"].fill_(-1)
+    b["mask"][src] = 1
+    b["visited"][src] = 1
+    b["cost"][src] = 0
+    level = 0
+    while level < max_levels:
+        b["over"].zero_()
+        b["updating"].zero_()
+        nb.nvbt_bfs_expand(ctx, tools, rowptr, col, n, b["mask"], b["visited"], b["updating"])
+        _sync(ctx)
+        dist.all_reduce(b["updating"], op=dist.ReduceOp.MAX, group=group)
+        nb.nvbt_bfs_update(ctx, tools, n, b["mask"], b["visited"], b["updating"], b["cost"], b["over"], level)
+        _sync(ctx)
+        dist.all_reduce(b["visited"], op=dist.ReduceOp.MAX, group=group)
+        dist.all_reduce(b["over"], op=dist.ReduceOp.MAX, group=group)
+        level += 1
+        if int(b["over"].item()) == 0:
+            break
+    dist.all_reduce(b["cost"], op=dist.ReduceOp.MAX, group=group)
+    return b["cost"], level
+
+
+def stencil_rows(n: int, rank: int, world: int):
+    """Grid rows [r0, r1) a rank computes in the partitioned stencil (CTA rows of 8 grid rows)."""
+    y0, y1 = cta_rows((n + 7) // 8, rank, world)
+    return min(8 * y0, n), min(8 * y1, n)
+
+
+def _exchange_halo(buf, n, rank, world, group):
+    """Every rank publishes its first and last own row; each then fills the row just above and just below
+    its slab from its neighbours. One int32 SUM all-reduce of a (world, 2, n) board (bit-exact: every slot
+    has one writer, the others add 0)."""
+    import torch
+    import torch.distributed as dist
+    r0, r1 = stencil_rows(n, rank, world)
+    board = torch.zeros((world, 2, n), dtype=torch.int32, device=buf.device)
+    g = buf.view(torch.int32)
+    if r1 > r0:
+        board[rank, 0] = g[r0]
+        board[rank, 1] = g[r1 - 1]
+    dist.all_reduce(board, op=dist.ReduceOp.SUM, group=group)
+    # nearest rank above with rows ends at r0; nearest below starts at r1
+    for q in range(rank - 1, -1, -1):
+        a0, a1 = stencil_rows(n, q, world)
+        if a1 > a0:
+            if r0 > 0 and a1 == r0:
+                g[r0 - 1] = board[q, 1]
+            break
+    for q in range(rank + 1, world):
+        a0, a1 = stencil_rows(n, q, world)
+        if a1 > a0:
+            if r1 < n and a0 == r1:
+                g[r1] = board[q, 0]
+            break
+
+
+def run_stencil_dist(ctx, tools, buf0, buf1, n, iters, rank, world, group=None, gather=True):
+    """C4 over `world` ranks: ctx is partitioned, so each rank runs the CTA rows of its own
+    row slab; after every iteration the 1-row halos are exchanged (_exchange_halo). With `gather`, the full
+    final grid is assembled on every rank at the end (one int32 SUM all-reduce, rows outside a rank's slab
+    zeroed first). Trace records stay on each rank's own channel; their digests add. Returns the final
+    buffer."""
+    import torch
+    import torch.distributed as dist
+    bufs = (buf0, buf1)
+    for it in range(iters):
+        _nb().nvbt_stencil(ctx, tools, bufs[it % 2], bufs[(it + 1) % 2], n)
+        _sync(ctx)
+        _exchange_halo(bufs[(it + 1) % 2], n, rank, world, group)
+    out = bufs[iters % 2]
+    if gather:
+        r0, r1 = stencil_rows(n, rank, world)
+        g = out.view(torch.int32)
+        g[:r0] = 0
+        g[r1:] = 0
+        dist.all_reduce(g, op=dist.ReduceOp.SUM, group=group)
+    return out
+
+
 def replay_range(ctx, seed, first, n, hdr, addr, chunk=None):
     """Generate-then-replay events [first, first + n) in chunks that fit the given stream buffers."""
     cap = hdr.numel() // 16 if chunk is None else chunk

@@ -96,6 +96,9 @@ _sigs = {
     "nvbt_sgemm": ([_P, _P, C.c_uint32, _P, _P, _P, C.c_int32, C.c_int32, C.c_int32], C.c_int),
     "nvbt_bfs_level": ([_P, _P, C.c_uint32, _P, _P, C.c_int32, _P, _P, _P, _P, _P, C.c_int32], C.c_int),
     "nvbt_stencil": ([_P, _P, C.c_uint32, _P, _P, C.c_int32], C.c_int),
+    "nvbt_bfs_expand": ([_P, _P, C.c_uint32, _P, _P, C.c_int32, _P, _P, _P], C.c_int),
+    "nvbt_bfs_update": ([_P, _P, C.c_uint32, C.c_int32, _P, _P, _P, _P, _P, C.c_int32], C.c_int),
+    "nvbt_set_partition": ([_P, C.c_uint32, C.c_uint32], C.c_int),
     "nvbt_wfft32": ([_P, _P, C.c_uint32, C.c_int32, _P, _P, C.c_int32, C.c_int32], C.c_int),
     "nvbt_wfft32_max_ctas": ([C.c_uint32, C.c_int32, C.c_int32, C.POINTER(C.c_int32)], C.c_int),
 }
@@ -419,3 +422,19 @@ def nvbt_wfft32_max_ctas(tools, variant, device=0):
     n = C.c_int32()
     _check(_lib.nvbt_wfft32_max_ctas(tools, variant, device, C.byref(n)))
     return n.value
+
+
+def nvbt_bfs_expand(ctx, tools, rowptr, col, n, mask, visited, updating, stream=None):
+    _check(_lib.nvbt_bfs_expand(_h(ctx), _s(ctx, stream), tools, _ptr(rowptr), _ptr(col), n, _ptr(mask),
+                                _ptr(visited), _ptr(updating)))
+
+
+def nvbt_bfs_update(ctx, tools, n, mask, visited, updating, cost, over, level, stream=None):
+    _check(_lib.nvbt_bfs_update(_h(ctx), _s(ctx, stream), tools, n, _ptr(mask), _ptr(visited), _ptr(updating),
+                                _ptr(cost), _ptr(over), level))
+
+
+def nvbt_set_partition(ctx, rank, world):
+    """Later workload launches through ctx run only `rank`'s share of their CTA grid."""
+    _check(_lib.nvbt_set_partition(ctx.handle, rank, world))
+    ctx.partition = (rank, world)
