@@ -33,7 +33,7 @@ int nvbt_workload_warps(int workload, const int64_t* args, uint32_t n_args, uint
  * (then stream is used); otherwise the context's program must be the vectorAdd program. */
 int nvbt_vectoradd(nvbt_ctx ctx, void* stream, uint32_t tools, const float* a, const float* b, float* c,
                    int32_t N);
-/* C2: naive row-fastest SGEMM C[M,N] = A[M,K] B[K,N], fp32 row-major, K >= 1 (EM §3.2). */
+/* C2: naive row-fastest SGEMM C[M,N] = A[M,K] B[K,N], fp32 row-major, K >= 1 (EM §3.2); ceil(N/8) <= 65535. */
 int nvbt_sgemm(nvbt_ctx ctx, void* stream, uint32_t tools, const float* A, const float* B, float* C,
                int32_t M, int32_t N, int32_t K);
 /* C3: one BFS level = kernel 1 (expand) then kernel 2 (update, writes cost = level + 1) (EM §3.3).
@@ -49,7 +49,7 @@ int nvbt_bfs_expand(nvbt_ctx ctx, void* stream, uint32_t tools, const int32_t* r
                     int32_t n, uint8_t* mask, const uint8_t* visited, uint8_t* updating);
 int nvbt_bfs_update(nvbt_ctx ctx, void* stream, uint32_t tools, int32_t n, uint8_t* mask, uint8_t* visited,
                     uint8_t* updating, int32_t* cost, int32_t* over, int32_t level);
-/* C4: one Jacobi iteration out = stencil(in) on an n x n fp32 grid (EM §3.4). */
+/* C4: one Jacobi iteration out = stencil(in) on an n x n fp32 grid (EM §3.4); ceil(n/8) <= 65535. */
 int nvbt_stencil(nvbt_ctx ctx, void* stream, uint32_t tools, const float* in, float* out, int32_t n);
 
 /* Multi-GPU partition ("partitioned ... by kernel and warp range"): every later workload

@@ -54,10 +54,10 @@ struct DevState {
   // ticket is exactly kRingChunk opens the stripe's next chunk from the global counter rheads[rstripes].
   unsigned long long* rheads;
   unsigned rstripes;
-  // multi-GPU partition (nvbt_set_partition): this launch runs logical CTAs cta_lo + blockIdx.x of a
-  // CTA grid grid_x wide (2D workloads derive ctaid.x = lin % grid_x, ctaid.y = lin / grid_x)
+  // multi-GPU partition (nvbt_set_partition): this launch runs the CTA rows from cta_y0 on; its logical
+  // linear CTA id is cta_lo + blockIdx.x + blockIdx.y * gridDim.x (cta_lo = cta_y0 * CTA-grid width)
   unsigned cta_lo;
-  unsigned grid_x;
+  unsigned cta_y0;
 };
 constexpr unsigned kRingChunk = 4096;
 constexpr unsigned kRingNoChunk = 0xFFFFFFFEu, kRingFull = 0xFFFFFFFFu;
@@ -295,7 +295,7 @@ struct Hooks {
     lanebit = 1u << lane;
     lmlt = lanemask_lt();
     const unsigned tid = threadIdx.x + threadIdx.y * blockDim.x;
-    gwarp = (st.cta_lo + blockIdx.x) * ((blockDim.x * blockDim.y) >> 5) + (tid >> 5);   // logical CTA (1D launches)
+    gwarp = (st.cta_lo + blockIdx.x + blockIdx.y * gridDim.x) * ((blockDim.x * blockDim.y) >> 5) + (tid >> 5);  // logical CTA
     scr = (unsigned)__cvta_generic_to_shared(sb + kScratchWord0 + SCRATCH_WORDS * ((tid >> 5) & (kMaxWarps - 1)));
     sbase = (unsigned)__cvta_generic_to_shared(sb);
     if constexpr (kOn) {
@@ -663,7 +663,7 @@ struct Hooks {
       constexpr int nt = kThreads;
       // this CTA's stripe of the global bins (spreads same-address atomics over st.stripes copies)
       // (logical CTA id: a partitioned launch fills the same stripes as the unpartitioned one)
-      const unsigned long long so = (unsigned long long)((st.cta_lo + blockIdx.x) & (st.stripes - 1u)) * st.stripe_words;
+      const unsigned long long so = (unsigned long long)((st.cta_lo + blockIdx.x + blockIdx.y * gridDim.x) & (st.stripes - 1u)) * st.stripe_words;
       for (int pc = tid; pc < NPC; pc += nt) {
         const unsigned* b = sb + pc * SITE_WORDS;
         if (b[0] | b[2]) {

@@ -246,7 +246,7 @@ extern "C" int nvbt_wfft32(nvbt_ctx ctx, void* stream, uint32_t tools, int32_t v
   if (rc) return rc;
   if (n_fft == 0 || lc.n_ctas == 0) return NVBT_OK;   // nothing launched (EM §3.6)
   rc = dispatch_wfft(tools, variant, [&](auto tag, auto var) {
-    k_wfft<decltype(tag)::value, decltype(var)::value><<<lc.n_ctas, 256, 0, lc.stream>>>(
+    k_wfft<decltype(tag)::value, decltype(var)::value><<<lc.grid, 256, 0, lc.stream>>>(
         static_cast<const float2*>(x), static_cast<float2*>(X), n_fft, ctas, lc.st);
   });
   return rc ? rc : done(ctx, 1);

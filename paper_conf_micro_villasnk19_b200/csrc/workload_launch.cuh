@@ -21,21 +21,24 @@ static inline int dispatch(uint32_t tools, F&& f) {
 struct LaunchCtx {
   cudaStream_t stream = nullptr;
   DevState st{};
-  unsigned n_ctas = 0;   // CTAs this launch runs (1D grid)
+  dim3 grid{0, 1, 1};    // the launch's share of the CTA grid
+  unsigned n_ctas = 0;
 };
 
 // Multi-GPU partition (nvbt_set_partition): a workload whose CTA grid has gy rows of gx
 // CTAs (1D grids: gx = 1) runs, on rank r of w, the whole CTA rows [gy r / w, gy (r + 1) / w), i.e. the
-// logical CTAs [gx gy r / w, ...) in linear order, launched as a 1D grid. Global warp ids, addresses and
-// hence every event are those of the unpartitioned launch, so per-rank results sum to the full result.
+// logical CTAs [gx gy r / w, ...) in linear order: 2D workloads launch (gx, rows) with ctaid.y offset by
+// cta_y0, 1D workloads launch (rows) with the CTA id offset by cta_lo. Global warp ids, addresses and hence
+// every event are those of the unpartitioned launch, so per-rank results sum to the full result.
 // Must follow prepare() (which rebuilds lc->st).
 static inline int partition(nvbt_ctx ctx, unsigned long long gx, unsigned long long gy, LaunchCtx* lc) {
   const unsigned long long r = ctx ? ctx->part_rank : 0, w = ctx ? ctx->part_world : 1;
   const unsigned long long y0 = gy * r / w, y1 = gy * (r + 1) / w;
-  if (gx * gy > 0x7fffffffull) return set_error(NVBT_EINVAL, "CTA grid too large");
+  if (gx * gy > 0x7fffffffull || (gx > 1 && gy > 65535)) return set_error(NVBT_EINVAL, "CTA grid too large");
   lc->st.cta_lo = (unsigned)(gx * y0);
-  lc->st.grid_x = (unsigned)gx;
+  lc->st.cta_y0 = (unsigned)y0;
   lc->n_ctas = (unsigned)(gx * (y1 - y0));
+  lc->grid = gx > 1 ? dim3((unsigned)gx, (unsigned)(y1 - y0), 1) : dim3((unsigned)(y1 - y0), 1, 1);
   return NVBT_OK;
 }
 

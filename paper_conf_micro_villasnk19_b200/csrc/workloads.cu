@@ -51,9 +51,8 @@ __global__ void __launch_bounds__(256, 6) k_sgemm(const float* __restrict__ A, c
   const auto m0 = h.active(true);
   const int tx = threadIdx.x;                  h.template at<0>(m0);
   const int ty = threadIdx.y;                  h.template at<1>(m0);
-  const unsigned lin = st.cta_lo + blockIdx.x;  // logical CTA (partitioned 1D launch)
-  const int bx = lin % st.grid_x;              h.template at<2>(m0);
-  const int by = lin / st.grid_x;              h.template at<3>(m0);
+  const int bx = blockIdx.x;                   h.template at<2>(m0);
+  const int by = st.cta_y0 + blockIdx.y;       h.template at<3>(m0);   // (partition: CTA-row offset)
   const int row = bx * 32 + tx;                h.template at<4>(m0);
   const int col = by * 8 + ty;                 h.template at<5>(m0);
   const bool p0 = row >= M || col >= N;        h.template at<6>(m0);
@@ -174,9 +173,8 @@ __global__ void __launch_bounds__(256) k_stencil(const float* __restrict__ in, f
   const auto m0 = h.active(true);
   const int tx = threadIdx.x;                  h.template at<0>(m0);
   const int ty = threadIdx.y;                  h.template at<1>(m0);
-  const unsigned lin = st.cta_lo + blockIdx.x;  // logical CTA (partitioned 1D launch)
-  const int bx = lin % st.grid_x;              h.template at<2>(m0);
-  const int by = lin / st.grid_x;              h.template at<3>(m0);
+  const int bx = blockIdx.x;                   h.template at<2>(m0);
+  const int by = st.cta_y0 + blockIdx.y;       h.template at<3>(m0);   // (partition: CTA-row offset)
   const int j = bx * 32 + tx;                  h.template at<4>(m0);
   const int i = by * 8 + ty;                   h.template at<5>(m0);
   const bool p0 = i >= n || j >= n;            h.template at<6>(m0);
@@ -237,7 +235,7 @@ int nvbt_vectoradd(nvbt_ctx ctx, void* stream, uint32_t tools, const float* a, c
   if (!rc) rc = partition(ctx, 1, (N + 255) / 256, &lc);
   if (rc) return rc;
   if (lc.n_ctas == 0) return NVBT_OK;
-  rc = dispatch(tools, [&](auto tag) { k_vectoradd<decltype(tag)::value><<<lc.n_ctas, 256, 0, lc.stream>>>(a, b, c, N, lc.st); });
+  rc = dispatch(tools, [&](auto tag) { k_vectoradd<decltype(tag)::value><<<lc.grid, 256, 0, lc.stream>>>(a, b, c, N, lc.st); });
   return rc ? rc : done(ctx, 1);
 }
 
@@ -250,7 +248,7 @@ int nvbt_sgemm(nvbt_ctx ctx, void* stream, uint32_t tools, const float* A, const
   if (rc) return rc;
   if (lc.n_ctas == 0) return NVBT_OK;
   const dim3 block(32, 8);
-  rc = dispatch(tools, [&](auto tag) { k_sgemm<decltype(tag)::value><<<lc.n_ctas, block, 0, lc.stream>>>(A, B, C, M, N, K, lc.st); });
+  rc = dispatch(tools, [&](auto tag) { k_sgemm<decltype(tag)::value><<<lc.grid, block, 0, lc.stream>>>(A, B, C, M, N, K, lc.st); });
   return rc ? rc : done(ctx, 1);
 }
 
@@ -275,8 +273,8 @@ static int bfs_launch(nvbt_ctx ctx, void* stream, uint32_t tools, int which, con
   if (nc == 0) return NVBT_OK;
   rc = dispatch(tools, [&](auto tag) {
     constexpr uint32_t TT = decltype(tag)::value;
-    if (which & 1) k_bfs_expand<TT><<<l1.n_ctas, 256, 0, l1.stream>>>(rowptr, col, n, mask, visited, updating, l1.st);
-    if (which & 2) k_bfs_update<TT><<<l2.n_ctas, 256, 0, l2.stream>>>(n, mask, visited, updating, cost, over, level, l2.st);
+    if (which & 1) k_bfs_expand<TT><<<l1.grid, 256, 0, l1.stream>>>(rowptr, col, n, mask, visited, updating, l1.st);
+    if (which & 2) k_bfs_update<TT><<<l2.grid, 256, 0, l2.stream>>>(n, mask, visited, updating, cost, over, level, l2.st);
   });
   return rc ? rc : done(ctx, which == 3 ? 2 : 1);
 }
@@ -306,7 +304,7 @@ int nvbt_stencil(nvbt_ctx ctx, void* stream, uint32_t tools, const float* in, fl
   if (rc) return rc;
   if (lc.n_ctas == 0) return NVBT_OK;
   const dim3 block(32, 8);
-  rc = dispatch(tools, [&](auto tag) { k_stencil<decltype(tag)::value><<<lc.n_ctas, block, 0, lc.stream>>>(in, out, n, lc.st); });
+  rc = dispatch(tools, [&](auto tag) { k_stencil<decltype(tag)::value><<<lc.grid, block, 0, lc.stream>>>(in, out, n, lc.st); });
   return rc ? rc : done(ctx, 1);
 }
 
