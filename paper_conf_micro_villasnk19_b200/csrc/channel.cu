@@ -338,7 +338,6 @@ int nvbt_channel_open(nvbt_ctx c, void* ring, size_t bytes, uint32_t record_byte
 // each owning a 4 KB block of 4 sector bits per line (8192 lines). The blocks cost 1/256 of the address
 // span a launch touches and stay L2-resident, so the kernel streams the records from HBM once.
 namespace nvbt {
-constexpr int kFpBatch = 8;                  // record address loads in flight per warp
 constexpr unsigned long long kFpEmpty = ~0ull;
 constexpr int kFpRegionShift = 20;           // 1 MB regions
 constexpr unsigned kFpWords = (1u << (kFpRegionShift - 7)) / 8;   // 32-bit words per block (8 lines each)
@@ -366,6 +365,31 @@ __device__ __forceinline__ bool fp_slot(unsigned long long k, unsigned long long
       if (v == kFpEmpty) v = atomicCAS(keys + h, kFpEmpty, k);
     }
     v = __shfl_sync(0xffffffffu, v, 0);
+    if (v == kFpEmpty || v == k) {
+      ck[1] = ck[0]; cs[1] = cs[0]; ck[0] = k; cs[0] = h;
+      slot = h;
+      return true;
+    }
+    h = (h + 1) & mask;
+  }
+  return false;
+}
+
+// Per-lane table lookup (divergent callers: each quad leader looks up its own record's region), with a
+// per-lane two-entry cache. Returns false if the table is full.
+__device__ __forceinline__ bool fp_slot_lane(unsigned long long k, unsigned long long* __restrict__ keys,
+                                             unsigned long long mask, unsigned long long (&ck)[2],
+                                             unsigned long long (&cs)[2], unsigned long long& slot) {
+  if (k == ck[0]) { slot = cs[0]; return true; }
+  if (k == ck[1]) {
+    slot = cs[1];
+    ck[1] = ck[0]; cs[1] = cs[0]; ck[0] = k; cs[0] = slot;
+    return true;
+  }
+  unsigned long long h = ((k * 0x9E3779B97F4A7C15ull) >> 24) & mask;
+  for (unsigned long long probes = 0; probes <= mask; ++probes) {
+    unsigned long long v = *reinterpret_cast<volatile unsigned long long*>(keys + h);
+    if (v == kFpEmpty) v = atomicCAS(keys + h, kFpEmpty, k);
     if (v == kFpEmpty || v == k) {
       ck[1] = ck[0]; cs[1] = cs[0]; ck[0] = k; cs[0] = h;
       slot = h;
@@ -447,7 +471,7 @@ __global__ void __launch_bounds__(256) k_fp_count(const unsigned long long* __re
 // Committed slots lie in the chunks handed out so far, [0, min(chunks * kRingChunk, cap)); slots never
 // written (the unused tail of each SM's last chunk, slots a warp reserved but did not use) have tag 0 and
 // are skipped. Each warp takes a contiguous range of slots, 32 at a time: lane i reads record i's
-// header, then the warp walks the 32 records (addresses coalesced, kFpBatch loads in flight).
+// header, then the warp walks the 32 records 8 at a time, 4 lanes per record (quad pass).
 __global__ void __launch_bounds__(256) k_footprint(const unsigned char* __restrict__ ring,
                                                     const unsigned long long* __restrict__ chunks,
                                                     unsigned long long cap,
@@ -464,14 +488,23 @@ __global__ void __launch_bounds__(256) k_footprint(const unsigned char* __restri
   unsigned cur = 0xFFFFFFFFu;
   unsigned long long nrec = 0;
   unsigned long long ck[2] = {kFpEmpty, kFpEmpty}, cs[2] = {0, 0};
+  // headers are loaded one 32-record group ahead
+  uint4 nh1 = make_uint4(0, 0, 0, 0);
+  unsigned nl = 0;
+  if (r0 + lane < r1) {
+    const unsigned char* rec = ring + 64 + (r0 + lane) * RECORD_BYTES;
+    nh1 = __ldcs(reinterpret_cast<const uint4*>(rec + 16));   // A P op|w|k tag
+    nl = __ldcs(reinterpret_cast<const unsigned*>(rec));
+  }
   for (unsigned long long base = r0; base < r1; base += 32) {
     const unsigned cnt = r1 - base < 32 ? (unsigned)(r1 - base) : 32u;
     unsigned lid = 0xFFFFFFFFu, E = 0;
-    if (lane < cnt) {
-      const unsigned char* rec = ring + 64 + (base + lane) * RECORD_BYTES;
-      const uint4 h1 = __ldcs(reinterpret_cast<const uint4*>(rec + 16));   // A P op|w|k tag
-      const unsigned l = __ldcs(reinterpret_cast<const unsigned*>(rec)) - first;
-      if (h1.w == 1u) { lid = l; E = h1.x & h1.y; }
+    if (lane < cnt && nh1.w == 1u) { lid = nl - first; E = nh1.x & nh1.y; }
+    nh1 = make_uint4(0, 0, 0, 0);
+    if (base + 32 + lane < r1) {
+      const unsigned char* rec = ring + 64 + (base + 32 + lane) * RECORD_BYTES;
+      nh1 = __ldcs(reinterpret_cast<const uint4*>(rec + 16));
+      nl = __ldcs(reinterpret_cast<const unsigned*>(rec));
     }
     const bool ok = lid < n_launches;
     const unsigned bad = __ballot_sync(0xffffffffu, lid != 0xFFFFFFFFu && !ok);
@@ -496,19 +529,70 @@ __global__ void __launch_bounds__(256) k_footprint(const unsigned char* __restri
       }
     }
     const unsigned live = __ballot_sync(0xffffffffu, ok && E != 0u);
-    for (unsigned j = 0; j < 32; j += kFpBatch) {
-      if (((live >> j) & ((1u << kFpBatch) - 1u)) == 0u) continue;   // uniform
-      unsigned long long a[kFpBatch];
+    // quad pass, 8 records at a time: lanes 4b..4b+3 read record j+b's 32 addresses (8 each, 4 x 16 B)
+    // and check that all lanes of E fall in one 1 KB word of one region; if so the quad's first lane ORs
+    // the record's sector bits with one atomic (common: a warp access covers <= 1 KB). Records spanning
+    // several words take the warp-cooperative fp_record().
+    const unsigned qb = lane >> 2, qq = lane & 3u;
+    for (unsigned j = 0; j < 32; j += 8) {
+      if (((live >> j) & 0xFFu) == 0u) continue;   // uniform
+      const unsigned jj = j + qb;
+      const bool qlive = (live >> jj) & 1u;
+      const unsigned qE = __shfl_sync(0xffffffffu, E, jj) >> (8u * qq);
+      const unsigned ql = __shfl_sync(0xffffffffu, lid, jj);
+      unsigned long long key = 0;
+      unsigned wd = 0, bits = 0;
+      bool have = false, same = true;
+      if (qlive) {
+        const uint4* src = reinterpret_cast<const uint4*>(ring + 64 + (base + jj) * RECORD_BYTES + 32 + 64 * qq);
+        uint4 va[4];
 #pragma unroll
-      for (int u = 0; u < kFpBatch; ++u) {
-        const unsigned jj = (live >> (j + u)) & 1u ? j + u : __ffs(live) - 1;   // keep loads in range
-        a[u] = __ldcs(reinterpret_cast<const unsigned long long*>(ring + 64 + (base + jj) * RECORD_BYTES + 32) + lane);
+        for (int k = 0; k < 4; ++k) va[k] = __ldcs(src + k);
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+          const uint4 v = va[k];
+          const unsigned long long a2[2] = {(unsigned long long)v.y << 32 | v.x, (unsigned long long)v.w << 32 | v.z};
+#pragma unroll
+          for (int t = 0; t < 2; ++t) {
+            if ((qE >> (2 * k + t)) & 1u) {
+              const unsigned long long a = a2[t];
+              const unsigned long long kk = ((unsigned long long)ql << (48 - kFpRegionShift)) | (a >> kFpRegionShift);
+              const unsigned line = (unsigned)(a >> 7) & (8 * kFpWords - 1);
+              same = same && (a >> 48) == 0ull && (!have || (kk == key && (line >> 3) == wd));
+              key = kk;
+              wd = line >> 3;
+              bits |= 1u << ((line & 7) * 4 + ((unsigned)(a >> 5) & 3));
+              have = true;
+            }
+          }
+        }
       }
+      // quad reduction: one (region, word) for the whole record?
 #pragma unroll
-      for (int u = 0; u < kFpBatch; ++u) {
-        const unsigned Ej = __shfl_sync(0xffffffffu, E, j + u);
-        const unsigned lj = __shfl_sync(0xffffffffu, lid, j + u);
-        if ((live >> (j + u)) & 1u) fp_record(lj, Ej, a[u], lane, keys, pool, mask, err, ck, cs);
+      for (unsigned d = 1; d <= 2; d <<= 1) {
+        const unsigned oh = __shfl_xor_sync(0xffffffffu, (unsigned)have, d);
+        const unsigned long long ok2 = __shfl_xor_sync(0xffffffffu, key, d);
+        const unsigned ow = __shfl_xor_sync(0xffffffffu, wd, d);
+        const unsigned ob = __shfl_xor_sync(0xffffffffu, bits, d);
+        const unsigned os = __shfl_xor_sync(0xffffffffu, (unsigned)same, d);
+        same = same && os != 0u && (!have || !oh || (ok2 == key && ow == wd));
+        if (!have && oh) { key = ok2; wd = ow; }
+        have = have || oh != 0u;
+        bits |= ob;
+      }
+      if (qlive && same && qq == 0) {
+        unsigned long long slot;
+        if (fp_slot_lane(key, keys, mask, ck, cs, slot)) atomicOr(pool + slot * kFpWords + wd, bits);
+        else atomicAdd(err, 1ull);
+      }
+      unsigned slow = __ballot_sync(0xffffffffu, qlive && !same && qq == 0);
+      while (slow) {
+        const unsigned b = (__ffs(slow) - 1) >> 2;
+        slow &= slow - 1;
+        const unsigned r = j + b;
+        const unsigned long long a = __ldcs(reinterpret_cast<const unsigned long long*>(ring + 64 + (base + r) * RECORD_BYTES + 32) + lane);
+        unsigned long long wck[2] = {kFpEmpty, kFpEmpty}, wcs[2] = {0, 0};
+        fp_record(__shfl_sync(0xffffffffu, lid, r), __shfl_sync(0xffffffffu, E, r), a, lane, keys, pool, mask, err, wck, wcs);
       }
     }
   }
