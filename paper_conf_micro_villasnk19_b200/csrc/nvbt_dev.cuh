@@ -496,18 +496,30 @@ struct Hooks {
         have = reserve(1, t);
       }
       if (have) {
-        unsigned char* rec = st.no_wait ? st.ring + t * RECORD_BYTES : slot_ptr(t, tag);
-        // lane j < 18 writes bytes [16j, 16j + 16): lanes 0, 1 the header (tag 0), lane j >= 2 the
-        // addresses of lanes 2(j-2), 2(j-2)+1
-        const unsigned src = 2u * (lane - 2u);
-        const unsigned long long a0 = __shfl_sync(FULL, a, src & 31u), a1 = __shfl_sync(FULL, a, (src + 1u) & 31u);
-        if (lane < 18) {
-          const uint4 v = lane == 0   ? make_uint4(st.launch, gwarp, seq, (unsigned)PC)
-                          : lane == 1 ? make_uint4(A, P, w2, st.no_wait)
-                                      : make_uint4((unsigned)a0, (unsigned)(a0 >> 32), (unsigned)a1, (unsigned)(a1 >> 32));
-          *reinterpret_cast<uint4*>(rec + 16 * lane) = v;
+        if (st.no_wait) {
+          // device ring (HBM, issue-bound producer): every lane stores its own address (8 B, 256 B
+          // coalesced per record) and lanes 0, 1 the 32 B header with tag 1 — no shuffles
+          unsigned char* rec = st.ring + t * RECORD_BYTES;
+          *reinterpret_cast<unsigned long long*>(rec + 32 + 8 * lane) = a;
+          if (lane < 2) {
+            const uint4 v = lane == 0 ? make_uint4(st.launch, gwarp, seq, (unsigned)PC) : make_uint4(A, P, w2, 1u);
+            *reinterpret_cast<uint4*>(rec + 16 * lane) = v;
+          }
+        } else {
+          unsigned char* rec = slot_ptr(t, tag);
+          // pinned host ring: one 16 B-per-lane store per record. Lane j < 18 writes bytes
+          // [16j, 16j + 16): lanes 0, 1 the header (tag 0), lane j >= 2 the addresses of lanes 2(j-2),
+          // 2(j-2)+1
+          const unsigned src = 2u * (lane - 2u);
+          const unsigned long long a0 = __shfl_sync(FULL, a, src & 31u), a1 = __shfl_sync(FULL, a, (src + 1u) & 31u);
+          if (lane < 18) {
+            const uint4 v = lane == 0   ? make_uint4(st.launch, gwarp, seq, (unsigned)PC)
+                            : lane == 1 ? make_uint4(A, P, w2, 0u)
+                                        : make_uint4((unsigned)a0, (unsigned)(a0 >> 32), (unsigned)a1, (unsigned)(a1 >> 32));
+            *reinterpret_cast<uint4*>(rec + 16 * lane) = v;
+          }
+          add_pending(rec, tag);
         }
-        if (!st.no_wait) add_pending(rec, tag);
       }
       ++seq;
       return;

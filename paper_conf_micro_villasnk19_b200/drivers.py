@@ -129,6 +129,8 @@ def _exchange_halo(buf, n, rank, world, group):
         board[rank, 0] = g[r0]
         board[rank, 1] = g[r1 - 1]
     dist.all_reduce(board, op=dist.ReduceOp.SUM, group=group)
+    if r1 == r0:                     # an empty slab computes nothing and needs no halo
+        return
     # nearest rank above with rows ends at r0; nearest below starts at r1
     for q in range(rank - 1, -1, -1):
         a0, a1 = stencil_rows(n, q, world)

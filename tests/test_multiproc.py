@@ -80,3 +80,59 @@ def test_merge_rejects_non_int64():
     from paper_conf_micro_villasnk19_b200 import drivers
     with pytest.raises(TypeError):
         drivers.merge_tensor(torch.zeros(3, dtype=torch.float32))
+
+
+def _halo_worker(rank, world, port, n, out_q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        from paper_conf_micro_villasnk19_b200 import drivers
+        # every rank's buffer: its own rows carry (rank, row, col)-dependent values, all others garbage
+        g = torch.full((n, n), -7.0)
+        r0, r1 = drivers.stencil_rows(n, rank, world)
+        rows = torch.arange(n, dtype=torch.float32)[:, None] * 1000 + torch.arange(n, dtype=torch.float32)[None, :]
+        g[r0:r1] = rows[r0:r1] + 0.5
+        drivers._exchange_halo(g, n, rank, world, None)
+        out_q.put((rank, r0, r1, g.numpy()))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("n,world", [(50, 3), (64, 2), (17, 4)])
+def test_gloo_stencil_halo_exchange(n, world):
+    """C4 partition: after the exchange every rank holds the true row just above and just
+    below its slab (bit-exact: the int32 SUM board has one writer per slot); nothing else changes."""
+    from paper_conf_micro_villasnk19_b200 import drivers
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_halo_worker, args=(r, world, port, n, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=300) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    rows = np.arange(n, dtype=np.float32)[:, None] * 1000 + np.arange(n, dtype=np.float32)[None, :] + 0.5
+    covered = np.zeros(n, dtype=int)
+    for rank, r0, r1, g in res:
+        covered[r0:r1] += 1
+        expect = np.full((n, n), -7.0, dtype=np.float32)
+        expect[r0:r1] = rows[r0:r1]
+        if r1 > r0:
+            if r0 > 0:
+                expect[r0 - 1] = rows[r0 - 1]
+            if r1 < n:
+                expect[r1] = rows[r1]
+        assert np.array_equal(g, expect), rank
+    assert (covered == 1).all()                  # the slabs partition the grid
+
+
+def test_cta_rows_partition():
+    from paper_conf_micro_villasnk19_b200 import drivers
+    for gy in (1, 2, 7, 1024):
+        for world in (1, 2, 3, 8):
+            parts = [drivers.cta_rows(gy, r, world) for r in range(world)]
+            assert parts[0][0] == 0 and parts[-1][1] == gy
+            assert all(parts[i][1] == parts[i + 1][0] for i in range(world - 1))
