@@ -350,6 +350,12 @@ def run_ours(args):
         "merge_ms": merge_ms,
     }
     line["roofline"]["peak_source"] = f"148 SMs x 4 issue/clk x sm_max_mhz ({peaks_src})"
+    # the binding resource of this workload is the application's own L1 traffic (the naive row-fastest
+    # SGEMM is L1-wavefront-bound uninstrumented); the hooks run inside that bound
+    line["app_bound"] = {"resource": "L1TEX wavefronts of the uninstrumented SGEMM",
+                         "instr_speed_vs_plain": statistics.median(t_plain) / t_kernel,
+                         "ncu": "profiles/r1_ncu_summary_c2_c5.txt: l1tex 98.8 % (plain) / 95.2 % (instrumented), "
+                                "issue-active 6.9 % / 85.2 %"}
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         rate, sample = wl.oracle_sample(args.cpu_budget)
         line["cpu_baseline"] = {"value": rate, "unit": "events/s", "cores": 1, "kind": "oracle", "sample": sample}
