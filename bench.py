@@ -428,32 +428,57 @@ def _timed_events(torch, fn, n):
 
 
 def run_c1(args, torch, nb, dr, local):
-    """C1: vectorAdd N = 65536, tools COUNT (instruction count + opcode histogram); a step is one launch."""
+    """C1: vectorAdd N = 65536, tools COUNT (instruction count + opcode histogram); a step is one launch.
+    A launch moves 786 KB, so launch overhead dominates: the launches are batched into one CUDA graph of
+    `reps` launches (captured on the context's stream) and each replay is timed."""
     from synth import uniform_f32
     N = 65536
-    ctx = nb.nvbt_init(nb.W_VECTORADD, nb.COUNT | nb.OPHIST)
+    s = torch.cuda.Stream()
+    ctx = nb.nvbt_init(nb.W_VECTORADD, nb.COUNT | nb.OPHIST, stream=s)
     a = torch.from_numpy(uniform_f32(N, 1)).cuda()
     b = torch.from_numpy(uniform_f32(N, 2)).cuda()
     c = torch.empty_like(a)
-    reps = 200   # launches per timed sample (a launch is a few microseconds)
-    f_plain = lambda: [nb.nvbt_vectoradd(ctx, nb.TOOL_NONE, a, b, c, N) for _ in range(reps)]
-    f_instr = lambda: [nb.nvbt_vectoradd(ctx, nb.TOOL_COUNT, a, b, c, N) for _ in range(reps)]
-    _timed_events(torch, f_instr, args.warmup)
-    _timed_events(torch, f_plain, args.warmup)
-    tp = _timed_events(torch, f_plain, args.steps)
+    reps = 200   # launches per graph
+    torch.cuda.synchronize()
+
+    def graph_of(tools):
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=s):
+            for _ in range(reps):
+                nb.nvbt_vectoradd(ctx, tools, a, b, c, N)
+        return g
+
+    g_plain, g_instr = graph_of(nb.TOOL_NONE), graph_of(nb.TOOL_COUNT)
+    nb.nvbt_reset(ctx)
+
+    def timed(g, n):
+        ts = []
+        for _ in range(n):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            with torch.cuda.stream(s):
+                e0.record(s)
+                g.replay()
+                e1.record(s)
+            e1.synchronize()
+            ts.append(e0.elapsed_time(e1) / 1e3)
+        return ts
+
+    timed(g_instr, args.warmup)
+    timed(g_plain, args.warmup)
+    tp = timed(g_plain, args.steps)
     nb.nvbt_reset(ctx)
     with ClockSampler(local) as clk:
-        ti = _timed_events(torch, f_instr, args.steps)
+        ti = timed(g_instr, args.steps)
     cnt = nb.nvbt_count(ctx)
     ev = int(cnt[2]) // (args.steps * reps)
     t_i, t_p = sum(ti) / (args.steps * reps), sum(tp) / (args.steps * reps)
     return {"metric": METRIC, "value": ev / t_i, "unit": "events/s", "n_gpus": 1, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": 1e3 * t_i, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-            "config": {"workload": "C1 vectorAdd N=65536, tools COUNT", "launches_per_sample": reps,
-                       "warp_events_per_launch": ev},
+            "config": {"workload": "C1 vectorAdd N=65536, tools COUNT", "launches_per_graph": reps,
+                       "warp_events_per_launch": ev, "counts_check": "ok" if ev == 26624 else f"{ev} != 26624"},
             "slowdown": t_i / t_p, "plain_us_per_launch": 1e6 * t_p, "instr_us_per_launch": 1e6 * t_i,
-            "bound": "launch latency (26,624 warp events per launch)", "clocks": clk.summary()}
+            "bound": "launch latency (26,624 warp events per launch; CUDA-graph replays)", "clocks": clk.summary()}
 
 
 def run_c3(args, torch, nb, dr, local):
