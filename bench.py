@@ -226,7 +226,7 @@ class ReplayBench:
     name = "c5"
     desc = "C5 trace replay of 10^10 generated events (counts, histograms, divergence), 2^27-event chunks"
 
-    def __init__(self, torch, nb, dr, world, rank, n_total=10**10, chunk=1 << 27):
+    def __init__(self, torch, nb, dr, world, rank, n_total=10**10, chunk=1 << 27, staged=True):
         self.torch, self.nb, self.dr = torch, nb, dr
         self.lo, self.hi = dr.shard_range(n_total, rank, world)
         self.n = self.hi - self.lo
@@ -234,8 +234,17 @@ class ReplayBench:
         self.ctx = nb.nvbt_init(nb.W_REPLAY, nb.COUNT | nb.OPHIST | nb.BB | nb.MEMDIV)
         self.hdr = torch.empty(chunk * 16, dtype=torch.uint8, device="cuda")
         self.addr = torch.empty(chunk * 256, dtype=torch.uint8, device="cuda")
+        # staged replay (two passes): the executed-memory-event list of one chunk (12 B per entry)
+        self.scratch = torch.empty(nb.nvbt_replay_scratch_size(self.ctx, chunk), dtype=torch.uint8,
+                                   device="cuda") if staged else None
         self.events = self.n
         self.kernels_per_step = -(-self.n // chunk)
+
+    def replay(self, m):
+        if self.scratch is None:
+            self.nb.nvbt_replay(self.ctx, self.hdr, self.addr, m)
+        else:
+            self.nb.nvbt_replay_staged(self.ctx, self.hdr, self.addr, m, self.scratch)
 
     def run(self, stream_events):
         """One step: generate (untimed) and replay (timed with events) every chunk."""
@@ -247,7 +256,7 @@ class ReplayBench:
             nb.nvbt_gen_events(self.ctx, 0x4E5642544E564254, self.lo + off, m, self.hdr, self.addr)
             e0, e1 = stream_events
             e0.record()
-            nb.nvbt_replay(self.ctx, self.hdr, self.addr, m)
+            self.replay(m)
             e1.record()
             e1.synchronize()
             t += e0.elapsed_time(e1) / 1e3
@@ -368,12 +377,12 @@ def run_ours(args):
 
 def run_replay(args, torch, nb, dr, rank, world, local, peaks, peaks_src):
     dev = torch.device("cuda", local)
-    wl = ReplayBench(torch, nb, dr, world, rank, n_total=args.replay_events)
+    wl = ReplayBench(torch, nb, dr, world, rank, n_total=args.replay_events, staged=args.replay_impl == "staged")
     evs = (torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
     # warm-up on one chunk
     for _ in range(args.warmup):
         nb.nvbt_gen_events(wl.ctx, 0x4E5642544E564254, 0, min(wl.chunk, wl.n), wl.hdr, wl.addr)
-        nb.nvbt_replay(wl.ctx, wl.hdr, wl.addr, min(wl.chunk, wl.n))
+        wl.replay(min(wl.chunk, wl.n))
     nb.nvbt_reset(wl.ctx)
     torch.cuda.synchronize()
     barrier(world)
@@ -774,6 +783,8 @@ def main():
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--replay-impl", choices=["staged", "single"], default="staged",
+                    help="C5: two-pass staged replay (default) or the single-pass kernel")
     ap.add_argument("--workload", choices=["c1", "c2", "c3", "c4", "c5", "f1", "f2", "f4"], default="c2")
     ap.add_argument("--fft-n", type=int, default=1 << 24, help="F4: transforms per launch")
     ap.add_argument("--fft-ctas", type=int, default=0, help="F4: grid (0 = one resident wave per kernel)")

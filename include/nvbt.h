@@ -187,6 +187,17 @@ int nvbt_gen_events(nvbt_ctx ctx, uint64_t seed, uint64_t first, uint64_t n, voi
 int nvbt_replay(nvbt_ctx ctx, const void* d_hdr, const void* d_addr, uint64_t n);
 int nvbt_replay_errors(nvbt_ctx ctx, uint64_t* bad_events);
 
+/* Staged replay: the same results as nvbt_replay (EM §2 items 1-4; north_star "trace-replay mode"),
+ * computed in two passes per block of events. Pass A streams the headers (items 1-3) and lists each
+ * executed memory event (slot index, E, pc: 12 B) in d_scratch; pass B streams the listed address slots
+ * and computes S/L (item 4, P:L187-213 (§6.1)). d_scratch: caller-owned device memory, 256-byte aligned,
+ * contents undefined between calls; a call processes n in blocks of as many events as the scratch holds.
+ * Without NVBT_MEMDIV no list is written and d_scratch may be null. ENOMEM if scratch_bytes is below
+ * nvbt_replay_scratch_size(ctx, 1). Asynchronous on the context's stream. */
+int nvbt_replay_scratch_size(nvbt_ctx ctx, uint64_t max_events_per_block, size_t* bytes);
+int nvbt_replay_staged(nvbt_ctx ctx, const void* d_hdr, const void* d_addr, uint64_t n, void* d_scratch,
+                       size_t scratch_bytes);
+
 /* Number of kernels this context launched since init (for the bench's gpu_launches claim). */
 int nvbt_launch_count(nvbt_ctx ctx, uint64_t* n);
 

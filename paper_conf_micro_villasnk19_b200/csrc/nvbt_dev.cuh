@@ -179,6 +179,68 @@ __device__ __forceinline__ uint2 sectors_lines_unsorted(unsigned long long addr,
   __syncwarp();
   return make_uint2(S, L);
 }
+// The same S/L for a caller that has already classified the access (the staged replay's lane scan knows
+// the minimum and maximum address of E): cls 0 = every address in one 1 KB word, cls 1 = every sector in
+// the 1024-sector window starting at sector `wbase` (32-aligned; all upper address words equal), cls 2 =
+// anything else (hashed all-distinct test, then the hash set). Same scratch contract as above.
+__device__ __forceinline__ uint2 sectors_lines_cls(unsigned long long addr, unsigned E, unsigned lanebit,
+                                                   unsigned lane, unsigned scr, unsigned cls, unsigned wbase) {
+  const bool act = (E & lanebit) != 0u;
+  const unsigned sk_lo = (unsigned)(addr >> 5);
+  if (cls == 0u) {
+    const unsigned word = __reduce_or_sync(FULL, act ? 1u << (sk_lo & 31u) : 0u);
+    const unsigned g = word | (word >> 1) | (word >> 2) | (word >> 3);
+    return make_uint2(__popc(word), __popc(g & 0x11111111u));
+  }
+  if (cls == 1u) {
+    const unsigned wv = ((unsigned)addr >> 5) - wbase;   // upper words equal: the low word orders the window
+    if (act) asm volatile("red.shared.and.b32 [%0], %1;" ::"r"(scr + 4u * (wv >> 5)), "r"(~(1u << (wv & 31u))) : "memory");
+    __syncwarp();
+    const unsigned word = ~lds_u32_(scr + 4u * lane);
+    asm volatile("st.shared.u32 [%0], %1;" ::"r"(scr + 4u * lane), "r"(0xffffffffu) : "memory");
+    __syncwarp();
+    const unsigned g = word | (word >> 1) | (word >> 2) | (word >> 3);
+    return make_uint2(__reduce_add_sync(FULL, __popc(word)), __reduce_add_sync(FULL, __popc(g & 0x11111111u)));
+  }
+  const unsigned long long line = addr >> 7;
+  const unsigned hh = ((unsigned)line ^ (unsigned)(line >> 32)) * 0x9E3779B1u;
+  if (act) asm volatile("red.shared.and.b32 [%0], %1;" ::"r"(scr + 4u * (hh >> 25)), "r"(~(1u << ((hh >> 20) & 31u))) : "memory");
+  __syncwarp();
+  {
+    unsigned w0, w1, w2, w3;
+    asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(w0), "=r"(w1), "=r"(w2), "=r"(w3) : "r"(scr + 16u * lane) : "memory");
+    asm volatile("st.shared.v4.u32 [%0], {%1, %1, %1, %1};" ::"r"(scr + 16u * lane), "r"(0xffffffffu) : "memory");
+    const unsigned used = __reduce_add_sync(FULL, __popc(~w0) + __popc(~w1) + __popc(~w2) + __popc(~w3));
+    __syncwarp();
+    if (used == (unsigned)__popc(E)) return make_uint2(used, used);
+  }
+  unsigned slot = hh >> 26;
+  bool pending = act, inserted = false;
+  while (__any_sync(FULL, pending)) {
+    if (pending) {
+      unsigned long long old;
+      asm volatile("atom.shared.cas.b64 %0, [%1], %2, %3;" : "=l"(old) : "r"(scr + 8u * slot), "l"(~0ull), "l"(line)
+                   : "memory");
+      if (old == ~0ull || old == line) {
+        pending = false;
+        inserted = old == ~0ull;
+      } else {
+        slot = (slot + 1u) & 63u;
+      }
+    }
+  }
+  if (act) asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(scr + 512u + 4u * slot), "r"(1u << (sk_lo & 3u)) : "memory");
+  const unsigned L = __popc(__ballot_sync(FULL, inserted));
+  __syncwarp();
+  unsigned m0, m1;
+  asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(m0), "=r"(m1) : "r"(scr + 512u + 8u * lane) : "memory");
+  asm volatile("st.shared.v2.u32 [%0], {%1, %1};" ::"r"(scr + 512u + 8u * lane), "r"(0u) : "memory");
+  asm volatile("st.shared.v4.u32 [%0], {%1, %1, %1, %1};" ::"r"(scr + 16u * lane), "r"(0xffffffffu) : "memory");
+  const unsigned S = __reduce_add_sync(FULL, __popc(m0) + __popc(m1));
+  __syncwarp();
+  return make_uint2(S, L);
+}
+
 static __device__ __noinline__ uint2 sectors_lines_unsorted_call(unsigned long long addr, unsigned E, unsigned lane,
                                                                  unsigned lanebit, unsigned scr) {
   return sectors_lines_unsorted(addr, E, lane, lanebit, scr);

@@ -169,14 +169,18 @@ def run_stencil_dist(ctx, tools, buf0, buf1, n, iters, rank, world, group=None, 
     return out
 
 
-def replay_range(ctx, seed, first, n, hdr, addr, chunk=None):
-    """Generate-then-replay events [first, first + n) in chunks that fit the given stream buffers."""
+def replay_range(ctx, seed, first, n, hdr, addr, chunk=None, scratch=None):
+    """Generate-then-replay events [first, first + n) in chunks that fit the given stream buffers; with a
+    scratch tensor the staged two-pass replay (nvbt_replay_staged) runs instead of the single pass."""
     cap = hdr.numel() // 16 if chunk is None else chunk
     done = 0
     while done < n:
         m = min(cap, n - done)
         _nb().nvbt_gen_events(ctx, seed, first + done, m, hdr, addr)
-        _nb().nvbt_replay(ctx, hdr, addr, m)
+        if scratch is None:
+            _nb().nvbt_replay(ctx, hdr, addr, m)
+        else:
+            _nb().nvbt_replay_staged(ctx, hdr, addr, m, scratch)
         done += m
 
 

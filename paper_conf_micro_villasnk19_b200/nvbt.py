@@ -88,6 +88,8 @@ _sigs = {
     "nvbt_gen_events": ([_P, C.c_uint64, C.c_uint64, C.c_uint64, _P, _P], C.c_int),
     "nvbt_replay": ([_P, _P, _P, C.c_uint64], C.c_int),
     "nvbt_replay_errors": ([_P, C.POINTER(C.c_uint64)], C.c_int),
+    "nvbt_replay_scratch_size": ([_P, C.c_uint64, C.POINTER(C.c_size_t)], C.c_int),
+    "nvbt_replay_staged": ([_P, _P, _P, C.c_uint64, _P, C.c_size_t], C.c_int),
     "nvbt_launch_count": ([_P, C.POINTER(C.c_uint64)], C.c_int),
     "nvbt_program": ([C.c_int, _P, C.c_uint32, C.POINTER(C.c_uint32), C.POINTER(C.c_uint32),
                       C.POINTER(C.c_uint32)], C.c_int),
@@ -376,6 +378,19 @@ def nvbt_gen_events(ctx, seed, first, n, hdr, addr):
 
 def nvbt_replay(ctx, hdr, addr, n):
     _check(_lib.nvbt_replay(ctx.handle, _ptr(hdr), _ptr(addr), n))
+
+
+def nvbt_replay_scratch_size(ctx, max_events_per_block):
+    b = C.c_size_t()
+    _check(_lib.nvbt_replay_scratch_size(ctx.handle, max_events_per_block, C.byref(b)))
+    return b.value
+
+
+def nvbt_replay_staged(ctx, hdr, addr, n, scratch):
+    """scratch: a device tensor (uint8) of at least nvbt_replay_scratch_size(ctx, 1) bytes, or None."""
+    nbytes = 0 if scratch is None else scratch.numel() * scratch.element_size()
+    _check(_lib.nvbt_replay_staged(ctx.handle, _ptr(hdr), _ptr(addr), n, None if scratch is None else _ptr(scratch),
+                                   nbytes))
 
 
 def nvbt_replay_errors(ctx):

@@ -316,15 +316,33 @@ def test_generator_bytes_match_oracle(nvbt):
         assert (ga == oaddr).all()   # non-memory slots are not written by either side (zeros here)
 
 
+# "staged" = nvbt_replay_staged (two passes, scratch list); digits = single-pass nvbt_replay kernel
+# variants selected through NVBT_REPLAY_VARIANT (read per call; 4 = default)
+REPLAY_VARIANTS = ["staged", "staged-small", "4", "7"]
+
+
+def _replay_scratch(nb, ctx, variant, monkeypatch):
+    """Scratch tensor for the staged variants (small: a few thousand events per block, so one call runs
+    several A/B pass pairs), else select the single-pass kernel variant."""
+    import torch
+    if not variant.startswith("staged"):
+        monkeypatch.setenv("NVBT_REPLAY_VARIANT", variant)
+        return None
+    per = 5000 if variant == "staged-small" else 1 << 20
+    return torch.empty(nb.nvbt_replay_scratch_size(ctx, per), dtype=torch.uint8, device="cuda")
+
+
+@pytest.mark.parametrize("variant", REPLAY_VARIANTS)
 @pytest.mark.parametrize("first,n", [(0, 1 << 18), (123456789, 100_003)])
-def test_replay_parity(nvbt, first, n):
+def test_replay_parity(nvbt, first, n, variant, monkeypatch):
     import torch
     nb, dr = nvbt.nvbt, nvbt.drivers
     ctx = nb.nvbt_init(nb.W_REPLAY, nb.COUNT | nb.OPHIST | nb.BB | nb.MEMDIV | nb.PER_WARP, n_warps=1 << 20)
+    scratch = _replay_scratch(nb, ctx, variant, monkeypatch)
     chunk = 1 << 16
     hdr = torch.empty(chunk * 16, dtype=torch.uint8, device="cuda")
     addr = torch.empty(chunk * 256, dtype=torch.uint8, device="cuda")
-    dr.replay_range(ctx, gen.SEED, first, n, hdr, addr)
+    dr.replay_range(ctx, gen.SEED, first, n, hdr, addr, scratch=scratch)
     g = read_all(nb, ctx, per_warp=True)
     acc = ev.Accumulator(programs.replay(), n_warps=1 << 20)
     gen.replay(acc, first, n)
@@ -387,17 +405,22 @@ def _adversarial_stream(n, seed):
     return pc.astype(np.int64), warp.astype(np.int64), A, P, addr
 
 
+@pytest.mark.parametrize("variant", REPLAY_VARIANTS)
 @pytest.mark.parametrize("seed", [1, 2])
-def test_replay_adversarial_addresses(nvbt, seed):
+def test_replay_adversarial_addresses(nvbt, seed, variant, monkeypatch):
     import torch
     nb = nvbt.nvbt
     n = 40_000
     pc, warp, A, P, addr = _adversarial_stream(n, seed)
     hdr = gen.header_bytes(pc, warp, A, P)
     ctx = nb.nvbt_init(nb.W_REPLAY, nb.COUNT | nb.MEMDIV)
+    scratch = _replay_scratch(nb, ctx, variant, monkeypatch)
     d_hdr = cuda(hdr.view(np.uint8).reshape(-1))
     d_addr = cuda(addr.view(np.uint8).reshape(-1))
-    nb.nvbt_replay(ctx, d_hdr, d_addr, n)
+    if scratch is None:
+        nb.nvbt_replay(ctx, d_hdr, d_addr, n)
+    else:
+        nb.nvbt_replay_staged(ctx, d_hdr, d_addr, n, scratch)
     g = read_all(nb, ctx)
     acc = ev.Accumulator(programs.replay())
     acc.add(0, warp, pc, A, P, addr)
@@ -461,6 +484,20 @@ def test_degenerate_shapes(nvbt):
     nb.nvbt_replay(rctx, d_h, d_a, 2)
     assert nb.nvbt_replay_errors(rctx) == 1
     assert nb.nvbt_count(rctx).tolist() == [32, 32, 1, 1]
+    # the staged replay: same degenerate behaviour, and a scratch too small for one block is ENOMEM
+    sctx = nb.nvbt_init(nb.W_REPLAY, nb.COUNT | nb.MEMDIV)
+    scratch = torch.empty(nb.nvbt_replay_scratch_size(sctx, 1), dtype=torch.uint8, device="cuda")
+    nb.nvbt_replay_staged(sctx, d_h, d_a, 0, scratch)
+    assert (nb.nvbt_count(sctx) == 0).all()
+    nb.nvbt_replay_staged(sctx, d_h, d_a, 2, scratch)
+    assert nb.nvbt_replay_errors(sctx) == 1
+    assert nb.nvbt_count(sctx).tolist() == [32, 32, 1, 1]
+    with pytest.raises(nb.NvbtError) as e:
+        nb.nvbt_replay_staged(sctx, d_h, d_a, 2, scratch[: scratch.numel() // 2])
+    assert e.value.code == nb.ENOMEM
+    cctx = nb.nvbt_init(nb.W_REPLAY, nb.COUNT)        # no MEMDIV: no list, scratch may be None
+    nb.nvbt_replay_staged(cctx, d_h, d_a, 2, None)
+    assert nb.nvbt_count(cctx).tolist() == [32, 32, 1, 1]
 
 
 def test_api_errors(nvbt):

@@ -28,7 +28,11 @@ if which in ("all", "c5"):
     hdr = torch.empty(n * 16, dtype=torch.uint8, device="cuda")
     addr = torch.empty(n * 256, dtype=torch.uint8, device="cuda")
     nb.nvbt_gen_events(rctx, 0x4E5642544E564254, 0, n, hdr, addr)
-    nb.nvbt_replay(rctx, hdr, addr, n)
+    if os.environ.get("NVBT_PROF_SINGLE"):
+        nb.nvbt_replay(rctx, hdr, addr, n)
+    else:   # staged two-pass replay (the bench default)
+        scratch = torch.empty(nb.nvbt_replay_scratch_size(rctx, n), dtype=torch.uint8, device="cuda")
+        nb.nvbt_replay_staged(rctx, hdr, addr, n, scratch)
     nb.nvbt_count(rctx)
 if which in ("all", "f4"):
     n_fft = 1 << 24
