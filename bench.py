@@ -375,6 +375,15 @@ def run_ours(args):
         dist.destroy_process_group()
 
 
+def _replay_traffic(chunk, staged):
+    """ncu DRAM bytes of one replay call on `chunk` events (captured at 2^26 events, scaled linearly)."""
+    names = ("k_rpA<0>", "k_rpB") if staged else ("k_replay4",)
+    tr = [load_traffic(k) for k in names]
+    if any(t is None for t in tr):
+        return None
+    return sum(t["traffic_bytes_per_launch"] for t in tr) / 67108864 * chunk
+
+
 def run_replay(args, torch, nb, dr, rank, world, local, peaks, peaks_src):
     dev = torch.device("cuda", local)
     wl = ReplayBench(torch, nb, dr, world, rank, n_total=args.replay_events, staged=args.replay_impl == "staged")
@@ -412,9 +421,10 @@ def run_replay(args, torch, nb, dr, rank, world, local, peaks, peaks_src):
         "roofline": {"bound": "hbm", "achieved": ach / 1e9, "peak": peaks["hbm_gbs"], "unit": "GB/s",
                      "frac": ach / 1e9 / peaks["hbm_gbs"], "peak_source": peaks_src,
                      "algorithmic_bytes_per_launch": bytes_rank * wl.chunk / wl.n,
-                     "traffic": (load_traffic("k_replay4") or {}).get("traffic_bytes_per_launch", 0) / 67108864 * wl.chunk
-                     if load_traffic("k_replay4") else None,
-                     "traffic_unit": "DRAM bytes per 2^27-event launch (ncu at 2^26, scaled; profiles/r1_traffic.json)"},
+                     "traffic": _replay_traffic(wl.chunk, staged=wl.scratch is not None),
+                     "traffic_unit": "DRAM bytes per 2^27-event replay call (ncu at 2^26, scaled; profiles/r1_traffic.json)",
+                     "kernel": "nvbt_replay_staged = k_rpA (headers, list) + k_rpB (slots)" if wl.scratch is not None
+                     else "k_replay4"},
         "gpu_launches": int(launches), "clocks": clk.summary(),
         "check": {"W_issued": int(cnt[2]), "expected": args.steps * n_all},
     }

@@ -189,7 +189,7 @@ int nvbt_replay_errors(nvbt_ctx ctx, uint64_t* bad_events);
 
 /* Staged replay: the same results as nvbt_replay (EM §2 items 1-4; north_star "trace-replay mode"),
  * computed in two passes per block of events. Pass A streams the headers (items 1-3) and lists each
- * executed memory event (slot index, E, pc: 12 B) in d_scratch; pass B streams the listed address slots
+ * executed memory event (E and a packed pc / tile / lane key: 8 B) in d_scratch; pass B streams the listed address slots
  * and computes S/L (item 4, P:L187-213 (§6.1)). d_scratch: caller-owned device memory, 256-byte aligned,
  * contents undefined between calls; a call processes n in blocks of as many events as the scratch holds.
  * Without NVBT_MEMDIV no list is written and d_scratch may be null. ENOMEM if scratch_bytes is below

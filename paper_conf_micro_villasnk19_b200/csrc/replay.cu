@@ -638,266 +638,22 @@ static size_t replay4_smem(unsigned P) {
   return (((6ull * P + 66 + 3) & ~3ull) + (size_t)L4_NW * L4_WARP_WORDS) * 4 + P + 16;
 }
 
-// ---------------------------------------------------------------- replay, pipelined lane-pair variant (V = 7)
-// The warp walks its header tiles as in V4, but the address slots of the executed memory events are not
-// analysed tile by tile: they are appended to a 16-row shared stage (cp.async.cg, 16 B per lane, two rows
-// per instruction) and a full stage is analysed while the other stage's copies are in flight (double
-// buffer, one cp.async group per stage). The analysis is lane-parallel: lanes 2j and 2j+1 take row j,
-// each scanning 16 of its 32 addresses from shared memory (8 x 16 B loads, rows swizzled so a quarter-warp
-// hits 8 distinct 16 B bank groups). The scan counts sector and line changes between consecutive lanes of
-// E — exact when the addresses of E are non-decreasing in lane order and share their upper 32 bits; the
-// two halves are joined with one exchange of (first, last, counts). Rows that fail the test (random
-// orders, 4 GB crossings) take the warp-cooperative exact path sectors_lines_unsorted().
-// Per executed memory event this is ~1/32 of the warp-cooperative monotone path's instructions.
-constexpr int L7_NW = 13;                  // warps per CTA (1 CTA per SM; bound by the 4096-pc shared bins)
-constexpr int L7_ROWS = 16;                // rows per stage
-constexpr int L7_STAGE_WORDS = L7_ROWS * 64;
-// per warp: 2 stages | meta [2][16] {E, pc} | rowsrc [32] | sectors_lines scratch
-constexpr int L7_WARP_WORDS = 2 * L7_STAGE_WORDS + 4 * L7_ROWS + 32 + SCRATCH_WORDS;
-static_assert(L7_WARP_WORDS % 4 == 0, "16 B aligned warp areas");
-
-// physical 16 B chunk of logical chunk c (0..15) in stage row j: quarter-warp reads of chunk 8h + q by
-// lanes (j, h) land on (2j + h) & 7 distinct bank groups
-__device__ __forceinline__ unsigned l7_chunk(unsigned j, unsigned c) { return c ^ ((2u * j + (c >> 3)) & 7u); }
-
-__device__ __forceinline__ void lds_v2(unsigned a, unsigned& x, unsigned& y) {
-  asm volatile("ld.shared.v2.u32 {%0,%1}, [%2];" : "=r"(x), "=r"(y) : "r"(a) : "memory");
-}
-
-// Analyse `nrows` staged rows of stage `stage` (base address) whose meta is at `meta`; adds S/L to the
-// CTA's per-pc sums and histograms.
-__device__ __forceinline__ void l7_process(unsigned stage, unsigned meta, unsigned nrows, unsigned lane,
-                                           unsigned lanebit, unsigned s_scr, unsigned s_sS, unsigned s_sL,
-                                           unsigned s_hist) {
-  const unsigned j = lane >> 1, h = lane & 1u;
-  const bool have = j < nrows;
-  unsigned E, pc;
-  lds_v2(meta + 8u * j, E, pc);
-  E = have ? E : 0u;
-  const unsigned Eh = h ? E >> 16 : E & 0xffffu;
-  const unsigned rowb = stage + 256u * j;
-  const unsigned f = (Eh ? (unsigned)__ffs(Eh) - 1u : 0u) + 16u * h;       // first active address of my half
-  unsigned f_lo, f_hi;
-  lds_v2(rowb + 16u * l7_chunk(j, f >> 1) + 8u * (f & 1u), f_lo, f_hi);
-  unsigned prev = f_lo, hb = 0, bs = 0, bl = 0, mn = f_lo, mx = f_lo;
-  bool viol = false;
-#pragma unroll
-  for (int q = 0; q < 8; ++q) {
-    uint4 v;
-    lds_v4(rowb + 16u * l7_chunk(j, 8u * h + q), v);
-#pragma unroll
-    for (int u = 0; u < 2; ++u) {
-      const bool act = (Eh >> (2 * q + u)) & 1u;
-      const unsigned lo = act ? (u ? v.z : v.x) : prev;
-      const unsigned hi = act ? (u ? v.w : v.y) : f_hi;
-      hb |= hi ^ f_hi;
-      viol |= lo < prev;
-      const unsigned x = lo ^ prev;
-      bs += x > 31u;
-      bl += x > 127u;
-      prev = lo;
-    }
-  }
-  // join the halves: lane 2j (h = 0) receives the upper half's first address, high word and counts
-  const unsigned pack = bs | bl << 8 | (unsigned)viol << 16 | (unsigned)(hb != 0u) << 17 | (unsigned)(Eh != 0u) << 18;
-  const unsigned o_pack = __shfl_xor_sync(FULL, pack, 1);
-  const unsigned o_lo = __shfl_xor_sync(FULL, f_lo, 1);
-  const unsigned o_hi = __shfl_xor_sync(FULL, f_hi, 1);
-  unsigned S = 1u + bs + (o_pack & 0xffu), L = 1u + bl + ((o_pack >> 8) & 0xffu);
-  bool slow = viol || hb != 0u || ((o_pack >> 16) & 3u) != 0u;
-  if (Eh != 0u && (o_pack >> 18) != 0u) {   // both halves active: boundary between my last and its first
-    const unsigned x = o_lo ^ prev;
-    S += x > 31u;
-    L += x > 127u;
-    slow |= o_lo < prev || o_hi != f_hi;
-  }
-  slow = slow && have && h == 0u;
-  unsigned hm = __ballot_sync(FULL, slow);
-  while (hm) {
-    const int src = __ffs(hm) - 1;
-    hm &= hm - 1;
-    const unsigned js = (unsigned)src >> 1;
-    const unsigned es = __shfl_sync(FULL, E, src);
-    unsigned long long a;
-    asm volatile("ld.shared.u64 %0, [%1];" : "=l"(a)
-                 : "r"(stage + 256u * js + 16u * l7_chunk(js, lane >> 1) + 8u * (lane & 1u)) : "memory");
-    const uint2 r = sectors_lines_unsorted(a, es, lane, lanebit, s_scr);
-    if (lane == (unsigned)src) { S = r.x; L = r.y; }
-  }
-  const bool own = have && h == 0u;
-  red_shared_add_if(own, s_sS + 4u * pc, S);
-  red_shared_add_if(own, s_sL + 4u * pc, L);
-  red_shared_add_if(own, s_hist + 4u * S, 1u);          // hS[S]
-  red_shared_add_if(own, s_hist + 4u * (33u + L), 1u);  // hL[L]
-  __syncwarp();
-}
-
-static __device__ __noinline__ void l7_process_call(unsigned stage, unsigned meta, unsigned nrows, unsigned lane,
-                                                    unsigned lanebit, unsigned s_scr, unsigned s_sS, unsigned s_sL,
-                                                    unsigned s_hist) {
-  l7_process(stage, meta, nrows, lane, lanebit, s_scr, s_sS, s_sL, s_hist);
-}
-
-template <bool PW>
-__global__ void __launch_bounds__(32 * L7_NW, 1)
-k_replay7(const uint4* __restrict__ hdr, const unsigned long long* __restrict__ addr, unsigned long long n,
-          unsigned P, const uint8_t* __restrict__ kind, DevState st, unsigned long long* err) {
-  extern __shared__ __align__(16) unsigned sm[];
-  const unsigned P4 = (6 * P + 66 + 3) & ~3u;
-  unsigned* sWarpAll = sm + P4;
-  uint8_t* sK = reinterpret_cast<uint8_t*>(sm + P4 + L7_NW * L7_WARP_WORDS);
-  for (unsigned i = threadIdx.x; i < P4; i += blockDim.x) sm[i] = 0;
-  constexpr unsigned kScr0 = 2 * L7_STAGE_WORDS + 4 * L7_ROWS + 32;
-  for (unsigned i = threadIdx.x; i < L7_NW * L7_WARP_WORDS; i += blockDim.x) {
-    const unsigned o = i % L7_WARP_WORDS;
-    sWarpAll[i] = o >= kScr0 ? scratch_init_word(o - kScr0) : 0u;
-  }
-  for (unsigned i = threadIdx.x; i < P; i += blockDim.x) sK[i] = is_mem_kind(kind[i]);
-  __syncthreads();
-
-  const unsigned lane = lane_id(), lmlt = lanemask_lt(), lanebit = 1u << lane;
-  const unsigned s_base = (unsigned)__cvta_generic_to_shared(sm);
-  const unsigned s_kind = (unsigned)__cvta_generic_to_shared(sK);
-  const unsigned s_w = (unsigned)__cvta_generic_to_shared(sWarpAll + (threadIdx.x >> 5) * L7_WARP_WORDS);
-  const unsigned s_stage = s_w;                                   // stage b at + 4096 b
-  const unsigned s_meta = s_w + 4u * 2u * L7_STAGE_WORDS;         // stage b's meta at + 128 b
-  const unsigned s_rowsrc = s_meta + 4u * 4u * L7_ROWS;
-  const unsigned s_scr = s_rowsrc + 4u * 32u;
-  const unsigned s_sS = s_base + 16u * P, s_sL = s_base + 20u * P, s_hist = s_base + 24u * P;
-  unsigned bad = 0, buf = 0, cnt = 0;
-  bool pending = false;
-  const unsigned long long warps = (unsigned long long)gridDim.x * L7_NW;
-  unsigned long long tile = (blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x) >> 5;
-  uint4 h = make_uint4(0, 0, 0, 0);
-  if (tile * 32 + lane < n) h = ld_nc_v4(hdr + tile * 32 + lane);
-  for (; tile * 32 < n; tile += warps) {
-    const bool valid = tile * 32 + lane < n;
-    const unsigned pc = h.x, A = h.z, E = h.z & h.w;
-    const unsigned long long nt = tile + warps;
-    uint4 hn = make_uint4(0, 0, 0, 0);
-    if (nt * 32 + lane < n) hn = ld_nc_v4(hdr + nt * 32 + lane);
-    const bool ok = valid && pc < P && A != 0u;
-    bad += valid && pc >= P;
-    const unsigned pcs = ok ? pc : 0u;
-    const unsigned a4 = s_base + 4u * pcs;
-    const unsigned pa = __popc(A), pe = __popc(E);
-    red_shared_add_if(ok, a4, pa);
-    red_shared_add_if(ok, a4 + 4u * P, 1u);
-    red_shared_add_if(ok && pa != pe, a4 + 8u * P, pa - pe);
-    red_shared_add_if(ok && E == 0u, a4 + 12u * P, 1u);
-    if constexpr (PW) {
-      const unsigned warp = h.y;
-      if (ok && warp < st.n_warps) {
-        atomicAdd(st.pw + warp, (unsigned long long)pe);
-        if (E) atomicAdd(st.pw + st.n_warps + warp, 1ull);
-      }
-    }
-    const bool mem = ok && E != 0u && lds_u8(s_kind + pcs) != 0u;
-    const unsigned mm = __ballot_sync(FULL, mem);
-    if (mm) {
-      const unsigned total = __popc(mm);
-      if (mem) sts_u32(s_rowsrc + 4u * __popc(mm & lmlt), lane);
-      __syncwarp();
-      const unsigned long long* tbase0 = addr + tile * 32 * 32 + 2u * (lane & 15u);
-      unsigned done = 0;
-      while (done < total) {
-        const unsigned take = min(total - done, (unsigned)L7_ROWS - cnt);
-        // meta of rows cnt .. cnt+take-1 from events done .. done+take-1 (lane i carries event done+i)
-        const unsigned srcl = lds_u32(s_rowsrc + 4u * min(done + lane, total - 1u));
-        const unsigned e_s = __shfl_sync(FULL, E, srcl), pc_s = __shfl_sync(FULL, pcs, srcl);
-        const unsigned mrow = s_meta + 128u * buf + 8u * (cnt + lane);
-        if (lane < take) asm volatile("st.shared.v2.u32 [%0], {%1, %2};" ::"r"(mrow), "r"(e_s), "r"(pc_s) : "memory");
-        // copies: two rows per instruction, lanes 0-15 the even row, 16-31 the odd one
-        const unsigned stg = s_stage + 4096u * buf;
-#pragma unroll 1
-        for (unsigned k = 0; k < take; k += 2) {
-          const unsigned rr = k + (lane >> 4);
-          if (rr < take) {
-            const unsigned src = lds_u32(s_rowsrc + 4u * (done + rr));
-            const unsigned row = cnt + rr;
-            asm volatile("cp.async.cg.shared.global [%0], [%1], 16;"
-                         ::"r"(stg + 256u * row + 16u * l7_chunk(row, lane & 15u)), "l"(tbase0 + src * 32u)
-                         : "memory");
-          }
-        }
-        cnt += take;
-        done += take;
-        if (cnt == (unsigned)L7_ROWS) {
-          asm volatile("cp.async.commit_group;" ::: "memory");
-          if (pending) {
-            asm volatile("cp.async.wait_group 1;" ::: "memory");
-            __syncwarp();
-            l7_process(s_stage + 4096u * (buf ^ 1u), s_meta + 128u * (buf ^ 1u), L7_ROWS, lane, lanebit, s_scr,
-                       s_sS, s_sL, s_hist);
-          }
-          pending = true;
-          buf ^= 1u;
-          cnt = 0;
-        }
-      }
-      __syncwarp();
-    }
-    h = hn;
-  }
-  asm volatile("cp.async.commit_group;" ::: "memory");
-  if (pending) {
-    asm volatile("cp.async.wait_group 1;" ::: "memory");
-    __syncwarp();
-    l7_process_call(s_stage + 4096u * (buf ^ 1u), s_meta + 128u * (buf ^ 1u), L7_ROWS, lane, lanebit, s_scr, s_sS,
-                    s_sL, s_hist);
-  }
-  if (cnt) {
-    asm volatile("cp.async.wait_group 0;" ::: "memory");
-    __syncwarp();
-    l7_process_call(s_stage + 4096u * buf, s_meta + 128u * buf, cnt, lane, lanebit, s_scr, s_sS, s_sL, s_hist);
-  }
-  bad = __reduce_add_sync(FULL, bad);
-  if (lane == 0 && bad) atomicAdd(err, (unsigned long long)bad);
-  __syncthreads();
-  const unsigned* sA = sm;
-  const unsigned* sW = sm + P;
-  const unsigned* sDT = sm + 2 * P;
-  const unsigned* sDW = sm + 3 * P;
-  const unsigned* sS = sm + 4 * P;
-  const unsigned* sL = sm + 5 * P;
-  const unsigned* sH = sm + 6 * P;
-  for (unsigned pc = threadIdx.x; pc < P; pc += blockDim.x) {
-    const unsigned a = sA[pc], w = sW[pc];
-    if (w) {
-      unsigned long long* s = st.site + 4 * pc;
-      atomicAdd(s + 0, (unsigned long long)a);
-      atomicAdd(s + 1, (unsigned long long)(a - sDT[pc]));
-      atomicAdd(s + 2, (unsigned long long)w);
-      atomicAdd(s + 3, (unsigned long long)(w - sDW[pc]));
-      if (sK[pc] && w != sDW[pc]) {
-        unsigned long long* m = st.mem + 3 * pc;
-        atomicAdd(m + 0, (unsigned long long)(w - sDW[pc]));
-        atomicAdd(m + 1, (unsigned long long)sS[pc]);
-        atomicAdd(m + 2, (unsigned long long)sL[pc]);
-      }
-    }
-  }
-  for (unsigned i = threadIdx.x; i < 66; i += blockDim.x)
-    if (sH[i]) atomicAdd(st.hist + i, (unsigned long long)sH[i]);
-}
-
-static size_t replay7_smem(unsigned P) {
-  return (((6ull * P + 66 + 3) & ~3ull) + (size_t)L7_NW * L7_WARP_WORDS) * 4 + P + 16;
-}
-
 // ---------------------------------------------------------------- staged replay (two passes per chunk)
 // The single-pass kernels hold 6 x 4096 u32 per-pc bins in shared memory, which leaves little room for
 // staging address slots. The staged replay splits the work along its two data streams:
-//   pass A (k_rpA): streams the 16 B headers with 32 warps per SM, does items 1-3 of EM §2 (per-pc
-//     issued/executed bins, per-warp arrays) and writes each executed memory event (slot index, E, pc:
-//     12 B) to the warp's region of a caller-owned list, compacted;
-//   pass B (k_rpB): streams the listed 256 B slots into per-warp shared stages (cp.async, double
-//     buffered, list entries prefetched a group ahead) and computes S/L lane-parallel (two lanes per
-//     slot, the scan of the V7 kernel) plus min/max of the addresses, so the rows that are not
-//     monotone go straight to the matching exact path (1 KB word, 32 KB window, hashed).
-// Extra traffic: 24 B per executed memory event (list write + read), ~7 % of the algorithmic bytes.
+//   pass A (k_rpA, 2 CTAs x 20 warps per SM): streams the 16 B headers through a per-warp cp.async ring
+//     (4 tiles in flight), does items 1-3 of EM §2 (per-pc issued/executed bins, per-warp arrays) and
+//     writes each executed memory event as one 8 B entry {E, pc | tile | lane} to its warp's region of a
+//     caller-owned list, compacted;
+//   pass B (k_rpB, 20 warps per SM): streams the listed 256 B slots into per-warp shared stages
+//     (cp.async, double buffered, list entries prefetched a group ahead) and computes S/L lane-parallel:
+//     two lanes per slot each scan 16 addresses, counting sector/line changes (exact when the addresses
+//     of E are non-decreasing within one 4 GB region) and their min/max, so the other rows go straight
+//     to the matching exact warp-cooperative path (1 KB word, 32 KB window, hashed).
+// Extra traffic: 16 B per executed memory event (list write + read), ~5 % of the algorithmic bytes.
 constexpr int RA_NW = 20;     // pass A warps per CTA (one list region per warp)
 constexpr int RB_NW = 20;     // pass B warps per CTA (warp w of pass B analyses region w)
+constexpr int RA_CTAS_PER_SM = 2;   // pass A CTAs per SM
 constexpr int RA_DEPTH = 4;   // pass A header tiles in flight per warp
 constexpr int RB_ROWS = 16;   // slots per stage
 constexpr int RB_STAGES = 2;
@@ -905,11 +661,16 @@ constexpr int RB_WARP_WORDS = RB_STAGES * (RB_ROWS * 64 + 2 * RB_ROWS) + SCRATCH
 constexpr size_t RS_COUNTS_BYTES = 65536;   // u32 per pass-A warp (<= 16384 warps)
 static_assert(RB_WARP_WORDS % 4 == 0, "16 B aligned warp areas");
 
+__device__ __forceinline__ void lds_v2(unsigned a, unsigned& x, unsigned& y) {
+  asm volatile("ld.shared.v2.u32 {%0,%1}, [%2];" : "=r"(x), "=r"(y) : "r"(a) : "memory");
+}
+
+// List entry of an executed memory event: {E, pc << 20 | k << 5 | lane}, where the event is lane `lane`
+// of the k-th tile of pass-A warp r (the entry's region): event index (r + k * warps) * 32 + lane.
 template <bool PW>
-__global__ void __launch_bounds__(32 * RA_NW, 1)
-k_rpA(const uint4* __restrict__ hdr, unsigned long long n, unsigned P, const uint8_t* __restrict__ kind,
-      DevState st, unsigned long long* err, unsigned* __restrict__ counts, unsigned* __restrict__ l_idx,
-      unsigned* __restrict__ l_E, unsigned* __restrict__ l_pc, unsigned region_cap) {
+__global__ void __launch_bounds__(32 * RA_NW, RA_CTAS_PER_SM)
+k_rpA(const uint4* __restrict__ hdr, unsigned n, unsigned P, const uint8_t* __restrict__ kind, DevState st,
+      unsigned long long* err, unsigned* __restrict__ counts, uint2* __restrict__ l_ent, unsigned region_cap) {
   extern __shared__ __align__(16) unsigned sm[];
   uint8_t* sK = reinterpret_cast<uint8_t*>(sm + 4 * P);
   for (unsigned i = threadIdx.x; i < 4 * P; i += blockDim.x) sm[i] = 0;
@@ -919,30 +680,28 @@ k_rpA(const uint4* __restrict__ hdr, unsigned long long n, unsigned P, const uin
   const unsigned s_base = (unsigned)__cvta_generic_to_shared(sm);
   const unsigned s_kind = (unsigned)__cvta_generic_to_shared(sK);
   const unsigned gw = blockIdx.x * RA_NW + (threadIdx.x >> 5);
-  const unsigned long long warps = (unsigned long long)gridDim.x * RA_NW;
-  const unsigned long long base = (unsigned long long)gw * region_cap;
-  unsigned cnt = 0, bad = 0;
-  unsigned long long tile = gw;
+  const unsigned warps = gridDim.x * RA_NW;
+  uint2* const ent = l_ent + (unsigned long long)gw * region_cap;
+  unsigned cnt = 0, bad = 0, k = 0;
   // headers RA_DEPTH tiles ahead: per-warp ring of 512 B tile slots filled by cp.async (16 B per lane;
   // each lane reads back only what it copied, so no warp barrier is needed)
   const unsigned s_hq = s_base + 16u * P + ((P + 15u) & ~15u) + 512u * RA_DEPTH * (threadIdx.x >> 5) + 16u * lane;
 #pragma unroll
   for (int d = 0; d < RA_DEPTH; ++d) {
-    const unsigned long long t = tile + d * warps;
-    if (t * 32 + lane < n)
-      asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(s_hq + 512u * d), "l"(hdr + t * 32 + lane) : "memory");
+    const unsigned i = (gw + d * warps) * 32 + lane;
+    if (i < n) asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(s_hq + 512u * d), "l"(hdr + i) : "memory");
     asm volatile("cp.async.commit_group;" ::: "memory");
   }
   // slot d holds tile (round + d); it is refilled with tile (round + d + DEPTH) once consumed
-  for (unsigned long long round = tile; round * 32 < n; round += RA_DEPTH * warps) {
+  for (unsigned round = gw; round * 32 < n; round += RA_DEPTH * warps) {
 #pragma unroll
    for (int d = 0; d < RA_DEPTH; ++d) {
-    tile = round + d * warps;
+    const unsigned tile = round + d * warps;
     if (tile * 32 >= n) break;
     asm volatile("cp.async.wait_group %0;" ::"n"(RA_DEPTH - 1) : "memory");
     uint4 h;
     lds_v4(s_hq + 512u * d, h);
-    const unsigned long long i = tile * 32 + lane;
+    const unsigned i = tile * 32 + lane;
     const bool valid = i < n;
     const unsigned pc = h.x, A = h.z, E = h.z & h.w;
     const bool ok = valid && pc < P && A != 0u;
@@ -963,16 +722,11 @@ k_rpA(const uint4* __restrict__ hdr, unsigned long long n, unsigned P, const uin
     }
     const bool mem = ok && E != 0u && lds_u8(s_kind + pcs) != 0u;
     const unsigned mm = __ballot_sync(FULL, mem);
-    if (mem && l_idx != nullptr) {
-      const unsigned long long pos = base + cnt + __popc(mm & lmlt);
-      l_idx[pos] = (unsigned)i;
-      l_E[pos] = E;
-      l_pc[pos] = pc;
-    }
+    if (mem && l_ent != nullptr) ent[cnt + __popc(mm & lmlt)] = make_uint2(E, pc << 20 | k << 5 | lane);
     cnt += __popc(mm);
-    const unsigned long long tn = tile + RA_DEPTH * warps;
-    if (tn * 32 + lane < n)
-      asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(s_hq + 512u * d), "l"(hdr + tn * 32 + lane) : "memory");
+    ++k;
+    const unsigned in = i + RA_DEPTH * warps * 32;
+    if (in < n) asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(s_hq + 512u * d), "l"(hdr + in) : "memory");
     asm volatile("cp.async.commit_group;" ::: "memory");
    }
   }
@@ -1081,8 +835,7 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
 
 __global__ void __launch_bounds__(32 * RB_NW, 1)
 k_rpB(const unsigned long long* __restrict__ addr, unsigned P, const uint8_t* __restrict__ kind, DevState st,
-      const unsigned* __restrict__ counts, unsigned n_regions, const unsigned* __restrict__ l_idx,
-      const unsigned* __restrict__ l_E, const unsigned* __restrict__ l_pc, unsigned region_cap) {
+      const unsigned* __restrict__ counts, unsigned n_regions, const uint2* __restrict__ l_ent, unsigned region_cap) {
   extern __shared__ __align__(16) unsigned sm[];
   const unsigned PB = (2 * P + 66 + 3) & ~3u;      // sS[P] | sL[P] | hist[66]
   unsigned* sWarpAll = sm + PB;
@@ -1105,7 +858,8 @@ k_rpB(const unsigned long long* __restrict__ addr, unsigned P, const uint8_t* __
   unsigned r = blockIdx.x * RB_NW + (threadIdx.x >> 5), off = 0;
   unsigned rcnt = r < n_regions ? counts[r] : 0u;
   // next group's list entries (row j in lanes j and j + 16), loaded one group ahead
-  unsigned nx_rows = 0, nx_idx = 0, nx_E = 0, nx_pc = 0;
+  unsigned nx_rows = 0, nx_r = 0;
+  uint2 nx_ent = make_uint2(0u, 0u);
   auto fetch = [&]() {
     while (r < n_regions && off >= rcnt) {
       r += WB;
@@ -1114,14 +868,14 @@ k_rpB(const unsigned long long* __restrict__ addr, unsigned P, const uint8_t* __
     }
     nx_rows = r < n_regions ? min(rcnt - off, (unsigned)RB_ROWS) : 0u;
     const unsigned long long p = (unsigned long long)r * region_cap + off + j;
-    const bool ld = j < nx_rows;
-    nx_idx = ld ? l_idx[p] : 0u;
-    nx_E = ld ? l_E[p] : 0u;
-    nx_pc = ld ? l_pc[p] : 0u;
+    nx_ent = j < nx_rows ? l_ent[p] : make_uint2(0u, 0u);   // decoded at issue time (load in flight)
+    nx_r = r;
     off += nx_rows;
   };
   // stage the fetched group into stage s (meta + slot copies), then fetch the next group
   auto issue = [&](unsigned s) {
+    const unsigned nx_E = nx_ent.x, nx_pc = nx_ent.y >> 20;
+    const unsigned nx_idx = (nx_r + ((nx_ent.y >> 5) & 0x7fffu) * n_regions) * 32u + (nx_ent.y & 31u);
     if (h == 0u)
       asm volatile("st.shared.v2.u32 [%0], {%1, %2};" ::"r"(s_meta + 128u * s + 8u * j), "r"(nx_E), "r"(nx_pc) : "memory");
     const unsigned stg = s_w + 4096u * s;
@@ -1339,34 +1093,10 @@ static int launch_replay4(nvbt_ctx c, const void* d_hdr, const void* d_addr, uin
   return NVBT_OK;
 }
 
-static int launch_replay7(nvbt_ctx c, const void* d_hdr, const void* d_addr, uint64_t n, const DevState& st) {
-  const size_t smem = replay7_smem(c->n_pcs);
-  static bool attr_set = false;
-  if (!attr_set) {
-    NVBT_CUDA(cudaFuncSetAttribute(k_replay7<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)replay7_smem(4096)));
-    NVBT_CUDA(cudaFuncSetAttribute(k_replay7<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)replay7_smem(4096)));
-    attr_set = true;
-  }
-  const unsigned long long kMaxPerLaunch = 1ull << 30;
-  const int sms = sm_count(c->device);
-  for (uint64_t off = 0; off < n; off += kMaxPerLaunch) {
-    const uint64_t m = std::min<uint64_t>(kMaxPerLaunch, n - off);
-    const unsigned long long tiles = (m + 31) / 32;
-    const int blocks = (int)std::min<unsigned long long>((tiles + 2 * L7_NW - 1) / (2 * L7_NW), (unsigned long long)sms);
-    auto kern = st.pw != nullptr ? k_replay7<true> : k_replay7<false>;
-    kern<<<blocks, 32 * L7_NW, smem, c->stream>>>(static_cast<const uint4*>(d_hdr) + off,
-                                                  static_cast<const unsigned long long*>(d_addr) + off * 32, m,
-                                                  c->n_pcs, c->d_kind, st, c->ctl + CTL_REPLAY_ERR);
-    NVBT_CUDA(cudaGetLastError());
-    c->launches++;
-  }
-  return NVBT_OK;
-}
-
-// Staged replay: scratch = counts [16384 u32] | idx [cap] | E [cap] | pc [cap]; passes of at most
+// Staged replay: scratch = counts [16384 u32] | entries [cap] (uint2, k_rpA); passes of at most
 // cap - 32 * (pass-A warps) events (every pass-A warp owns a region of 32 * ceil(tiles / warps) entries).
 static unsigned long long staged_cap(size_t bytes) {
-  return bytes > RS_COUNTS_BYTES ? ((bytes - RS_COUNTS_BYTES) / 12) & ~63ull : 0ull;
+  return bytes > RS_COUNTS_BYTES ? ((bytes - RS_COUNTS_BYTES) / 8) & ~63ull : 0ull;
 }
 
 static int launch_staged(nvbt_ctx c, const void* d_hdr, const void* d_addr, uint64_t n, const DevState& st,
@@ -1381,7 +1111,7 @@ static int launch_staged(nvbt_ctx c, const void* d_hdr, const void* d_addr, uint
   const int sms = sm_count(c->device);
   const bool memdiv = (c->flags & NVBT_MEMDIV) != 0;
   const unsigned long long cap = staged_cap(scratch_bytes);
-  const unsigned long long max_warps = (unsigned long long)sms * RA_NW;
+  const unsigned long long max_warps = (unsigned long long)sms * RA_CTAS_PER_SM * RA_NW;
   unsigned long long pass = 1ull << 30;   // keeps every CTA's u32 bins far from overflow
   if (memdiv) {
     if (scratch == nullptr || cap <= 32ull * max_warps)
@@ -1390,25 +1120,30 @@ static int launch_staged(nvbt_ctx c, const void* d_hdr, const void* d_addr, uint
     pass = std::min(pass, (cap - 32ull * max_warps) & ~31ull);
   }
   unsigned* counts = static_cast<unsigned*>(scratch);
-  unsigned* l_idx = memdiv ? reinterpret_cast<unsigned*>(static_cast<char*>(scratch) + RS_COUNTS_BYTES) : nullptr;
-  unsigned* l_E = memdiv ? l_idx + cap : nullptr;
-  unsigned* l_pc = memdiv ? l_E + cap : nullptr;
+  uint2* l_ent = memdiv ? reinterpret_cast<uint2*>(static_cast<char*>(scratch) + RS_COUNTS_BYTES) : nullptr;
   for (uint64_t off = 0; off < n; off += pass) {
     const uint64_t m = std::min<uint64_t>(pass, n - off);
     const unsigned long long tiles = (m + 31) / 32;
-    const int blocks = (int)std::min<unsigned long long>((tiles + 2 * RA_NW - 1) / (2 * RA_NW), (unsigned long long)sms);
+    // pass A: up to RA_CTAS_PER_SM CTAs per SM (its shared footprint allows 2), pass B: one per SM; a
+    // pass-B warp takes the regions gw, gw + warps_B, ... (exactly RA_CTAS_PER_SM each on full grids)
+    const int blocks = (int)std::min<unsigned long long>((tiles + 2 * RA_NW - 1) / (2 * RA_NW),
+                                                         (unsigned long long)sms * RA_CTAS_PER_SM);
+    const int blocks_b = std::min(blocks, sms);
     const unsigned warps = (unsigned)blocks * RA_NW;
     const unsigned region_cap = (unsigned)(32 * ((tiles + warps - 1) / warps));
+    // list keys hold the tile ordinal within a warp in 15 bits (pass <= 2^30 events on >= 1024 warps, or
+    // fewer events on small grids)
+    if (region_cap / 32 > 32768u) return set_error(NVBT_EINVAL, "staged replay: %u tiles per warp", region_cap / 32);
     auto ka = st.pw != nullptr ? k_rpA<true> : k_rpA<false>;
     ka<<<blocks, 32 * RA_NW, rpA_smem(c->n_pcs), c->stream>>>(
-        static_cast<const uint4*>(d_hdr) + off, m, c->n_pcs, c->d_kind, st, c->ctl + CTL_REPLAY_ERR,
-        memdiv ? counts : nullptr, l_idx, l_E, l_pc, region_cap);
+        static_cast<const uint4*>(d_hdr) + off, (unsigned)m, c->n_pcs, c->d_kind, st, c->ctl + CTL_REPLAY_ERR,
+        memdiv ? counts : nullptr, l_ent, region_cap);
     NVBT_CUDA(cudaGetLastError());
     c->launches++;
     if (!memdiv) continue;
-    k_rpB<<<blocks, 32 * RB_NW, rpB_smem(c->n_pcs), c->stream>>>(
-        static_cast<const unsigned long long*>(d_addr) + off * 32, c->n_pcs, c->d_kind, st, counts, warps, l_idx,
-        l_E, l_pc, region_cap);
+    k_rpB<<<blocks_b, 32 * RB_NW, rpB_smem(c->n_pcs), c->stream>>>(
+        static_cast<const unsigned long long*>(d_addr) + off * 32, c->n_pcs, c->d_kind, st, counts, warps, l_ent,
+        region_cap);
     NVBT_CUDA(cudaGetLastError());
     c->launches++;
   }
@@ -1420,8 +1155,8 @@ extern "C" {
 int nvbt_replay_scratch_size(nvbt_ctx c, uint64_t max_events, size_t* bytes) {
   if (!c || !bytes) return set_error(NVBT_EINVAL, "null argument");
   const unsigned long long per = std::min<unsigned long long>(std::max<uint64_t>(max_events, 1), 1ull << 30);
-  const unsigned long long cap = ((per + 31) & ~31ull) + 32ull * sm_count(c->device) * RA_NW + 64;
-  *bytes = RS_COUNTS_BYTES + 12 * cap;
+  const unsigned long long cap = ((per + 31) & ~31ull) + 32ull * sm_count(c->device) * RA_CTAS_PER_SM * RA_NW + 64;
+  *bytes = RS_COUNTS_BYTES + 8 * cap;
   return NVBT_OK;
 }
 
@@ -1454,7 +1189,6 @@ int nvbt_replay(nvbt_ctx c, const void* d_hdr, const void* d_addr, uint64_t n) {
     g_replay_variant = e && *e ? atoi(e) : 4;
   }
   switch (g_replay_variant) {
-    case 7: return launch_replay7(c, d_hdr, d_addr, n, st);
     case 0: return launch_replay<0>(c, d_hdr, d_addr, n, st);
     case 2: return launch_replay<2>(c, d_hdr, d_addr, n, st);
     case 3: return launch_replay_lane(c, d_hdr, d_addr, n, st);
