@@ -241,6 +241,30 @@ __device__ __forceinline__ uint2 sectors_lines_cls(unsigned long long addr, unsi
   return make_uint2(S, L);
 }
 
+// The three classes of sectors_lines_cls() as separate functions (callers that loop per class):
+// sl_word: all lanes of E in one 1 KB word (only the low address word is needed);
+__device__ __forceinline__ uint2 sl_word(unsigned a_lo, bool act) {
+  const unsigned word = __reduce_or_sync(FULL, act ? 1u << ((a_lo >> 5) & 31u) : 0u);
+  const unsigned g = word | (word >> 1) | (word >> 2) | (word >> 3);
+  return make_uint2(__popc(word), __popc(g & 0x11111111u));
+}
+// sl_window: all sectors of E in the 1024-sector window from sector wbase (32-aligned, upper words equal);
+__device__ __forceinline__ uint2 sl_window(unsigned a_lo, bool act, unsigned lane, unsigned scr, unsigned wbase) {
+  const unsigned wv = (a_lo >> 5) - wbase;
+  if (act) asm volatile("red.shared.and.b32 [%0], %1;" ::"r"(scr + 4u * (wv >> 5)), "r"(~(1u << (wv & 31u))) : "memory");
+  __syncwarp();
+  const unsigned word = ~lds_u32_(scr + 4u * lane);
+  asm volatile("st.shared.u32 [%0], %1;" ::"r"(scr + 4u * lane), "r"(0xffffffffu) : "memory");
+  __syncwarp();
+  const unsigned g = word | (word >> 1) | (word >> 2) | (word >> 3);
+  return make_uint2(__reduce_add_sync(FULL, __popc(word)), __reduce_add_sync(FULL, __popc(g & 0x11111111u)));
+}
+// sl_wide: anything else (class 2 of sectors_lines_cls).
+__device__ __forceinline__ uint2 sl_wide(unsigned long long addr, unsigned E, unsigned lanebit, unsigned lane,
+                                         unsigned scr) {
+  return sectors_lines_cls(addr, E, lanebit, lane, scr, 2u, 0u);
+}
+
 static __device__ __noinline__ uint2 sectors_lines_unsorted_call(unsigned long long addr, unsigned E, unsigned lane,
                                                                  unsigned lanebit, unsigned scr) {
   return sectors_lines_unsorted(addr, E, lane, lanebit, scr);

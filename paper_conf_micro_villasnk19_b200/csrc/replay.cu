@@ -811,20 +811,39 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
   const unsigned wbase = (rmn >> 5) & ~31u;
   const unsigned cls = hb_row ? 2u : (rmn >> 10) == (rmx >> 10) ? 0u : ((rmx >> 5) - wbase < 1024u ? 1u : 2u);
   const bool own = h == 0u && E != 0u;
-  // rows that are not monotone within one 4 GB region: exact warp-cooperative path, classified by the
-  // row's address range (one 1 KB word / a 32 KB window / anything else)
-  unsigned hm = __ballot_sync(FULL, own && slow);
-  while (hm) {
-    const int src = __ffs(hm) - 1;
-    hm &= hm - 1;
+  // rows that are not monotone within one 4 GB region: exact warp-cooperative paths, one loop per class of
+  // the row's address range (one 1 KB word / a 32 KB window / anything else); lane l reads address l
+  const unsigned l8 = 8u * lane;
+  unsigned m0 = __ballot_sync(FULL, own && slow && cls == 0u);
+  unsigned m1 = __ballot_sync(FULL, own && slow && cls == 1u);
+  unsigned m2 = __ballot_sync(FULL, own && slow && cls == 2u);
+  while (m0) {
+    const unsigned src = 31u - __clz(m0);
+    m0 ^= 1u << src;
     const unsigned es = __shfl_sync(FULL, E, src);
-    const unsigned cs = __shfl_sync(FULL, cls, src), wb = __shfl_sync(FULL, wbase, src);
+    const unsigned a_lo = lds_u32(stage + 256u * src + (l8 ^ (16u * (src & 7u))));
+    const uint2 r = sl_word(a_lo, (es & lanebit) != 0u);
+    S = lane == src ? r.x : S;
+    L = lane == src ? r.y : L;
+  }
+  while (m1) {
+    const unsigned src = 31u - __clz(m1);
+    m1 ^= 1u << src;
+    const unsigned es = __shfl_sync(FULL, E, src), wb = __shfl_sync(FULL, wbase, src);
+    const unsigned a_lo = lds_u32(stage + 256u * src + (l8 ^ (16u * (src & 7u))));
+    const uint2 r = sl_window(a_lo, (es & lanebit) != 0u, lane, s_scr, wb);
+    S = lane == src ? r.x : S;
+    L = lane == src ? r.y : L;
+  }
+  while (m2) {
+    const unsigned src = 31u - __clz(m2);
+    m2 ^= 1u << src;
+    const unsigned es = __shfl_sync(FULL, E, src);
     unsigned long long a;
-    asm volatile("ld.shared.u64 %0, [%1];" : "=l"(a)
-                 : "r"(stage + 256u * (unsigned)src + 16u * ((lane >> 1) ^ ((unsigned)src & 7u)) + 8u * (lane & 1u))
-                 : "memory");
-    const uint2 r = sectors_lines_cls(a, es, lanebit, lane, s_scr, cs, wb);
-    if (lane == (unsigned)src) { S = r.x; L = r.y; }
+    asm volatile("ld.shared.u64 %0, [%1];" : "=l"(a) : "r"(stage + 256u * src + (l8 ^ (16u * (src & 7u)))) : "memory");
+    const uint2 r = sl_wide(a, es, lanebit, lane, s_scr);
+    S = lane == src ? r.x : S;
+    L = lane == src ? r.y : L;
   }
   red_shared_add_if(own, s_sS + 4u * pc, S);
   red_shared_add_if(own, s_sL + 4u * pc, L);
