@@ -350,20 +350,23 @@ def test_replay_parity(nvbt, first, n, variant, monkeypatch):
     assert nb.nvbt_replay_errors(ctx) == 0
 
 
-def test_replay_merge_equals_single(nvbt):
-    """a8: two partitions merged by summing the packed accumulator region equal one run (I-6)."""
+@pytest.mark.parametrize("staged", [False, True])
+def test_replay_merge_equals_single(nvbt, staged):
+    """a8: three partitions merged by summing the packed accumulator region equal one run (I-6); the
+    single run uses the other replay path, so the two paths also agree with each other."""
     import torch
     nb, dr = nvbt.nvbt, nvbt.drivers
     n = 200_000
     hdr = torch.empty((1 << 16) * 16, dtype=torch.uint8, device="cuda")
     addr = torch.empty((1 << 16) * 256, dtype=torch.uint8, device="cuda")
     whole = nb.nvbt_init(nb.W_REPLAY, nb.COUNT | nb.MEMDIV)
-    dr.replay_range(whole, gen.SEED, 0, n, hdr, addr)
+    scratch = torch.empty(nb.nvbt_replay_scratch_size(whole, 1 << 16), dtype=torch.uint8, device="cuda")
+    dr.replay_range(whole, gen.SEED, 0, n, hdr, addr, scratch=None if staged else scratch)
     parts = []
     for r in range(3):
         lo, hi = dr.shard_range(n, r, 3)
         c = nb.nvbt_init(nb.W_REPLAY, nb.COUNT | nb.MEMDIV)
-        dr.replay_range(c, gen.SEED, lo, hi - lo, hdr, addr)
+        dr.replay_range(c, gen.SEED, lo, hi - lo, hdr, addr, scratch=scratch if staged else None)
         parts.append(c)
     v0 = nb.nvbt_accum_view(parts[0])
     v0 += nb.nvbt_accum_view(parts[1]) + nb.nvbt_accum_view(parts[2])
