@@ -43,6 +43,17 @@ def load_traffic(kernel):
         return None
 
 
+def load_counters(kernel, keys=("warp_inst_per_unit", "dram_bytes_per_unit", "shared_atomic_wavefronts_per_unit",
+                                 "global_atomic_sectors_per_unit", "issue_active_pct")):
+    """ncu counters per unit of work of `kernel` from the committed capture (profiles/r1_ncu_counters.json)."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "r1_ncu_counters.json")) as f:
+            d = json.load(f).get(kernel)
+    except Exception:
+        return None
+    return None if d is None else {k: d[k] for k in keys if k in d}
+
+
 def load_peaks():
     try:
         with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
@@ -365,6 +376,9 @@ def run_ours(args):
                          "instr_speed_vs_plain": statistics.median(t_plain) / t_kernel,
                          "ncu": "profiles/r1_ncu_summary_c2_c5.txt: l1tex 98.8 % (plain) / 95.2 % (instrumented), "
                                 "issue-active 6.9 % / 85.2 %"}
+    # ncu evidence per warp event (the north_star's instructions per event and atomic traffic)
+    line["ncu_per_event"] = {"instrumented": load_counters("k_sgemm<6>"), "plain": load_counters("k_sgemm<0>"),
+                             "source": "profiles/r1_ncu_counters.json (ncu --set full, tools/prof_step.py c2)"}
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         rate, sample = wl.oracle_sample(args.cpu_budget)
         line["cpu_baseline"] = {"value": rate, "unit": "events/s", "cores": 1, "kind": "oracle", "sample": sample}
@@ -425,6 +439,8 @@ def run_replay(args, torch, nb, dr, rank, world, local, peaks, peaks_src):
                      "traffic_unit": "DRAM bytes per 2^27-event replay call (ncu at 2^26, scaled; profiles/r1_traffic.json)",
                      "kernel": "nvbt_replay_staged = k_rpA (headers, list) + k_rpB (slots)" if wl.scratch is not None
                      else "k_replay4"},
+        "ncu_per_event": {"k_rpA": load_counters("k_rpA"), "k_rpB": load_counters("k_rpB"),
+                          "source": "profiles/r1_ncu_counters.json (ncu --set full, tools/prof_step.py c5)"},
         "gpu_launches": int(launches), "clocks": clk.summary(),
         "check": {"W_issued": int(cnt[2]), "expected": args.steps * n_all},
     }
