@@ -2,15 +2,13 @@
 //
 // Replay applies EM §2 items 1-4 to an HBM-resident stream of 16 B event headers and 256 B address
 // slots. It is HBM-bound: the algorithmic bytes are 16 per header plus 256 per executed memory event
-// (the only slots that must be read). Layout of the work:
-//   * persistent grid (2 CTAs x 512 threads per SM), each warp strides over 32-event tiles; lane l owns
-//     header tile*32+l (one 16 B non-coherent load per lane = 512 B coalesced per warp);
-//   * per-pc counters are privatised per CTA in shared memory (u32; t_issued, w_issued and the two
-//     "predicated-off" deltas that only exist when E != A) and folded into the global u64 bins once per
-//     CTA at the end (a8);
-//   * executed memory events of the tile (ballot) are processed by the whole warp: the 256 B slot is
-//     read by 32 lanes (8 B each, coalesced), S/L come from two __match_any_sync + leader ballots, the
-//     S/L histograms live in lane-distributed registers (lane l counts S == l + 1).
+// (the only slots that must be read). Two paths, same results:
+//   * nvbt_replay (k_replay4): one pass, one CTA of 32 warps per SM; each warp strides over 32-event tiles
+//     (lane l owns header tile*32+l), counts into per-CTA shared per-pc bins (folded into the global u64
+//     bins once per CTA, a8), and analyses the tile's executed memory events warp-cooperatively
+//     (sectors_lines(), slots staged by cp.async);
+//   * nvbt_replay_staged (k_rpA + k_rpB): a header pass that lists the executed memory events and a slot
+//     pass that analyses them lane-parallel from double-buffered shared stages (section below).
 #include <cstdlib>
 #include <cstring>
 
@@ -89,8 +87,6 @@ __global__ void __launch_bounds__(256) k_gen(GenConsts G, unsigned long long fir
 }
 
 // ---------------------------------------------------------------- replay
-constexpr int RP_BATCH = 8;  // memory events whose slots are loaded before processing
-
 __device__ __forceinline__ void red_shared_add(unsigned saddr, unsigned v) {
   asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(saddr), "r"(v) : "memory");
 }
@@ -104,195 +100,8 @@ __device__ __forceinline__ uint4 ld_nc_v4(const uint4* p) {
                : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
   return r;
 }
-__device__ __forceinline__ unsigned long long ld_nc_u64(const unsigned long long* p) {
-  unsigned long long r;
-  asm volatile("ld.global.nc.L1::no_allocate.u64 %0, [%1];" : "=l"(r) : "l"(p));
-  return r;
-}
 
-// Replay kernel variants (same results, different staging of the address slots):
-//   V = 0: 8 slot loads per batch into registers, batch processing unrolled (large code);
-//   V = 1: 8 slot loads per batch into registers, rolled processing loop (register select);
-//   V = 2: slots staged into shared memory with cp.async (8 B per lane), rolled processing loop.
-template <int V> struct ReplayCfg;
-template <> struct ReplayCfg<0> { static constexpr int THREADS = 512, MINB = 2; };
-template <> struct ReplayCfg<1> { static constexpr int THREADS = 512, MINB = 2; };
-template <> struct ReplayCfg<2> { static constexpr int THREADS = 1024, MINB = 1; };
-
-__device__ __forceinline__ void cp_async8(unsigned saddr, const void* g) {
-  asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(saddr), "l"(g) : "memory");
-}
-
-template <int V, bool PW>
-__global__ void __launch_bounds__(ReplayCfg<V>::THREADS, ReplayCfg<V>::MINB)
-k_replay(const uint4* __restrict__ hdr, const unsigned long long* __restrict__ addr, unsigned long long n, unsigned P,
-         const uint8_t* __restrict__ kind, DevState st, unsigned long long* err) {
-  constexpr int NW = ReplayCfg<V>::THREADS / 32;
-  extern __shared__ __align__(16) unsigned sm[];
-  unsigned* sA = sm;            // t_issued
-  unsigned* sW = sm + P;        // w_issued
-  unsigned* sDT = sm + 2 * P;   // popc(A & ~E)
-  unsigned* sDW = sm + 3 * P;   // [A != 0 && E == 0]
-  unsigned* sS = sm + 4 * P;
-  unsigned* sL = sm + 5 * P;
-  unsigned* sH = sm + 6 * P;    // hS[33], hL[33]
-  unsigned* sScr = sm + ((6 * P + 66 + 3) & ~3u);   // per-warp scratch of sectors_lines() (16 B aligned)
-  unsigned long long* sStage = reinterpret_cast<unsigned long long*>(sScr + SCRATCH_WORDS * NW);  // V2: [NW][8][32]
-  uint8_t* sK = reinterpret_cast<uint8_t*>(sScr + SCRATCH_WORDS * NW + (V == 2 ? 2 * NW * RP_BATCH * 32 : 0));
-  for (unsigned i = threadIdx.x; i < 6 * P + 66; i += blockDim.x) sm[i] = 0;
-  for (unsigned i = threadIdx.x; i < SCRATCH_WORDS * NW; i += blockDim.x) sScr[i] = scratch_init_word(i % SCRATCH_WORDS);
-  for (unsigned i = threadIdx.x; i < P; i += blockDim.x) sK[i] = is_mem_kind(kind[i]);
-  __syncthreads();
-
-  const unsigned lane = lane_id(), lmlt = lanemask_lt(), lanebit = 1u << lane;
-  const unsigned s_base = (unsigned)__cvta_generic_to_shared(sm);
-  const unsigned s_scr = (unsigned)__cvta_generic_to_shared(sScr + SCRATCH_WORDS * (threadIdx.x >> 5));
-  const unsigned s_stage = (unsigned)__cvta_generic_to_shared(sStage + (threadIdx.x >> 5) * RP_BATCH * 32 + lane);
-  unsigned hS = 0, hL = 0;
-  unsigned bad = 0;
-  const unsigned long long warps = (unsigned long long)gridDim.x * (blockDim.x >> 5);
-  unsigned long long tile = (blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x) >> 5;
-  uint4 h = make_uint4(0, 0, 0, 0);
-  if (tile * 32 + lane < n) h = ld_nc_v4(hdr + tile * 32 + lane);
-
-  auto process = [&](unsigned long long a, int src, unsigned E) {
-    const unsigned es = __shfl_sync(FULL, E, src);
-    const unsigned ps = __shfl_sync(FULL, h.x, src);
-    unsigned S, L;
-    sectors_lines<true, false>(a, es, lane, lanebit, lmlt, s_scr, S, L);
-    red_shared_add_if(lane == 0, s_base + 4u * (4 * P + ps), S);   // sS[ps]
-    red_shared_add_if(lane == 0, s_base + 4u * (5 * P + ps), L);   // sL[ps]
-    inc_if_eq(hS, S, lane + 1u);
-    inc_if_eq(hL, L, lane + 1u);
-  };
-
-  for (; tile * 32 < n; tile += warps) {
-    const bool valid = tile * 32 + lane < n;
-    const unsigned pc = h.x, A = h.z, E = h.z & h.w, warp = h.y;
-    // prefetch the next tile's header
-    const unsigned long long nt = tile + warps;
-    uint4 hn = make_uint4(0, 0, 0, 0);
-    if (nt * 32 + lane < n) hn = ld_nc_v4(hdr + nt * 32 + lane);
-    const bool ok = valid && pc < P && A != 0u;
-    bad += valid && pc >= P;
-    {  // branch-free: predicated shared reductions (E = A & P, so popc(A) - popc(E) = popc(A & ~E))
-      const unsigned a4 = s_base + 4u * (ok ? pc : 0u);
-      const unsigned pa = __popc(A), pe = __popc(E);
-      red_shared_add_if(ok, a4, pa);                         // sA[pc]
-      red_shared_add_if(ok, a4 + 4u * P, 1u);                // sW[pc]
-      red_shared_add_if(ok && pa != pe, a4 + 8u * P, pa - pe);   // sDT[pc]
-      red_shared_add_if(ok && E == 0u, a4 + 12u * P, 1u);    // sDW[pc]
-      if constexpr (PW) {
-        if (ok && warp < st.n_warps) {
-          atomicAdd(st.pw + warp, (unsigned long long)pe);
-          if (E) atomicAdd(st.pw + st.n_warps + warp, 1ull);
-        }
-      }
-    }
-    unsigned mm = __ballot_sync(FULL, ok && E != 0u && sK[ok ? pc : 0]);
-    const unsigned long long* tbase = addr + tile * 32 * 32 + lane;
-    while (mm) {
-      if constexpr (V == 0) {
-        int src[RP_BATCH];
-        unsigned long long a[RP_BATCH];
-#pragma unroll
-        for (int b = 0; b < RP_BATCH; ++b) {
-          src[b] = mm ? __ffs(mm) - 1 : -1;
-          if (mm) mm &= mm - 1;
-          if (src[b] >= 0) a[b] = ld_nc_u64(tbase + src[b] * 32);
-        }
-#pragma unroll
-        for (int b = 0; b < RP_BATCH; ++b) {
-          if (src[b] < 0) break;
-          process(a[b], src[b], E);
-        }
-      } else if constexpr (V == 1) {
-        unsigned long long a[RP_BATCH];
-        const unsigned batch = mm;
-        int nb = 0;
-#pragma unroll
-        for (int b = 0; b < RP_BATCH; ++b) {
-          if (mm) {
-            a[b] = ld_nc_u64(tbase + (__ffs(mm) - 1) * 32);
-            mm &= mm - 1;
-            ++nb;
-          }
-        }
-        unsigned rest = batch;
-#pragma unroll 1
-        for (int b = 0; b < nb; ++b) {
-          const int src = __ffs(rest) - 1;
-          rest &= rest - 1;
-          unsigned long long x = a[0];
-#pragma unroll
-          for (int k = 1; k < RP_BATCH; ++k) x = (b == k) ? a[k] : x;
-          process(x, src, E);
-        }
-      } else {
-        const unsigned batch = mm;
-        int nb = 0;
-#pragma unroll
-        for (int b = 0; b < RP_BATCH; ++b) {
-          if (mm) {
-            cp_async8(s_stage + 8u * 32u * b, tbase + (__ffs(mm) - 1) * 32);
-            mm &= mm - 1;
-            ++nb;
-          }
-        }
-        asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
-        __syncwarp();
-        unsigned rest = batch;
-#pragma unroll 1
-        for (int b = 0; b < nb; ++b) {
-          const int src = __ffs(rest) - 1;
-          rest &= rest - 1;
-          unsigned long long x;
-          asm volatile("ld.shared.u64 %0, [%1];" : "=l"(x) : "r"(s_stage + 8u * 32u * b) : "memory");
-          process(x, src, E);
-        }
-        __syncwarp();
-      }
-    }
-    h = hn;
-  }
-  if (hS) atomicAdd(&sH[1 + lane], hS);
-  if (hL) atomicAdd(&sH[34 + lane], hL);
-  bad = __reduce_add_sync(FULL, bad);
-  if (lane == 0 && bad) atomicAdd(err, (unsigned long long)bad);
-  __syncthreads();
-  for (unsigned pc = threadIdx.x; pc < P; pc += blockDim.x) {
-    const unsigned a = sA[pc], w = sW[pc];
-    if (w) {
-      unsigned long long* s = st.site + 4 * pc;
-      atomicAdd(s + 0, (unsigned long long)a);
-      atomicAdd(s + 1, (unsigned long long)(a - sDT[pc]));
-      atomicAdd(s + 2, (unsigned long long)w);
-      atomicAdd(s + 3, (unsigned long long)(w - sDW[pc]));
-      if (sK[pc] && w != sDW[pc]) {
-        unsigned long long* m = st.mem + 3 * pc;
-        atomicAdd(m + 0, (unsigned long long)(w - sDW[pc]));
-        atomicAdd(m + 1, (unsigned long long)sS[pc]);
-        atomicAdd(m + 2, (unsigned long long)sL[pc]);
-      }
-    }
-  }
-  for (unsigned i = threadIdx.x; i < 66; i += blockDim.x)
-    if (sH[i]) atomicAdd(st.hist + i, (unsigned long long)sH[i]);
-}
-
-// ---------------------------------------------------------------- replay, lane-per-event variant (V = 3)
-// Each warp takes 128 consecutive events per round (4 header tiles). Headers are counted as in the
-// other variants; the executed memory events of the round are compacted into a per-warp list, their
-// 256 B address slots gathered with coalesced 8 B/lane loads into a shared-memory stage (one 272 B row
-// per event), and then every LANE analyses one event on its own, reading its row with 16 B shared loads:
-// one pass over the 32 addresses counts sector/line boundaries (valid if the addresses are
-// non-decreasing) and sets bits in a per-lane 512-sector window bitmap (valid if they span < 16 KB);
-// events that are neither (wide random patterns) fall back to the warp-cooperative sectors_lines().
-// Per event this costs ~1/32 of the warp-cooperative instruction count for the common paths.
-constexpr int L3_NW = 10;                    // warps per CTA (1 CTA per SM)
-constexpr int L3_ROW = 68;                   // words per stage row (272 B: conflict-free 16 B lane reads)
-constexpr int L3_WARP_WORDS = 3 * 128 + 32 * L3_ROW + SCRATCH_WORDS;
-
+// shared-memory helpers (32-bit shared addresses)
 __device__ __forceinline__ void lds_v4(unsigned a, uint4& v) {
   asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a));
 }
@@ -308,188 +117,7 @@ __device__ __forceinline__ void sts_u64(unsigned a, unsigned long long v) {
   asm volatile("st.shared.u64 [%0], %1;" ::"r"(a), "l"(v) : "memory");
 }
 
-template <bool PW>
-__global__ void __launch_bounds__(32 * L3_NW, 1)
-k_replay_lane(const uint4* __restrict__ hdr, const unsigned long long* __restrict__ addr, unsigned long long n,
-              unsigned P, const uint8_t* __restrict__ kind, DevState st, unsigned long long* err) {
-  extern __shared__ __align__(16) unsigned sm[];
-  const unsigned P4 = (6 * P + 66 + 3) & ~3u;
-  unsigned* sH = sm + 6 * P;
-  unsigned* sWarp = sm + P4 + (threadIdx.x >> 5) * L3_WARP_WORDS;
-  uint8_t* sK = reinterpret_cast<uint8_t*>(sm + P4 + L3_NW * L3_WARP_WORDS);
-  for (unsigned i = threadIdx.x; i < P4; i += blockDim.x) sm[i] = 0;
-  for (unsigned i = threadIdx.x; i < L3_NW * L3_WARP_WORDS; i += blockDim.x) {
-    const unsigned o = i % L3_WARP_WORDS;
-    const unsigned s0 = 3 * 128 + 32 * L3_ROW;
-    sm[P4 + i] = o >= s0 ? scratch_init_word(o - s0) : 0u;
-  }
-  for (unsigned i = threadIdx.x; i < P; i += blockDim.x) sK[i] = is_mem_kind(kind[i]);
-  __syncthreads();
-
-  const unsigned lane = lane_id(), lmlt = lanemask_lt(), lanebit = 1u << lane;
-  const unsigned s_base = (unsigned)__cvta_generic_to_shared(sm);
-  const unsigned s_list = (unsigned)__cvta_generic_to_shared(sWarp);            // [128][3]: idx, E, pc
-  const unsigned s_stage = s_list + 4u * 3u * 128u;                              // [32][L3_ROW]
-  const unsigned s_scr = s_stage + 4u * 32u * L3_ROW;                            // hash scratch
-  const unsigned my_row = s_stage + 4u * L3_ROW * lane;
-  unsigned bad = 0;
-  const unsigned long long warps = (unsigned long long)gridDim.x * L3_NW;
-  unsigned long long round = (blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x) >> 5;
-  uint4 h[4];
-#pragma unroll
-  for (int t = 0; t < 4; ++t) {
-    const unsigned long long i = round * 128 + t * 32 + lane;
-    h[t] = i < n ? ld_nc_v4(hdr + i) : make_uint4(0, 0, 0, 0);
-  }
-  for (; round * 128 < n; round += warps) {
-    // ---- headers: counts (predicated shared reductions) and the compacted memory-event list
-    unsigned c = 0;
-#pragma unroll
-    for (int t = 0; t < 4; ++t) {
-      const unsigned long long i = round * 128 + t * 32 + lane;
-      const bool valid = i < n;
-      const unsigned pc = h[t].x, A = h[t].z, E = h[t].z & h[t].w;
-      const bool ok = valid && pc < P && A != 0u;
-      bad += valid && pc >= P;
-      const unsigned a4 = s_base + 4u * (ok ? pc : 0u);
-      const unsigned pa = __popc(A), pe = __popc(E);
-      red_shared_add_if(ok, a4, pa);
-      red_shared_add_if(ok, a4 + 4u * P, 1u);
-      red_shared_add_if(ok && pa != pe, a4 + 8u * P, pa - pe);
-      red_shared_add_if(ok && E == 0u, a4 + 12u * P, 1u);
-      if constexpr (PW) {
-        const unsigned warp = h[t].y;
-        if (ok && warp < st.n_warps) {
-          atomicAdd(st.pw + warp, (unsigned long long)pe);
-          if (E) atomicAdd(st.pw + st.n_warps + warp, 1ull);
-        }
-      }
-      const bool mem = ok && E != 0u && sK[ok ? pc : 0];
-      const unsigned m = __ballot_sync(FULL, mem);
-      if (mem) {
-        const unsigned e = s_list + 12u * (c + __popc(m & lmlt));
-        sts_u32(e, (unsigned)(i - round * 128));   // event offset within the round
-        sts_u32(e + 4, E);
-        sts_u32(e + 8, pc);
-      }
-      c += __popc(m);
-    }
-    // prefetch the next round's headers
-    const unsigned long long nr = round + warps;
-#pragma unroll
-    for (int t = 0; t < 4; ++t) {
-      const unsigned long long i = nr * 128 + t * 32 + lane;
-      h[t] = i < n ? ld_nc_v4(hdr + i) : make_uint4(0, 0, 0, 0);
-    }
-    __syncwarp();
-    const unsigned long long* rbase = addr + round * 128 * 32 + lane;
-    for (unsigned r0 = 0; r0 < c; r0 += 32) {
-      const unsigned nrows = min(32u, c - r0);
-      // ---- gather: row s <- slot of list[r0 + s], lane l loads address l (256 B coalesced per row)
-      for (unsigned s = 0; s < nrows; s += 8) {
-        unsigned long long v[8];
-#pragma unroll
-        for (int k = 0; k < 8; ++k) {
-          const unsigned row = min(s + k, nrows - 1);
-          const unsigned off = lds_u32(s_list + 12u * (r0 + row));
-          v[k] = ld_nc_u64(rbase + off * 32ull);
-        }
-#pragma unroll
-        for (int k = 0; k < 8; ++k)
-          if (s + k < nrows) sts_u64(s_stage + 4u * L3_ROW * (s + k) + 8u * lane, v[k]);
-      }
-      __syncwarp();
-      // ---- per-lane analysis of row `lane`
-      const bool have = lane < nrows;
-      const unsigned E = have ? lds_u32(s_list + 12u * (r0 + lane) + 4) : 0u;
-      const unsigned pc = have ? lds_u32(s_list + 12u * (r0 + lane) + 8) : 0u;
-      unsigned S = 0, L = 0;
-      bool hard = false;
-      if (have) {
-        const int f = __ffs(E) - 1;
-        const unsigned f_lo = lds_u32(my_row + 8u * f), f_hi = lds_u32(my_row + 8u * f + 4);
-        unsigned prev = f_lo, hb = 0, bs = 0, bl = 0;
-        bool viol = false;
-#pragma unroll
-        for (int q = 0; q < 16; ++q) {
-          uint4 v;
-          lds_v4(my_row + 16u * q, v);
-#pragma unroll
-          for (int u = 0; u < 2; ++u) {
-            const int l = 2 * q + u;
-            const bool act = (E >> l) & 1u;
-            const unsigned lo = act ? (u ? v.z : v.x) : prev;
-            const unsigned hi = act ? (u ? v.w : v.y) : f_hi;
-            hb |= hi ^ f_hi;
-            viol |= lo < prev;
-            const unsigned x = lo ^ prev;
-            bs += (x & ~31u) != 0u;
-            bl += (x & ~127u) != 0u;
-            prev = lo;
-          }
-        }
-        if (hb == 0u && !viol) {
-          S = bs + 1u;
-          L = bl + 1u;
-        } else {
-          hard = true;
-        }
-      }
-      // ---- hard rows: warp-cooperative exact path
-      unsigned hm = __ballot_sync(FULL, hard);
-      while (hm) {
-        const int src = __ffs(hm) - 1;
-        hm &= hm - 1;
-        const unsigned es = __shfl_sync(FULL, E, src);
-        unsigned long long a;
-        asm volatile("ld.shared.u64 %0, [%1];" : "=l"(a) : "r"(s_stage + 4u * L3_ROW * src + 8u * lane));
-        unsigned s2, l2;
-        sectors_lines<true, false>(a, es, lane, lanebit, lmlt, s_scr, s2, l2);
-        if (lane == (unsigned)src) { S = s2; L = l2; }
-      }
-      if (have) {
-        red_shared_add(s_base + 4u * (4 * P + pc), S);
-        red_shared_add(s_base + 4u * (5 * P + pc), L);
-        red_shared_add(s_base + 4u * (6 * P + S), 1u);        // hS[S]
-        red_shared_add(s_base + 4u * (6 * P + 33 + L), 1u);   // hL[L]
-      }
-      __syncwarp();
-    }
-  }
-  bad = __reduce_add_sync(FULL, bad);
-  if (lane == 0 && bad) atomicAdd(err, (unsigned long long)bad);
-  __syncthreads();
-  const unsigned* sA = sm;
-  const unsigned* sW = sm + P;
-  const unsigned* sDT = sm + 2 * P;
-  const unsigned* sDW = sm + 3 * P;
-  const unsigned* sS = sm + 4 * P;
-  const unsigned* sL = sm + 5 * P;
-  for (unsigned pc = threadIdx.x; pc < P; pc += blockDim.x) {
-    const unsigned a = sA[pc], w = sW[pc];
-    if (w) {
-      unsigned long long* s = st.site + 4 * pc;
-      atomicAdd(s + 0, (unsigned long long)a);
-      atomicAdd(s + 1, (unsigned long long)(a - sDT[pc]));
-      atomicAdd(s + 2, (unsigned long long)w);
-      atomicAdd(s + 3, (unsigned long long)(w - sDW[pc]));
-      if (sK[pc] && w != sDW[pc]) {
-        unsigned long long* m = st.mem + 3 * pc;
-        atomicAdd(m + 0, (unsigned long long)(w - sDW[pc]));
-        atomicAdd(m + 1, (unsigned long long)sS[pc]);
-        atomicAdd(m + 2, (unsigned long long)sL[pc]);
-      }
-    }
-  }
-  for (unsigned i = threadIdx.x; i < 66; i += blockDim.x)
-    if (sH[i]) atomicAdd(st.hist + i, (unsigned long long)sH[i]);
-}
-
-static size_t replay_lane_smem(unsigned P) {
-  return (((6ull * P + 66 + 3) & ~3ull) + (size_t)L3_NW * L3_WARP_WORDS) * 4 + P + 16;
-}
-
-// ---------------------------------------------------------------- replay, lean warp-cooperative variant (V = 4)
+// ---------------------------------------------------------------- single-pass replay (nvbt_replay)
 // One CTA of 32 warps per SM. Per 32-event tile: predicated shared reductions for the counts (no
 // branches), then the tile's executed memory events in batches of 8: cp.async (8 B per lane) stages the
 // 8 address slots into the warp's shared rows, and a rolled loop runs sectors_lines() per event with
@@ -949,12 +577,6 @@ static int sm_count(int dev) {
   return g_sms > 0 ? g_sms : 148;
 }
 
-template <int V>
-static size_t replay_smem(unsigned P) {
-  constexpr int NW = ReplayCfg<V>::THREADS / 32;
-  return (((6ull * P + 66 + 3) & ~3ull) + SCRATCH_WORDS * NW + (V == 2 ? 2ull * NW * RP_BATCH * 32 : 0)) * 4 + P + 16;
-}
-static int g_replay_variant = -1;
 
 }  // namespace nvbt
 
@@ -1036,57 +658,6 @@ int nvbt_gen_events(nvbt_ctx c, uint64_t seed, uint64_t first, uint64_t n, void*
 }
 
 }  // extern "C"
-
-template <int V>
-static int launch_replay(nvbt_ctx c, const void* d_hdr, const void* d_addr, uint64_t n, const DevState& st) {
-  const size_t smem = replay_smem<V>(c->n_pcs);
-  static bool attr_set = false;
-  if (!attr_set) {
-    NVBT_CUDA(cudaFuncSetAttribute(k_replay<V, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)replay_smem<V>(4096)));
-    NVBT_CUDA(cudaFuncSetAttribute(k_replay<V, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)replay_smem<V>(4096)));
-    attr_set = true;
-  }
-  const unsigned long long kMaxPerLaunch = 1ull << 30;  // keeps every CTA's u32 bins far from overflow
-  const int sms = sm_count(c->device);
-  const int per_sm = ReplayCfg<V>::MINB;
-  for (uint64_t off = 0; off < n; off += kMaxPerLaunch) {
-    const uint64_t m = std::min<uint64_t>(kMaxPerLaunch, n - off);
-    const unsigned long long tiles = (m + 31) / 32;
-    const int wpc = ReplayCfg<V>::THREADS / 32;
-    const int blocks = (int)std::min<unsigned long long>((tiles + 2 * wpc - 1) / (2 * wpc), (unsigned long long)sms * per_sm);
-    auto kern = st.pw != nullptr ? k_replay<V, true> : k_replay<V, false>;
-    kern<<<blocks, ReplayCfg<V>::THREADS, smem, c->stream>>>(
-        static_cast<const uint4*>(d_hdr) + off, static_cast<const unsigned long long*>(d_addr) + off * 32, m,
-        c->n_pcs, c->d_kind, st, c->ctl + CTL_REPLAY_ERR);
-    NVBT_CUDA(cudaGetLastError());
-    c->launches++;
-  }
-  return NVBT_OK;
-}
-
-static int launch_replay_lane(nvbt_ctx c, const void* d_hdr, const void* d_addr, uint64_t n, const DevState& st) {
-  const size_t smem = replay_lane_smem(c->n_pcs);
-  static bool attr_set = false;
-  if (!attr_set) {
-    NVBT_CUDA(cudaFuncSetAttribute(k_replay_lane<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)replay_lane_smem(4096)));
-    NVBT_CUDA(cudaFuncSetAttribute(k_replay_lane<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)replay_lane_smem(4096)));
-    attr_set = true;
-  }
-  const unsigned long long kMaxPerLaunch = 1ull << 30;
-  const int sms = sm_count(c->device);
-  for (uint64_t off = 0; off < n; off += kMaxPerLaunch) {
-    const uint64_t m = std::min<uint64_t>(kMaxPerLaunch, n - off);
-    const unsigned long long rounds = (m + 127) / 128;
-    const int blocks = (int)std::min<unsigned long long>((rounds + L3_NW - 1) / L3_NW, (unsigned long long)sms);
-    auto kern = st.pw != nullptr ? k_replay_lane<true> : k_replay_lane<false>;
-    kern<<<blocks, 32 * L3_NW, smem, c->stream>>>(static_cast<const uint4*>(d_hdr) + off,
-                                                  static_cast<const unsigned long long*>(d_addr) + off * 32, m,
-                                                  c->n_pcs, c->d_kind, st, c->ctl + CTL_REPLAY_ERR);
-    NVBT_CUDA(cudaGetLastError());
-    c->launches++;
-  }
-  return NVBT_OK;
-}
 
 static int launch_replay4(nvbt_ctx c, const void* d_hdr, const void* d_addr, uint64_t n, const DevState& st) {
   const size_t smem = replay4_smem(c->n_pcs);
@@ -1203,17 +774,7 @@ int nvbt_replay(nvbt_ctx c, const void* d_hdr, const void* d_addr, uint64_t n) {
   if (rc) return rc;
   if (n == 0) return NVBT_OK;
   NVBT_CUDA(cudaSetDevice(c->device));
-  {  // read per call so tests can compare variants in one process
-    const char* e = getenv("NVBT_REPLAY_VARIANT");
-    g_replay_variant = e && *e ? atoi(e) : 4;
-  }
-  switch (g_replay_variant) {
-    case 0: return launch_replay<0>(c, d_hdr, d_addr, n, st);
-    case 2: return launch_replay<2>(c, d_hdr, d_addr, n, st);
-    case 3: return launch_replay_lane(c, d_hdr, d_addr, n, st);
-    case 4: return launch_replay4(c, d_hdr, d_addr, n, st);
-    default: return launch_replay<1>(c, d_hdr, d_addr, n, st);
-  }
+  return launch_replay4(c, d_hdr, d_addr, n, st);
 }
 
 }  // extern "C"

@@ -316,17 +316,15 @@ def test_generator_bytes_match_oracle(nvbt):
         assert (ga == oaddr).all()   # non-memory slots are not written by either side (zeros here)
 
 
-# "staged" = nvbt_replay_staged (two passes, scratch list); digits = single-pass nvbt_replay kernel
-# variants selected through NVBT_REPLAY_VARIANT (read per call; 4 = default)
-REPLAY_VARIANTS = ["staged", "staged-small", "4"]
+# "staged" = nvbt_replay_staged (two passes, scratch list; "staged-small": a few thousand events per
+# block, so one call runs several pass pairs); "single" = the single-pass nvbt_replay
+REPLAY_VARIANTS = ["staged", "staged-small", "single"]
 
 
 def _replay_scratch(nb, ctx, variant, monkeypatch):
-    """Scratch tensor for the staged variants (small: a few thousand events per block, so one call runs
-    several A/B pass pairs), else select the single-pass kernel variant."""
+    """Scratch tensor for the staged variants, None for the single pass."""
     import torch
     if not variant.startswith("staged"):
-        monkeypatch.setenv("NVBT_REPLAY_VARIANT", variant)
         return None
     per = 5000 if variant == "staged-small" else 1 << 20
     return torch.empty(nb.nvbt_replay_scratch_size(ctx, per), dtype=torch.uint8, device="cuda")
