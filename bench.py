@@ -469,7 +469,7 @@ def run_c1(args, torch, nb, dr, local):
     from synth import uniform_f32
     N = 65536
     s = torch.cuda.Stream()
-    ctx = nb.nvbt_init(nb.W_VECTORADD, nb.COUNT | nb.OPHIST, stream=s)
+    ctx = nb.nvbt_init(nb.W_VECTORADD, nb.COUNT | nb.OPHIST | nb.BB, stream=s)
     a = torch.from_numpy(uniform_f32(N, 1)).cuda()
     b = torch.from_numpy(uniform_f32(N, 2)).cuda()
     c = torch.empty_like(a)
@@ -483,7 +483,9 @@ def run_c1(args, torch, nb, dr, local):
                 nb.nvbt_vectoradd(ctx, tools, a, b, c, N)
         return g
 
-    g_plain, g_instr = graph_of(nb.TOOL_NONE), graph_of(nb.TOOL_COUNT)
+    # per-pc counts two ways, identical results (I-5): a hook at every instruction (COUNT) or at block
+    # leaders and guarded pcs only (BBCOUNT, the paper's basic-block instrumentation)
+    g_plain, g_cnt, g_bb = graph_of(nb.TOOL_NONE), graph_of(nb.TOOL_COUNT), graph_of(nb.TOOL_BBCOUNT)
     nb.nvbt_reset(ctx)
 
     def timed(g, n):
@@ -498,22 +500,34 @@ def run_c1(args, torch, nb, dr, local):
             ts.append(e0.elapsed_time(e1) / 1e3)
         return ts
 
-    timed(g_instr, args.warmup)
-    timed(g_plain, args.warmup)
+    for g in (g_cnt, g_bb, g_plain):
+        timed(g, args.warmup)
     tp = timed(g_plain, args.steps)
-    nb.nvbt_reset(ctx)
-    with ClockSampler(local) as clk:
-        ti = timed(g_instr, args.steps)
-    cnt = nb.nvbt_count(ctx)
+    res = {}
+    for name, g in (("COUNT", g_cnt), ("BBCOUNT", g_bb)):
+        nb.nvbt_reset(ctx)
+        with ClockSampler(local) as clk:
+            ti = timed(g, args.steps)
+        cnt = nb.nvbt_count(ctx)
+        ht, hw = nb.nvbt_opcode_hist(ctx)
+        res[name] = (ti, cnt, ht, hw, clk.summary())
+    ok = all((res["COUNT"][1] == res["BBCOUNT"][1]).all() and (res["COUNT"][k] == res["BBCOUNT"][k]).all()
+             for k in (2, 3))
+    ti, cnt, _, _, clocks = res["BBCOUNT"]
     ev = int(cnt[2]) // (args.steps * reps)
     t_i, t_p = sum(ti) / (args.steps * reps), sum(tp) / (args.steps * reps)
+    t_c = sum(res["COUNT"][0]) / (args.steps * reps)
     return {"metric": METRIC, "value": ev / t_i, "unit": "events/s", "n_gpus": 1, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": 1e3 * t_i, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-            "config": {"workload": "C1 vectorAdd N=65536, tools COUNT", "launches_per_graph": reps,
-                       "warp_events_per_launch": ev, "counts_check": "ok" if ev == 26624 else f"{ev} != 26624"},
+            "config": {"workload": "C1 vectorAdd N=65536, instruction counts + opcode histogram (tools BBCOUNT)",
+                       "launches_per_graph": reps, "warp_events_per_launch": ev,
+                       "counts_check": ("ok" if ev == 26624 else f"{ev} != 26624") +
+                                       ("; COUNT == BBCOUNT counts and opcode histograms" if ok else "; COUNT != BBCOUNT")},
             "slowdown": t_i / t_p, "plain_us_per_launch": 1e6 * t_p, "instr_us_per_launch": 1e6 * t_i,
-            "bound": "launch latency (26,624 warp events per launch; CUDA-graph replays)", "clocks": clk.summary()}
+            "per_instruction_hooks": {"tools": "COUNT", "instr_us_per_launch": 1e6 * t_c, "slowdown": t_c / t_p,
+                                      "value": ev / t_c},
+            "bound": "launch latency (26,624 warp events per launch; CUDA-graph replays)", "clocks": clocks}
 
 
 def run_c3(args, torch, nb, dr, local):

@@ -353,6 +353,7 @@ struct Hooks {
   static constexpr bool kOn = T != 0;
   static constexpr bool kCount = (T & (TOOL_COUNT | TOOL_BB)) != 0;
   static constexpr bool kBB = (T & TOOL_BB) != 0;
+  static constexpr bool kLoopFree = Prog::REG_LO > Prog::REG_HI;   // no register-mode (loop) sites
   static constexpr int kMaxWarps = 8;  // workload CTAs have 256 threads
   static constexpr int kThreads = 32 * kMaxWarps;
   static constexpr int kScratchWord0 = (NPC * SITE_WORDS + 66 + 3) & ~3;  // 16-byte aligned
@@ -430,12 +431,27 @@ struct Hooks {
             dW[PC] += wa - we;
           }
         } else {
+          // one lane adds the hook's bins. Loop-free programs group the reductions under one branch
+          // (ptxas does not predicate shared atomics: each separately predicated one costs its own
+          // branch); programs with register-mode loops keep them separate (grouping raises the register
+          // pressure of their loop bodies)
           const unsigned b = sbase + 4u * (PC * SITE_WORDS);
-          red_if(lane == 0u, b, pa);
-          red_if(lane == 0u, b + 8u, wa);
-          if constexpr (d.guarded) {
-            red_if(lane == 0u, b + 4u, pa - pe);
-            red_if(lane == 0u, b + 12u, wa - we);
+          if constexpr (kLoopFree) {
+            if (lane == 0u) {
+              red(b, pa);
+              red(b + 8u, wa);
+              if constexpr (d.guarded) {
+                red(b + 4u, pa - pe);
+                red(b + 12u, wa - we);
+              }
+            }
+          } else {
+            red_if(lane == 0u, b, pa);
+            red_if(lane == 0u, b + 8u, wa);
+            if constexpr (d.guarded) {
+              red_if(lane == 0u, b + 4u, pa - pe);
+              red_if(lane == 0u, b + 12u, wa - we);
+            }
           }
           // this warp's executed totals (PER_WARP); register sites add theirs at retire()
           if constexpr ((T & TOOL_COUNT) != 0) {
@@ -463,9 +479,17 @@ struct Hooks {
               mN[PC] += 1u; mS[PC] += S; mL[PC] += L;
             } else {
               const unsigned b = sbase + 4u * (PC * SITE_WORDS);
-              red_if(lane == 0u, b + 16u, 1u);
-              red_if(lane == 0u, b + 20u, S);
-              red_if(lane == 0u, b + 24u, L);
+              if constexpr (kLoopFree) {
+                if (lane == 0u) {
+                  red(b + 16u, 1u);
+                  red(b + 20u, S);
+                  red(b + 24u, L);
+                }
+              } else {
+                red_if(lane == 0u, b + 16u, 1u);
+                red_if(lane == 0u, b + 20u, S);
+                red_if(lane == 0u, b + 24u, L);
+              }
             }
             inc_if_eq(hS, S, lane1);
             inc_if_eq(hL, L, lane1);
@@ -476,6 +500,9 @@ struct Hooks {
     }
   }
 
+  __device__ __forceinline__ static void red(unsigned saddr, unsigned v) {
+    asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(saddr), "r"(v) : "memory");
+  }
   __device__ __forceinline__ static void red_if(bool p, unsigned saddr, unsigned v) {
     asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q red.shared.add.u32 [%0], %1;\n\t}"
                  ::"r"(saddr), "r"(v), "r"((unsigned)p) : "memory");

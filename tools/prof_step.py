@@ -22,6 +22,16 @@ if which in ("all", "c2"):
     nb.nvbt_sgemm(ctx, nb.TOOL_COUNT | nb.TOOL_MEMDIV, A, B, C, M, N, K)
     nb.nvbt_sgemm(ctx, nb.TOOL_BBCOUNT | nb.TOOL_MEMDIV, A, B, C, M, N, K)
     nb.nvbt_count(ctx)
+if which in ("all", "c1"):
+    from synth import uniform_f32 as _u
+    N = 65536
+    c1 = nb.nvbt_init(nb.W_VECTORADD, nb.COUNT | nb.OPHIST)
+    a, b = torch.from_numpy(_u(N, 1)).cuda(), torch.from_numpy(_u(N, 2)).cuda()
+    c = torch.empty_like(a)
+    for _ in range(3):
+        nb.nvbt_vectoradd(c1, nb.TOOL_NONE, a, b, c, N)
+        nb.nvbt_vectoradd(c1, nb.TOOL_COUNT, a, b, c, N)
+    nb.nvbt_count(c1)
 if which in ("all", "c5"):
     n = 1 << 26
     rctx = nb.nvbt_init(nb.W_REPLAY, nb.COUNT | nb.MEMDIV)
