@@ -401,7 +401,15 @@ struct Hooks {
   // every pc of a basic block ("each thread will execute without change in control flow", P:L116 (§4)),
   // so kernels take one ballot per block instance and hand it to that block's hooks.
   struct Act { unsigned A; };
+  // Debug builds (libnvbt_debug.so, -DNVBT_CHECK_CONVERGED) check the converged-hook discipline at every
+  // hook: all 32 lanes of the warp must arrive together (R-15); a violation traps the kernel.
+  __device__ __forceinline__ static void check_converged() {
+#ifdef NVBT_CHECK_CONVERGED
+    if (__activemask() != FULL) __trap();
+#endif
+  }
   __device__ __forceinline__ Act active(bool in_flow) const {
+    check_converged();
     if constexpr (kOn) return Act{__ballot_sync(FULL, in_flow)};
     else return Act{0u};
   }
@@ -416,6 +424,7 @@ struct Hooks {
     constexpr bool div = mem && (T & TOOL_MEM);
     constexpr bool trc = mem && (T & TOOL_TRACE);
     constexpr bool reg = PC >= Prog::REG_LO && PC <= Prog::REG_HI;   // loop site: register counters
+    check_converged();
     if constexpr (cnt || div || trc) {
       const unsigned A = m.A;
       const unsigned P = d.guarded ? (__ballot_sync(FULL, pred) & A) : A;

@@ -13,7 +13,8 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libnvbt.so")
+# NVBT_LIB selects another build of the library (tests load libnvbt_debug.so, the converged-hook check)
+LIB_PATH = os.environ.get("NVBT_LIB") or os.path.join(_HERE, "libnvbt.so")
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"libnvbt.so not built at {LIB_PATH}; run __graft_entry__.build()")
