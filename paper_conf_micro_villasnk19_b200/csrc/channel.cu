@@ -472,7 +472,7 @@ __global__ void __launch_bounds__(256) k_fp_count(const unsigned long long* __re
 // written (the unused tail of each SM's last chunk, slots a warp reserved but did not use) have tag 0 and
 // are skipped. Each warp takes a contiguous range of slots, 32 at a time: lane i reads record i's
 // header, then the warp walks the 32 records 8 at a time, 4 lanes per record (quad pass).
-__global__ void __launch_bounds__(256) k_footprint(const unsigned char* __restrict__ ring,
+__global__ void __launch_bounds__(256, 4) k_footprint(const unsigned char* __restrict__ ring,
                                                     const unsigned long long* __restrict__ chunks,
                                                     unsigned long long cap,
                                                     unsigned long long* __restrict__ keys, unsigned* __restrict__ pool,
@@ -540,9 +540,10 @@ __global__ void __launch_bounds__(256) k_footprint(const unsigned char* __restri
       const bool qlive = (live >> jj) & 1u;
       const unsigned qE = __shfl_sync(0xffffffffu, E, jj) >> (8u * qq);
       const unsigned ql = __shfl_sync(0xffffffffu, lid, jj);
-      unsigned long long key = 0;
-      unsigned wd = 0, bits = 0;
-      bool have = false, same = true;
+      // per lane: the first active address is the reference; every active address must lie in the
+      // reference's 1 KB word (same a >> 10); sector bit = (a >> 5) & 31 within that word
+      unsigned ref_lo = 0, ref_hi = 0, nd = 0, bits = 0;
+      bool have = false;
       if (qlive) {
         const uint4* src = reinterpret_cast<const uint4*>(ring + 64 + (base + jj) * RECORD_BYTES + 32 + 64 * qq);
         uint4 va[4];
@@ -550,36 +551,36 @@ __global__ void __launch_bounds__(256) k_footprint(const unsigned char* __restri
         for (int k = 0; k < 4; ++k) va[k] = __ldcs(src + k);
 #pragma unroll
         for (int k = 0; k < 4; ++k) {
-          const uint4 v = va[k];
-          const unsigned long long a2[2] = {(unsigned long long)v.y << 32 | v.x, (unsigned long long)v.w << 32 | v.z};
 #pragma unroll
           for (int t = 0; t < 2; ++t) {
-            if ((qE >> (2 * k + t)) & 1u) {
-              const unsigned long long a = a2[t];
-              const unsigned long long kk = ((unsigned long long)ql << (48 - kFpRegionShift)) | (a >> kFpRegionShift);
-              const unsigned line = (unsigned)(a >> 7) & (8 * kFpWords - 1);
-              same = same && (a >> 48) == 0ull && (!have || (kk == key && (line >> 3) == wd));
-              key = kk;
-              wd = line >> 3;
-              bits |= 1u << ((line & 7) * 4 + ((unsigned)(a >> 5) & 3));
-              have = true;
-            }
+            const bool act = (qE >> (2 * k + t)) & 1u;
+            const unsigned lo = t ? va[k].z : va[k].x, hi = t ? va[k].w : va[k].y;
+            const bool first = act && !have;
+            ref_lo = first ? lo : ref_lo;
+            ref_hi = first ? hi : ref_hi;
+            have = have || act;
+            nd |= act ? (((lo ^ ref_lo) >> 10) | (hi ^ ref_hi)) : 0u;
+            bits |= act ? 1u << ((lo >> 5) & 31u) : 0u;
           }
         }
       }
-      // quad reduction: one (region, word) for the whole record?
+      // quad reduction: one 1 KB word (below 2^48) for the whole record?
+      bool same = nd == 0u && (ref_hi >> 16) == 0u;
 #pragma unroll
       for (unsigned d = 1; d <= 2; d <<= 1) {
         const unsigned oh = __shfl_xor_sync(0xffffffffu, (unsigned)have, d);
-        const unsigned long long ok2 = __shfl_xor_sync(0xffffffffu, key, d);
-        const unsigned ow = __shfl_xor_sync(0xffffffffu, wd, d);
+        const unsigned olo = __shfl_xor_sync(0xffffffffu, ref_lo, d);
+        const unsigned ohi = __shfl_xor_sync(0xffffffffu, ref_hi, d);
         const unsigned ob = __shfl_xor_sync(0xffffffffu, bits, d);
         const unsigned os = __shfl_xor_sync(0xffffffffu, (unsigned)same, d);
-        same = same && os != 0u && (!have || !oh || (ok2 == key && ow == wd));
-        if (!have && oh) { key = ok2; wd = ow; }
+        same = same && os != 0u && (!have || !oh || (((olo ^ ref_lo) >> 10) | (ohi ^ ref_hi)) == 0u);
+        if (!have && oh) { ref_lo = olo; ref_hi = ohi; }
         have = have || oh != 0u;
         bits |= ob;
       }
+      const unsigned long long key =
+          ((unsigned long long)ql << (48 - kFpRegionShift)) | ((((unsigned long long)ref_hi << 32) | ref_lo) >> kFpRegionShift);
+      const unsigned wd = (ref_lo >> 10) & (kFpWords - 1u);
       if (qlive && same && qq == 0) {
         unsigned long long slot;
         if (fp_slot_lane(key, keys, mask, ck, cs, slot)) atomicOr(pool + slot * kFpWords + wd, bits);
