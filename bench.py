@@ -251,6 +251,19 @@ class ReplayBench:
         self.events = self.n
         self.kernels_per_step = -(-self.n // chunk)
 
+    def oracle_sample(self, budget_s):
+        """The oracle (generator + per-event definitions) on a bounded sample of the same event stream:
+        consecutive 2^16-event chunks from the rank's first event until the budget is spent."""
+        from oracle import events as ev, gen, programs
+        acc = ev.Accumulator(programs.replay())
+        t0 = time.perf_counter()
+        done = 0
+        while time.perf_counter() - t0 < budget_s:
+            gen.replay(acc, self.lo + done, 1 << 16)
+            done += 1 << 16
+        dt = time.perf_counter() - t0
+        return done / dt, f"{done} generated events from event {self.lo} (oracle replay incl. generation, 1 core)"
+
     def replay(self, m):
         if self.scratch is None:
             self.nb.nvbt_replay(self.ctx, self.hdr, self.addr, m)
@@ -444,6 +457,9 @@ def run_replay(args, torch, nb, dr, rank, world, local, peaks, peaks_src):
         "gpu_launches": int(launches), "clocks": clk.summary(),
         "check": {"W_issued": int(cnt[2]), "expected": args.steps * n_all},
     }
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        rate, sample = wl.oracle_sample(min(args.cpu_budget, 10.0))
+        line["cpu_baseline"] = {"value": rate, "unit": "events/s", "cores": 1, "kind": "oracle", "sample": sample}
     if rank == 0:
         print(json.dumps(line), flush=True)
 
