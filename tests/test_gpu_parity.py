@@ -581,3 +581,41 @@ def test_kernel_sampling_error_on_data_dependent_kernels(nvbt):
     exact, est = nb.nvbt_count(full).astype(np.int64), nb.nvbt_count(samp).astype(np.int64)
     assert est[2] != exact[2]                               # sampling is not exact here
     assert exact[2] > 0 and abs(est[2] - exact[2]) / exact[2] < 10.0
+
+
+def test_replay_full_size_c5(nvbt):
+    """C5 at BASELINE.json's full size in the bench's launch configuration (10^10 generated events in
+    2^27-event chunks, staged replay with a 2^27-event scratch): W_issued = 10^10 and the I-2 invariants;
+    the single-pass kernel over the same 10^10 events gives identical bins (two independent divergence
+    implementations agreeing at full size); and three 2^16-event windows (start, middle, end of the
+    stream) through the same launch configuration equal the oracle element by element."""
+    import torch
+    nb, dr = nvbt.nvbt, nvbt.drivers
+    n, chunk = 10**10, 1 << 27
+    flags = nb.COUNT | nb.OPHIST | nb.BB | nb.MEMDIV
+    hdr = torch.empty(chunk * 16, dtype=torch.uint8, device="cuda")
+    addr = torch.empty(chunk * 256, dtype=torch.uint8, device="cuda")
+    staged = nb.nvbt_init(nb.W_REPLAY, flags)
+    single = nb.nvbt_init(nb.W_REPLAY, flags)
+    scratch = torch.empty(nb.nvbt_replay_scratch_size(staged, chunk), dtype=torch.uint8, device="cuda")
+    done = 0
+    while done < n:
+        m = min(chunk, n - done)
+        nb.nvbt_gen_events(staged, gen.SEED, done, m, hdr, addr)
+        nb.nvbt_replay_staged(staged, hdr, addr, m, scratch)
+        nb.nvbt_replay(single, hdr, addr, m)
+        done += m
+    g = read_all(nb, staged)
+    assert int(g["counts"][2]) == n
+    gpu_invariants(g)
+    assert_same(g, read_all(nb, single), what="staged vs single-pass replay, 10^10 events")
+    assert nb.nvbt_replay_errors(staged) == 0 and nb.nvbt_replay_errors(single) == 0
+    for first in (0, n // 2 - 12345, n - (1 << 16)):
+        ctx = nb.nvbt_init(nb.W_REPLAY, flags)
+        nb.nvbt_gen_events(ctx, gen.SEED, first, 1 << 16, hdr, addr)
+        nb.nvbt_replay_staged(ctx, hdr, addr, 1 << 16, scratch)
+        acc = ev.Accumulator(programs.replay())
+        gen.replay(acc, first, 1 << 16)
+        assert_same(read_all(nb, ctx), acc.result(), COUNT_KEYS + MEM_KEYS, f"window at {first}")
+    del hdr, addr, scratch
+    torch.cuda.empty_cache()
