@@ -619,3 +619,35 @@ def test_replay_full_size_c5(nvbt):
         assert_same(read_all(nb, ctx), acc.result(), COUNT_KEYS + MEM_KEYS, f"window at {first}")
     del hdr, addr, scratch
     torch.cuda.empty_cache()
+
+
+def test_bfs_full_size_c3(nvbt):
+    """C3 at BASELINE.json's full size (R-MAT scale 20, edge factor 16, the bench's graph): BFS distances
+    equal scipy's unweighted shortest paths, the BB-entry run and the per-instruction run give identical
+    per-pc counts (I-5 at full size), the I-2 invariants hold, and every kernel-1 launch is entered by
+    every warp (Ent_w of the first block = levels x warps)."""
+    import torch
+    from scipy.sparse import csr_matrix
+    from scipy.sparse.csgraph import shortest_path
+    nb, dr = nvbt.nvbt, nvbt.drivers
+    rowptr, col = rmat_csr(20, 16, seed=3)
+    n = len(rowptr) - 1
+    src = bfs_source(rowptr)
+    nw = nb.nvbt_workload_warps(nb.W_BFS, n)
+    rp, cl = cuda(rowptr), cuda(col)
+    res = {}
+    for name, tools in (("bb", nb.TOOL_BBCOUNT), ("count", nb.TOOL_COUNT | nb.TOOL_MEMDIV)):
+        ctx = nb.nvbt_init(nb.W_BFS, nb.COUNT | nb.BB | nb.MEMDIV)
+        bufs = dr.bfs_buffers(n, "cuda")
+        cost, levels = dr.run_bfs(ctx, tools, rp, cl, src, bufs)
+        res[name] = (read_all(nb, ctx), cost.cpu().numpy(), levels)
+    g_bb, cost, levels = res["bb"]
+    g_ct = res["count"][0]
+    assert res["count"][2] == levels and (res["count"][1] == cost).all()
+    A = csr_matrix((np.ones(len(col), dtype=np.int8), col, rowptr), shape=(n, n))
+    d = shortest_path(A, unweighted=True, indices=src)
+    exp = np.where(np.isinf(d), -1, d).astype(np.int64)
+    assert (cost.astype(np.int64) == exp).all()
+    assert_same(g_bb, g_ct, COUNT_KEYS, "BFS scale 20: BBCOUNT vs COUNT")
+    gpu_invariants(g_ct)
+    assert int(g_bb["Ent_w"][0]) == levels * nw
