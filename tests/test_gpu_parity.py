@@ -651,3 +651,39 @@ def test_bfs_full_size_c3(nvbt):
     assert_same(g_bb, g_ct, COUNT_KEYS, "BFS scale 20: BBCOUNT vs COUNT")
     gpu_invariants(g_ct)
     assert int(g_bb["Ent_w"][0]) == levels * nw
+
+
+def test_stencil_trace_full_size_c4(nvbt):
+    """C4 at BASELINE.json's full size (8192^2 stencil, 100 iterations, every global LD/ST traced through
+    the pinned-host channel and drained with the digest callback, the bench's configuration): the number
+    of records equals the closed form iters x (2 n^2/32 + 4 (n-2) n/32), none dropped, W_issued of the
+    traced memory pcs equals the record count plus the predicated-off events (COUNT tool alongside), and
+    the traced run computes exactly the uninstrumented run's grid."""
+    import torch
+    nb, dr = nvbt.nvbt, nvbt.drivers
+    n, iters = 8192, 100
+    ctx = nb.nvbt_init(nb.W_STENCIL, nb.COUNT | nb.TRACE)
+    x0 = cuda(uniform_f32((n, n), 4))
+    a0, a1 = x0.clone(), torch.empty_like(x0)
+    dr.run_stencil(ctx, nb.TOOL_NONE, a0, a1, n, iters)
+    plain = (a0 if iters % 2 == 0 else a1).clone()
+    nb.nvbt_reset(ctx)
+    ring = torch.empty(64 + 288 * (1 << 22), dtype=torch.uint8, pin_memory=True)
+    ch = nb.nvbt_channel_open(ctx, ring)
+    b0, b1 = x0.clone(), torch.empty_like(x0)
+    dr.run_stencil(ctx, nb.TOOL_TRACE | nb.TOOL_COUNT, b0, b1, n, iters)
+    d = nb.nvbt_channel_drain_digest(ch, timeout_us=600_000_000)
+    torch.cuda.synchronize()
+    expect = iters * (2 * (n * n // 32) + 4 * (n - 2) * (n // 32))
+    assert d.n_rec == expect and nb.nvbt_channel_dropped(ch) == 0
+    assert torch.equal(b0 if iters % 2 == 0 else b1, plain)
+    g = read_all(nb, ctx)
+    gpu_invariants(g)
+    # every executed warp-level event of a memory pc is one record (EM §5): the warp-executed histogram
+    # over the memory opcodes (used by no other pc) counts the records
+    prog = programs.stencil()
+    mem_ops = np.unique(prog["opcode"][programs.is_mem(prog)])
+    other_ops = np.unique(prog["opcode"][~programs.is_mem(prog)])
+    assert len(np.intersect1d(mem_ops, other_ops)) == 0
+    assert int(g["H_w"][mem_ops].sum()) == expect
+    del ring
