@@ -28,6 +28,9 @@ constexpr unsigned FULL = 0xffffffffu;
 constexpr uint32_t TOOL_COUNT = NVBT_TOOL_COUNT, TOOL_BB = NVBT_TOOL_BBCOUNT, TOOL_MEM = NVBT_TOOL_MEMDIV,
                    TOOL_TRACE = NVBT_TOOL_TRACE;
 constexpr int RECORD_BYTES = 288;
+// internal tool bit (not in the ABI): TRACE into a device-memory ring (F2), chosen at launch time when the
+// context's channel lives in HBM, so the producer's path is selected at compile time
+constexpr uint32_t TOOL_TRACE_DEV = 1u << 8;
 constexpr int SITE_WORDS = 7;  // per-pc shared bins: tA, dT, wI, dW, mN, mS, mL
 
 // POD handed by value to every instrumented kernel (kernel parameter space).
@@ -330,21 +333,19 @@ __device__ __forceinline__ void inc_if_eq(unsigned& h, unsigned v, unsigned ref)
 }
 
 // Ring backpressure: ticket t may be written once t < tail + cap. has_room() is the
-// cheap check against the device-side cache of the host's consumer index; wait_room() spins on the host
-// index (PCIe reads) and returns false if the host never freed a slot within ~2 s or another producer
-// already gave up (the record is then dropped and counted, never hangs the GPU).
+// cheap check against the device-side cache of the host's consumer index; reserve() then waits on the host
+// index (PCIe reads, poll_room() in a warp-uniform loop) and gives up if the host never freed a slot within
+// ~2 s or another producer already gave up (the record is then dropped and counted, never hangs the GPU).
 __device__ __forceinline__ bool has_room(const DevState& st, unsigned long long t) {
   return t < *(volatile const unsigned long long*)st.tail_cache + st.cap;
 }
-__device__ __forceinline__ bool wait_room(const DevState& st, unsigned long long t) {
-  if (*(volatile const unsigned long long*)st.dropped != 0) return false;
-  const unsigned long long t0 = globaltimer();
-  for (;;) {
-    const unsigned long long tl = *(volatile const unsigned long long*)st.tail;
-    if (t < tl + st.cap) { atomicMax(st.tail_cache, tl); return true; }
-    if (globaltimer() - t0 > 2000000000ull || *(volatile const unsigned long long*)st.dropped != 0) return false;
-    __nanosleep(500);
-  }
+// One poll of the host index for ticket t (waiting since t0): 1 = room (tail cache refreshed), -1 = give up
+// (~2 s without progress, or another producer already gave up), 0 = keep waiting.
+__device__ __forceinline__ int poll_room(const DevState& st, unsigned long long t, unsigned long long t0) {
+  if (*(volatile const unsigned long long*)st.dropped != 0) return -1;
+  const unsigned long long tl = *(volatile const unsigned long long*)st.tail;
+  if (t < tl + st.cap) { atomicMax(st.tail_cache, tl); return 1; }
+  return globaltimer() - t0 > 2000000000ull ? -1 : 0;
 }
 
 template <uint32_t T, class Prog>
@@ -368,6 +369,7 @@ struct Hooks {
   unsigned seq;               // records emitted by this warp in this launch
   unsigned long long hslot;   // device ring: next slot this warp holds, `held` slots from there
   unsigned held;
+  unsigned char* dptr = nullptr;   // device ring (TOOL_TRACE_DEV): this lane's address word of the next held slot
   unsigned npend = 0;         // uncommitted records of this warp (warp-uniform)
   unsigned pend_val = 0;      // lane k: tag value of the k-th uncommitted record
   unsigned char* pend_tag = nullptr;
@@ -527,38 +529,49 @@ struct Hooks {
   // of 16 full addresses each when the warp's addresses span more than ±2 GB.
   // Device ring (F2): k contiguous slots from this SM's current chunk; the warp whose range covers the
   // chunk's end opens the stripe's next chunk. No backpressure: a ring without free chunks drops.
+  // The whole warp runs the (rarely repeated) loop; lane 0 does the atomics and broadcasts, so no lane
+  // is left behind in a divergent retry loop (the hooks that follow need the warp converged, R-15).
   __device__ __forceinline__ bool reserve_dev(unsigned k, unsigned long long& t) {
-    unsigned long long tt = 0;
-    int ok = 1;
-    if (lane == 0) {
-      const unsigned sm = smid();
-      unsigned long long* w = st.rheads + (sm < st.rstripes ? sm : sm % st.rstripes);
-      const unsigned long long t0 = globaltimer();
-      for (;;) {
-        const unsigned long long v = atomicAdd(w, (unsigned long long)k);
-        const unsigned ck = (unsigned)(v >> 32), off = (unsigned)v;
-        if (ck == kRingFull) { ok = 0; break; }
-        if (off + k <= kRingChunk) {
-          tt = (unsigned long long)ck * kRingChunk + off;
-          ok = tt + k <= st.cap;
-          break;
-        }
-        if (off <= kRingChunk) {   // this warp's range covers the chunk end: open the next chunk
-          const unsigned long long nc = atomicAdd(st.rheads + st.rstripes, 1ull);
-          if (nc * kRingChunk >= st.cap) { atomicExch(w, (unsigned long long)kRingFull << 32); ok = 0; break; }
-          atomicExch(w, (nc << 32) | k);
-          tt = nc * kRingChunk;
-          ok = tt + k <= st.cap;
-          break;
-        }
-        // another warp is opening the next chunk: wait until the stripe word moves on
-        while ((unsigned)(*(volatile unsigned long long*)w >> 32) == ck && globaltimer() - t0 < 2000000000ull) {}
-        if (globaltimer() - t0 >= 2000000000ull) { ok = 0; break; }
+    const unsigned sm = smid();
+    unsigned long long* w = st.rheads + (sm < st.rstripes ? sm : sm % st.rstripes);
+    const unsigned long long t0 = globaltimer();
+    bool ok = false;
+    for (;;) {
+      unsigned long long v = 0;
+      if (lane == 0) v = atomicAdd(w, (unsigned long long)k);
+      v = __shfl_sync(FULL, v, 0);
+      const unsigned ck = (unsigned)(v >> 32), off = (unsigned)v;
+      if (ck == kRingFull) break;
+      if (off + k <= kRingChunk) {
+        t = (unsigned long long)ck * kRingChunk + off;
+        ok = t + k <= st.cap;
+        break;
       }
-      if (!ok) atomicAdd(st.dropped, 1ull);
+      if (off <= kRingChunk) {   // this warp's range covers the chunk end: open the next chunk
+        unsigned long long nc = 0;
+        if (lane == 0) nc = atomicAdd(st.rheads + st.rstripes, 1ull);
+        nc = __shfl_sync(FULL, nc, 0);
+        if (nc * kRingChunk >= st.cap) {
+          if (lane == 0) atomicExch(w, (unsigned long long)kRingFull << 32);
+          break;
+        }
+        if (lane == 0) atomicExch(w, (nc << 32) | k);
+        t = nc * kRingChunk;
+        ok = t + k <= st.cap;
+        break;
+      }
+      // another warp is opening the next chunk: wait until the stripe word moves on
+      bool moved = false;
+      while (!moved && globaltimer() - t0 < 2000000000ull) {
+        unsigned c = 0;
+        if (lane == 0) c = (unsigned)(*(volatile unsigned long long*)w >> 32);
+        moved = __shfl_sync(FULL, c, 0) != ck;
+      }
+      if (!moved) break;
     }
-    t = __shfl_sync(FULL, tt, 0);
-    return __shfl_sync(FULL, ok, 0) != 0;
+    if (!ok && lane == 0) atomicAdd(st.dropped, 1ull);
+    __syncwarp();
+    return ok;
   }
 
   __device__ __forceinline__ bool reserve(unsigned k, unsigned long long& t) {
@@ -570,12 +583,25 @@ struct Hooks {
     t = __shfl_sync(FULL, t, 0);
     if (!__shfl_sync(FULL, room, 0)) {
       commit();
-      int ok = 1;
-      if (lane == 0) ok = st.no_wait ? 0 : wait_room(st, t + k - 1);
-      if (!__shfl_sync(FULL, ok, 0)) {
+      // wait for the host to free the slot: the whole warp loops (lane 0 polls, then broadcasts), so
+      // no lane stays behind in a divergent spin (R-15)
+      int ok = 0;
+      if (!st.no_wait) {
+        const unsigned long long t0 = globaltimer();
+        for (;;) {
+          int r = 0;   // 1: room, -1: give up, 0: keep waiting
+          if (lane == 0) r = poll_room(st, t + k - 1, t0);
+          r = __shfl_sync(FULL, r, 0);
+          if (r != 0) { ok = r > 0; break; }
+          __nanosleep(500);
+        }
+      }
+      if (!ok) {
         if (lane == 0) atomicAdd(st.dropped, 1ull);
+        __syncwarp();
         return false;
       }
+      __syncwarp();
     }
     return true;
   }
@@ -599,6 +625,33 @@ struct Hooks {
     constexpr nvbt_instr_desc d = Prog::t[PC];
     const unsigned w2 = (unsigned)d.opcode | ((unsigned)d.width << 16) | ((unsigned)d.kind << 24);
     const unsigned long long a = act ? addr : 0ull;
+    if constexpr ((T & TOOL_TRACE_DEV) != 0) {
+      // device ring, selected at compile time: a warp reserves the slots of the rest of its basic block
+      // at once (x4 in loops) and walks them with a per-lane pointer (+288 B per record); every lane
+      // stores its address (8 B, 256 B coalesced per record) and lanes 0, 1 the 32 B header with tag 1
+      // in one predicated 16 B store each. Every slot is lap 1 and the consumer is a later kernel: no
+      // fence, no commit.
+      constexpr unsigned K = (unsigned)mem_left<Prog>(PC) * ((PC >= Prog::REG_LO && PC <= Prog::REG_HI) ? 4u : 1u);
+      if (held == 0u) {   // warp-uniform
+        unsigned long long t0;
+        if (reserve_dev(K, t0)) {
+          held = K;
+          dptr = st.ring + t0 * RECORD_BYTES + 32u + 8u * lane;
+        }
+      }
+      if (held != 0u) {
+        --held;
+        asm volatile("st.global.u64 [%0], %1;" ::"l"(dptr), "l"(a) : "memory");
+        const bool l0 = lane == 0u;
+        asm volatile("{\n\t.reg .pred p;\n\tsetp.lt.u32 p, %0, 2;\n\t@p st.global.v4.u32 [%1], {%2, %3, %4, %5};\n\t}"
+                     ::"r"(lane), "l"(dptr + (8 * (int)lane - 32)), "r"(l0 ? st.launch : A), "r"(l0 ? gwarp : P),
+                     "r"(l0 ? seq : w2), "r"(l0 ? (unsigned)PC : 1u) : "memory");
+        __syncwarp();   // ptxas may branch around the predicated store: rejoin before the next hook (R-15)
+        dptr += RECORD_BYTES;
+      }
+      ++seq;
+      return;
+    }
     unsigned long long t;
     unsigned tag;
     if (!st.compact) {

@@ -18,6 +18,21 @@ static inline int dispatch(uint32_t tools, F&& f) {
 #undef NVBT_CASE
 }
 
+// Workloads that trace into device rings (F2: stencil, BFS) also have TRACE variants with the device-ring
+// producer selected at compile time (TOOL_TRACE_DEV); other contexts take the run-time channel path.
+template <class F>
+static inline int dispatch_trace(uint32_t tools, bool dev_ring, F&& f) {
+  if ((tools & NVBT_TOOL_TRACE) != 0 && dev_ring) {
+#define NVBT_CASE(v) case v: f(std::integral_constant<uint32_t, v | TOOL_TRACE_DEV>{}); return NVBT_OK;
+    switch (tools) {
+      NVBT_CASE(8) NVBT_CASE(9) NVBT_CASE(10) NVBT_CASE(12) NVBT_CASE(13) NVBT_CASE(14)
+      default: return set_error(NVBT_EINVAL, "unsupported tools combination 0x%x", tools);
+    }
+#undef NVBT_CASE
+  }
+  return dispatch(tools, f);
+}
+
 struct LaunchCtx {
   cudaStream_t stream = nullptr;
   DevState st{};

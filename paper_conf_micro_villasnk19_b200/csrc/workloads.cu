@@ -271,7 +271,7 @@ static int bfs_launch(nvbt_ctx ctx, void* stream, uint32_t tools, int which, con
   if (rc) return rc;
   const unsigned nc = (which & 1) ? l1.n_ctas : l2.n_ctas;
   if (nc == 0) return NVBT_OK;
-  rc = dispatch(tools, [&](auto tag) {
+  rc = dispatch_trace(tools, ((which & 1) ? l1.st : l2.st).no_wait != 0u, [&](auto tag) {
     constexpr uint32_t TT = decltype(tag)::value;
     if (which & 1) k_bfs_expand<TT><<<l1.grid, 256, 0, l1.stream>>>(rowptr, col, n, mask, visited, updating, l1.st);
     if (which & 2) k_bfs_update<TT><<<l2.grid, 256, 0, l2.stream>>>(n, mask, visited, updating, cost, over, level, l2.st);
@@ -304,7 +304,9 @@ int nvbt_stencil(nvbt_ctx ctx, void* stream, uint32_t tools, const float* in, fl
   if (rc) return rc;
   if (lc.n_ctas == 0) return NVBT_OK;
   const dim3 block(32, 8);
-  rc = dispatch(tools, [&](auto tag) { k_stencil<decltype(tag)::value><<<lc.grid, block, 0, lc.stream>>>(in, out, n, lc.st); });
+  rc = dispatch_trace(tools, lc.st.no_wait != 0u, [&](auto tag) {
+    k_stencil<decltype(tag)::value><<<lc.grid, block, 0, lc.stream>>>(in, out, n, lc.st);
+  });
   return rc ? rc : done(ctx, 1);
 }
 

@@ -32,6 +32,19 @@ if which in ("all", "c1"):
         nb.nvbt_vectoradd(c1, nb.TOOL_NONE, a, b, c, N)
         nb.nvbt_vectoradd(c1, nb.TOOL_COUNT, a, b, c, N)
     nb.nvbt_count(c1)
+if which == "f2":   # traced stencil into an HBM ring (F2 producer), 8192^2 x 2 launches, then the consumer
+    from synth import uniform_f32 as _u
+    n, iters = 8192, 2
+    fctx = nb.nvbt_init(nb.W_STENCIL, nb.COUNT | nb.TRACE)
+    x0 = torch.from_numpy(_u((n, n), 4)).cuda()
+    b0, b1 = x0.clone(), torch.empty_like(x0)
+    cap = iters * (2 * (n * n // 32) + 4 * (n - 2) * (n // 32))
+    cap += cap // 50 + 148 * 4096
+    ring = torch.zeros(64 + 288 * cap, dtype=torch.uint8, device="cuda")
+    ch = nb.nvbt_channel_open(fctx, ring)
+    dr.run_stencil(fctx, nb.TOOL_NONE, b0, b1, n, iters)
+    dr.run_stencil(fctx, nb.TOOL_TRACE, b0, b1, n, iters)
+    torch.cuda.synchronize()
 if which in ("all", "c5"):
     n = 1 << 26
     rctx = nb.nvbt_init(nb.W_REPLAY, nb.COUNT | nb.MEMDIV)
