@@ -380,6 +380,12 @@ k_rpA(const uint4* __restrict__ hdr, unsigned n, unsigned P, const uint8_t* __re
   }
 }
 
+// c += (x > K) as a predicated add (the compiler's select-based form costs ~3 instructions)
+template <unsigned K>
+__device__ __forceinline__ void inc_if_gt(unsigned& c, unsigned x) {
+  asm("{\n\t.reg .pred p;\n\tsetp.gt.u32 p, %1, %2;\n\t@p add.u32 %0, %0, 1;\n\t}" : "+r"(c) : "r"(x), "n"(K));
+}
+
 // Pass B analysis of one stage (up to 16 slots; meta E = 0 marks an empty row). Lane (j, h) = (lane & 15,
 // lane >> 4) scans addresses 16h .. 16h+15 of row j; 16 B chunk c of row j is stored at chunk c ^ (j & 7),
 // so the 8 lanes of a quarter-warp (consecutive j, same h) read 8 distinct bank groups.
@@ -407,8 +413,8 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
       hb |= hi ^ f_hi;
       viol |= lo < prev;
       const unsigned x = lo ^ prev;
-      bs += x > 31u;
-      bl += x > 127u;
+      inc_if_gt<31>(bs, x);
+      inc_if_gt<127>(bl, x);
       mn = min(mn, lo);
       mx = max(mx, lo);
       prev = lo;
