@@ -493,8 +493,8 @@ __global__ void __launch_bounds__(256, 4) k_footprint(const unsigned char* __res
   unsigned nl = 0;
   if (r0 + lane < r1) {
     const unsigned char* rec = ring + 64 + (r0 + lane) * RECORD_BYTES;
-    nh1 = __ldcs(reinterpret_cast<const uint4*>(rec + 16));   // A P op|w|k tag
-    nl = __ldcs(reinterpret_cast<const unsigned*>(rec));
+    nh1 = __ldg(reinterpret_cast<const uint4*>(rec + 16));   // A P op|w|k tag
+    nl = __ldg(reinterpret_cast<const unsigned*>(rec));
   }
   for (unsigned long long base = r0; base < r1; base += 32) {
     const unsigned cnt = r1 - base < 32 ? (unsigned)(r1 - base) : 32u;
@@ -503,8 +503,8 @@ __global__ void __launch_bounds__(256, 4) k_footprint(const unsigned char* __res
     nh1 = make_uint4(0, 0, 0, 0);
     if (base + 32 + lane < r1) {
       const unsigned char* rec = ring + 64 + (base + 32 + lane) * RECORD_BYTES;
-      nh1 = __ldcs(reinterpret_cast<const uint4*>(rec + 16));
-      nl = __ldcs(reinterpret_cast<const unsigned*>(rec));
+      nh1 = __ldg(reinterpret_cast<const uint4*>(rec + 16));
+      nl = __ldg(reinterpret_cast<const unsigned*>(rec));
     }
     const bool ok = lid < n_launches;
     const unsigned bad = __ballot_sync(0xffffffffu, lid != 0xFFFFFFFFu && !ok);
