@@ -443,7 +443,8 @@ def run_replay(args, torch, nb, dr, rank, world, local, peaks, peaks_src):
         "metric": "replayed warp-instr events/sec", "value": value, "unit": "events/s", "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * t_total / args.steps,
         "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-        "config": {"workload": wl.desc, "events": args.replay_events, "chunk": wl.chunk,
+        "config": {"workload": wl.desc.replace("10^10", f"{args.replay_events:.3g}" if args.replay_events != 10**10 else "10^10"),
+                   "events": args.replay_events, "chunk": wl.chunk,
                    "l2": "inputs (36.5 GB per chunk) larger than L2"},
         "roofline": {"bound": "hbm", "achieved": ach / 1e9, "peak": peaks["hbm_gbs"], "unit": "GB/s",
                      "frac": ach / 1e9 / peaks["hbm_gbs"], "peak_source": peaks_src,
