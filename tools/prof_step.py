@@ -28,9 +28,11 @@ if which in ("all", "c1"):
     c1 = nb.nvbt_init(nb.W_VECTORADD, nb.COUNT | nb.OPHIST)
     a, b = torch.from_numpy(_u(N, 1)).cuda(), torch.from_numpy(_u(N, 2)).cuda()
     c = torch.empty_like(a)
+    c1b = nb.nvbt_init(nb.W_VECTORADD, nb.COUNT | nb.OPHIST | nb.BB)
     for _ in range(3):
         nb.nvbt_vectoradd(c1, nb.TOOL_NONE, a, b, c, N)
         nb.nvbt_vectoradd(c1, nb.TOOL_COUNT, a, b, c, N)
+        nb.nvbt_vectoradd(c1b, nb.TOOL_BBCOUNT, a, b, c, N)
     nb.nvbt_count(c1)
 if which == "f2":   # traced stencil into an HBM ring (F2 producer), 8192^2 x 2 launches, then the consumer
     from synth import uniform_f32 as _u
