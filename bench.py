@@ -602,9 +602,12 @@ def run_c4(args, torch, nb, dr, local):
             e0.record()
             dr.run_stencil(ctx, nb.TOOL_TRACE, buf0, buf1, n, iters)
             e1.record()
-            d = nb.nvbt_channel_drain_digest(ch, timeout_us=600_000_000)
+            if args.drain == "discard":
+                nrec = nb.nvbt_channel_drain_discard(ch, timeout_us=600_000_000)
+            else:
+                nrec = nb.nvbt_channel_drain_digest(ch, timeout_us=600_000_000).n_rec
             torch.cuda.synchronize()
-            res.append((time.perf_counter() - t0, d.n_rec, e0.elapsed_time(e1) / 1e3))
+            res.append((time.perf_counter() - t0, nrec, e0.elapsed_time(e1) / 1e3))
     dropped = nb.nvbt_channel_dropped(ch)
     recs = res[-1][1]
     t_tr = sum(r[0] for r in res) / len(res)
@@ -614,7 +617,8 @@ def run_c4(args, torch, nb, dr, local):
             "unit": "records/s", "n_gpus": 1, "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * t_tr,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
             "config": {"workload": f"C4 stencil {n}^2 x {iters}, tools TRACE", "ring_slots": args.ring_records,
-                       "transport": "compact 176 B slots (EM 5.1)" if args.compact else "288 B records"},
+                       "transport": "compact 176 B slots (EM 5.1)" if args.compact else "288 B records",
+                       "host_callback": args.drain},
             "records_per_run": recs, "records_expected": expect, "dropped": dropped,
             "gpu_s_per_run": sum(r[2] for r in res) / len(res),
             "host_threads": os.environ.get("NVBT_DRAIN_THREADS", str(os.cpu_count())),
@@ -840,6 +844,8 @@ def main():
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--drain", choices=["digest", "discard"], default="digest",
+                    help="C4: host callback (digest of every record, or discard: the transport alone)")
     ap.add_argument("--replay-impl", choices=["staged", "single"], default="staged",
                     help="C5: two-pass staged replay (default) or the single-pass kernel")
     ap.add_argument("--workload", choices=["c1", "c2", "c3", "c4", "c5", "f1", "f2", "f4"], default="c2")

@@ -170,6 +170,8 @@ typedef struct { uint64_t n_rec, d1, d2; } nvbt_digest;         /* EM §5 multis
 int nvbt_drain_digest(const void* records, uint64_t n_records, void* user /* nvbt_digest* */);
 typedef struct { void* dst; uint64_t capacity; uint64_t n; } nvbt_copy_sink;   /* dst: host [capacity*288] */
 int nvbt_drain_copy(const void* records, uint64_t n_records, void* user /* nvbt_copy_sink* */);
+/* Counts and discards the records (user: nullable uint64_t* count): measures the transport alone. */
+int nvbt_drain_discard(const void* records, uint64_t n_records, void* user /* uint64_t* */);
 /* Host-side digest of an array of records (for checking copies). */
 int nvbt_digest_records(const void* records, uint64_t n_records, nvbt_digest* out);
 /* Decodes n_slots 176 B transport slots (EM §5.1; tags ignored) into EM §5 records at out (capacity

@@ -279,6 +279,7 @@ using namespace nvbt;
 extern "C" {
 int nvbt_drain_digest(const void* records, uint64_t n_records, void* user);
 int nvbt_drain_copy(const void* records, uint64_t n_records, void* user);
+int nvbt_drain_discard(const void* records, uint64_t n_records, void* user);
 }
 
 extern "C" {
@@ -666,7 +667,7 @@ int nvbt_channel_drain(nvbt_channel ch, nvbt_drain_fn fn, void* user, int64_t ti
   const auto t0 = std::chrono::steady_clock::now();
   const uint64_t kBatch = 1u << 17;
   volatile uint64_t* tail = reinterpret_cast<volatile uint64_t*>(ch->host);
-  const bool builtin = fn == nvbt_drain_digest || fn == nvbt_drain_copy;
+  const bool builtin = fn == nvbt_drain_digest || fn == nvbt_drain_copy || fn == nvbt_drain_discard;
   uint64_t delivered = 0;
   int rc = NVBT_OK;
   for (;;) {
@@ -750,6 +751,11 @@ int nvbt_channel_drain(nvbt_channel ch, nvbt_drain_fn fn, void* user, int64_t ti
   }
   if (n_drained) *n_drained = delivered;
   return rc;
+}
+
+int nvbt_drain_discard(const void*, uint64_t n, void* user) {
+  if (user) *static_cast<uint64_t*>(user) += n;
+  return 0;
 }
 
 int nvbt_drain_digest(const void* records, uint64_t n, void* user) {

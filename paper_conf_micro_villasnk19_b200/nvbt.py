@@ -109,9 +109,10 @@ for _name, (_args, _res) in _sigs.items():
     _f = getattr(_lib, _name)
     _f.argtypes = _args
     _f.restype = _res
-EXPORTED = tuple(_sigs) + ("nvbt_drain_digest", "nvbt_drain_copy")
+EXPORTED = tuple(_sigs) + ("nvbt_drain_digest", "nvbt_drain_copy", "nvbt_drain_discard")
 _DRAIN_DIGEST = C.cast(_lib.nvbt_drain_digest, C.c_void_p).value
 _DRAIN_COPY = C.cast(_lib.nvbt_drain_copy, C.c_void_p).value
+_DRAIN_DISCARD = C.cast(_lib.nvbt_drain_discard, C.c_void_p).value
 
 
 class NvbtError(RuntimeError):
@@ -350,6 +351,14 @@ def nvbt_channel_drain_digest(ch, timeout_us=-1, digest=None):
     n = C.c_uint64()
     _check(_lib.nvbt_channel_drain(ch.handle, C.c_void_p(_DRAIN_DIGEST), C.byref(d), timeout_us, C.byref(n)))
     return d
+
+
+def nvbt_channel_drain_discard(ch, timeout_us=-1):
+    """Drain with the built-in discard callback (transport only); returns the number of records."""
+    cnt = C.c_uint64()
+    n = C.c_uint64()
+    _check(_lib.nvbt_channel_drain(ch.handle, C.c_void_p(_DRAIN_DISCARD), C.byref(cnt), timeout_us, C.byref(n)))
+    return n.value
 
 
 def nvbt_channel_drain_copy(ch, dst, timeout_us=-1):
