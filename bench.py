@@ -586,7 +586,7 @@ def run_c4(args, torch, nb, dr, local):
     x0 = torch.from_numpy(uniform_f32((n, n), 4)).cuda()
     buf0, buf1 = x0.clone(), torch.empty_like(x0)
     slot = 176 if args.compact else 288
-    ring = torch.empty(64 + slot * args.ring_records, dtype=torch.uint8, pin_memory=True)
+    ring = torch.empty(nb.nvbt_channel_bytes(args.ring_records, compact=args.compact), dtype=torch.uint8, pin_memory=True)
     ch = nb.nvbt_channel_open(ctx, ring, compact=args.compact)
     # plain baseline
     for _ in range(args.warmup):

@@ -4,11 +4,13 @@
 // or sent to the CPU for further processing" (P:L187 (§6.1)). The paper gives no mechanism; this one:
 //  * producers (warps, nvbt_dev.cuh emit<>) take a ticket t = atomicAdd(head, 1) in device memory, wait
 //    while t >= tail + cap (tail = consumer index the host publishes in the ring's first 64 bytes, cached
-//    in device memory), write the 288 B record into slot t % cap over PCIe with coalesced stores, then a
-//    system-scope fence and a 16 B store carrying the tag (t / cap) + 1;
+//    in device memory), write the 288 B record (reserved field 0) into slot t % cap over PCIe with
+//    coalesced stores, then a system-scope fence and a 4 B store of the tag (t / cap) + 1 into word t % cap
+//    of a dense tag array that follows the slots (tags of neighbouring tickets share PCIe lines; a tag in
+//    the record's own header line cost one extra partial-line write per record, see DESIGN §5 C4);
 //  * the consumer (nvbt_channel_drain, calling thread) delivers slots in ticket order as soon as their tag
-//    matches, zeroes the tag field (EM §5 "reserved = 0"), calls the user callback on contiguous batches
-//    and publishes tail.
+//    matches (a tag of an earlier lap never equals the current one, so tags are never cleared), calls the
+//    user callback on contiguous batches and publishes tail.
 #include <chrono>
 #include <condition_variable>
 #include <cstring>
@@ -25,6 +27,7 @@ struct nvbt_chan_s {
   unsigned char* host = nullptr;      // ring base (host view)
   unsigned char* dev = nullptr;       // ring base (device view)
   unsigned char* slots = nullptr;     // host view of slot 0
+  const uint32_t* tags = nullptr;     // host ring: host view of the tag array (cap words after the slots)
   uint64_t cap = 0;
   uint64_t consumed = 0;
   unsigned slot = 288;                 // bytes per ring slot (288 full, 176 compact)
@@ -46,6 +49,7 @@ void channel_state(nvbt_chan_s* ch, DevState* st) {
   st->ring = ch->dev + HDR;
   st->tail = reinterpret_cast<const unsigned long long*>(ch->dev);
   st->cap = ch->cap;
+  st->tags = ch->on_device ? nullptr : reinterpret_cast<unsigned*>(ch->dev + HDR + ch->cap * ch->slot);
   st->slot_bytes = ch->slot;
   // compact = 1; 2 forces the wide form for every record (NVBT_COMPACT_FORCE_WIDE=1, tests only)
   st->compact = ch->slot == COMPACT_BYTES ? (ch->force_wide ? 2u : 1u) : 0u;
@@ -75,7 +79,7 @@ static void digest_serial(const unsigned char* rec, uint64_t n, uint64_t* d1, ui
   for (uint64_t r = 0; r < n; ++r) {
     uint64_t x[36];
     std::memcpy(x, rec + r * RECORD_BYTES, RECORD_BYTES);
-    x[3] &= 0x00000000ffffffffull;  // bytes 28..31: ring tag, delivered as 0 (EM §5 reserved)
+    x[3] &= 0x00000000ffffffffull;  // bytes 28..31: EM §5 reserved, delivered as 0
     uint64_t h1 = 0, h2 = 0;
     for (int j = 0; j < 36; ++j) { h1 += x[j] * kDig.c1[j]; h2 += x[j] * kDig.c2[j]; }
     s1 += mix64(h1);
@@ -165,21 +169,21 @@ static void digest_range(const unsigned char* rec, uint64_t n, uint64_t* d1, uin
 
 // Length of the prefix of slots [0, lim) whose tag equals `lap` (written and committed). Scans a short
 // window serially and, when that is all ready, the rest of the batch in parallel on the pool.
-static inline bool slot_ready(const unsigned char* rec, uint32_t lap) {
-  return *reinterpret_cast<volatile const uint32_t*>(rec + 28) == lap;
+static inline bool slot_ready(const uint32_t* tag, uint32_t lap) {
+  return *reinterpret_cast<volatile const uint32_t*>(tag) == lap;
 }
-static uint64_t ready_prefix(const unsigned char* base, uint64_t lim, uint32_t lap, unsigned sb) {
+static uint64_t ready_prefix(const uint32_t* base, uint64_t lim, uint32_t lap) {
   const uint64_t w = std::min<uint64_t>(lim, 2048);
   uint64_t n = 0;
-  while (n < w && slot_ready(base + n * sb, lap)) ++n;
+  while (n < w && slot_ready(base + n, lap)) ++n;
   if (n < w || n == lim) return n;
   Pool& pool = Pool::get();
   const uint64_t rest = lim - n;
   std::vector<uint64_t> first(pool.size(), UINT64_MAX);
-  const unsigned char* b2 = base + n * sb;
+  const uint32_t* b2 = base + n;
   pool.parallel_for(rest, [&](unsigned id, uint64_t lo, uint64_t hi) {
     uint64_t i = lo;
-    while (i < hi && slot_ready(b2 + i * sb, lap)) ++i;
+    while (i < hi && slot_ready(b2 + i, lap)) ++i;
     first[id] = i < hi ? i : UINT64_MAX;
   });
   uint64_t stop = rest;
@@ -266,12 +270,6 @@ static uint64_t digest_compact(const unsigned char* sl, uint64_t n, uint64_t* d1
   return c;
 }
 
-static void clear_tags(unsigned char* base, uint64_t n) {
-  Pool::get().parallel_for(n, [&](unsigned, uint64_t lo, uint64_t hi) {
-    for (uint64_t r = lo; r < hi; ++r) std::memset(base + r * RECORD_BYTES + 28, 0, 4);
-  });
-}
-
 }  // namespace nvbt
 
 using namespace nvbt;
@@ -284,6 +282,10 @@ int nvbt_drain_discard(const void* records, uint64_t n_records, void* user);
 
 extern "C" {
 
+size_t nvbt_channel_bytes(uint32_t record_bytes, uint64_t slots, int on_device) {
+  return HDR + slots * (record_bytes + (on_device ? 0u : 4u));
+}
+
 int nvbt_channel_open(nvbt_ctx c, void* ring, size_t bytes, uint32_t record_bytes, nvbt_channel* out) {
   if (!c || !ring || !out) return set_error(NVBT_EINVAL, "null argument");
   if (!(c->flags & NVBT_TRACE)) return set_error(NVBT_ESTATE, "NVBT_TRACE not enabled at init");
@@ -291,7 +293,7 @@ int nvbt_channel_open(nvbt_ctx c, void* ring, size_t bytes, uint32_t record_byte
   if (record_bytes != RECORD_BYTES && record_bytes != COMPACT_BYTES)
     return set_error(NVBT_EINVAL, "record_bytes %u is neither 288 nor 176", record_bytes);
   if (reinterpret_cast<uintptr_t>(ring) % 64) return set_error(NVBT_EINVAL, "ring not 64-byte aligned");
-  if (bytes < HDR + 2 * record_bytes) return set_error(NVBT_ENOMEM, "ring of %zu bytes holds < 2 slots", bytes);
+  if (bytes < HDR + 2 * (record_bytes + 4)) return set_error(NVBT_ENOMEM, "ring of %zu bytes holds < 2 slots", bytes);
   NVBT_CUDA(cudaSetDevice(c->device));
   cudaPointerAttributes pa{};
   NVBT_CUDA(cudaPointerGetAttributes(&pa, ring));
@@ -309,7 +311,9 @@ int nvbt_channel_open(nvbt_ctx c, void* ring, size_t bytes, uint32_t record_byte
   ch->slots = on_device ? nullptr : ch->host + HDR;
   ch->slot = record_bytes;
   { const char* e = getenv("NVBT_COMPACT_FORCE_WIDE"); ch->force_wide = e && atoi(e) != 0; }
-  ch->cap = (bytes - HDR) / record_bytes;
+  // host rings: each slot has a 4 B tag in the array after the slots; device rings carry the tag in-record
+  ch->cap = (bytes - HDR) / (record_bytes + (on_device ? 0u : 4u));
+  ch->tags = on_device ? nullptr : reinterpret_cast<const uint32_t*>(ch->host + HDR + ch->cap * record_bytes);
   if (on_device) {
     int sms = 148;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, c->device);
@@ -317,7 +321,7 @@ int nvbt_channel_open(nvbt_ctx c, void* ring, size_t bytes, uint32_t record_byte
   }
   cudaError_t e = cudaSuccess;
   if (on_device) e = cudaMemsetAsync(ring, 0, HDR + ch->cap * record_bytes, c->stream);
-  else std::memset(ch->host, 0, HDR + ch->cap * record_bytes);
+  else std::memset(ch->host, 0, HDR + ch->cap * (record_bytes + 4));
   if (on_device && e == cudaSuccess) {   // every stripe starts without a chunk; chunk counter 0
     std::vector<unsigned long long> w(ch->rstripes + 1, ((unsigned long long)kRingNoChunk << 32) | kRingChunk);
     w.back() = 0;
@@ -667,7 +671,6 @@ int nvbt_channel_drain(nvbt_channel ch, nvbt_drain_fn fn, void* user, int64_t ti
   const auto t0 = std::chrono::steady_clock::now();
   const uint64_t kBatch = 1u << 17;
   volatile uint64_t* tail = reinterpret_cast<volatile uint64_t*>(ch->host);
-  const bool builtin = fn == nvbt_drain_digest || fn == nvbt_drain_copy || fn == nvbt_drain_discard;
   uint64_t delivered = 0;
   int rc = NVBT_OK;
   for (;;) {
@@ -675,11 +678,10 @@ int nvbt_channel_drain(nvbt_channel ch, nvbt_drain_fn fn, void* user, int64_t ti
     const uint32_t lap = static_cast<uint32_t>(ch->consumed / ch->cap) + 1u;
     const uint64_t lim = std::min<uint64_t>(ch->cap - slot, kBatch);
     const unsigned sb = ch->slot;
-    const uint64_t n = ready_prefix(ch->slots + slot * sb, lim, lap, sb);
+    const uint64_t n = ready_prefix(ch->tags + slot, lim, lap);
     if (n && sb == RECORD_BYTES) {
       std::atomic_thread_fence(std::memory_order_acquire);
       unsigned char* base = ch->slots + slot * RECORD_BYTES;
-      if (!builtin) clear_tags(base, n);   // built-in callbacks ignore / clear the tag themselves
       const int urc = fn(base, n, user);
       ch->consumed += n;
       delivered += n;

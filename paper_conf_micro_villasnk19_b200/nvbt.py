@@ -79,6 +79,7 @@ _sigs = {
     "nvbt_opcode_hist": ([_P, _P, _P, C.c_uint32], C.c_int),
     "nvbt_bb_count": ([_P, _P, C.c_uint32], C.c_int),
     "nvbt_mem_divergence": ([_P, _P, C.c_uint32, C.POINTER(MemDivTotal)], C.c_int),
+    "nvbt_channel_bytes": ([C.c_uint32, C.c_uint64, C.c_int], C.c_size_t),
     "nvbt_channel_open": ([_P, _P, C.c_size_t, C.c_uint32, C.POINTER(_P)], C.c_int),
     "nvbt_channel_drain": ([_P, _P, _P, C.c_int64, C.POINTER(C.c_uint64)], C.c_int),
     "nvbt_channel_close": ([_P], C.c_int),
@@ -303,6 +304,12 @@ def nvbt_launch_count(ctx):
 class Channel:
     def __init__(self, handle, ctx, ring):
         self.handle, self.ctx, self.ring = handle, ctx, ring
+
+
+def nvbt_channel_bytes(slots, compact=False, on_device=False):
+    """Ring size (bytes) that holds `slots` slots: 64 + slots * (record + 4-byte tag) for host rings."""
+    rb = COMPACT_RECORD_BYTES if compact else RECORD_BYTES
+    return int(_lib.nvbt_channel_bytes(rb, slots, 1 if on_device else 0))
 
 
 def nvbt_channel_open(ctx, ring, compact=False):

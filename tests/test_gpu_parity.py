@@ -153,7 +153,7 @@ def _stencil_case(nvbt, n, iters, ring_records, tools_names=("TRACE", "MEMDIV", 
     ctx = nb.nvbt_init(nb.W_STENCIL, nb.COUNT | nb.MEMDIV | nb.TRACE)
     x0 = cuda(uniform_f32((n, n), 4))
     buf0, buf1 = x0.clone(), torch.zeros_like(x0)
-    ring = torch.empty(64 + (176 if compact else 288) * ring_records, dtype=torch.uint8, pin_memory=True)
+    ring = torch.empty(nb.nvbt_channel_bytes(ring_records, compact=compact), dtype=torch.uint8, pin_memory=True)
     ring.view(torch.int32).fill_(1)            # stale "lap 1" tags everywhere: open must clear them
     ch = nb.nvbt_channel_open(ctx, ring, compact=compact)
     dr.run_stencil(ctx, t, buf0, buf1, n, iters)
@@ -203,7 +203,7 @@ def test_channel_digest_drain(nvbt):
     ctx = nb.nvbt_init(nb.W_STENCIL, nb.TRACE)
     x0 = cuda(uniform_f32((n, n), 4))
     buf0, buf1 = x0.clone(), torch.zeros_like(x0)
-    ring = torch.empty(64 + 288 * 1000, dtype=torch.uint8, pin_memory=True)
+    ring = torch.empty(nb.nvbt_channel_bytes(1000), dtype=torch.uint8, pin_memory=True)
     ch = nb.nvbt_channel_open(ctx, ring)
     dr.run_stencil(ctx, nb.TOOL_TRACE, buf0, buf1, n, iters)
     d = nb.nvbt_channel_drain_digest(ch, timeout_us=60_000_000)
@@ -668,7 +668,7 @@ def test_stencil_trace_full_size_c4(nvbt):
     dr.run_stencil(ctx, nb.TOOL_NONE, a0, a1, n, iters)
     plain = (a0 if iters % 2 == 0 else a1).clone()
     nb.nvbt_reset(ctx)
-    ring = torch.empty(64 + 288 * (1 << 22), dtype=torch.uint8, pin_memory=True)
+    ring = torch.empty(nb.nvbt_channel_bytes(1 << 22), dtype=torch.uint8, pin_memory=True)
     ch = nb.nvbt_channel_open(ctx, ring)
     b0, b1 = x0.clone(), torch.empty_like(x0)
     dr.run_stencil(ctx, nb.TOOL_TRACE | nb.TOOL_COUNT, b0, b1, n, iters)

@@ -172,7 +172,7 @@ def _worker(rank, world, port, q):
         sn, iters = 96, 3
         sctx = nb.nvbt_init(nb.W_STENCIL, nb.COUNT | nb.MEMDIV | nb.TRACE)
         nb.nvbt_set_partition(sctx, rank, world)
-        ring = torch.empty(64 + 288 * (1 << 14), dtype=torch.uint8, pin_memory=True)
+        ring = torch.empty(nb.nvbt_channel_bytes(1 << 14), dtype=torch.uint8, pin_memory=True)
         ch = nb.nvbt_channel_open(sctx, ring)
         x0 = cuda(uniform_f32((sn, sn), 4))
         b0, b1 = x0.clone(), torch.zeros_like(x0)

@@ -158,7 +158,7 @@ def test_wfft_trace_records(nvbt):
     nb = nvbt.nvbt
     n_fft, ctas = 333, 4
     ctx = nb.nvbt_init(nb.W_WFFT_EMU, nb.COUNT | nb.TRACE)
-    ring = torch.empty(64 + 288 * 4096, dtype=torch.uint8, pin_memory=True)
+    ring = torch.empty(nb.nvbt_channel_bytes(4096), dtype=torch.uint8, pin_memory=True)
     ch = nb.nvbt_channel_open(ctx, ring)
     x, X = inputs(n_fft, seed=8)
     nb.nvbt_wfft32(ctx, nb.TOOL_EMU | nb.TOOL_TRACE | nb.TOOL_COUNT, nb.WFFT_PROXY, x, X, n_fft, ctas)
