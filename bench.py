@@ -617,7 +617,7 @@ def run_c4(args, torch, nb, dr, local):
             "unit": "records/s", "n_gpus": 1, "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * t_tr,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
             "config": {"workload": f"C4 stencil {n}^2 x {iters}, tools TRACE", "ring_slots": args.ring_records,
-                       "transport": "compact 176 B slots (EM 5.1)" if args.compact else "288 B records",
+                       "transport": "compact 176 B slots at a 192 B stride (EM 5.1)" if args.compact else "288 B records",
                        "host_callback": args.drain},
             "records_per_run": recs, "records_expected": expect, "dropped": dropped,
             "gpu_s_per_run": sum(r[2] for r in res) / len(res),

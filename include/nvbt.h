@@ -126,9 +126,11 @@ int nvbt_mem_divergence(nvbt_ctx ctx, nvbt_memdiv* per_pc, uint32_t n_pcs, nvbt_
 
 /* ---- trace channel (a6; "sent to the CPU for further processing", P:L187 (§6.1)) ----
  * pinned_ring: caller-owned pinned, device-mapped host memory (cudaHostAlloc / torch pin_memory), at
- * least 64 + 2 * (record_bytes + 4) bytes, 64-byte aligned. Its first 64 bytes hold the consumer index the
- * producers read for backpressure; the rest is cap = floor((ring_bytes - 64) / (record_bytes + 4)) slots
- * followed by cap 4-byte commit tags (one per slot, written by the producer after its record). A CUDA
+ * least 64 + 2 * (stride + 4) bytes, 64-byte aligned, where stride = 288 for 288 B records and 192 for
+ * 176 B compact slots (padded so that two slots cover three 128 B lines). Its first 64 bytes hold the
+ * consumer index the producers read for backpressure; the rest is cap = floor((ring_bytes - 64) /
+ * (stride + 4)) slots followed by cap 4-byte commit tags (one per slot, written by the producer after its
+ * record). A CUDA
  * device buffer instead (F2, on-GPU consumers) has no tag array: cap = floor((ring_bytes - 64) / 288).
  * nvbt_channel_bytes gives the ring_bytes that hold `slots` slots. */
 size_t nvbt_channel_bytes(uint32_t record_bytes, uint64_t slots, int on_device);

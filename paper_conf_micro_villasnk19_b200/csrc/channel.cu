@@ -44,6 +44,11 @@ namespace nvbt {
 
 static constexpr size_t HDR = 64;
 static constexpr unsigned COMPACT_BYTES = NVBT_COMPACT_RECORD_BYTES;
+// Ring stride of a compact slot: the 176 B slot padded to 192 B (pairs of slots cover 3 whole lines; PCIe
+// D2H of SM stores, tools/peaks/d2h_pattern.cu: 176 B at a 176 B stride 33.0 GB/s of slot bytes, at a 192 B
+// stride 36.5). The pad is never written or read.
+static constexpr unsigned COMPACT_STRIDE = 192;
+static inline unsigned slot_stride(uint32_t record_bytes) { return record_bytes == COMPACT_BYTES ? COMPACT_STRIDE : record_bytes; }
 
 void channel_state(nvbt_chan_s* ch, DevState* st) {
   st->ring = ch->dev + HDR;
@@ -52,7 +57,7 @@ void channel_state(nvbt_chan_s* ch, DevState* st) {
   st->tags = ch->on_device ? nullptr : reinterpret_cast<unsigned*>(ch->dev + HDR + ch->cap * ch->slot);
   st->slot_bytes = ch->slot;
   // compact = 1; 2 forces the wide form for every record (NVBT_COMPACT_FORCE_WIDE=1, tests only)
-  st->compact = ch->slot == COMPACT_BYTES ? (ch->force_wide ? 2u : 1u) : 0u;
+  st->compact = ch->slot == COMPACT_STRIDE ? (ch->force_wide ? 2u : 1u) : 0u;
   st->no_wait = ch->on_device ? 1u : 0u;   // nobody frees device-ring slots: drop instead of waiting
   st->rheads = ch->on_device ? ch->ctx->ctl + CTL_RHEAD : nullptr;
   st->rstripes = ch->rstripes;
@@ -220,10 +225,10 @@ static void decode_wide_pair(const unsigned char* s0, const unsigned char* s1, u
 
 // Decodes slots [0, n) into records; a wide-first at the end must not occur (caller keeps pairs whole).
 // Parallel: count records per part, prefix, decode. Returns the record count.
-static uint64_t decode_batch(const unsigned char* sl, uint64_t n, unsigned char* out) {
+static uint64_t decode_batch(const unsigned char* sl, uint64_t n, unsigned char* out, unsigned ss) {
   Pool& pool = Pool::get();
   std::vector<uint64_t> cnt(pool.size() + 1, 0), lo_of(pool.size(), 0), hi_of(pool.size(), 0);
-  auto is_rec = [&](uint64_t i) { return slot_flags(sl + (size_t)i * COMPACT_BYTES) != 0x20u; };
+  auto is_rec = [&](uint64_t i) { return slot_flags(sl + (size_t)i * ss) != 0x20u; };
   pool.parallel_for(n, [&](unsigned id, uint64_t lo, uint64_t hi) {
     uint64_t c = 0;
     for (uint64_t i = lo; i < hi; ++i) c += is_rec(i);
@@ -235,11 +240,11 @@ static uint64_t decode_batch(const unsigned char* sl, uint64_t n, unsigned char*
   pool.parallel_for(n, [&](unsigned id, uint64_t lo, uint64_t hi) {
     uint64_t o = cnt[id];
     for (uint64_t i = lo; i < hi; ++i) {
-      const unsigned char* s0 = sl + (size_t)i * COMPACT_BYTES;
+      const unsigned char* s0 = sl + (size_t)i * ss;
       const unsigned f = slot_flags(s0);
       if (f == 0x20u) continue;
       unsigned char* r = out + (size_t)o * RECORD_BYTES;
-      if (f == 0x40u) decode_wide_pair(s0, s0 + COMPACT_BYTES, r);
+      if (f == 0x40u) decode_wide_pair(s0, s0 + ss, r);
       else decode_compact_slot(s0, r);
       ++o;
     }
@@ -248,17 +253,17 @@ static uint64_t decode_batch(const unsigned char* sl, uint64_t n, unsigned char*
 }
 
 // Digest of the records encoded in slots [0, n) without materialising them (built-in digest callback).
-static uint64_t digest_compact(const unsigned char* sl, uint64_t n, uint64_t* d1, uint64_t* d2) {
+static uint64_t digest_compact(const unsigned char* sl, uint64_t n, uint64_t* d1, uint64_t* d2, unsigned ss) {
   Pool& pool = Pool::get();
   std::vector<uint64_t> p1(pool.size(), 0), p2(pool.size(), 0), pc(pool.size(), 0);
   pool.parallel_for(n, [&](unsigned id, uint64_t lo, uint64_t hi) {
     alignas(16) unsigned char rec[RECORD_BYTES];
     uint64_t s1 = 0, s2 = 0, c = 0;
     for (uint64_t i = lo; i < hi; ++i) {
-      const unsigned char* s0 = sl + (size_t)i * COMPACT_BYTES;
+      const unsigned char* s0 = sl + (size_t)i * ss;
       const unsigned f = slot_flags(s0);
       if (f == 0x20u) continue;
-      if (f == 0x40u) decode_wide_pair(s0, s0 + COMPACT_BYTES, rec);
+      if (f == 0x40u) decode_wide_pair(s0, s0 + ss, rec);
       else decode_compact_slot(s0, rec);
       digest_serial(rec, 1, &s1, &s2);
       ++c;
@@ -283,7 +288,7 @@ int nvbt_drain_discard(const void* records, uint64_t n_records, void* user);
 extern "C" {
 
 size_t nvbt_channel_bytes(uint32_t record_bytes, uint64_t slots, int on_device) {
-  return HDR + slots * (record_bytes + (on_device ? 0u : 4u));
+  return HDR + slots * (slot_stride(record_bytes) + (on_device ? 0u : 4u));
 }
 
 int nvbt_channel_open(nvbt_ctx c, void* ring, size_t bytes, uint32_t record_bytes, nvbt_channel* out) {
@@ -293,7 +298,7 @@ int nvbt_channel_open(nvbt_ctx c, void* ring, size_t bytes, uint32_t record_byte
   if (record_bytes != RECORD_BYTES && record_bytes != COMPACT_BYTES)
     return set_error(NVBT_EINVAL, "record_bytes %u is neither 288 nor 176", record_bytes);
   if (reinterpret_cast<uintptr_t>(ring) % 64) return set_error(NVBT_EINVAL, "ring not 64-byte aligned");
-  if (bytes < HDR + 2 * (record_bytes + 4)) return set_error(NVBT_ENOMEM, "ring of %zu bytes holds < 2 slots", bytes);
+  if (bytes < HDR + 2 * (slot_stride(record_bytes) + 4)) return set_error(NVBT_ENOMEM, "ring of %zu bytes holds < 2 slots", bytes);
   NVBT_CUDA(cudaSetDevice(c->device));
   cudaPointerAttributes pa{};
   NVBT_CUDA(cudaPointerGetAttributes(&pa, ring));
@@ -309,11 +314,11 @@ int nvbt_channel_open(nvbt_ctx c, void* ring, size_t bytes, uint32_t record_byte
   ch->host = on_device ? nullptr : static_cast<unsigned char*>(ring);
   ch->dev = static_cast<unsigned char*>(on_device ? ring : pa.devicePointer);
   ch->slots = on_device ? nullptr : ch->host + HDR;
-  ch->slot = record_bytes;
+  ch->slot = slot_stride(record_bytes);
   { const char* e = getenv("NVBT_COMPACT_FORCE_WIDE"); ch->force_wide = e && atoi(e) != 0; }
   // host rings: each slot has a 4 B tag in the array after the slots; device rings carry the tag in-record
-  ch->cap = (bytes - HDR) / (record_bytes + (on_device ? 0u : 4u));
-  ch->tags = on_device ? nullptr : reinterpret_cast<const uint32_t*>(ch->host + HDR + ch->cap * record_bytes);
+  ch->cap = (bytes - HDR) / (ch->slot + (on_device ? 0u : 4u));
+  ch->tags = on_device ? nullptr : reinterpret_cast<const uint32_t*>(ch->host + HDR + ch->cap * ch->slot);
   if (on_device) {
     int sms = 148;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, c->device);
@@ -321,7 +326,7 @@ int nvbt_channel_open(nvbt_ctx c, void* ring, size_t bytes, uint32_t record_byte
   }
   cudaError_t e = cudaSuccess;
   if (on_device) e = cudaMemsetAsync(ring, 0, HDR + ch->cap * record_bytes, c->stream);
-  else std::memset(ch->host, 0, HDR + ch->cap * (record_bytes + 4));
+  else std::memset(ch->host, 0, HDR + ch->cap * (ch->slot + 4));
   if (on_device && e == cudaSuccess) {   // every stripe starts without a chunk; chunk counter 0
     std::vector<unsigned long long> w(ch->rstripes + 1, ((unsigned long long)kRingNoChunk << 32) | kRingChunk);
     w.back() = 0;
@@ -716,11 +721,11 @@ int nvbt_channel_drain(nvbt_channel ch, nvbt_drain_fn fn, void* user, int64_t ti
       if (fn == nvbt_drain_digest && user) {   // fused decode + digest, no staging of records
         auto* dg = static_cast<nvbt_digest*>(user);
         if (o) urc = fn(out, o, user);
-        const uint64_t k = digest_compact(base + first * sb, end - first, &dg->d1, &dg->d2);
+        const uint64_t k = digest_compact(base + first * sb, end - first, &dg->d1, &dg->d2, sb);
         dg->n_rec += k;
         o += k;
       } else {
-        o += decode_batch(base + first * sb, end - first, out + o * RECORD_BYTES);
+        o += decode_batch(base + first * sb, end - first, out + o * RECORD_BYTES, sb);
         urc = o ? fn(out, o, user) : 0;
       }
       ch->consumed += consume;

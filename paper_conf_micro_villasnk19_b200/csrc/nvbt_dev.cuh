@@ -50,7 +50,7 @@ struct DevState {
   unsigned n_warps;
   unsigned stripes;                // site/mem/hist repeat `stripes` times, stride stripe_words
   unsigned long long stripe_words;
-  unsigned slot_bytes;             // 288, or 176 for compact channels (EM §5.1)
+  unsigned slot_bytes;             // slot stride: 288, or 192 for compact channels (176 B slots, EM §5.1, padded)
   unsigned compact;
   unsigned no_wait;                // device-memory ring (F2): drop when full instead of waiting
   // device ring (F2): slots are handed out in chunks of kRingChunk. Each SM owns a stripe word

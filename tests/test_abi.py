@@ -124,12 +124,12 @@ def test_compact_decode_matches_records():
 
 
 def test_channel_bytes_layout():
-    """nvbt_channel_bytes follows include/nvbt.h: 64-byte header, then per slot the record plus a 4-byte
-    commit tag for pinned host rings; device rings (F2) carry no tag array."""
+    """nvbt_channel_bytes follows include/nvbt.h: 64-byte header, then per slot the record (compact: 176 B
+    padded to 192) plus a 4-byte commit tag for pinned host rings; device rings (F2) carry no tag array."""
     lib = C.CDLL(LIB)
     f = lib.nvbt_channel_bytes
     f.argtypes, f.restype = [C.c_uint32, C.c_uint64, C.c_int], C.c_size_t
     assert f(288, 5, 0) == 64 + 5 * 292
-    assert f(176, 7, 0) == 64 + 7 * 180
+    assert f(176, 7, 0) == 64 + 7 * (192 + 4)      # compact slots padded to a 192 B stride
     assert f(288, 1 << 22, 1) == 64 + 288 * (1 << 22)
     assert f(288, 0, 0) == 64

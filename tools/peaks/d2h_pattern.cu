@@ -31,6 +31,13 @@ int main() {
       {288, 384, 0, "288 B records in 384 B slots (3 lines each)"},
       {1152, 1152, 0, "1152 B blocks (4 x 288 B, 9 full lines)"},
       {176, 176, 64, "176 B compact slots at +64"},
+      {176, 176, 0, "176 B compact slots at +0"},
+      {176, 192, 0, "176 B compact records in 192 B slots at +0"},
+      {176, 192, 64, "176 B compact records in 192 B slots at +64"},
+      {176, 192, 128, "176 B compact records in 192 B slots at +128"},
+      {176, 256, 0, "176 B compact records in 256 B slots at +0"},
+      {128, 128, 0, "128 B records, 128 B stride (one line each)"},
+      {256, 256, 64, "256 B records, 256 B stride at +64"},
   };
   cudaEvent_t e0, e1;
   cudaEventCreate(&e0); cudaEventCreate(&e1);
