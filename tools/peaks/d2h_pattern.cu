@@ -37,6 +37,8 @@ int main() {
       {176, 192, 128, "176 B compact records in 192 B slots at +128"},
       {176, 256, 0, "176 B compact records in 256 B slots at +0"},
       {128, 128, 0, "128 B records, 128 B stride (one line each)"},
+      {288, 320, 0, "288 B records in 320 B slots at +0 (pairs of slots = 5 lines)"},
+      {288, 320, 64, "288 B records in 320 B slots at +64"},
       {256, 256, 64, "256 B records, 256 B stride at +64"},
   };
   cudaEvent_t e0, e1;
