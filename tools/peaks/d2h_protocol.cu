@@ -9,7 +9,7 @@
 #include <cstdio>
 #include <cuda_runtime.h>
 
-enum { PER_RECORD_TICKET = 1, COMMIT = 2, BLOCK_TAG = 4, TAG_ARRAY = 8, NO_FENCE = 16 };
+enum { PER_RECORD_TICKET = 1, COMMIT = 2, BLOCK_TAG = 4, TAG_ARRAY = 8, NO_FENCE = 16, DATA_AT_128 = 32 };
 
 __global__ void k_emit(unsigned char* ring, unsigned* tags, unsigned long long* head, unsigned long long n_warp_blocks, unsigned R,
                        unsigned mode) {
@@ -29,7 +29,7 @@ __global__ void k_emit(unsigned char* ring, unsigned* tags, unsigned long long* 
         if (lane == 0) t = atomicAdd(head, 1ull);
         t = __shfl_sync(0xffffffffu, t, 0);
       }
-      unsigned char* rec = ring + 64 + t * 288;
+      unsigned char* rec = ring + ((mode & DATA_AT_128) ? 128 : 64) + t * 288;
       if (lane == r) tagp = (mode & TAG_ARRAY) ? reinterpret_cast<unsigned char*>(tags + t) : rec + 28;
       if (lane < 18) *reinterpret_cast<uint4*>(rec + 16 * lane) = make_uint4((unsigned)t, r, lane, 0u);
     }
@@ -66,6 +66,8 @@ int main() {
       {6, PER_RECORD_TICKET | COMMIT | TAG_ARRAY, "ticket per record, fence + 4 B tag per record in a dense tag array"},
       {6, PER_RECORD_TICKET | COMMIT | TAG_ARRAY | NO_FENCE, "ticket per record, 4 B tag per record in a dense tag array, no fence"},
       {6, COMMIT | TAG_ARRAY, "6 tickets per warp, fence + 6 tags (24 B) in a dense tag array"},
+      {4, COMMIT | TAG_ARRAY | DATA_AT_128, "4 tickets per warp, data at +128, fence + 4 tags in a dense tag array"},
+      {4, DATA_AT_128, "4 tickets per warp, data at +128, no commit"},
   };
   cudaEvent_t e0, e1;
   cudaEventCreate(&e0); cudaEventCreate(&e1);
