@@ -305,7 +305,23 @@ int nvbt_stencil(nvbt_ctx ctx, void* stream, uint32_t tools, const float* in, fl
   if (lc.n_ctas == 0) return NVBT_OK;
   const dim3 block(32, 8);
   rc = dispatch_trace(tools, lc.st.no_wait != 0u, [&](auto tag) {
-    k_stencil<decltype(tag)::value><<<lc.grid, block, 0, lc.stream>>>(in, out, n, lc.st);
+    constexpr uint32_t T = decltype(tag)::value;
+    size_t dyn = 0;
+    if constexpr ((T & TOOL_TRACE) && !(T & TOOL_TRACE_DEV)) {
+      // Host-channel producer: at most 3 CTAs (24 warps) per SM, enforced by padding dynamic shared memory
+      // (4 CTAs would need more than the SM has). The PCIe link is saturated; fewer warps fencing and
+      // writing partial lines at once move more records (C4: 147 -> 151 M records/s, compact 205 -> 214;
+      // 6 CTAs per SM: 134 / 182).
+      static const size_t pad = [&] {
+        int per_sm = 0;
+        cudaDeviceGetAttribute(&per_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, ctx->device);
+        const size_t p = (size_t)per_sm * 2 / 7 - 8192;
+        cudaFuncSetAttribute(k_stencil<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p);
+        return p;
+      }();
+      dyn = pad;
+    }
+    k_stencil<T><<<lc.grid, block, dyn, lc.stream>>>(in, out, n, lc.st);
   });
   return rc ? rc : done(ctx, 1);
 }
