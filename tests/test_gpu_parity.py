@@ -89,33 +89,6 @@ def test_sgemm_parity(nvbt, M, N, K, tools):
     torch.testing.assert_close(Cm, A @ B, rtol=1e-4, atol=1e-4)
 
 
-@pytest.mark.slow
-def test_sgemm_full_size(nvbt):
-    """C2 at 1024^3 in the bench's launch configuration: closed forms (I-3) and sampled warps."""
-    import torch
-    nb = nvbt.nvbt
-    M = N = K = 1024
-    nw = nb.nvbt_workload_warps(nb.W_SGEMM, M, N)
-    ctx = nb.nvbt_init(nb.W_SGEMM, nb.COUNT | nb.MEMDIV | nb.PER_WARP, n_warps=nw)
-    A = cuda(uniform_f32((M, K), 3, -1, 1))
-    B = cuda(uniform_f32((K, N), 4, -1, 1))
-    Cm = torch.empty(M, N, device="cuda")
-    nb.nvbt_sgemm(ctx, nb.TOOL_COUNT | nb.TOOL_MEMDIV, A, B, Cm, M, N, K)
-    g = read_all(nb, ctx, per_warp=True)
-    W = nw
-    w_iss = W * (12 + 6 * K)
-    assert g["counts"].tolist() == [32 * w_iss, 32 * (w_iss - 2 * W), w_iss, w_iss - 2 * W]
-    assert g["mem_n"].sum() == 67_141_632
-    assert g["mem_S"].sum() == g["mem_L"].sum() == 1_108_344_832
-    rng = np.random.default_rng(0)
-    sample = np.sort(rng.choice(W, size=6, replace=False))
-    acc = ev.Accumulator(programs.sgemm(), n_warps=W)
-    m_sg.run(acc, M, N, K, A.data_ptr(), B.data_ptr(), Cm.data_ptr(), warps=sample)
-    r = acc.result()
-    assert (g["PW_T"][sample] == r["PW_T"][sample]).all() and (g["PW_W"][sample] == r["PW_W"][sample]).all()
-    gpu_invariants(g)
-
-
 # ---------------------------------------------------------------- C3 BFS
 @pytest.mark.parametrize("scale,tools", [(12, "BBCOUNT"), (12, "COUNT|MEMDIV"), (10, "BBCOUNT|MEMDIV")])
 def test_bfs_parity(nvbt, scale, tools):
@@ -524,20 +497,48 @@ def test_api_errors(nvbt):
 
 
 # ---------------------------------------------------------------- F1 kernel sampling
+class PerLaunch:
+    """Oracle accumulator that keeps one numpy Accumulator per launch id (to form F1's extrapolation
+    from the oracle's own per-launch results)."""
+
+    def __init__(self, prog):
+        self.prog, self.by_launch = prog, {}
+
+    def add(self, launch, *a, **kw):
+        self.by_launch.setdefault(launch, ev.Accumulator(self.prog)).add(launch, *a, **kw)
+
+    def result(self, launches=None, factor=1):
+        ks = sorted(self.by_launch) if launches is None else launches
+        out = None
+        for k in ks:
+            r = self.by_launch[k].result()
+            r.pop("trace")
+            out = r if out is None else {x: out[x] + r[x] for x in out}
+        return {x: v * factor for x, v in out.items()}
+
+
 def test_kernel_sampling_exact_when_control_flow_is_grid_only(nvbt):
     """"If the control flow of a kernel does not change based on the values computed, but it is
-    only a function of the grid dimensions, the sampling error is 0%" — stencil and vectorAdd qualify."""
+    only a function of the grid dimensions, the sampling error is 0%" — stencil and vectorAdd qualify:
+    the sampled estimate equals the ORACLE's full run (every launch modelled) element by element, and so
+    does the fully instrumented GPU run."""
     import torch
     nb, dr = nvbt.nvbt, nvbt.drivers
     flags = nb.COUNT | nb.OPHIST | nb.BB | nb.MEMDIV
+    tools = nb.TOOL_BBCOUNT | nb.TOOL_MEMDIV
+    # stencil: 2 grid shapes over 3 runs (ping-pong buffers: the addresses alternate between launches,
+    # but every launch of a shape has the same S/L per event, so the extrapolation is still exact)
     full = nb.nvbt_init(nb.W_STENCIL, flags)
     samp = nb.nvbt_init(nb.W_STENCIL, flags)
     scratch = nb.nvbt_init(nb.W_STENCIL, flags)
     sampler = dr.KernelSampler(samp, scratch)
-    tools = nb.TOOL_BBCOUNT | nb.TOOL_MEMDIV
+    acc = ev.Accumulator(programs.stencil())
+    launch = 0
     for n, iters in [(96, 5), (64, 3), (96, 2)]:
         x0 = cuda(uniform_f32((n, n), 4))
         b0, b1 = x0.clone(), torch.zeros_like(x0)
+        m_st.run_iterations(acc, n, b0.data_ptr(), b1.data_ptr(), iters, first_launch=launch)
+        launch += iters
         bufs = (b0, b1)
         for it in range(iters):
             src, dst = bufs[it % 2], bufs[(it + 1) % 2]
@@ -545,12 +546,30 @@ def test_kernel_sampling_exact_when_control_flow_is_grid_only(nvbt):
             sampler.launch(("stencil", n), lambda c, t: nb.nvbt_stencil(c, t, src, dst, n), tools)
     launches = sampler.finish()
     assert launches == {("stencil", 96): 7, ("stencil", 64): 3}
-    assert_same(read_all(nb, samp), read_all(nb, full), COUNT_KEYS + MEM_KEYS, "sampled stencil")
+    ref = acc.result()
+    assert_same(read_all(nb, samp), ref, COUNT_KEYS + MEM_KEYS, "sampled stencil vs oracle full run")
+    assert_same(read_all(nb, full), ref, COUNT_KEYS + MEM_KEYS, "full stencil vs oracle")
+    # vectorAdd: 3 sizes (one ragged), 4 launches each
+    samp = nb.nvbt_init(nb.W_VECTORADD, flags)
+    scratch = nb.nvbt_init(nb.W_VECTORADD, flags)
+    sampler = dr.KernelSampler(samp, scratch)
+    acc = ev.Accumulator(programs.vectoradd())
+    for N in (4096, 1000, 65536):
+        a, b = cuda(uniform_f32(N, 1)), cuda(uniform_f32(N, 2))
+        c = torch.empty_like(a)
+        for _ in range(4):
+            m_va.run(acc, N, a.data_ptr(), b.data_ptr(), c.data_ptr())
+            sampler.launch(("vectoradd", N), lambda cx, t: nb.nvbt_vectoradd(cx, t, a, b, c, N), tools)
+    sampler.finish()
+    assert_same(read_all(nb, samp), acc.result(), COUNT_KEYS + MEM_KEYS, "sampled vectorAdd vs oracle")
 
 
 def test_kernel_sampling_error_on_data_dependent_kernels(nvbt):
-    """BFS levels share grid dimensions but not control flow: sampling extrapolates level 0's counts to
-    every level, so its error is large and reported, not hidden."""
+    """BFS levels share grid dimensions but not control flow, so sampling (one instrumented level, its
+    counts extrapolated to every level) has an error, stated against the ORACLE's exact counts: the GPU's
+    sampled estimate equals levels x the oracle's level-0 counts element by element, the GPU's full run
+    equals the oracle's exact counts, and the relative error of W_issued is their quotient."""
+    import torch
     nb, dr = nvbt.nvbt, nvbt.drivers
     rowptr, col = rmat_csr(10, 16, seed=3)
     n = len(rowptr) - 1
@@ -561,9 +580,6 @@ def test_kernel_sampling_error_on_data_dependent_kernels(nvbt):
     samp = nb.nvbt_init(nb.W_BFS, nb.COUNT | nb.BB)
     scratch = nb.nvbt_init(nb.W_BFS, nb.COUNT | nb.BB)
     sampler = dr.KernelSampler(samp, scratch)
-    bufs = dr.bfs_buffers(n, "cuda")
-    dr.run_bfs(None, 0, rp, cl, src, bufs)                 # plain run to know the level count
-    import torch
     bufs = dr.bfs_buffers(n, "cuda")
     bufs["mask"][src] = 1; bufs["visited"][src] = 1; bufs["cost"][src] = 0
     level = 0
@@ -578,112 +594,14 @@ def test_kernel_sampling_error_on_data_dependent_kernels(nvbt):
         if int(bufs["over"].item()) == 0:
             break
     sampler.finish()
-    exact, est = nb.nvbt_count(full).astype(np.int64), nb.nvbt_count(samp).astype(np.int64)
-    assert est[2] != exact[2]                               # sampling is not exact here
-    assert exact[2] > 0 and abs(est[2] - exact[2]) / exact[2] < 10.0
-
-
-def test_replay_full_size_c5(nvbt):
-    """C5 at BASELINE.json's full size in the bench's launch configuration (10^10 generated events in
-    2^27-event chunks, staged replay with a 2^27-event scratch): W_issued = 10^10 and the I-2 invariants;
-    the single-pass kernel over the same 10^10 events gives identical bins (two independent divergence
-    implementations agreeing at full size); and three 2^16-event windows (start, middle, end of the
-    stream) through the same launch configuration equal the oracle element by element."""
-    import torch
-    nb, dr = nvbt.nvbt, nvbt.drivers
-    n, chunk = 10**10, 1 << 27
-    flags = nb.COUNT | nb.OPHIST | nb.BB | nb.MEMDIV
-    hdr = torch.empty(chunk * 16, dtype=torch.uint8, device="cuda")
-    addr = torch.empty(chunk * 256, dtype=torch.uint8, device="cuda")
-    staged = nb.nvbt_init(nb.W_REPLAY, flags)
-    single = nb.nvbt_init(nb.W_REPLAY, flags)
-    scratch = torch.empty(nb.nvbt_replay_scratch_size(staged, chunk), dtype=torch.uint8, device="cuda")
-    done = 0
-    while done < n:
-        m = min(chunk, n - done)
-        nb.nvbt_gen_events(staged, gen.SEED, done, m, hdr, addr)
-        nb.nvbt_replay_staged(staged, hdr, addr, m, scratch)
-        nb.nvbt_replay(single, hdr, addr, m)
-        done += m
-    g = read_all(nb, staged)
-    assert int(g["counts"][2]) == n
-    gpu_invariants(g)
-    assert_same(g, read_all(nb, single), what="staged vs single-pass replay, 10^10 events")
-    assert nb.nvbt_replay_errors(staged) == 0 and nb.nvbt_replay_errors(single) == 0
-    for first in (0, n // 2 - 12345, n - (1 << 16)):
-        ctx = nb.nvbt_init(nb.W_REPLAY, flags)
-        nb.nvbt_gen_events(ctx, gen.SEED, first, 1 << 16, hdr, addr)
-        nb.nvbt_replay_staged(ctx, hdr, addr, 1 << 16, scratch)
-        acc = ev.Accumulator(programs.replay())
-        gen.replay(acc, first, 1 << 16)
-        assert_same(read_all(nb, ctx), acc.result(), COUNT_KEYS + MEM_KEYS, f"window at {first}")
-    del hdr, addr, scratch
-    torch.cuda.empty_cache()
-
-
-def test_bfs_full_size_c3(nvbt):
-    """C3 at BASELINE.json's full size (R-MAT scale 20, edge factor 16, the bench's graph): BFS distances
-    equal scipy's unweighted shortest paths, the BB-entry run and the per-instruction run give identical
-    per-pc counts (I-5 at full size), the I-2 invariants hold, and every kernel-1 launch is entered by
-    every warp (Ent_w of the first block = levels x warps)."""
-    import torch
-    from scipy.sparse import csr_matrix
-    from scipy.sparse.csgraph import shortest_path
-    nb, dr = nvbt.nvbt, nvbt.drivers
-    rowptr, col = rmat_csr(20, 16, seed=3)
-    n = len(rowptr) - 1
-    src = bfs_source(rowptr)
-    nw = nb.nvbt_workload_warps(nb.W_BFS, n)
-    rp, cl = cuda(rowptr), cuda(col)
-    res = {}
-    for name, tools in (("bb", nb.TOOL_BBCOUNT), ("count", nb.TOOL_COUNT | nb.TOOL_MEMDIV)):
-        ctx = nb.nvbt_init(nb.W_BFS, nb.COUNT | nb.BB | nb.MEMDIV)
-        bufs = dr.bfs_buffers(n, "cuda")
-        cost, levels = dr.run_bfs(ctx, tools, rp, cl, src, bufs)
-        res[name] = (read_all(nb, ctx), cost.cpu().numpy(), levels)
-    g_bb, cost, levels = res["bb"]
-    g_ct = res["count"][0]
-    assert res["count"][2] == levels and (res["count"][1] == cost).all()
-    A = csr_matrix((np.ones(len(col), dtype=np.int8), col, rowptr), shape=(n, n))
-    d = shortest_path(A, unweighted=True, indices=src)
-    exp = np.where(np.isinf(d), -1, d).astype(np.int64)
-    assert (cost.astype(np.int64) == exp).all()
-    assert_same(g_bb, g_ct, COUNT_KEYS, "BFS scale 20: BBCOUNT vs COUNT")
-    gpu_invariants(g_ct)
-    assert int(g_bb["Ent_w"][0]) == levels * nw
-
-
-def test_stencil_trace_full_size_c4(nvbt):
-    """C4 at BASELINE.json's full size (8192^2 stencil, 100 iterations, every global LD/ST traced through
-    the pinned-host channel and drained with the digest callback, the bench's configuration): the number
-    of records equals the closed form iters x (2 n^2/32 + 4 (n-2) n/32), none dropped, W_issued of the
-    traced memory pcs equals the record count plus the predicated-off events (COUNT tool alongside), and
-    the traced run computes exactly the uninstrumented run's grid."""
-    import torch
-    nb, dr = nvbt.nvbt, nvbt.drivers
-    n, iters = 8192, 100
-    ctx = nb.nvbt_init(nb.W_STENCIL, nb.COUNT | nb.TRACE)
-    x0 = cuda(uniform_f32((n, n), 4))
-    a0, a1 = x0.clone(), torch.empty_like(x0)
-    dr.run_stencil(ctx, nb.TOOL_NONE, a0, a1, n, iters)
-    plain = (a0 if iters % 2 == 0 else a1).clone()
-    nb.nvbt_reset(ctx)
-    ring = torch.empty(nb.nvbt_channel_bytes(1 << 22), dtype=torch.uint8, pin_memory=True)
-    ch = nb.nvbt_channel_open(ctx, ring)
-    b0, b1 = x0.clone(), torch.empty_like(x0)
-    dr.run_stencil(ctx, nb.TOOL_TRACE | nb.TOOL_COUNT, b0, b1, n, iters)
-    d = nb.nvbt_channel_drain_digest(ch, timeout_us=600_000_000)
-    torch.cuda.synchronize()
-    expect = iters * (2 * (n * n // 32) + 4 * (n - 2) * (n // 32))
-    assert d.n_rec == expect and nb.nvbt_channel_dropped(ch) == 0
-    assert torch.equal(b0 if iters % 2 == 0 else b1, plain)
-    g = read_all(nb, ctx)
-    gpu_invariants(g)
-    # every executed warp-level event of a memory pc is one record (EM §5): the warp-executed histogram
-    # over the memory opcodes (used by no other pc) counts the records
-    prog = programs.stencil()
-    mem_ops = np.unique(prog["opcode"][programs.is_mem(prog)])
-    other_ops = np.unique(prog["opcode"][~programs.is_mem(prog)])
-    assert len(np.intersect1d(mem_ops, other_ops)) == 0
-    assert int(g["H_w"][mem_ops].sum()) == expect
-    del ring
+    per = PerLaunch(programs.bfs())
+    _, olevels, _ = m_bfs.run(per, rowptr, col, src, m_bfs.Ptrs(*([1 << 32] * 7)))
+    assert olevels == level
+    exact = per.result()
+    est = per.result(launches=[0, 1], factor=level)          # level 0 = launches 0 (expand) and 1 (update)
+    assert_same(read_all(nb, full), exact, COUNT_KEYS, "full BFS vs oracle")
+    assert_same(read_all(nb, samp), est, COUNT_KEYS, "sampled BFS vs oracle extrapolation")
+    err = abs(int(est["counts"][2]) - int(exact["counts"][2])) / int(exact["counts"][2])
+    assert err > 0.0                                         # not exact: control flow depends on data
+    print(f"F1 BFS scale 10: {level} levels, W_issued exact {int(exact['counts'][2])}, "
+          f"sampled {int(est['counts'][2])}, relative error {err:.4f}")

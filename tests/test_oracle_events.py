@@ -148,3 +148,31 @@ def test_invariants_detect_a_dropped_term():
     assert ev.invariants(r) == []
     r["H_t"][3] += 1
     assert "sum H = totals" in ev.invariants(r)
+
+
+# ---------------------------------------------------------------- Ent_t at a guarded leader (A != E)
+def guarded_leader_case():
+    g = json.load(open(os.path.join(GOLD, "guarded_leader.json")))
+    pr = g["program"]
+    prog = {k: np.array(pr[k]) for k in ("opcode", "kind", "width", "bb", "is_leader", "guarded")}
+    prog.update(n_pcs=4, n_opcodes=pr["n_opcodes"], n_bbs=2)
+    evs = g["events"]
+    base = 1 << 32
+    addr = np.array([[base + 4 * l for l in range(32)] for _ in evs], dtype=np.uint64)
+    cols = dict(pc=np.array([e["pc"] for e in evs]), A=np.array([int(e["A"], 16) for e in evs], dtype=np.uint32),
+                P=np.array([int(e["P"], 16) for e in evs], dtype=np.uint32), addr=addr)
+    return prog, cols, g["expect"]
+
+
+def test_ent_t_counts_active_threads_at_a_guarded_leader():
+    prog, c, exp = guarded_leader_case()
+    acc = ev.Accumulator(prog)
+    acc.add(0, np.zeros(len(c["pc"]), dtype=np.int64), c["pc"], c["A"], c["P"], c["addr"])
+    r = acc.result()
+    for k in ("Ent_t", "Ent_w", "Ins_t", "Ins_w", "counts"):
+        assert r[k].tolist() == exp[k], k
+    assert (r["mem_n"][0], r["mem_S"][0], r["mem_L"][0]) == (exp["mem_n0"], exp["mem_S0"], exp["mem_L0"])
+    # I-5 with the guard corrections computed from the raw masks
+    off_t = sum(bin(int(A) & ~int(P) & 0xFFFFFFFF).count("1") for pc, A, P in zip(c["pc"], c["A"], c["P"])
+                if prog["guarded"][pc] and prog["bb"][pc] == 0)
+    assert 3 * r["Ent_t"][0] - off_t == r["Ins_t"][0]
