@@ -116,57 +116,91 @@ def stencil_rows(n: int, rank: int, world: int):
     return min(8 * y0, n), min(8 * y1, n)
 
 
+def slab_neighbours(n: int, rank: int, world: int):
+    """Nearest ranks above and below `rank` whose row slabs are non-empty (None at the grid's edges). A
+    rank with an empty slab sits between them with r0 == r1, so the neighbour above ends exactly at my
+    first row and the one below starts right after my last row."""
+    up = next((q for q in range(rank - 1, -1, -1) if stencil_rows(n, q, world)[1] > stencil_rows(n, q, world)[0]), None)
+    down = next((q for q in range(rank + 1, world) if stencil_rows(n, q, world)[1] > stencil_rows(n, q, world)[0]), None)
+    return up, down
+
+
+def _backend(group):
+    import torch.distributed as dist
+    return dist.get_backend(group)
+
+
 def _exchange_halo(buf, n, rank, world, group):
-    """Every rank publishes its first and last own row; each then fills the row just above and just below
-    its slab from its neighbours. One int32 SUM all-reduce of a (world, 2, n) board (bit-exact: every slot
-    has one writer, the others add 0)."""
+    """1-row halos with the two slab neighbours ("1-row halos (32 KiB) via P2P send/recv"):
+    send my first row up and my last row down, receive the row above my slab and the row below it.
+    NCCL: one batched isend/irecv group, stream-ordered after the iteration's kernel (no host sync, so
+    the trace drain keeps running); other backends (gloo, CPU tests) stage the rows through the host."""
     import torch
     import torch.distributed as dist
     r0, r1 = stencil_rows(n, rank, world)
-    board = torch.zeros((world, 2, n), dtype=torch.int32, device=buf.device)
-    g = buf.view(torch.int32)
-    if r1 > r0:
-        board[rank, 0] = g[r0]
-        board[rank, 1] = g[r1 - 1]
-    dist.all_reduce(board, op=dist.ReduceOp.SUM, group=group)
     if r1 == r0:                     # an empty slab computes nothing and needs no halo
         return
-    # nearest rank above with rows ends at r0; nearest below starts at r1
-    for q in range(rank - 1, -1, -1):
-        a0, a1 = stencil_rows(n, q, world)
-        if a1 > a0:
-            if r0 > 0 and a1 == r0:
-                g[r0 - 1] = board[q, 1]
-            break
-    for q in range(rank + 1, world):
-        a0, a1 = stencil_rows(n, q, world)
-        if a1 > a0:
-            if r1 < n and a0 == r1:
-                g[r1] = board[q, 0]
-            break
+    up, down = slab_neighbours(n, rank, world)
+    g = buf.view(torch.int32)
+    nccl = _backend(group) == "nccl"
+    pairs = []                        # (peer, row to send, row to receive into)
+    if up is not None:
+        pairs.append((up, r0, r0 - 1))
+    if down is not None:
+        pairs.append((down, r1 - 1, r1))
+    if not pairs:
+        return
+    gr = (lambda q: q) if group is None else (lambda q: dist.get_global_rank(group, q))
+    if nccl:
+        ops = []
+        for peer, srow, rrow in pairs:
+            ops.append(dist.P2POp(dist.isend, g[srow], gr(peer), group))
+            ops.append(dist.P2POp(dist.irecv, g[rrow], gr(peer), group))
+        for w in dist.batch_isend_irecv(ops):
+            w.wait()
+        return
+    host = [(peer, g[srow].cpu(), torch.empty(n, dtype=torch.int32), rrow) for peer, srow, rrow in pairs]
+    ops = []
+    for peer, sbuf, rbuf, _ in host:
+        ops.append(dist.P2POp(dist.isend, sbuf, gr(peer), group))
+        ops.append(dist.P2POp(dist.irecv, rbuf, gr(peer), group))
+    for w in dist.batch_isend_irecv(ops):
+        w.wait()
+    for _, _, rbuf, rrow in host:
+        g[rrow].copy_(rbuf)
 
 
 def run_stencil_dist(ctx, tools, buf0, buf1, n, iters, rank, world, group=None, gather=True):
     """C4 over `world` ranks: ctx is partitioned, so each rank runs the CTA rows of its own
-    row slab; after every iteration the 1-row halos are exchanged (_exchange_halo). With `gather`, the full
-    final grid is assembled on every rank at the end (one int32 SUM all-reduce, rows outside a rank's slab
-    zeroed first). Trace records stay on each rank's own channel; their digests add. Returns the final
-    buffer."""
+    row slab; after every iteration the 1-row halos go to and come from the slab neighbours
+    (_exchange_halo). Under NCCL nothing here waits on the host, so a caller can enqueue all iterations
+    and drain the trace channel while they run. With `gather`, the full final grid is assembled on every
+    rank at the end (one int32 SUM all-reduce, rows outside a rank's slab zeroed first). Trace records stay
+    on each rank's own channel; their digests add. Returns the final buffer."""
     import torch
     import torch.distributed as dist
     bufs = (buf0, buf1)
-    for it in range(iters):
-        _nb().nvbt_stencil(ctx, tools, bufs[it % 2], bufs[(it + 1) % 2], n)
-        _sync(ctx)
-        _exchange_halo(bufs[(it + 1) % 2], n, rank, world, group)
-    out = bufs[iters % 2]
-    if gather:
-        r0, r1 = stencil_rows(n, rank, world)
-        g = out.view(torch.int32)
-        g[:r0] = 0
-        g[r1:] = 0
-        dist.all_reduce(g, op=dist.ReduceOp.SUM, group=group)
+    stream = getattr(ctx, "stream", None)
+    with torch.cuda.stream(stream) if stream is not None else _null():
+        for it in range(iters):
+            _nb().nvbt_stencil(ctx, tools, bufs[it % 2], bufs[(it + 1) % 2], n)
+            _exchange_halo(bufs[(it + 1) % 2], n, rank, world, group)
+        out = bufs[iters % 2]
+        if gather:
+            r0, r1 = stencil_rows(n, rank, world)
+            g = out.view(torch.int32)
+            g[:r0] = 0
+            g[r1:] = 0
+            dist.all_reduce(g, op=dist.ReduceOp.SUM, group=group)
     return out
+
+
+class _null:
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        return False
 
 
 def replay_range(ctx, seed, first, n, hdr, addr, chunk=None, scratch=None):

@@ -102,7 +102,8 @@ def _halo_worker(rank, world, port, n, out_q):
 @pytest.mark.parametrize("n,world", [(50, 3), (64, 2), (17, 4)])
 def test_gloo_stencil_halo_exchange(n, world):
     """C4 partition: after the exchange every rank holds the true row just above and just
-    below its slab (bit-exact: the int32 SUM board has one writer per slot); nothing else changes."""
+    below its slab (P2P send/recv with the nearest non-empty slabs, including across a rank whose slab is
+    empty: n = 17 has 3 CTA rows for 4 ranks); nothing else changes.""""
     from paper_conf_micro_villasnk19_b200 import drivers
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
