@@ -1,23 +1,33 @@
 #!/usr/bin/env python
-"""nvbt benchmark: instrumented warp-instruction events/s and slowdown vs the uninstrumented kernel.
+"""nvbt benchmark: instrumented warp-instruction events/s and slowdown vs the uninstrumented kernel
+(BASELINE.json metric), on all five BASELINE.json configs.
 
-Default workload (BASELINE.json configs[1]): C2 — naive row-fastest SGEMM 1024^3 with the full tool set
-compiled in (counts, opcode/BB histograms, per-instruction memory divergence), one step = one
-instrumented launch; with N > 1 each rank runs its own instance and the counters are merged once by an
-int64 all-reduce after the timed steps. Other workloads
-(`--workload c1|c3|c4|c5`) are for profiling; the driver's bench line is C2.
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--configs c1,c3,c4,c5]
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload c2] [--impl ours|reference]
+One JSON line. `value` is the headline config C2 (configs[1]: naive row-fastest SGEMM 1024^3 with the
+bench tool set BBCOUNT|MEMDIV: counts, opcode/BB histograms via basic-block-entry hooks, per-instruction
+memory divergence), one step = one instrumented launch; `configs` holds the other four configs measured in
+the same run (C1 vectorAdd, C3 BFS on R-MAT scale 20, C4 the 8192^2 x 100 stencil traced through the
+pinned-host channel, C5 the replay of 10^10 generated events), each with its value, slowdown, roofline
+fraction and a result check.
 
-Multi-GPU (weak scaling): torchrun, one rank per GPU, every rank runs its own instance; the time of
-the job is the max over ranks. Timing: CUDA events on the context's stream around each step, L2
-flushed (256 MiB write) between steps, clocks sampled with nvidia-smi during the timed region.
+Multi-GPU: one process per GPU. Without torchrun, `--gpus N` (N > 1) re-launches itself
+under torch.distributed.run. Work is partitioned, total work fixed ("strong"): C1/C2 by CTA rows of the
+same launch (nvbt_set_partition), C3 by vertex range with its per-level MAX exchanges, C4 by row slab with
+P2P halos and one channel per rank, C5 by event-index range; the per-GPU counters are merged by one int64
+SUM all-reduce (a8) and checked against the closed forms. Timing: CUDA events on the launching stream,
+max over ranks; L2 flushed (256 MiB write) between C2 steps; clocks sampled with nvidia-smi during the
+timed region.
+
+`--impl reference`: the reference arm of this tier is the CPU oracle: the multithreaded C
+oracle (oracle/c) on all host cores, one whole C2 launch per step.
 """
 from __future__ import annotations
 
 import argparse
 import json
 import os
+import socket
 import statistics
 import subprocess
 import sys
@@ -32,35 +42,53 @@ sys.path.insert(0, ROOT)
 PEAKS_FALLBACK = {"hbm_gbs": 6650.0, "sm_max_mhz": 1965.0}
 N_SM = 148
 METRIC = "instrumented warp-instr events/sec and slowdown vs uninstrumented"
+SEED = 0x4E5642544E564254
+
+
+def _profile_json(name):
+    try:
+        with open(os.path.join(ROOT, "profiles", name)) as f:
+            return json.load(f)
+    except Exception:
+        return None
 
 
 def load_traffic(kernel):
     """DRAM bytes per launch of `kernel` from the committed ncu capture (profiles/r1_traffic.json)."""
-    try:
-        with open(os.path.join(ROOT, "profiles", "r1_traffic.json")) as f:
-            return json.load(f).get(kernel)
-    except Exception:
-        return None
+    d = _profile_json("r1_traffic.json")
+    return None if d is None else d.get(kernel)
 
 
 def load_counters(kernel, keys=("warp_inst_per_unit", "dram_bytes_per_unit", "shared_atomic_wavefronts_per_unit",
                                  "global_atomic_sectors_per_unit", "issue_active_pct")):
     """ncu counters per unit of work of `kernel` from the committed capture (profiles/r1_ncu_counters.json)."""
-    try:
-        with open(os.path.join(ROOT, "profiles", "r1_ncu_counters.json")) as f:
-            d = json.load(f).get(kernel)
-    except Exception:
-        return None
+    d = (_profile_json("r1_ncu_counters.json") or {}).get(kernel)
     return None if d is None else {k: d[k] for k in keys if k in d}
 
 
 def load_peaks():
     try:
         with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
-            p = json.load(f)
-        return p, "measured"
+            return json.load(f), "measured (MEASURED_PEAKS.json)"
     except Exception:
-        return PEAKS_FALLBACK, "fallback"
+        return PEAKS_FALLBACK, "fallback (B200_PROFILING.md)"
+
+
+def d2h_peak():
+    """Measured SM-store bandwidth into pinned host memory (tools/peaks/peaks.cu, profiles/r1_box_peaks.json)."""
+    d = _profile_json("r1_box_peaks.json") or {}
+    return float(d.get("sm_store16_host_GBs_occ4", 52.7))
+
+
+def cpu_model():
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return "unknown"
 
 
 # --------------------------------------------------------------------------- clocks
@@ -110,6 +138,22 @@ class ClockSampler:
 
 
 # --------------------------------------------------------------------------- distributed
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def spawn_ranks(n):
+    """`--gpus N` without torchrun: re-launch this script under torch.distributed.run (one rank per GPU)."""
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
+           "--master-addr", "127.0.0.1", "--master-port", str(_free_port()), os.path.abspath(__file__),
+           *sys.argv[1:]]
+    return subprocess.call(cmd)
+
+
 def dist_setup(args):
     import torch
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -117,12 +161,13 @@ def dist_setup(args):
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if os.environ.get("NVBT_BENCH_SAME_GPU"):   # test hook: all ranks on GPU 0 (with a gloo backend)
         local = 0
-    if args.impl == "ours":
-        torch.cuda.set_device(local)
+    torch.cuda.set_device(local)
     if world > 1:
         import torch.distributed as dist
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
-        backend = os.environ.get("NVBT_BENCH_BACKEND", "nccl" if args.impl == "ours" else "gloo")
+        os.environ.setdefault("NCCL_DEBUG", "INFO")          # communicator init log (ranks, NVLS, channels)
+        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+        backend = os.environ.get("NVBT_BENCH_BACKEND", "nccl")
         kw = {"device_id": torch.device("cuda", local)} if backend == "nccl" else {}
         dist.init_process_group(backend, **kw)
     return rank, world, local
@@ -134,342 +179,61 @@ def barrier(world):
         dist.barrier()
 
 
-def max_over_ranks(x, world, device=None):
+def _reduce(x, world, op):
     if world == 1:
         return x
     import torch
     import torch.distributed as dist
-    t = torch.tensor([x], dtype=torch.float64, device=device)
-    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    dev = torch.device("cuda", torch.cuda.current_device()) if dist.get_backend() == "nccl" else "cpu"
+    t = torch.tensor([x], dtype=torch.float64, device=dev)
+    dist.all_reduce(t, op=op)
     return float(t.item())
+
+
+def max_over_ranks(x, world, device=None):
+    import torch.distributed as dist
+    return _reduce(x, world, dist.ReduceOp.MAX if world > 1 else None)
 
 
 def sum_over_ranks(x, world, device=None):
-    if world == 1:
-        return x
+    import torch.distributed as dist
+    return _reduce(x, world, dist.ReduceOp.SUM if world > 1 else None)
+
+
+def merge(dr, ctx, world):
+    """a8: one int64 SUM all-reduce of the packed accumulator region (after the timed region)."""
+    if world > 1:
+        dr.merge(ctx)
+
+
+def allreduce_latency(world):
+    """int64 SUM all-reduce latency of 8 KB / 64 KB / 1 MB messages (the merge's
+    sizes), median of 20 after 5 warm-ups, device-timed, max over ranks."""
     import torch
     import torch.distributed as dist
-    t = torch.tensor([x], dtype=torch.float64, device=device)
-    dist.all_reduce(t, op=dist.ReduceOp.SUM)
-    return float(t.item())
-
-
-# --------------------------------------------------------------------------- C2 SGEMM
-class SgemmBench:
-    name = "c2"
-    M = N = K = 1024
-    desc = "C2 naive row-fastest SGEMM 1024^3 (fp32), tools BBCOUNT|MEMDIV (counts, opcode+BB histograms via BB-entry hooks, divergence)"
-
-    def __init__(self, torch, nb, dr, world):
-        self.torch, self.nb, self.dr, self.world = torch, nb, dr, world
-        from synth import uniform_f32
-        M, N, K = self.M, self.N, self.K
-        self.nw = nb.nvbt_workload_warps(nb.W_SGEMM, M, N)
-        self.ctx = nb.nvbt_init(nb.W_SGEMM, nb.COUNT | nb.OPHIST | nb.BB | nb.MEMDIV)
-        self.tools = nb.TOOL_BBCOUNT | nb.TOOL_MEMDIV
-        self.hA = torch.from_numpy(uniform_f32((M, K), 3, -1, 1)).pin_memory()
-        self.hB = torch.from_numpy(uniform_f32((K, N), 4, -1, 1)).pin_memory()
-        self.A, self.B = self.hA.cuda(), self.hB.cuda()
-        self.C = torch.empty(M, N, device="cuda")
-        # events per launch (EM §3.2): every warp runs 12 + 6K warp-level instructions
-        self.events = self.nw * (12 + 6 * K)
-        self.kernels_per_step = 1
-
-    def plain(self):
-        self.nb.nvbt_sgemm(self.ctx, self.nb.TOOL_NONE, self.A, self.B, self.C, self.M, self.N, self.K)
-
-    def instr(self):
-        self.nb.nvbt_sgemm(self.ctx, self.tools, self.A, self.B, self.C, self.M, self.N, self.K)
-
-    def e2e_step(self, out_host):
-        """Through the public API with host buffers: H2D inputs, instrumented launch, read results."""
-        nb = self.nb
-        self.A.copy_(self.hA, non_blocking=True)
-        self.B.copy_(self.hB, non_blocking=True)
-        nb.nvbt_sgemm(self.ctx, self.tools, self.A, self.B, self.C, self.M, self.N, self.K)
-        out_host["counts"] = nb.nvbt_count(self.ctx)
-        out_host["memdiv"] = nb.nvbt_mem_divergence(self.ctx)
-        out_host["ophist"] = nb.nvbt_opcode_hist(self.ctx)
-        return self.hA.numel() * 4 + self.hB.numel() * 4, 8 * (4 + 3 * 18 + 3 + 66 + 2 * 16)
-
-    def roofline(self, t_kernel_s, peaks):
-        """Issue roofline ("alu"): algorithmic warp-instructions per launch ÷ launch time vs
-        148 SMs x 4 schedulers x 1 warp-instr/clk at the max SM clock."""
-        K, W = self.K, self.nw
-        # app instructions (one per warp-level event) + BB-entry hooks at the 3 + K leaders + guard
-        # hooks at pc7 and K x pc15 + divergence hooks at the 2K + 1 global LD/ST events
-        per_warp = (12 + 6 * K) + (K + 3) * HOOK_OPS["count"] + (K + 1) * HOOK_OPS["guard"] + \
-            (2 * K + 1) * HOOK_OPS["mem"]
-        ops = W * per_warp
-        peak = N_SM * 4 * peaks.get("sm_max_mhz", 1965.0) * 1e6
-        ach = ops / t_kernel_s
-        t = load_traffic("k_sgemm<6>")
-        return {"bound": "alu", "achieved": ach / 1e9, "peak": peak / 1e9, "unit": "Gwarp-inst/s",
-                "frac": ach / peak, "traffic": t["traffic_bytes_per_launch"] if t else None,
-                "traffic_unit": "DRAM bytes per launch (ncu, profiles/r1_traffic.json)",
-                "algorithmic_warp_inst_per_launch": ops}
-
-    def oracle_sample(self, budget_s):
-        """The oracle on a bounded sample of the same workload: whole warps, full K."""
-        from oracle import events as ev, programs
-        from oracle.models import sgemm as m_sg
-        acc = ev.Accumulator(programs.sgemm())
-        rng = np.random.default_rng(1)
-        warps = np.sort(rng.choice(self.nw, size=64, replace=False))
-        t0 = time.perf_counter()
-        done = 0
-        while True:
-            m_sg.run(acc, self.M, self.N, self.K, self.A.data_ptr(), self.B.data_ptr(), self.C.data_ptr(),
-                     warps=warps)
-            done += len(warps) * (12 + 6 * self.K)
-            if time.perf_counter() - t0 > budget_s:
-                break
-        dt = time.perf_counter() - t0
-        return done / dt, f"{done} warp events: SGEMM 1024^3 oracle model on 64 sampled warps x full K"
-
-
-# hook instruction costs per event used for the issue roofline (DESIGN.md §5, minimal SASS per hook)
-HOOK_OPS = {"count": 4, "guard": 6, "mem": 23}
-
-
-# --------------------------------------------------------------------------- C5 replay
-class ReplayBench:
-    name = "c5"
-    desc = "C5 trace replay of 10^10 generated events (counts, histograms, divergence), 2^27-event chunks"
-
-    def __init__(self, torch, nb, dr, world, rank, n_total=10**10, chunk=1 << 27, staged=True):
-        self.torch, self.nb, self.dr = torch, nb, dr
-        self.lo, self.hi = dr.shard_range(n_total, rank, world)
-        self.n = self.hi - self.lo
-        self.chunk = chunk
-        self.ctx = nb.nvbt_init(nb.W_REPLAY, nb.COUNT | nb.OPHIST | nb.BB | nb.MEMDIV)
-        self.hdr = torch.empty(chunk * 16, dtype=torch.uint8, device="cuda")
-        self.addr = torch.empty(chunk * 256, dtype=torch.uint8, device="cuda")
-        # staged replay (two passes): the executed-memory-event list of one chunk (12 B per entry)
-        self.scratch = torch.empty(nb.nvbt_replay_scratch_size(self.ctx, chunk), dtype=torch.uint8,
-                                   device="cuda") if staged else None
-        self.events = self.n
-        self.kernels_per_step = -(-self.n // chunk)
-
-    def oracle_sample(self, budget_s):
-        """The oracle (generator + per-event definitions) on a bounded sample of the same event stream:
-        consecutive 2^16-event chunks from the rank's first event until the budget is spent."""
-        from oracle import events as ev, gen, programs
-        acc = ev.Accumulator(programs.replay())
-        t0 = time.perf_counter()
-        done = 0
-        while time.perf_counter() - t0 < budget_s:
-            gen.replay(acc, self.lo + done, 1 << 16)
-            done += 1 << 16
-        dt = time.perf_counter() - t0
-        return done / dt, f"{done} generated events from event {self.lo} (oracle replay incl. generation, 1 core)"
-
-    def replay(self, m):
-        if self.scratch is None:
-            self.nb.nvbt_replay(self.ctx, self.hdr, self.addr, m)
-        else:
-            self.nb.nvbt_replay_staged(self.ctx, self.hdr, self.addr, m, self.scratch)
-
-    def run(self, stream_events):
-        """One step: generate (untimed) and replay (timed with events) every chunk."""
-        torch, nb = self.torch, self.nb
-        t = 0.0
-        off = 0
-        while off < self.n:
-            m = min(self.chunk, self.n - off)
-            nb.nvbt_gen_events(self.ctx, 0x4E5642544E564254, self.lo + off, m, self.hdr, self.addr)
-            e0, e1 = stream_events
-            e0.record()
-            self.replay(m)
-            e1.record()
-            e1.synchronize()
-            t += e0.elapsed_time(e1) / 1e3
-            off += m
-        return t
-
-
-# --------------------------------------------------------------------------- main
-def run_ours(args):
-    import torch
-    rank, world, local = dist_setup(args)
-    import paper_conf_micro_villasnk19_b200 as pkg
-    nb, dr = pkg.nvbt, pkg.drivers
-    peaks, peaks_src = load_peaks()
-    dev = torch.device("cuda", local)
-    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
-
-    if args.workload == "c5":
-        return run_replay(args, torch, nb, dr, rank, world, local, peaks, peaks_src)
-    if args.workload in ("c1", "c3", "c4", "f1", "f2", "f4"):
-        line = {"c1": run_c1, "c3": run_c3, "c4": run_c4, "f1": run_f1, "f2": run_f2, "f4": run_f4}[args.workload](
-            args, torch, nb, dr, local)
-        if rank == 0:
-            print(json.dumps(line), flush=True)
-        return
-
-    wl = SgemmBench(torch, nb, dr, world)
-    launches0 = nb.nvbt_launch_count(wl.ctx)
-
-    def timed(fn, n):
+    out = {}
+    for nbytes in (8 << 10, 64 << 10, 1 << 20):
+        t = torch.zeros(nbytes // 8, dtype=torch.int64, device="cuda")
+        for _ in range(5):
+            dist.all_reduce(t)
         ts = []
-        for _ in range(n):
-            flush.zero_()
+        for _ in range(20):
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record()
-            fn()
+            dist.all_reduce(t)
             e1.record()
             e1.synchronize()
-            ts.append(e0.elapsed_time(e1) / 1e3)
-        return ts
-
-    # warm-up (untimed), plain baseline
-    timed(wl.instr, args.warmup)
-    timed(wl.plain, max(args.warmup, 3))
-    t_plain = timed(wl.plain, args.steps)
-    nb.nvbt_reset(wl.ctx)
-    barrier(world)
-    torch.cuda.synchronize()
-    l0 = nb.nvbt_launch_count(wl.ctx)
-    with ClockSampler(local) as clk:
-        barrier(world)
-        torch.cuda.synchronize()
-        t_instr = timed(wl.instr, args.steps)
-        torch.cuda.synchronize()
-        barrier(world)
-    gpu_launches = nb.nvbt_launch_count(wl.ctx) - l0
-    # a8 merge: the per-GPU accumulators are summed once, by one int64 all-reduce (EM §4)
-    merge_ms = 0.0
-    if world > 1:
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record()
-        dr.merge(wl.ctx)
-        e1.record()
-        e1.synchronize()
-        merge_ms = e0.elapsed_time(e1)
-    # result check of the timed steps: exactly K x the per-launch closed form (I-3)
-    cnt = nb.nvbt_count(wl.ctx)
-    expect = wl.events * args.steps * (world if world > 1 else 1)
-    ok = int(cnt[2]) == expect
-    tot_instr = max_over_ranks(sum(t_instr), world, dev)
-    tot_plain = max_over_ranks(sum(t_plain), world, dev)
-    events_all = wl.events * args.steps * world
-    value = events_all / tot_instr
-    slowdown = tot_instr / tot_plain
-    t_kernel = statistics.median(t_instr)
-    # e2e through the public API with host buffers
-    out = {}
-    for _ in range(2):
-        wl.e2e_step(out)
-    torch.cuda.synchronize()
-    t0 = time.perf_counter()
-    e2e_steps = max(3, min(args.steps, 10))
-    for _ in range(e2e_steps):
-        h2d, d2h = wl.e2e_step(out)
-    torch.cuda.synchronize()
-    e2e_t = max_over_ranks(time.perf_counter() - t0, world, dev)
-    e2e_value = wl.events * e2e_steps * world / e2e_t
-    line = {
-        "metric": METRIC, "value": value, "unit": "events/s", "n_gpus": world, "steps": args.steps,
-        "warmup": args.warmup, "ms_per_step": 1e3 * tot_instr / args.steps, "higher_is_better": True,
-        "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-        "config": {"workload": wl.desc, "M": wl.M, "N": wl.N, "K": wl.K, "warp_events_per_launch": wl.events,
-                   "tools": "BBCOUNT|MEMDIV", "l2": "flushed between steps (256 MiB write)",
-                   "parallelism": f"replicas x{world}, one int64 all-reduce merge of the counters" if world > 1 else "1 GPU"},
-        "slowdown": slowdown, "plain_ms_per_launch": 1e3 * statistics.median(t_plain),
-        "instr_ms_per_launch": 1e3 * t_kernel, "counts_check": "ok" if ok else f"mismatch {int(cnt[2])} != {expect}",
-        "roofline": wl.roofline(t_kernel, peaks),
-        "e2e": {"value": e2e_value, "unit": "events/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h},
-        "gpu_launches": int(gpu_launches), "clocks": clk.summary(), "peaks_source": peaks_src,
-        "merge_ms": merge_ms,
-    }
-    line["roofline"]["peak_source"] = f"148 SMs x 4 issue/clk x sm_max_mhz ({peaks_src})"
-    # the binding resource of this workload is the application's own L1 traffic (the naive row-fastest
-    # SGEMM is L1-wavefront-bound uninstrumented); the hooks run inside that bound
-    line["app_bound"] = {"resource": "L1TEX wavefronts of the uninstrumented SGEMM",
-                         "instr_speed_vs_plain": statistics.median(t_plain) / t_kernel,
-                         "ncu": "profiles/r1_ncu_summary_c2_c5.txt: l1tex 98.8 % (plain) / 95.2 % (instrumented), "
-                                "issue-active 6.9 % / 85.2 %"}
-    # ncu evidence per warp event (the north_star's instructions per event and atomic traffic)
-    line["ncu_per_event"] = {"instrumented": load_counters("k_sgemm<6>"), "plain": load_counters("k_sgemm<0>"),
-                             "source": "profiles/r1_ncu_counters.json (ncu --set full, tools/prof_step.py c2)"}
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        rate, sample = wl.oracle_sample(args.cpu_budget)
-        line["cpu_baseline"] = {"value": rate, "unit": "events/s", "cores": 1, "kind": "oracle", "sample": sample}
-    if rank == 0:
-        print(json.dumps(line), flush=True)
-    if world > 1:
-        import torch.distributed as dist
-        dist.destroy_process_group()
+            ts.append(e0.elapsed_time(e1) * 1e3)
+        out[f"{nbytes >> 10}KiB_us"] = max_over_ranks(statistics.median(ts), world)
+    return out
 
 
-def _replay_traffic(chunk, staged):
-    """ncu DRAM bytes of one replay call on `chunk` events (captured at 2^26 events, scaled linearly)."""
-    names = ("k_rpA<0>", "k_rpB") if staged else ("k_replay4",)
-    tr = [load_traffic(k) for k in names]
-    if any(t is None for t in tr):
-        return None
-    return sum(t["traffic_bytes_per_launch"] for t in tr) / 67108864 * chunk
-
-
-def run_replay(args, torch, nb, dr, rank, world, local, peaks, peaks_src):
-    dev = torch.device("cuda", local)
-    wl = ReplayBench(torch, nb, dr, world, rank, n_total=args.replay_events, staged=args.replay_impl == "staged")
-    evs = (torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
-    # warm-up on one chunk
-    for _ in range(args.warmup):
-        nb.nvbt_gen_events(wl.ctx, 0x4E5642544E564254, 0, min(wl.chunk, wl.n), wl.hdr, wl.addr)
-        wl.replay(min(wl.chunk, wl.n))
-    nb.nvbt_reset(wl.ctx)
-    torch.cuda.synchronize()
-    barrier(world)
-    l0 = nb.nvbt_launch_count(wl.ctx)
-    with ClockSampler(local) as clk:
-        ts = [wl.run(evs) for _ in range(args.steps)]
-        if world > 1:
-            dr.merge(wl.ctx)
-        torch.cuda.synchronize()
-        barrier(world)
-    launches = nb.nvbt_launch_count(wl.ctx) - l0
-    per, tot, hs, hl = nb.nvbt_mem_divergence(wl.ctx)
-    cnt = nb.nvbt_count(wl.ctx)
-    t_total = max_over_ranks(sum(ts), world, dev)
-    n_all = wl.n * world if world > 1 else wl.n
-    value = args.steps * sum_over_ranks(wl.n, world, dev) / t_total
-    # algorithmic bytes: 16 B per header + 256 B per executed memory event (slots that must be read)
-    mem_exec = int(tot[0]) // max(1, world if world > 1 else 1)
-    bytes_rank = 16 * wl.n + 256 * (mem_exec // args.steps)
-    ach = bytes_rank * args.steps / (sum(ts))
-    line = {
-        "metric": "replayed warp-instr events/sec", "value": value, "unit": "events/s", "n_gpus": world,
-        "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * t_total / args.steps,
-        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-        "config": {"workload": wl.desc.replace("10^10", f"{args.replay_events:.3g}" if args.replay_events != 10**10 else "10^10"),
-                   "events": args.replay_events, "chunk": wl.chunk,
-                   "l2": "inputs (36.5 GB per chunk) larger than L2"},
-        "roofline": {"bound": "hbm", "achieved": ach / 1e9, "peak": peaks["hbm_gbs"], "unit": "GB/s",
-                     "frac": ach / 1e9 / peaks["hbm_gbs"], "peak_source": peaks_src,
-                     "algorithmic_bytes_per_launch": bytes_rank * wl.chunk / wl.n,
-                     "traffic": _replay_traffic(wl.chunk, staged=wl.scratch is not None),
-                     "traffic_unit": "DRAM bytes per 2^27-event replay call (ncu at 2^26, scaled; profiles/r1_traffic.json)",
-                     "kernel": "nvbt_replay_staged = k_rpA (headers, list) + k_rpB (slots)" if wl.scratch is not None
-                     else "k_replay4"},
-        "ncu_per_event": {"k_rpA": load_counters("k_rpA"), "k_rpB": load_counters("k_rpB"),
-                          "source": "profiles/r1_ncu_counters.json (ncu --set full, tools/prof_step.py c5)"},
-        "gpu_launches": int(launches), "clocks": clk.summary(),
-        "check": {"W_issued": int(cnt[2]), "expected": args.steps * n_all},
-    }
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        rate, sample = wl.oracle_sample(min(args.cpu_budget, 10.0))
-        line["cpu_baseline"] = {"value": rate, "unit": "events/s", "cores": 1, "kind": "oracle", "sample": sample}
-    if rank == 0:
-        print(json.dumps(line), flush=True)
-
-
-
-# --------------------------------------------------------------------------- C1 / C3 / C4 (profiling lines)
-def _timed_events(torch, fn, n):
+def timed_steps(torch, fn, n, flush=None):
+    """n steps, each bracketed by CUDA events on the current stream (the contexts' stream)."""
     ts = []
     for _ in range(n):
+        if flush is not None:
+            flush.zero_()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record()
         fn()
@@ -479,31 +243,216 @@ def _timed_events(torch, fn, n):
     return ts
 
 
-def run_c1(args, torch, nb, dr, local):
-    """C1: vectorAdd N = 65536, tools COUNT (instruction count + opcode histogram); a step is one launch.
-    A launch moves 786 KB, so launch overhead dominates: the launches are batched into one CUDA graph of
-    `reps` launches (captured on the context's stream) and each replay is timed."""
+def _timed_events(torch, fn, n):
+    return timed_steps(torch, fn, n)
+
+
+# --------------------------------------------------------------------------- C2 SGEMM (headline)
+# hook instruction minima per event used for the issue roofline (minimal SASS per hook)
+HOOK_OPS = {"count": 4, "guard": 6, "mem": 23}
+
+
+class SgemmBench:
+    name = "c2"
+    M = N = K = 1024
+    desc = ("C2 naive row-fastest SGEMM 1024^3 (fp32), tools BBCOUNT|MEMDIV (counts, opcode+BB histograms via "
+            "BB-entry hooks, per-instruction divergence)")
+
+    def __init__(self, torch, nb, dr, rank, world):
+        self.torch, self.nb, self.dr = torch, nb, dr
+        from synth import uniform_f32
+        M, N, K = self.M, self.N, self.K
+        self.nw = nb.nvbt_workload_warps(nb.W_SGEMM, M, N)
+        self.ctx = nb.nvbt_init(nb.W_SGEMM, nb.COUNT | nb.OPHIST | nb.BB | nb.MEMDIV)
+        if world > 1:   # this rank runs CTA rows [y0, y1) of the one 1024^3 launch
+            nb.nvbt_set_partition(self.ctx, rank, world)
+        gx, gy = -(-M // 32), -(-N // 8)
+        y0, y1 = dr.cta_rows(gy, rank, world)
+        self.rank_warps = (y1 - y0) * gx * 8
+        self.tools = nb.TOOL_BBCOUNT | nb.TOOL_MEMDIV
+        self.hA = torch.from_numpy(uniform_f32((M, K), 3, -1, 1)).pin_memory()
+        self.hB = torch.from_numpy(uniform_f32((K, N), 4, -1, 1)).pin_memory()
+        self.A, self.B = self.hA.cuda(), self.hB.cuda()
+        self.C = torch.empty(M, N, device="cuda")
+        # events per launch (EM §3.2): every warp runs 12 + 6K warp-level instructions
+        self.per_warp = 12 + 6 * K
+        self.events = self.nw * self.per_warp
+        self.launched = 0
+
+    def plain(self):
+        self.nb.nvbt_sgemm(self.ctx, self.nb.TOOL_NONE, self.A, self.B, self.C, self.M, self.N, self.K)
+
+    def instr(self):
+        self.nb.nvbt_sgemm(self.ctx, self.tools, self.A, self.B, self.C, self.M, self.N, self.K)
+        self.launched += 1
+
+    def reset(self):
+        self.nb.nvbt_reset(self.ctx)
+        self.launched = 0   # instrumented launches accumulated in the context since the reset
+
+    def e2e_step(self, out_host):
+        """Through the public API with host buffers: H2D inputs, instrumented launch, read results."""
+        nb = self.nb
+        self.A.copy_(self.hA, non_blocking=True)
+        self.B.copy_(self.hB, non_blocking=True)
+        nb.nvbt_sgemm(self.ctx, self.tools, self.A, self.B, self.C, self.M, self.N, self.K)
+        self.launched += 1
+        out_host["counts"] = nb.nvbt_count(self.ctx)
+        out_host["memdiv"] = nb.nvbt_mem_divergence(self.ctx)
+        out_host["ophist"] = nb.nvbt_opcode_hist(self.ctx)
+        return self.hA.numel() * 4 + self.hB.numel() * 4, 8 * (4 + 3 * 18 + 3 + 66 + 2 * 16)
+
+    def roofline(self, t_kernel_s, peaks):
+        """Issue roofline ("alu") on the METHOD's own work: the minimal hook instructions of this rank's
+        launch (BB-entry hooks at the K + 3 block instances, guard hooks at pc 7 and K x pc 15, divergence
+        hooks at the 2K + 1 global LD/ST events per warp) ÷ the instrumented kernel time,
+        against 148 SMs x 4 schedulers x 1 warp-instr/clk at the max SM clock. The SGEMM's own 12 + 6K
+        instructions per warp are not the method's work and are excluded (reported beside it)."""
+        K, W = self.K, self.rank_warps
+        hooks = (K + 3) * HOOK_OPS["count"] + (K + 1) * HOOK_OPS["guard"] + (2 * K + 1) * HOOK_OPS["mem"]
+        ops = W * hooks
+        peak = N_SM * 4 * peaks.get("sm_max_mhz", 1965.0) * 1e6
+        ach = ops / t_kernel_s
+        t = load_traffic("k_sgemm<6>")
+        return {"bound": "alu", "achieved": ach / 1e9, "peak": peak / 1e9, "unit": "Gwarp-inst/s",
+                "frac": ach / peak, "traffic": t["traffic_bytes_per_launch"] if t else None,
+                "traffic_unit": "DRAM bytes per launch (ncu, profiles/r1_traffic.json)",
+                "algorithmic_hook_warp_inst_per_launch": ops,
+                "with_app_instructions_frac": (ops + W * self.per_warp) / t_kernel_s / peak}
+
+
+def run_c2(args, torch, nb, dr, rank, world, local, peaks, peaks_src):
+    wl = SgemmBench(torch, nb, dr, rank, world)
+    dev = torch.device("cuda", local)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    timed_steps(torch, wl.instr, args.warmup, flush)
+    timed_steps(torch, wl.plain, args.warmup, flush)
+    t_plain = timed_steps(torch, wl.plain, args.steps, flush)
+    wl.reset()
+    barrier(world)
+    torch.cuda.synchronize()
+    l0 = nb.nvbt_launch_count(wl.ctx)
+    with ClockSampler(local) as clk:
+        barrier(world)
+        torch.cuda.synchronize()
+        t_instr = timed_steps(torch, wl.instr, args.steps, flush)
+        torch.cuda.synchronize()
+        barrier(world)
+    gpu_launches = nb.nvbt_launch_count(wl.ctx) - l0
+    merge_ms = 0.0
+    if world > 1:
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        merge(dr, wl.ctx, world)
+        e1.record()
+        e1.synchronize()
+        merge_ms = max_over_ranks(e0.elapsed_time(e1), world)
+    # the timed steps' merged result: exactly K x the per-launch closed form (I-3)
+    cnt = nb.nvbt_count(wl.ctx)
+    _, tot, _, _ = nb.nvbt_mem_divergence(wl.ctx)
+    K = args.steps
+    ok = (int(cnt[2]) == wl.events * K and int(tot[0]) == 67_141_632 * K and
+          int(tot[1]) == int(tot[2]) == 1_108_344_832 * K)
+    tot_instr = max_over_ranks(sum(t_instr), world)
+    tot_plain = max_over_ranks(sum(t_plain), world)
+    t_kernel = max_over_ranks(statistics.median(t_instr), world)
+    value = wl.events * K / tot_instr
+    # e2e through the public API with host buffers
+    out = {}
+    for _ in range(2):
+        wl.e2e_step(out)
+    torch.cuda.synchronize()
+    barrier(world)
+    e2e_steps = max(3, min(args.steps, 10))
+    t0 = time.perf_counter()
+    for _ in range(e2e_steps):
+        h2d, d2h = wl.e2e_step(out)
+    torch.cuda.synchronize()
+    e2e_t = max_over_ranks(time.perf_counter() - t0, world)
+    line = {
+        "metric": METRIC, "value": value, "unit": "events/s", "n_gpus": world, "steps": K,
+        "warmup": args.warmup, "ms_per_step": 1e3 * tot_instr / K, "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+        "config": {"workload": wl.desc, "M": wl.M, "N": wl.N, "K": wl.K, "warp_events_per_launch": wl.events,
+                   "tools": "BBCOUNT|MEMDIV", "l2": "flushed between steps (256 MiB write)",
+                   "parallelism": (f"CTA-row partition of the launch over {world} GPUs (nvbt_set_partition), "
+                                   "one int64 all-reduce merge") if world > 1 else "1 GPU"},
+        "slowdown": tot_instr / tot_plain, "plain_ms_per_launch": 1e3 * max_over_ranks(statistics.median(t_plain), world),
+        "instr_ms_per_launch": 1e3 * t_kernel,
+        "counts_check": "ok" if ok else f"mismatch W_issued {int(cnt[2])} != {wl.events * K}",
+        "roofline": wl.roofline(statistics.median(t_instr), peaks),
+        "e2e": {"value": wl.events * e2e_steps / e2e_t, "unit": "events/s", "h2d_bytes_per_step": h2d,
+                "d2h_bytes_per_step": d2h},
+        "gpu_launches": int(gpu_launches), "clocks": clk.summary(), "peaks_source": peaks_src,
+        "merge_ms": merge_ms,
+    }
+    line["roofline"]["peak_source"] = f"148 SMs x 4 issue/clk x sm_max_mhz ({peaks_src})"
+    # the binding resource of this workload is the application's own L1 traffic (the naive row-fastest
+    # SGEMM is L1-wavefront-bound uninstrumented); the hooks run inside that bound
+    line["app_bound"] = {"resource": "L1TEX wavefronts of the uninstrumented SGEMM",
+                         "instr_speed_vs_plain": statistics.median(t_plain) / statistics.median(t_instr),
+                         "ncu": "profiles/r1_ncu_summary_c2_c5.txt: l1tex 98.8 % (plain) / 95.2 % (instrumented), "
+                                "issue-active 6.9 % / 85.2 %"}
+    line["ncu_per_event"] = {"instrumented": load_counters("k_sgemm<6>"), "plain": load_counters("k_sgemm<0>"),
+                             "source": "profiles/r1_ncu_counters.json (ncu --set full, tools/prof_step.py c2)"}
+    return line, wl
+
+
+def c2_cpu_baseline(wl, nb):
+    """cpu_baseline leg: the C oracle (all host cores) over the WHOLE C2 launch (same buffers, so the same
+    events), timed; plus its 1-thread rate on a 1 % slice; its result must equal the GPU's per launch."""
+    from oracle import coracle as co, programs
+    prog = programs.sgemm()
+    T = co.host_threads()
+    a, b, c = wl.A.data_ptr(), wl.B.data_ptr(), wl.C.data_ptr()
+    co.sgemm(prog, 64, 64, 64, a, b, c, threads=T)          # load + build outside the timing
+    t0 = time.perf_counter()
+    r = co.sgemm(prog, wl.M, wl.N, wl.K, a, b, c, threads=T)
+    dt = time.perf_counter() - t0
+    sl = wl.nw // 100
+    t1 = time.perf_counter()
+    co.sgemm(prog, wl.M, wl.N, wl.K, a, b, c, warps=(0, sl), threads=1)
+    dt1 = time.perf_counter() - t1
+    cnt = nb.nvbt_count(wl.ctx).astype(np.int64)
+    per, tot, hs, hl = nb.nvbt_mem_divergence(wl.ctx)
+    steps = wl.launched
+    match = (np.array_equal(cnt, steps * r["counts"]) and np.array_equal(per[:, 1].astype(np.int64), steps * r["mem_S"])
+             and np.array_equal(per[:, 2].astype(np.int64), steps * r["mem_L"])
+             and np.array_equal(hs.astype(np.int64), steps * r["hS"]))
+    return {"value": wl.events / dt, "unit": "events/s", "cores": T, "kind": "oracle",
+            "sample": f"the whole C2 launch ({wl.events} warp events), C oracle (oracle/c) on {T} threads",
+            "cpu_model": cpu_model(), "one_thread_value": sl * wl.per_warp / dt1,
+            "one_thread_sample": f"warps [0, {sl}) (1 %) on 1 thread", "matches_gpu": bool(match)}
+
+
+# --------------------------------------------------------------------------- C1 vectorAdd
+def run_c1(args, torch, nb, dr, rank, world, local, steps):
+    """C1: vectorAdd N = 65536, instruction counts + opcode histogram. A launch moves 786 KB, so launch
+    overhead dominates: launches are batched into one CUDA graph of `reps` launches (captured on the
+    context's stream) and each replay is timed. Counts two ways, identical results (I-5): BBCOUNT (hooks at
+    block leaders and guarded pcs) is the config's value, COUNT (a hook at every pc) beside it."""
     from synth import uniform_f32
-    N = 65536
+    N, reps = 65536, 200
     s = torch.cuda.Stream()
-    ctx = nb.nvbt_init(nb.W_VECTORADD, nb.COUNT | nb.OPHIST | nb.BB, stream=s)
+    ctxs = {}
+    for name in ("COUNT", "BBCOUNT"):
+        ctxs[name] = nb.nvbt_init(nb.W_VECTORADD, nb.COUNT | nb.OPHIST | nb.BB, stream=s)
+        if world > 1:
+            nb.nvbt_set_partition(ctxs[name], rank, world)
     a = torch.from_numpy(uniform_f32(N, 1)).cuda()
     b = torch.from_numpy(uniform_f32(N, 2)).cuda()
     c = torch.empty_like(a)
-    reps = 200   # launches per graph
     torch.cuda.synchronize()
 
-    def graph_of(tools):
+    def graph_of(ctx, tools):
         g = torch.cuda.CUDAGraph()
         with torch.cuda.graph(g, stream=s):
             for _ in range(reps):
                 nb.nvbt_vectoradd(ctx, tools, a, b, c, N)
         return g
 
-    # per-pc counts two ways, identical results (I-5): a hook at every instruction (COUNT) or at block
-    # leaders and guarded pcs only (BBCOUNT, the paper's basic-block instrumentation, P:L89)
-    g_plain, g_cnt, g_bb = graph_of(nb.TOOL_NONE), graph_of(nb.TOOL_COUNT), graph_of(nb.TOOL_BBCOUNT)
-    nb.nvbt_reset(ctx)
+    graphs = {"plain": graph_of(ctxs["COUNT"], nb.TOOL_NONE), "COUNT": graph_of(ctxs["COUNT"], nb.TOOL_COUNT),
+              "BBCOUNT": graph_of(ctxs["BBCOUNT"], nb.TOOL_BBCOUNT)}
 
     def timed(g, n):
         ts = []
@@ -517,116 +466,220 @@ def run_c1(args, torch, nb, dr, local):
             ts.append(e0.elapsed_time(e1) / 1e3)
         return ts
 
-    for g in (g_cnt, g_bb, g_plain):
-        timed(g, args.warmup)
-    tp = timed(g_plain, args.steps)
+    for g in graphs.values():
+        timed(g, 3)
+    t = {}
+    for name in ("plain", "COUNT", "BBCOUNT"):
+        if name != "plain":
+            nb.nvbt_reset(ctxs[name])
+        barrier(world)
+        t[name] = max_over_ranks(sum(timed(graphs[name], steps)), world) / (steps * reps)
     res = {}
-    for name, g in (("COUNT", g_cnt), ("BBCOUNT", g_bb)):
-        nb.nvbt_reset(ctx)
-        with ClockSampler(local) as clk:
-            ti = timed(g, args.steps)
-        cnt = nb.nvbt_count(ctx)
-        ht, hw = nb.nvbt_opcode_hist(ctx)
-        res[name] = (ti, cnt, ht, hw, clk.summary())
-    ok = all((res["COUNT"][1] == res["BBCOUNT"][1]).all() and (res["COUNT"][k] == res["BBCOUNT"][k]).all()
-             for k in (2, 3))
-    ti, cnt, _, _, clocks = res["BBCOUNT"]
-    ev = int(cnt[2]) // (args.steps * reps)
-    t_i, t_p = sum(ti) / (args.steps * reps), sum(tp) / (args.steps * reps)
-    t_c = sum(res["COUNT"][0]) / (args.steps * reps)
-    return {"metric": METRIC, "value": ev / t_i, "unit": "events/s", "n_gpus": 1, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": 1e3 * t_i, "higher_is_better": True, "scaling": "weak",
-            "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-            "config": {"workload": "C1 vectorAdd N=65536, instruction counts + opcode histogram (tools BBCOUNT)",
-                       "launches_per_graph": reps, "warp_events_per_launch": ev,
-                       "counts_check": ("ok" if ev == 26624 else f"{ev} != 26624") +
-                                       ("; COUNT == BBCOUNT counts and opcode histograms" if ok else "; COUNT != BBCOUNT")},
-            "slowdown": t_i / t_p, "plain_us_per_launch": 1e6 * t_p, "instr_us_per_launch": 1e6 * t_i,
-            "per_instruction_hooks": {"tools": "COUNT", "instr_us_per_launch": 1e6 * t_c, "slowdown": t_c / t_p,
-                                      "value": ev / t_c},
-            "bound": "launch latency (26,624 warp events per launch; CUDA-graph replays)", "clocks": clocks}
+    for name in ("COUNT", "BBCOUNT"):
+        merge(dr, ctxs[name], world)
+        res[name] = (nb.nvbt_count(ctxs[name]), nb.nvbt_opcode_hist(ctxs[name]))
+    same = (np.array_equal(res["COUNT"][0], res["BBCOUNT"][0]) and
+            all(np.array_equal(x, y) for x, y in zip(res["COUNT"][1], res["BBCOUNT"][1])))
+    ev = int(res["BBCOUNT"][0][2]) // (steps * reps)
+    ok = ev == 26624 and int(res["BBCOUNT"][0][3]) == 24576 * steps * reps and same
+    return {"value": 26624 / t["BBCOUNT"], "unit": "events/s", "steps": steps, "launches_per_step": reps,
+            "workload": "C1 vectorAdd N=65536 (256 thr/CTA), counts + opcode histogram, tools BBCOUNT",
+            "slowdown": t["BBCOUNT"] / t["plain"], "plain_us_per_launch": 1e6 * t["plain"],
+            "instr_us_per_launch": 1e6 * t["BBCOUNT"],
+            "per_instruction_hooks": {"tools": "COUNT", "value": 26624 / t["COUNT"], "slowdown": t["COUNT"] / t["plain"]},
+            "counts_check": ("ok: W_issued 26,624 and W_exec 24,576 per launch (I-3), COUNT == BBCOUNT counts "
+                             "and opcode histograms") if ok else f"mismatch: {ev} events per launch, same={same}",
+            "roofline": {"bound": "launch", "note": "26,624 warp events per launch: launch latency, not a "
+                         "throughput roofline (CUDA-graph replays)"}}
 
 
-def run_c3(args, torch, nb, dr, local):
-    """C3: BFS on an R-MAT scale-20 graph with BB-entry counting; a step is one whole BFS."""
+# --------------------------------------------------------------------------- C3 BFS
+def run_c3(args, torch, nb, dr, rank, world, local, steps):
+    """C3: BFS on the R-MAT scale-20 graph (edge factor 16) with BB-entry counting; a step is one whole
+    BFS. N > 1: vertex-range partition with the per-level MAX exchanges (drivers.run_bfs_dist)."""
     from synth import rmat_csr, bfs_source
     rowptr, col = rmat_csr(args.bfs_scale, 16, seed=3)
     n = len(rowptr) - 1
     src = bfs_source(rowptr)
+    nw = nb.nvbt_workload_warps(nb.W_BFS, n)
     rp, cl = torch.from_numpy(rowptr).cuda(), torch.from_numpy(col).cuda()
     ctx = nb.nvbt_init(nb.W_BFS, nb.COUNT | nb.BB)
+    if world > 1:
+        nb.nvbt_set_partition(ctx, rank, world)
     bufs = dr.bfs_buffers(n, "cuda")
-    f_plain = lambda: dr.run_bfs(ctx, nb.TOOL_NONE, rp, cl, src, bufs)
-    f_instr = lambda: dr.run_bfs(ctx, nb.TOOL_BBCOUNT, rp, cl, src, bufs)
-    for _ in range(args.warmup):
-        f_plain(); f_instr()
-    tp = _timed_events(torch, f_plain, args.steps)
+    if world > 1:
+        bfs = lambda t: dr.run_bfs_dist(ctx, t, rp, cl, src, bufs)
+    else:
+        bfs = lambda t: dr.run_bfs(ctx, t, rp, cl, src, bufs)
+    for _ in range(2):
+        bfs(nb.TOOL_NONE)
+        bfs(nb.TOOL_BBCOUNT)
+    barrier(world)
+    tp = max_over_ranks(sum(timed_steps(torch, lambda: bfs(nb.TOOL_NONE), steps)), world)
     nb.nvbt_reset(ctx)
-    with ClockSampler(local) as clk:
-        ti = _timed_events(torch, f_instr, args.steps)
+    barrier(world)
+    ti = max_over_ranks(sum(timed_steps(torch, lambda: bfs(nb.TOOL_BBCOUNT), steps)), world)
+    _, levels = bfs(nb.TOOL_NONE)
+    merge(dr, ctx, world)
     cnt = nb.nvbt_count(ctx)
-    ev = int(cnt[2]) // args.steps
-    _, levels = f_plain()
-    return {"metric": METRIC, "value": ev * args.steps / sum(ti), "unit": "events/s", "n_gpus": 1,
-            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * sum(ti) / args.steps,
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-            "config": {"workload": f"C3 BFS R-MAT scale {args.bfs_scale} ef16, tools BBCOUNT",
-                       "vertices": n, "directed_edges": int(len(col)), "levels": levels,
-                       "warp_events_per_bfs": ev},
-            "slowdown": sum(ti) / sum(tp), "plain_ms_per_bfs": 1e3 * sum(tp) / args.steps,
-            "bound": "latency of the hub warp's serial edge loop", "clocks": clk.summary()}
+    bb = nb.nvbt_bb_count(ctx)
+    ev = int(cnt[2]) // steps
+    # every kernel-1 launch is entered by every warp: Ent_w(block 0) = levels x warps per BFS
+    ok = int(bb[0, 0]) == levels * nw * steps
+    return {"value": ev * steps / ti, "unit": "events/s", "steps": steps,
+            "workload": f"C3 BFS R-MAT scale {args.bfs_scale} ef16 (Graph500 a,b,c), tools BBCOUNT",
+            "vertices": n, "directed_edges": int(len(col)), "levels": levels, "warp_events_per_bfs": ev,
+            "slowdown": ti / tp, "plain_ms_per_bfs": 1e3 * tp / steps, "instr_ms_per_bfs": 1e3 * ti / steps,
+            "counts_check": "ok: Ent_w(kernel 1 entry block) = levels x warps" if ok else
+                            f"mismatch Ent_w {int(bb[0, 0])} != {levels * nw * steps}",
+            "roofline": {"bound": "latency", "note": "the hub warp's serial edge loop (max degree ~6.5e4) "
+                         "bounds both the plain and the instrumented BFS"}}
 
 
-def run_c4(args, torch, nb, dr, local):
-    """C4: 8192^2 5-point stencil x 100 iterations, every global LD/ST traced through the channel and
-    drained to pinned host memory (digest callback on all host cores); a step is the whole run."""
+# --------------------------------------------------------------------------- C4 stencil + channel
+def run_c4(args, torch, nb, dr, rank, world, local, steps):
+    """C4: 8192^2 5-point stencil x 100 iterations, every executed global LD/ST traced through the pinned
+    host channel (288 B records, EM §5) and digested on the host; a step is the whole traced run. The
+    drain runs on a host thread while the iterations are enqueued (N > 1: row slabs with P2P halos, one
+    channel per rank). Device time from the first launch to the last kernel's end (the producers wait on
+    the host ring, so it includes the transport), max over ranks."""
     from synth import uniform_f32
     n, iters = args.stencil_n, args.stencil_iters
     ctx = nb.nvbt_init(nb.W_STENCIL, nb.COUNT | nb.TRACE)
+    if world > 1:
+        nb.nvbt_set_partition(ctx, rank, world)
     x0 = torch.from_numpy(uniform_f32((n, n), 4)).cuda()
     buf0, buf1 = x0.clone(), torch.empty_like(x0)
-    slot = 176 if args.compact else 288
-    ring = torch.empty(nb.nvbt_channel_bytes(args.ring_records, compact=args.compact), dtype=torch.uint8, pin_memory=True)
-    ch = nb.nvbt_channel_open(ctx, ring, compact=args.compact)
-    # plain baseline
-    for _ in range(args.warmup):
-        dr.run_stencil(ctx, nb.TOOL_NONE, buf0, buf1, n, iters)
-    tp = _timed_events(torch, lambda: dr.run_stencil(ctx, nb.TOOL_NONE, buf0, buf1, n, iters), args.steps)
-    # traced runs: wall time from first launch to the last record drained
-    res = []
-    with ClockSampler(local) as clk:
-        for _ in range(args.steps):
-            torch.cuda.synchronize()
-            t0 = time.perf_counter()
+    ring = torch.empty(nb.nvbt_channel_bytes(args.ring_records), dtype=torch.uint8, pin_memory=True)
+    ch = nb.nvbt_channel_open(ctx, ring)
+    if world > 1:
+        run = lambda t, it: dr.run_stencil_dist(ctx, t, buf0, buf1, n, it, rank, world, gather=False)
+    else:
+        run = lambda t, it: dr.run_stencil(ctx, t, buf0, buf1, n, it)
+
+    def traced(it):
+        d = nb.Digest()
+        done = threading.Event()
+        err = []
+
+        def drain():   # the drain returns whenever the stream is idle with everything delivered
+            try:
+                while True:
+                    fin = done.is_set()
+                    nb.nvbt_channel_drain_digest(ch, timeout_us=900_000_000, digest=d)
+                    if fin:
+                        return
+            except Exception as e:  # noqa: BLE001 - reported by the caller
+                err.append(e)
+        th = threading.Thread(target=drain)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        t0 = time.perf_counter()
+        e0.record()
+        th.start()
+        run(nb.TOOL_TRACE, it)
+        e1.record()
+        done.set()
+        th.join()
+        torch.cuda.synchronize()
+        if err:
+            raise err[0]
+        return e0.elapsed_time(e1) / 1e3, time.perf_counter() - t0, d.n_rec
+
+    run(nb.TOOL_NONE, iters)
+    tp = max_over_ranks(sum(timed_steps(torch, lambda: run(nb.TOOL_NONE, iters), max(steps, 3))), world) / max(steps, 3)
+    traced(max(1, iters // 10))                                  # warm-up: 10 % of the iterations
+    barrier(world)
+    res = [traced(iters) for _ in range(steps)]
+    dropped = nb.nvbt_channel_dropped(ch)
+    t_dev = max_over_ranks(sum(r[0] for r in res), world) / steps
+    t_wall = max_over_ranks(sum(r[1] for r in res), world) / steps
+    recs = sum_over_ranks(res[-1][2], world)
+    G = n // 32
+    expect = iters * (4 * G + 6 * G * (n - 2))                   # SURVEY I-3 closed form
+    dropped_all = sum_over_ranks(dropped, world)
+    ok = int(recs) == expect and dropped_all == 0
+    gbs = recs * (288 + 4) / t_dev / 1e9 / world                 # records + commit tags per GPU link
+    peak = d2h_peak()
+    nb.nvbt_channel_close(ch)
+    del ring
+    return {"value": recs / t_dev, "unit": "records/s", "steps": steps,
+            "workload": f"C4 stencil {n}^2 x {iters}, tools TRACE, 288 B records to pinned host, digest drain",
+            "records_per_run": int(recs), "records_expected": expect, "dropped": int(dropped_all),
+            "slowdown": t_dev / tp, "plain_ms": 1e3 * tp, "traced_s": t_dev, "traced_wall_s": t_wall,
+            "ring_slots": args.ring_records,
+            "counts_check": "ok: records = iters x (4G + 6G(n-2)) (I-3), none dropped" if ok else
+                            f"mismatch: {int(recs)} records, expected {expect}, dropped {int(dropped_all)}",
+            "roofline": {"bound": "pcie", "achieved": gbs, "peak": peak, "unit": "GB/s", "frac": gbs / peak,
+                         "peak_source": "measured SM-store D2H into pinned memory (profiles/r1_box_peaks.json)",
+                         "algorithmic_bytes_per_record": 292}}
+
+
+# --------------------------------------------------------------------------- C5 replay
+def _replay_traffic(chunk):
+    """ncu DRAM bytes of one staged replay call on `chunk` events (captured at 2^26 events, scaled)."""
+    tr = [load_traffic(k) for k in ("k_rpA<0>", "k_rpB")]
+    if any(t is None for t in tr):
+        return None
+    return sum(t["traffic_bytes_per_launch"] for t in tr) / 67108864 * chunk
+
+
+def run_c5(args, torch, nb, dr, rank, world, local, steps, peaks, peaks_src):
+    """C5: staged replay (counts, histograms, divergence) of 10^10 generated events in 2^27-event chunks;
+    generation is not timed; N > 1: contiguous event-index ranges per rank. Inputs (36.5 GB per chunk)
+    exceed L2."""
+    n_total, chunk = args.replay_events, 1 << 27
+    lo, hi = dr.shard_range(n_total, rank, world)
+    n = hi - lo
+    ctx = nb.nvbt_init(nb.W_REPLAY, nb.COUNT | nb.OPHIST | nb.BB | nb.MEMDIV)
+    hdr = torch.empty(chunk * 16, dtype=torch.uint8, device="cuda")
+    addr = torch.empty(chunk * 256, dtype=torch.uint8, device="cuda")
+    scratch = torch.empty(nb.nvbt_replay_scratch_size(ctx, chunk), dtype=torch.uint8, device="cuda")
+    for _ in range(2):
+        nb.nvbt_gen_events(ctx, SEED, lo, min(chunk, n), hdr, addr)
+        nb.nvbt_replay_staged(ctx, hdr, addr, min(chunk, n), scratch)
+    nb.nvbt_reset(ctx)
+    torch.cuda.synchronize()
+    barrier(world)
+
+    def step():
+        t = 0.0
+        off = 0
+        while off < n:
+            m = min(chunk, n - off)
+            nb.nvbt_gen_events(ctx, SEED, lo + off, m, hdr, addr)
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record()
-            dr.run_stencil(ctx, nb.TOOL_TRACE, buf0, buf1, n, iters)
+            nb.nvbt_replay_staged(ctx, hdr, addr, m, scratch)
             e1.record()
-            if args.drain == "discard":
-                nrec = nb.nvbt_channel_drain_discard(ch, timeout_us=600_000_000)
-            else:
-                nrec = nb.nvbt_channel_drain_digest(ch, timeout_us=600_000_000).n_rec
-            torch.cuda.synchronize()
-            res.append((time.perf_counter() - t0, nrec, e0.elapsed_time(e1) / 1e3))
-    dropped = nb.nvbt_channel_dropped(ch)
-    recs = res[-1][1]
-    t_tr = sum(r[0] for r in res) / len(res)
-    G = n // 32
-    expect = iters * (2 * (n * n // 32) + 4 * (n - 2) * G)
-    return {"metric": "traced warp-level memory events/sec (records drained to host)", "value": recs / t_tr,
-            "unit": "records/s", "n_gpus": 1, "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * t_tr,
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-            "config": {"workload": f"C4 stencil {n}^2 x {iters}, tools TRACE", "ring_slots": args.ring_records,
-                       "transport": "compact 176 B slots at a 192 B stride (EM 5.1)" if args.compact else "288 B records",
-                       "host_callback": args.drain},
-            "records_per_run": recs, "records_expected": expect, "dropped": dropped,
-            "gpu_s_per_run": sum(r[2] for r in res) / len(res),
-            "host_threads": os.environ.get("NVBT_DRAIN_THREADS", str(os.cpu_count())),
-            "GB_per_s_to_host": recs * slot / t_tr / 1e9, "record_GB_per_s": recs * 288 / t_tr / 1e9, "slowdown": t_tr / (sum(tp) / len(tp)),
-            "plain_ms": 1e3 * sum(tp) / len(tp), "bound": "PCIe D2H (measured 52.7 GB/s SM stores to pinned memory)",
-            "clocks": clk.summary()}
+            e1.synchronize()
+            t += e0.elapsed_time(e1) / 1e3
+            off += m
+        return t
+
+    ts = [step() for _ in range(steps)]
+    _, tot, _, _ = nb.nvbt_mem_divergence(ctx)
+    mem_exec = int(tot[0]) // steps
+    t_rank = sum(ts) / steps
+    ach = (16 * n + 256 * mem_exec) / t_rank / 1e9
+    merge(dr, ctx, world)
+    cnt = nb.nvbt_count(ctx)
+    t_all = max_over_ranks(t_rank, world)
+    ok = int(cnt[2]) == steps * n_total
+    del hdr, addr, scratch
+    torch.cuda.empty_cache()
+    return {"value": n_total / t_all, "unit": "events/s", "steps": steps,
+            "workload": f"C5 staged trace replay of {n_total:.3g} generated events (counts, histograms, divergence)",
+            "ms_per_step": 1e3 * t_all, "chunk": chunk,
+            "counts_check": "ok: W_issued = events" if ok else f"mismatch W_issued {int(cnt[2])}",
+            "roofline": {"bound": "hbm", "achieved": ach, "peak": float(peaks["hbm_gbs"]), "unit": "GB/s",
+                         "frac": ach / float(peaks["hbm_gbs"]), "peak_source": peaks_src,
+                         "algorithmic_bytes": "16 per header + 256 per executed memory event (per rank)",
+                         "traffic": _replay_traffic(chunk),
+                         "traffic_unit": "DRAM bytes per 2^27-event call (ncu at 2^26, scaled)",
+                         "kernel": "nvbt_replay_staged = k_rpA (headers, list) + k_rpB (slots)"}}
 
 
+# --------------------------------------------------------------------------- NEXT-row profiling lines (F1, F2, F4)
 def run_f2(args, torch, nb, dr, local):
     """F2: C4's traced stencil (8192^2, --f2-iters iterations) with the trace kept in an HBM ring and
     analysed on the GPU (per-launch footprint) instead of drained to the host. A step = traced run
@@ -801,38 +854,75 @@ def run_f4(args, torch, nb, dr, local):
             "paper_context": "21 vs 150 instructions per warp with and without WFFT32 (P:L295), parity-unpinned"}
 
 
-def run_reference(args):
-    """Reference arm = the CPU oracle (this tier has no runnable reference)."""
-    rank = int(os.environ.get("RANK", "0"))
-    if rank != 0:
+# --------------------------------------------------------------------------- main
+def run_ours(args):
+    import torch
+    rank, world, local = dist_setup(args)
+    import paper_conf_micro_villasnk19_b200 as pkg
+    nb, dr = pkg.nvbt, pkg.drivers
+    peaks, peaks_src = load_peaks()
+    if args.workload in ("f1", "f2", "f4"):
+        line = {"f1": run_f1, "f2": run_f2, "f4": run_f4}[args.workload](args, torch, nb, dr, local)
+        if rank == 0:
+            print(json.dumps(line), flush=True)
         return
-    from oracle import events as ev, programs
-    from oracle.models import sgemm as m_sg
+    line, wl = run_c2(args, torch, nb, dr, rank, world, local, peaks, peaks_src)
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        line["cpu_baseline"] = c2_cpu_baseline(wl, nb)
+    del wl
+    torch.cuda.empty_cache()
+    wanted = [c for c in args.configs.split(",") if c and c != "none"]
+    cfg = {}
+    for c in wanted:
+        if c == "c1":
+            cfg["c1"] = run_c1(args, torch, nb, dr, rank, world, local, args.steps)
+        elif c == "c3":
+            cfg["c3"] = run_c3(args, torch, nb, dr, rank, world, local, min(args.steps, 5))
+        elif c == "c4":
+            cfg["c4"] = run_c4(args, torch, nb, dr, rank, world, local, args.c4_steps)
+        elif c == "c5":
+            cfg["c5"] = run_c5(args, torch, nb, dr, rank, world, local, args.c5_steps, peaks, peaks_src)
+        torch.cuda.empty_cache()
+    if cfg:
+        line["configs"] = cfg
+    if world > 1:
+        line["allreduce_latency"] = allreduce_latency(world)
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        import torch.distributed as dist
+        dist.destroy_process_group()
+
+
+def run_reference(args):
+    """Reference arm = the CPU oracle (this tier has no runnable reference): the C oracle
+    (oracle/c, multithreaded, plain event-by-event EM §2) on all host cores; one step = one whole C2 launch
+    (the same 201,719,808 warp events the GPU step instruments)."""
+    if int(os.environ.get("RANK", "0")) != 0:
+        return
+    from oracle import coracle as co, programs
+    prog = programs.sgemm()
     M = N = K = 1024
-    nw = (M // 32) * (N // 8) * 8
-    events_per_launch = nw * (12 + 6 * K)
+    T = co.host_threads()
+    events = (M // 32) * (N // 8) * 8 * (12 + 6 * K)
     base = 1 << 32
-    rng = np.random.default_rng(1)
-    warps = np.sort(rng.choice(nw, size=16, replace=False))
-    per_step_events = len(warps) * (12 + 6 * K)
+    ptrs = (base, base + (8 << 20), base + (16 << 20))
     for _ in range(args.warmup):
-        acc = ev.Accumulator(programs.sgemm())
-        m_sg.run(acc, M, N, K, base, base + (8 << 20), base + (16 << 20), warps=warps[:2])
+        co.sgemm(prog, M, N, K, *ptrs, threads=T, warps=(0, 3276))
     ts = []
     for _ in range(args.steps):
-        acc = ev.Accumulator(programs.sgemm())
         t0 = time.perf_counter()
-        m_sg.run(acc, M, N, K, base, base + (8 << 20), base + (16 << 20), warps=warps)
+        co.sgemm(prog, M, N, K, *ptrs, threads=T)
         ts.append(time.perf_counter() - t0)
-    value = per_step_events * args.steps / sum(ts)
-    sample = (f"{per_step_events} warp events per step: 16 sampled warps (full K) of C2 SGEMM 1024^3 "
-              f"({events_per_launch} events per launch)")
+    value = events * args.steps / sum(ts)
+    sample = f"the whole C2 launch ({events} warp events) per step, C oracle on {T} threads"
     line = {
-        "metric": METRIC, "value": value, "unit": "events/s", "n_gpus": int(os.environ.get("WORLD_SIZE", "1")),
+        "metric": METRIC, "value": value, "unit": "events/s", "n_gpus": int(os.environ.get("WORLD_SIZE", args.gpus)),
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * sum(ts) / args.steps,
-        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
         "config": {"workload": SgemmBench.desc, "M": M, "N": N, "K": K}, "impl": "reference",
-        "cpu_baseline": {"value": value, "unit": "events/s", "cores": 1, "kind": "oracle", "sample": sample},
+        "cpu_baseline": {"value": value, "unit": "events/s", "cores": T, "kind": "oracle", "sample": sample,
+                         "cpu_model": cpu_model()},
         "e2e": {"value": value, "unit": "events/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
@@ -844,11 +934,11 @@ def main():
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--drain", choices=["digest", "discard"], default="digest",
-                    help="C4: host callback (digest of every record, or discard: the transport alone)")
-    ap.add_argument("--replay-impl", choices=["staged", "single"], default="staged",
-                    help="C5: two-pass staged replay (default) or the single-pass kernel")
-    ap.add_argument("--workload", choices=["c1", "c2", "c3", "c4", "c5", "f1", "f2", "f4"], default="c2")
+    ap.add_argument("--workload", choices=["c2", "f1", "f2", "f4"], default="c2",
+                    help="c2: the headline line with --configs beside it; f1/f2/f4: NEXT-row profiling lines")
+    ap.add_argument("--configs", default="c1,c3,c4,c5", help="configs measured beside C2 ('none' for C2 only)")
+    ap.add_argument("--c4-steps", type=int, default=2)
+    ap.add_argument("--c5-steps", type=int, default=3)
     ap.add_argument("--fft-n", type=int, default=1 << 24, help="F4: transforms per launch")
     ap.add_argument("--fft-ctas", type=int, default=0, help="F4: grid (0 = one resident wave per kernel)")
     ap.add_argument("--f2-iters", type=int, default=10, help="F2: stencil iterations kept in the HBM ring")
@@ -856,15 +946,15 @@ def main():
     ap.add_argument("--stencil-n", type=int, default=8192)
     ap.add_argument("--stencil-iters", type=int, default=100)
     ap.add_argument("--ring-records", type=int, default=1 << 22)
-    ap.add_argument("--compact", action="store_true", help="C4: compact 176 B transport slots (F3)")
     ap.add_argument("--replay-events", type=int, default=10**10)
-    ap.add_argument("--cpu-budget", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
     if args.impl == "reference":
         run_reference(args)
+    elif args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        sys.exit(spawn_ranks(args.gpus))
     else:
         run_ours(args)
 

@@ -147,7 +147,12 @@ int nvbt_channel_open(nvbt_ctx ctx, void* pinned_ring, size_t ring_bytes, uint32
 typedef int (*nvbt_drain_fn)(const void* records, uint64_t n_records, void* user);
 /* Consumes records in ticket order until the context's stream is idle and every reserved record has
  * been delivered, or timeout_us elapses (-1 = no limit; NVBT_ETIMEDOUT). Runs on the calling thread,
- * concurrently with kernels already enqueued. *n_drained (nullable) = records delivered by this call. */
+ * concurrently with kernels already enqueued; it never synchronises the context's stream, so a drain
+ * thread may run while another thread keeps enqueueing producers (it returns whenever it sees the stream
+ * idle with everything delivered: call it again until the producer thread is done). *n_drained
+ * (nullable) = records delivered by this call. A producer that waits ~2 s on a full ring gives up: its
+ * record is dropped and counted (nvbt_channel_dropped), the drain then reports NVBT_ETIMEDOUT, and the
+ * channel must be closed and reopened (the dropped ticket leaves a hole that is never committed). */
 int nvbt_channel_drain(nvbt_channel ch, nvbt_drain_fn fn, void* user, int64_t timeout_us,
                        uint64_t* n_drained);
 int nvbt_channel_close(nvbt_channel ch);
@@ -206,6 +211,32 @@ int nvbt_replay_errors(nvbt_ctx ctx, uint64_t* bad_events);
 int nvbt_replay_scratch_size(nvbt_ctx ctx, uint64_t max_events_per_block, size_t* bytes);
 int nvbt_replay_staged(nvbt_ctx ctx, const void* d_hdr, const void* d_addr, uint64_t n, void* d_scratch,
                        size_t scratch_bytes);
+
+/* ---- public device API (include/nvbt_dev.cuh): kernels outside the library instrument themselves ----
+ * The compiled-in analogue of nvbit_insert_call / nvbit_add_call_arg (P:L123 (§4); Listing 8,
+ * P:L243-246 (§6.1)): a kernel receives this POD by value and calls nvbt_on_instr / nvbt_on_bb /
+ * nvbt_on_mem / nvbt_cta_flush at its injection points (pcs of the context's program table). Pointers
+ * are device addresses inside the context's workspace (caller-owned, valid until nvbt_fini). */
+#define NVBT_DEV_STATE_VERSION 1
+typedef struct {
+  uint32_t version;             /* NVBT_DEV_STATE_VERSION */
+  uint32_t tools;               /* the tool set the hooks record: NVBT_TOOL_COUNT or NVBT_TOOL_BBCOUNT,
+                                   and/or NVBT_TOOL_MEMDIV */
+  unsigned long long* site;     /* per pc 4 u64 (t_issued, t_exec, w_issued, w_exec) at site + 4 pc, in
+                                   each of `stripes` copies stripe_words apart (CTA c uses copy c % stripes) */
+  unsigned long long* mem;      /* per pc 3 u64 (n, sectors, lines) at mem + 3 pc, striped the same way */
+  unsigned long long* hist;     /* 66 u64 (hS[0..32], hL[0..32]), striped the same way */
+  unsigned long long* per_warp; /* [2][n_warps] (executed thread / warp instructions) or NULL */
+  uint64_t stripe_words;
+  uint32_t stripes;             /* a power of two */
+  uint32_t n_pcs;
+  uint32_t n_warps;             /* per_warp length (0 without NVBT_PER_WARP) */
+  uint32_t launch;              /* launch id this state was issued for (EM §5) */
+} nvbt_dev_state;
+/* Fills *out (pod_bytes must be sizeof(nvbt_dev_state)) for ONE instrumented launch of an external kernel
+ * with `tools` (COUNT xor BBCOUNT, optionally MEMDIV; TRACE is not offered to external kernels: EINVAL);
+ * takes the context's next launch id. ESTATE if a tool's flag was not enabled at init. Host-only. */
+int nvbt_device_state(nvbt_ctx ctx, uint32_t tools, void* out_pod, size_t pod_bytes);
 
 /* Number of kernels this context launched since init (for the bench's gpu_launches claim). */
 int nvbt_launch_count(nvbt_ctx ctx, uint64_t* n);

@@ -38,6 +38,13 @@ struct nvbt_chan_s {
   bool have_half = false;              // compact: first half of a wide pair seen at the ring end
   unsigned char half[176];
   std::vector<unsigned char> scratch;  // compact: decoded records of one batch
+  // host rings: a private non-blocking stream for the drain's reads of the ticket counter. The drain never
+  // synchronises the context's stream: another thread may be enqueueing producers on it, and waiting for
+  // them would deadlock against the ring they are waiting on.
+  cudaStream_t qs = nullptr;
+  ~nvbt_chan_s() {
+    if (qs) cudaStreamDestroy(qs);
+  }
 };
 
 namespace nvbt {
@@ -335,6 +342,7 @@ int nvbt_channel_open(nvbt_ctx c, void* ring, size_t bytes, uint32_t record_byte
   }
   if (e == cudaSuccess) e = cudaMemsetAsync(c->ctl + CTL_HEAD, 0, 3 * 8, c->stream);  // head, tail_cache, dropped
   if (e == cudaSuccess) e = cudaStreamSynchronize(c->stream);
+  if (e == cudaSuccess && !on_device) e = cudaStreamCreateWithFlags(&ch->qs, cudaStreamNonBlocking);
   if (e != cudaSuccess) { delete ch; return set_error(NVBT_ECUDA, "channel reset: %s", cudaGetErrorString(e)); }
   ch->open = true;
   c->chan = ch;
@@ -737,9 +745,11 @@ int nvbt_channel_drain(nvbt_channel ch, nvbt_drain_fn fn, void* user, int64_t ti
     }
     const cudaError_t q = cudaStreamQuery(c->stream);
     if (q == cudaSuccess) {
+      // the producers enqueued before the query have finished, so head is final for them (read on the
+      // channel's own stream: never wait on the context's stream, see nvbt_chan_s::qs)
       uint64_t ctl[3];
-      NVBT_CUDA(cudaMemcpyAsync(ctl, c->ctl + CTL_HEAD, sizeof ctl, cudaMemcpyDeviceToHost, c->stream));
-      NVBT_CUDA(cudaStreamSynchronize(c->stream));
+      NVBT_CUDA(cudaMemcpyAsync(ctl, c->ctl + CTL_HEAD, sizeof ctl, cudaMemcpyDeviceToHost, ch->qs));
+      NVBT_CUDA(cudaStreamSynchronize(ch->qs));
       if (ch->consumed >= ctl[0]) break;  // every ticket handed out has been delivered
       if (ctl[2] != 0) {
         rc = set_error(NVBT_ETIMEDOUT, "%llu records dropped by producers (ring full, no consumer)",

@@ -361,6 +361,32 @@ int nvbt_replay_errors(nvbt_ctx c, uint64_t* bad) {
   return NVBT_OK;
 }
 
+int nvbt_device_state(nvbt_ctx c, uint32_t tools, void* out_pod, size_t pod_bytes) {
+  if (!c || !out_pod) return set_error(NVBT_EINVAL, "null argument");
+  if (pod_bytes != sizeof(nvbt_dev_state))
+    return set_error(NVBT_EINVAL, "pod_bytes %zu != sizeof(nvbt_dev_state) %zu", pod_bytes, sizeof(nvbt_dev_state));
+  if (tools & (NVBT_TOOL_TRACE | NVBT_TOOL_EMU))
+    return set_error(NVBT_EINVAL, "external kernels get COUNT / BBCOUNT / MEMDIV hooks only");
+  std::lock_guard<std::mutex> g(c->mu);
+  DevState st;
+  int rc = make_state(c, tools, &st);
+  if (rc) return rc;
+  nvbt_dev_state d{};
+  d.version = NVBT_DEV_STATE_VERSION;
+  d.tools = tools;
+  d.site = st.site;
+  d.mem = st.mem;
+  d.hist = st.hist;
+  d.per_warp = st.pw;
+  d.stripe_words = st.stripe_words;
+  d.stripes = st.stripes;
+  d.n_pcs = c->n_pcs;
+  d.n_warps = st.pw ? c->n_warps : 0;
+  d.launch = st.launch;
+  std::memcpy(out_pod, &d, sizeof d);
+  return NVBT_OK;
+}
+
 int nvbt_launch_count(nvbt_ctx c, uint64_t* n) {
   if (!c || !n) return set_error(NVBT_EINVAL, "null argument");
   *n = c->launches.load();

@@ -11,7 +11,7 @@
 #include <vector>
 
 #include "nvbt.h"
-#include "nvbt_dev.cuh"
+#include "nvbt_hooks.cuh"
 
 namespace nvbt {
 

@@ -63,6 +63,13 @@ class CopySink(C.Structure):
     _fields_ = [("dst", C.c_void_p), ("capacity", C.c_uint64), ("n", C.c_uint64)]
 
 
+class DevState(C.Structure):
+    """nvbt_dev_state (include/nvbt.h): the POD an external instrumented kernel receives by value."""
+    _fields_ = [("version", C.c_uint32), ("tools", C.c_uint32), ("site", C.c_void_p), ("mem", C.c_void_p),
+                ("hist", C.c_void_p), ("per_warp", C.c_void_p), ("stripe_words", C.c_uint64),
+                ("stripes", C.c_uint32), ("n_pcs", C.c_uint32), ("n_warps", C.c_uint32), ("launch", C.c_uint32)]
+
+
 DRAIN_FN = C.CFUNCTYPE(C.c_int, C.c_void_p, C.c_uint64, C.c_void_p)
 
 _P = C.c_void_p
@@ -103,6 +110,7 @@ _sigs = {
     "nvbt_bfs_expand": ([_P, _P, C.c_uint32, _P, _P, C.c_int32, _P, _P, _P], C.c_int),
     "nvbt_bfs_update": ([_P, _P, C.c_uint32, C.c_int32, _P, _P, _P, _P, _P, C.c_int32], C.c_int),
     "nvbt_set_partition": ([_P, C.c_uint32, C.c_uint32], C.c_int),
+    "nvbt_device_state": ([_P, C.c_uint32, _P, C.c_size_t], C.c_int),
     "nvbt_wfft32": ([_P, _P, C.c_uint32, C.c_int32, _P, _P, C.c_int32, C.c_int32], C.c_int),
     "nvbt_wfft32_max_ctas": ([C.c_uint32, C.c_int32, C.c_int32, C.POINTER(C.c_int32)], C.c_int),
 }
@@ -470,3 +478,11 @@ def nvbt_set_partition(ctx, rank, world):
     """Later workload launches through ctx run only `rank`'s share of their CTA grid."""
     _check(_lib.nvbt_set_partition(ctx.handle, rank, world))
     ctx.partition = (rank, world)
+
+
+def nvbt_device_state(ctx, tools):
+    """The nvbt_dev_state POD for one launch of an external kernel instrumented with include/nvbt_dev.cuh
+    (tools: COUNT or BBCOUNT, optionally MEMDIV). Pass C.byref(result) to the kernel's launcher."""
+    st = DevState()
+    _check(_lib.nvbt_device_state(ctx.handle, tools, C.byref(st), C.sizeof(DevState)))
+    return st

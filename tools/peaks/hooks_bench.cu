@@ -5,7 +5,7 @@
 //             -I../../paper_conf_micro_villasnk19_b200/csrc -o hooks_bench hooks_bench.cu
 #include <cstdio>
 #include <cstdlib>
-#include "nvbt_dev.cuh"
+#include "nvbt_hooks.cuh"
 
 #define CK(x) do { cudaError_t e_ = (x); if (e_ != cudaSuccess) { printf("CUDA %s line %d\n", cudaGetErrorString(e_), __LINE__); exit(1);} } while (0)
 using namespace nvbt;
