@@ -114,6 +114,9 @@ class Pool {
   void parallel_for(uint64_t n, const std::function<void(unsigned, uint64_t, uint64_t)>& fn) {
     const unsigned T = size();
     if (T == 1 || n < 4096) { fn(0, 0, n); return; }
+    // one call at a time: the job slot (fn_, n_, pending_) is shared by the workers, so two drains on two
+    // threads (or a digest during a drain) take turns instead of overwriting each other's job
+    std::lock_guard<std::mutex> one(call_);
     {
       std::lock_guard<std::mutex> g(m_);
       fn_ = &fn; n_ = n; parts_ = T; pending_ = T - 1; ++gen_;
@@ -160,7 +163,7 @@ class Pool {
     }
   }
   std::vector<std::thread> workers_;
-  std::mutex m_;
+  std::mutex m_, call_;
   std::condition_variable cv_, done_;
   const std::function<void(unsigned, uint64_t, uint64_t)>* fn_ = nullptr;
   uint64_t n_ = 0, gen_ = 0;

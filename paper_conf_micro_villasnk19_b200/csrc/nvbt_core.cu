@@ -119,6 +119,30 @@ __global__ void fold_kernel(const nvbt_instr_desc* __restrict__ prog, const uint
   }
 }
 
+int device_sms(int dev) {
+  static std::mutex m;
+  static std::vector<int> sms;
+  std::lock_guard<std::mutex> g(m);
+  if (dev < 0) return 148;
+  if ((size_t)dev >= sms.size()) sms.resize((size_t)dev + 1, 0);
+  if (sms[dev] == 0) cudaDeviceGetAttribute(&sms[dev], cudaDevAttrMultiProcessorCount, dev);
+  return sms[dev] > 0 ? sms[dev] : 148;
+}
+
+int func_smem(const void* fn, int dev, size_t bytes) {
+  static std::mutex m;
+  static std::vector<std::pair<const void*, int>> done;   // (function, device) pairs already set
+  std::lock_guard<std::mutex> g(m);
+  for (auto& d : done)
+    if (d.first == fn && d.second == dev) return NVBT_OK;
+  const cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
+  if (e != cudaSuccess)
+    return set_error(NVBT_ECUDA, "cudaFuncSetAttribute(%zu B dynamic shared) on device %d: %s", bytes, dev,
+                     cudaGetErrorString(e));
+  done.emplace_back(fn, dev);
+  return NVBT_OK;
+}
+
 int fold(nvbt_ctx c) {
   NVBT_CUDA(cudaSetDevice(c->device));
   NVBT_CUDA(cudaMemsetAsync(c->out, 0, c->lay.out_words * 8, c->stream));

@@ -119,6 +119,7 @@ struct Hooks {
   unsigned tA[NPC], dT[NPC], wI[NPC], dW[NPC], mN[NPC], mS[NPC], mL[NPC];
   unsigned hS, hL;            // lane-distributed: lane l counts events with S (L) == l + 1
   unsigned pwT, pwW;          // this warp's executed thread / warp instructions (PER_WARP)
+  unsigned iters = 0;         // loop instances since the last spill() (warp-uniform)
   unsigned seq;               // records emitted by this warp in this launch
   unsigned long long hslot;   // device ring: next slot this warp holds, `held` slots from there
   unsigned held;
@@ -592,6 +593,70 @@ struct Hooks {
     }
   }
 
+  // Overflow guard for loops. Every register / lane counter grows by at most 32 per loop instance and
+  // per pc, and the CTA's shared bins hold 8 warps' worth, so all stay far below 2^32 as long as no warp
+  // keeps more than 2^16 instances in them: kernels call tick() once per loop instance, and every 2^16th
+  // call moves this warp's register-mode counters, divergence histogram lanes and per-warp totals
+  // straight into the global 64-bit bins (lane-parallel atomics, warp-uniform branch, taken once per 2^16
+  // instances) and zeroes them. Without it an SGEMM with K >= 2^24 (or a BFS hub of that degree) would
+  // wrap a u32 bin silently.
+  static constexpr unsigned kSpillEvery = 1u << 16;
+  __device__ __forceinline__ void tick() {
+    if constexpr (kOn && !kLoopFree) {
+      if (++iters == kSpillEvery) {
+        iters = 0;
+        spill();
+      }
+    }
+  }
+  __device__ __forceinline__ unsigned long long stripe_off() const {
+    return (unsigned long long)((st.cta_lo + blockIdx.x + blockIdx.y * gridDim.x) & (st.stripes - 1u)) * st.stripe_words;
+  }
+  __device__ __forceinline__ void spill() {
+    if constexpr (kOn && !kLoopFree) {
+      constexpr int LO = Prog::REG_LO, HI = Prog::REG_HI;
+      const unsigned long long so = stripe_off();
+      if constexpr (kCount) {
+        unsigned t = 0, w = 0;
+        retire_sum<LO, HI>(t, w);
+        pwT += t; pwW += w;
+        if (st.pw != nullptr && lane == 0 && gwarp < st.n_warps) {
+          if (pwT) atomicAdd(st.pw + gwarp, (unsigned long long)pwT);
+          if (pwW) atomicAdd(st.pw + st.n_warps + gwarp, (unsigned long long)pwW);
+        }
+        pwT = pwW = 0;
+      }
+      spill_round<LO, HI, LO>(so);
+      zero_range<LO, HI>();
+      if (hS) atomicAdd(st.hist + so + 1 + lane, (unsigned long long)hS);
+      if (hL) atomicAdd(st.hist + so + 34 + lane, (unsigned long long)hL);
+      hS = hL = 0;
+      __syncwarp();
+    }
+  }
+  template <int LO, int HI, int BASE>
+  __device__ __forceinline__ void spill_round(unsigned long long so) {
+    if constexpr (BASE <= HI) {
+      unsigned v[SITE_WORDS] = {0, 0, 0, 0, 0, 0, 0};
+      select_lane<BASE, (HI < BASE + 31 ? HI : BASE + 31), BASE>(v);
+      if (BASE + (int)lane <= HI) {
+        const int pc = BASE + (int)lane;
+        unsigned long long* s = st.site + so + 4 * pc;
+        if (v[0]) atomicAdd(s + 0, (unsigned long long)v[0]);
+        if (v[0] - v[1]) atomicAdd(s + 1, (unsigned long long)(v[0] - v[1]));
+        if (v[2]) atomicAdd(s + 2, (unsigned long long)v[2]);
+        if (v[2] - v[3]) atomicAdd(s + 3, (unsigned long long)(v[2] - v[3]));
+        if (v[4]) {
+          unsigned long long* m = st.mem + so + 3 * pc;
+          atomicAdd(m + 0, (unsigned long long)v[4]);
+          atomicAdd(m + 1, (unsigned long long)v[5]);
+          atomicAdd(m + 2, (unsigned long long)v[6]);
+        }
+      }
+      spill_round<LO, HI, BASE + 32>(so);
+    }
+  }
+
   // CTA epilogue (nvbt_cta_flush): registers -> shared bins -> one global atomic per non-zero bin.
   // Must be reached by every thread of the CTA.
   __device__ __forceinline__ void finish() {
@@ -611,7 +676,7 @@ struct Hooks {
       constexpr int nt = kThreads;
       // this CTA's stripe of the global bins (spreads same-address atomics over st.stripes copies)
       // (logical CTA id: a partitioned launch fills the same stripes as the unpartitioned one)
-      const unsigned long long so = (unsigned long long)((st.cta_lo + blockIdx.x + blockIdx.y * gridDim.x) & (st.stripes - 1u)) * st.stripe_words;
+      const unsigned long long so = stripe_off();
       for (int pc = tid; pc < NPC; pc += nt) {
         const unsigned* b = sb + pc * SITE_WORDS;
         if (b[0] | b[2]) {

@@ -83,4 +83,9 @@ int check_program(nvbt_ctx ctx, const nvbt_instr_desc* prog, int n, const char* 
 void channel_state(nvbt_chan_s* ch, DevState* st);
 bool channel_open(nvbt_chan_s* ch);
 int fold(nvbt_ctx ctx);  // runs the fold kernel and copies the result to host-visible staging
+// Per-device facts and one-time function attributes (both are per device: a process may drive several
+// GPUs). device_sms: SM count of `dev`, cached. func_smem: cudaFuncSetAttribute(MaxDynamicSharedMemorySize)
+// once per (function, device), errors reported as NVBT_ECUDA.
+int device_sms(int dev);
+int func_smem(const void* fn, int dev, size_t bytes);
 }  // namespace nvbt

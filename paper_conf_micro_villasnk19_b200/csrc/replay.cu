@@ -577,11 +577,7 @@ k_rpB(const unsigned long long* __restrict__ addr, unsigned P, const uint8_t* __
 static size_t rpA_smem(unsigned P) { return 16ull * P + ((P + 15ull) & ~15ull) + 512ull * RA_DEPTH * RA_NW; }
 static size_t rpB_smem(unsigned P) { return (((2ull * P + 66 + 3) & ~3ull) + (size_t)RB_NW * RB_WARP_WORDS) * 4; }
 
-static int g_sms = 0;
-static int sm_count(int dev) {
-  if (g_sms == 0) cudaDeviceGetAttribute(&g_sms, cudaDevAttrMultiProcessorCount, dev);
-  return g_sms > 0 ? g_sms : 148;
-}
+static int sm_count(int dev) { return device_sms(dev); }
 
 
 }  // namespace nvbt
@@ -667,12 +663,9 @@ int nvbt_gen_events(nvbt_ctx c, uint64_t seed, uint64_t first, uint64_t n, void*
 
 static int launch_replay4(nvbt_ctx c, const void* d_hdr, const void* d_addr, uint64_t n, const DevState& st) {
   const size_t smem = replay4_smem(c->n_pcs);
-  static bool attr_set = false;
-  if (!attr_set) {
-    NVBT_CUDA(cudaFuncSetAttribute(k_replay4<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)replay4_smem(4096)));
-    NVBT_CUDA(cudaFuncSetAttribute(k_replay4<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)replay4_smem(4096)));
-    attr_set = true;
-  }
+  int rc = func_smem((const void*)k_replay4<false>, c->device, replay4_smem(4096));
+  if (!rc) rc = func_smem((const void*)k_replay4<true>, c->device, replay4_smem(4096));
+  if (rc) return rc;
   const unsigned long long kMaxPerLaunch = 1ull << 30;
   const int sms = sm_count(c->device);
   for (uint64_t off = 0; off < n; off += kMaxPerLaunch) {
@@ -697,13 +690,10 @@ static unsigned long long staged_cap(size_t bytes) {
 
 static int launch_staged(nvbt_ctx c, const void* d_hdr, const void* d_addr, uint64_t n, const DevState& st,
                          void* scratch, size_t scratch_bytes) {
-  static bool attr_set = false;
-  if (!attr_set) {
-    NVBT_CUDA(cudaFuncSetAttribute(k_rpA<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)rpA_smem(4096)));
-    NVBT_CUDA(cudaFuncSetAttribute(k_rpA<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)rpA_smem(4096)));
-    NVBT_CUDA(cudaFuncSetAttribute(k_rpB, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)rpB_smem(4096)));
-    attr_set = true;
-  }
+  int arc = func_smem((const void*)k_rpA<false>, c->device, rpA_smem(4096));
+  if (!arc) arc = func_smem((const void*)k_rpA<true>, c->device, rpA_smem(4096));
+  if (!arc) arc = func_smem((const void*)k_rpB, c->device, rpB_smem(4096));
+  if (arc) return arc;
   const int sms = sm_count(c->device);
   const bool memdiv = (c->flags & NVBT_MEMDIV) != 0;
   const unsigned long long cap = staged_cap(scratch_bytes);

@@ -186,6 +186,7 @@ __global__ void __launch_bounds__(256) k_wfft(const float2* __restrict__ x, floa
                                                              h.template at<S + 2>(m1);
                                                              h.template at<S + 3>(m1);
                                                              h.template at<S + 4>(m1, k + 1 < kw);  // @P1 BRA
+      h.tick();
     }
   }
   asm volatile("cp.async.wait_group 0;" ::: "memory");

@@ -5,6 +5,7 @@
 // reached by all 32 lanes and A/P are exact ballots (EM §1, reading R-15). Loops whose trip count
 // varies per lane run warp-uniformly to the warp's maximum (SIMT-stack / IPDOM semantics). The
 // template parameter T selects the instrumentation variant; T = 0 is the uninstrumented baseline.
+#include <tuple>
 #include <type_traits>
 
 #include "nvbt_internal.h"
@@ -75,6 +76,7 @@ __global__ void __launch_bounds__(256, 6) k_sgemm(const float* __restrict__ A, c
                                                h.template at<13>(m1);
                                                h.template at<14>(m1);
                                                h.template at<15>(m1, k + 1 < K);  // @P1 BRA
+      h.tick();
     }
   }
   float* pc = C + (size_t)row * N + col;
@@ -130,6 +132,7 @@ __global__ void __launch_bounds__(256) k_bfs_expand(const int* __restrict__ rowp
                                                h.template at<20>(m3, p4);  // @P4 BRA loop
     if (in_loop) e = e1;
     in_loop = in_loop && p4;
+    h.tick();
   }
                                                h.template at<21>(m1);
   h.finish();
@@ -203,6 +206,38 @@ __global__ void __launch_bounds__(256) k_stencil(const float* __restrict__ in, f
 }  // namespace nvbt
 
 using namespace nvbt;
+
+// Dynamic shared memory that caps k_stencil<T> (256 threads) at 3 CTAs per SM on `dev`: 4 x (dyn + static
+// + per-block reserved) must exceed the SM's shared memory, 3 x must fit. Derived from the kernel's own
+// static size and the device's limits, checked with the occupancy calculator, cached per (kernel, device).
+static int stencil_pad(const void* fn, int dev, size_t* dyn) {
+  static std::mutex m;
+  static std::vector<std::tuple<const void*, int, size_t>> cache;
+  {
+    std::lock_guard<std::mutex> g(m);
+    for (auto& c : cache)
+      if (std::get<0>(c) == fn && std::get<1>(c) == dev) { *dyn = std::get<2>(c); return NVBT_OK; }
+  }
+  cudaFuncAttributes fa{};
+  int per_sm = 0, reserved = 0;
+  NVBT_CUDA(cudaFuncGetAttributes(&fa, fn));
+  NVBT_CUDA(cudaDeviceGetAttribute(&per_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, dev));
+  NVBT_CUDA(cudaDeviceGetAttribute(&reserved, cudaDevAttrReservedSharedMemoryPerBlock, dev));
+  const size_t used = fa.sharedSizeBytes + (size_t)reserved;
+  const size_t quarter = (size_t)per_sm / 4 + 128;              // 4 CTAs of this size exceed the SM
+  const size_t d = quarter > used ? ((quarter - used + 127) & ~size_t(127)) : 0;
+  if (3 * (d + used) > (size_t)per_sm) return set_error(NVBT_ECUDA, "stencil pad: 3 CTAs do not fit (%zu B)", d);
+  int rc = func_smem(fn, dev, d);
+  if (rc) return rc;
+  int blocks = 0;
+  NVBT_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks, fn, 256, d));
+  if (blocks > 3 || blocks < 1)
+    return set_error(NVBT_ECUDA, "stencil pad %zu B gives %d CTAs per SM, expected <= 3", d, blocks);
+  std::lock_guard<std::mutex> g(m);
+  cache.emplace_back(fn, dev, d);
+  *dyn = d;
+  return NVBT_OK;
+}
 
 extern "C" {
 
@@ -304,25 +339,22 @@ int nvbt_stencil(nvbt_ctx ctx, void* stream, uint32_t tools, const float* in, fl
   if (rc) return rc;
   if (lc.n_ctas == 0) return NVBT_OK;
   const dim3 block(32, 8);
+  int pad_rc = NVBT_OK;
   rc = dispatch_trace(tools, lc.st.no_wait != 0u, [&](auto tag) {
     constexpr uint32_t T = decltype(tag)::value;
     size_t dyn = 0;
     if constexpr ((T & TOOL_TRACE) && !(T & TOOL_TRACE_DEV)) {
       // Host-channel producer: at most 3 CTAs (24 warps) per SM, enforced by padding dynamic shared memory
-      // (4 CTAs would need more than the SM has). The PCIe link is saturated; fewer warps fencing and
-      // writing partial lines at once move more records (C4: 147 -> 151 M records/s, compact 205 -> 214;
-      // 6 CTAs per SM: 134 / 182).
-      static const size_t pad = [&] {
-        int per_sm = 0;
-        cudaDeviceGetAttribute(&per_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, ctx->device);
-        const size_t p = (size_t)per_sm * 2 / 7 - 8192;
-        cudaFuncSetAttribute(k_stencil<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p);
-        return p;
-      }();
-      dyn = pad;
+      // just past a quarter of the SM's shared memory (so 4 CTAs never fit, and as much as possible stays
+      // L1). The PCIe link is saturated; fewer warps fencing and writing partial lines at once move more
+      // records (C4 measured in round 1: uncapped 147 M records/s, 3 CTAs 151, 2 CTAs 154 / compact 205,
+      // 214, 199-221; 6 CTAs per SM 134 / 182).
+      pad_rc = stencil_pad((const void*)k_stencil<T>, ctx->device, &dyn);
+      if (pad_rc) return;
     }
     k_stencil<T><<<lc.grid, block, dyn, lc.stream>>>(in, out, n, lc.st);
   });
+  if (pad_rc) return pad_rc;
   return rc ? rc : done(ctx, 1);
 }
 
