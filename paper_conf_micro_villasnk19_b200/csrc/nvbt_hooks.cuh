@@ -594,13 +594,13 @@ struct Hooks {
   }
 
   // Overflow guard for loops. Every register / lane counter grows by at most 32 per loop instance and
-  // per pc, and the CTA's shared bins hold 8 warps' worth, so all stay far below 2^32 as long as no warp
-  // keeps more than 2^16 instances in them: kernels call tick() once per loop instance, and every 2^16th
-  // call moves this warp's register-mode counters, divergence histogram lanes and per-warp totals
-  // straight into the global 64-bit bins (lane-parallel atomics, warp-uniform branch, taken once per 2^16
-  // instances) and zeroes them. Without it an SGEMM with K >= 2^24 (or a BFS hub of that degree) would
-  // wrap a u32 bin silently.
-  static constexpr unsigned kSpillEvery = 1u << 16;
+  // per pc, and the CTA's shared bins hold 8 warps' worth, so all stay below 2^28 as long as no warp
+  // keeps more than 2^20 instances in them: kernels run their loops in chunks of kSpillEvery instances
+  // and call spill() between chunks (or tick() once per instance), which moves this warp's register-mode
+  // counters, divergence histogram lanes and per-warp totals straight into the global 64-bit bins
+  // (lane-parallel atomics) and zeroes them. Without it an SGEMM with K >= 2^24 (or a BFS hub of that
+  // degree) would wrap a u32 bin silently.
+  static constexpr unsigned kSpillEvery = 1u << 20;
   __device__ __forceinline__ void tick() {
     if constexpr (kOn && !kLoopFree) {
       if (++iters == kSpillEvery) {

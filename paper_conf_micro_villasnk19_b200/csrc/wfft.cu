@@ -159,8 +159,7 @@ __global__ void __launch_bounds__(256) k_wfft(const float2* __restrict__ x, floa
 #pragma unroll
     for (int d = 0; d < kRing; ++d)
       ring_copy(lane, slot0 + 256u * d, x + (size_t)(f0 + d * W) * 32, d < kw);
-#pragma unroll 1
-    for (int k = 0; k < kw; ++k) {                    // warp-uniform: one loop instance per transform
+    auto instance = [&](int k) {                      // warp-uniform: one loop instance per transform
       const int ff = f0 + k * W;
       const unsigned sl = (unsigned)k & (kRing - 1u);
       const float2* px = x + (size_t)ff * 32 + lane;        h.template at<LO>(m1);
@@ -186,7 +185,19 @@ __global__ void __launch_bounds__(256) k_wfft(const float2* __restrict__ x, floa
                                                              h.template at<S + 2>(m1);
                                                              h.template at<S + 3>(m1);
                                                              h.template at<S + 4>(m1, k + 1 < kw);  // @P1 BRA
-      h.tick();
+    };
+    constexpr int kChunk = (int)decltype(h)::kSpillEvery;
+    if (kw <= kChunk) {                               // the u32 counters cannot wrap: the plain loop
+#pragma unroll 1
+      for (int k = 0; k < kw; ++k) instance(k);
+    } else {                                          // chunks of kChunk instances, counters spilled between
+#pragma unroll 1
+      for (int k0 = 0; k0 < kw; k0 += kChunk) {
+        const int k1 = kw - k0 > kChunk ? k0 + kChunk : kw;
+#pragma unroll 1
+        for (int k = k0; k < k1; ++k) instance(k);
+        if (k1 < kw) h.spill();
+      }
     }
   }
   asm volatile("cp.async.wait_group 0;" ::: "memory");

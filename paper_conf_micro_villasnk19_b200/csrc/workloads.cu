@@ -68,7 +68,7 @@ __global__ void __launch_bounds__(256, 6) k_sgemm(const float* __restrict__ A, c
   if (__any_sync(FULL, live)) {
     const float* pa = A + (size_t)row * K;
     const float* pb = B + col;
-    for (int k = 0; k < K; ++k) {
+    auto instance = [&](int k) {               // BB2, instance k
       float x = 0.f, y = 0.f;
       if (live) x = pa[k];                     h.template at<10>(m1, true, (unsigned long long)(pa + k));
       if (live) y = pb[(size_t)k * N];         h.template at<11>(m1, true, (unsigned long long)(pb + (size_t)k * N));
@@ -76,7 +76,16 @@ __global__ void __launch_bounds__(256, 6) k_sgemm(const float* __restrict__ A, c
                                                h.template at<13>(m1);
                                                h.template at<14>(m1);
                                                h.template at<15>(m1, k + 1 < K);  // @P1 BRA
-      h.tick();
+    };
+    constexpr int kChunk = (int)Hooks<T, ProgSgemm>::kSpillEvery;
+    if (K <= kChunk) {                         // the u32 counters cannot wrap: the plain loop
+      for (int k = 0; k < K; ++k) instance(k);
+    } else {                                   // chunks of kChunk instances, counters spilled in between
+      for (int k0 = 0; k0 < K; k0 += kChunk) {
+        const int k1 = K - k0 > kChunk ? k0 + kChunk : K;
+        for (int k = k0; k < k1; ++k) instance(k);
+        if (k1 < K) h.spill();
+      }
     }
   }
   float* pc = C + (size_t)row * N + col;
@@ -116,7 +125,7 @@ __global__ void __launch_bounds__(256) k_bfs_expand(const int* __restrict__ rowp
   h.template retire<8, 12>();
   bool in_loop = front && !p2;
   int e = start;
-  while (__any_sync(FULL, in_loop)) {          // warp-uniform edge loop; instance k has e = start + k
+  auto instance = [&]() {                      // warp-uniform edge loop; instance k has e = start + k
     const auto m3 = h.active(in_loop);         // BB3 and BB5 of this instance
     int nb = 0;
     if (in_loop) nb = colidx[e];               h.template at<13>(m3, true, (unsigned long long)(colidx + e));
@@ -132,7 +141,20 @@ __global__ void __launch_bounds__(256) k_bfs_expand(const int* __restrict__ rowp
                                                h.template at<20>(m3, p4);  // @P4 BRA loop
     if (in_loop) e = e1;
     in_loop = in_loop && p4;
-    h.tick();
+  };
+  constexpr int kChunk = (int)Hooks<T, ProgBfs>::kSpillEvery;
+  if (!__any_sync(FULL, in_loop && end - start > kChunk)) {   // degrees <= kChunk: the plain loop
+    while (__any_sync(FULL, in_loop)) instance();
+  } else {                                     // a hub: chunks of kChunk instances, counters spilled
+    for (;;) {
+      int it = 0;
+      while (it < kChunk && __any_sync(FULL, in_loop)) {
+        instance();
+        ++it;
+      }
+      if (!__any_sync(FULL, in_loop)) break;
+      h.spill();
+    }
   }
                                                h.template at<21>(m1);
   h.finish();

@@ -1,7 +1,7 @@
 """Exactness of the privatised counters past 2^32: per-site counters live in u32
 registers and CTA shared bins before the 64-bit global flush, so long loops must spill them before they
 can wrap (nvbt_hooks.cuh Hooks::tick, every 2^16 loop instances). SGEMM with M = 32, N = 8 (one CTA, 8
-warps) and K = 2^24 + 3: every warp runs 6K + 12 > 10^8 warp instructions, its executed-thread count
+warps) and K = 2^25 + 3: every warp runs 6K + 12 > 2 x 10^8 warp instructions, its executed-thread count
 32 (6K + 10) > 2^32, and the CTA's A-load sector sum 8 x 32K > 2^32. All results equal the closed form
 (EM §3.2) and the C oracle exactly."""
 import numpy as np
@@ -18,7 +18,7 @@ pytestmark = [pytest.mark.gpu, pytest.mark.slow]
 def test_sgemm_k_beyond_u32(nvbt, tools):
     import torch
     nb = nvbt.nvbt
-    M, N, K = 32, 8, (1 << 24) + 3
+    M, N, K = 32, 8, (1 << 25) + 3
     t = 0
     for x in tools.split("|"):
         t |= getattr(nb, "TOOL_" + x)
@@ -43,6 +43,6 @@ def test_sgemm_k_beyond_u32(nvbt, tools):
     assert g["hS"][32] == W * K + W and g["hS"][1] == W * K and g["hL"][8] == W
     r = co.sgemm(programs.sgemm(), M, N, K, A.data_ptr(), B.data_ptr(), Cm.data_ptr(), per_warp=True)
     assert_same(g, r, ["counts", "H_t", "H_w", "Ent_w", "Ent_t", "Ins_w", "Ins_t", "mem_n", "mem_S", "mem_L",
-                       "hS", "hL", "PW_T", "PW_W"], f"SGEMM K = 2^24 + 3 {tools}")
+                       "hS", "hL", "PW_T", "PW_W"], f"SGEMM K = 2^25 + 3 {tools}")
     # fp32 accumulation of K ones saturates at 2^24 (2^24 + 1 rounds to even): the computed product
     assert torch.all(Cm == float(1 << 24))
