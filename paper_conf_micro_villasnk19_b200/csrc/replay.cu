@@ -126,6 +126,9 @@ __device__ __forceinline__ void sts_u64(unsigned a, unsigned long long v) {
 constexpr int L4_NW = 32;  // warps per CTA (1 CTA per SM)
 constexpr int L4_WARP_WORDS = SCRATCH_WORDS + 4 + 8 * 64 + 32;   // scratch + pad + 8 stage rows + row sources
 
+__device__ __forceinline__ void sts_u8(unsigned a, unsigned v) {
+  asm volatile("st.shared.u8 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
 __device__ __forceinline__ unsigned lds_u8(unsigned a) {
   unsigned v;
   asm volatile("ld.shared.u8 %0, [%1];" : "=r"(v) : "r"(a));
@@ -281,11 +284,20 @@ static size_t replay4_smem(unsigned P) {
 // Extra traffic: 16 B per executed memory event (list write + read), ~5 % of the algorithmic bytes.
 constexpr int RA_NW = 20;     // pass A warps per CTA (one list region per warp)
 constexpr int RB_NW = 20;     // pass B warps per CTA (warp w of pass B analyses region w)
+#ifndef NVBT_RPB_EXPERIMENT
+#define NVBT_RPB_EXPERIMENT 0   // timing experiments (tools/replay_ab.py), never in a product build
+#endif
+#ifndef NVBT_RPB_TAGS
+#define NVBT_RPB_TAGS 1        // slow rows by tag arrays (0: round-1 atomics + reductions, for A/B)
+#endif
 constexpr int RA_CTAS_PER_SM = 2;   // pass A CTAs per SM
 constexpr int RA_DEPTH = 4;   // pass A header tiles in flight per warp
 constexpr int RB_ROWS = 16;   // slots per stage
 constexpr int RB_STAGES = 2;
-constexpr int RB_WARP_WORDS = RB_STAGES * (RB_ROWS * 64 + 2 * RB_ROWS) + SCRATCH_WORDS;
+// per-warp scratch, 1280 B: the slow rows' tag arrays (1 KB sector / hash tags + 256 B line tags); the
+// A/B build without them (NVBT_RPB_TAGS=0) uses its first SCRATCH_WORDS words as sectors_lines_cls scratch
+constexpr int RB_SCR2 = 128;
+constexpr int RB_WARP_WORDS = RB_STAGES * (RB_ROWS * 64 + 2 * RB_ROWS) + SCRATCH_WORDS + RB_SCR2;
 constexpr size_t RS_COUNTS_BYTES = 65536;   // u32 per pass-A warp (<= 16384 warps)
 static_assert(RB_WARP_WORDS % 4 == 0, "16 B aligned warp areas");
 
@@ -392,6 +404,7 @@ __device__ __forceinline__ void inc_if_gt(unsigned& c, unsigned x) {
 __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsigned lane, unsigned lanebit,
                                            unsigned s_scr, unsigned s_sS, unsigned s_sL, unsigned s_hist) {
   const unsigned j = lane & 15u, h = lane >> 4, sw = j & 7u;
+  constexpr unsigned kWin = NVBT_RPB_TAGS ? 512u : 1024u;   // window sectors (tags build: two rows in flight)
   unsigned E, pc;
   lds_v2(meta + 8u * j, E, pc);
   const unsigned Eh = h ? E >> 16 : E & 0xffffu;
@@ -400,9 +413,10 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
   unsigned f_lo, f_hi;
   lds_v2(rowb + 16u * ((f >> 1) ^ sw) + 8u * (f & 1u), f_lo, f_hi);
   unsigned prev = f_lo, hb = 0, bs = 0, bl = 0, mn = f_lo, mx = f_lo;
+  unsigned sbits = 0;   // (tags build) the 1 KB-word sector bits of the scanned addresses (bit (a >> 5) & 31)
   bool viol = false;
 #pragma unroll
-  for (int q = 0; q < 8; ++q) {
+  for (int q = 0; q < ((NVBT_RPB_EXPERIMENT & 2) ? 1 : 8); ++q) {   // (experiment 2: scan 2 addresses only)
     uint4 v;
     lds_v4(rowb + 16u * ((8u * h + q) ^ sw), v);
 #pragma unroll
@@ -417,6 +431,9 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
       inc_if_gt<127>(bl, x);
       mn = min(mn, lo);
       mx = max(mx, lo);
+#if NVBT_RPB_TAGS
+      sbits |= __funnelshift_l(0u, 1u, lo >> 5);   // 1 << ((lo >> 5) & 31): one SHF.L.W
+#endif
       prev = lo;
     }
   }
@@ -428,6 +445,9 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
   const unsigned o_hi = __shfl_xor_sync(FULL, f_hi, 16);
   const unsigned o_mn = __shfl_xor_sync(FULL, mn, 16);
   const unsigned o_mx = __shfl_xor_sync(FULL, mx, 16);
+#if NVBT_RPB_TAGS
+  const unsigned o_sb = __shfl_xor_sync(FULL, sbits, 16);
+#endif
   const bool other = (o_pack >> 18) != 0u;
   unsigned S = 1u + bs + (o_pack & 0xffu), L = 1u + bl + ((o_pack >> 8) & 0xffu);
   bool hb_row = hb != 0u || ((o_pack >> 17) & 1u) != 0u;
@@ -443,14 +463,117 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
   const unsigned rmn = mine ? (other ? min(mn, o_mn) : mn) : o_mn;
   const unsigned rmx = mine ? (other ? max(mx, o_mx) : mx) : o_mx;
   const unsigned wbase = (rmn >> 5) & ~31u;
-  const unsigned cls = hb_row ? 2u : (rmn >> 10) == (rmx >> 10) ? 0u : ((rmx >> 5) - wbase < 1024u ? 1u : 2u);
+  // classes: 0 = one 1 KB word, 1 = a window of kWin sectors from wbase, 2 = anything else
+  const unsigned cls = hb_row ? 2u : (rmn >> 10) == (rmx >> 10) ? 0u : ((rmx >> 5) - wbase < kWin ? 1u : 2u);
   const bool own = h == 0u && E != 0u;
-  // rows that are not monotone within one 4 GB region: exact warp-cooperative paths, one loop per class of
-  // the row's address range (one 1 KB word / a 32 KB window / anything else); lane l reads address l
+  // rows that are not monotone within one 4 GB region: exact paths, one loop per class of the row's
+  // address range (one 1 KB word / a 32 KB window / anything else)
+  // (NVBT_RPB_EXPERIMENT bits 1, 4, 8, 16: timing experiments only, wrong results: drop all / class-0 /
+  // class-1 / class-2 slow rows)
+#if NVBT_RPB_TAGS
+  if (slow && cls == 0u) {   // one 1 KB word: the scan's sector bits are exact (no loop below)
+    const unsigned word = (mine ? sbits : 0u) | (other ? o_sb : 0u);
+    const unsigned g = word | (word >> 1) | (word >> 2) | (word >> 3);
+    S = __popc(word);
+    L = __popc(g & 0x11111111u);
+  }
+  const unsigned cm0 = 0u;
+#else
+  const unsigned cm0 = (NVBT_RPB_EXPERIMENT & 5) ? 0u : __ballot_sync(FULL, own && slow && cls == 0u);
+#endif
+  const unsigned cm1 = (NVBT_RPB_EXPERIMENT & 9) ? 0u : __ballot_sync(FULL, own && slow && cls == 1u);
+  const unsigned cm2 = (NVBT_RPB_EXPERIMENT & 17) ? 0u : __ballot_sync(FULL, own && slow && cls == 2u);
+#if NVBT_RPB_TAGS
+  // Exact distinct counts without atomics or reductions: every active lane stores its lane id (u8) at its
+  // key's slot of a per-warp tag array and reads the slot back after a __syncwarp; of the lanes sharing a
+  // slot exactly one (the last writer) reads its own id, so the number of distinct slots = popc(ballot(own
+  // id read)). Stale tags from earlier rows never matter: every lane that reads a slot wrote it this row.
+  //  * rows within one 1 KB word (class 0) are settled from the scan's sector bits above;
+  //  * window rows (all sectors of E in the 512-sector window from wbase, upper words equal; class 1):
+  //    the slot is the sector's offset in the window (512 B of tags) and, for lines, offset >> 2 (128 B):
+  //    S and L exactly; two rows per iteration;
+  //  * wide rows (class 2): all lines distinct? slots = a hash of the line into 1280 buckets, up to three
+  //    independent hashes; all lanes owning their slot proves every line (hence sector) distinct: S = L =
+  //    |E|. Rows that collide three times (~3 %) take an exact bitonic sort of the sector keys.
+  const unsigned stag = s_scr, ltag = s_scr + 1024u;
   const unsigned l8 = 8u * lane;
-  unsigned m0 = __ballot_sync(FULL, own && slow && cls == 0u);
-  unsigned m1 = __ballot_sync(FULL, own && slow && cls == 1u);
-  unsigned m2 = __ballot_sync(FULL, own && slow && cls == 2u);
+  const unsigned long long kInvalid = ~0ull;
+  unsigned mw = cm0 | cm1, mwide = cm2;
+  // two window rows per iteration (independent chains; 512-sector window and 128 line tags per row)
+  while (mw) {
+    const unsigned ra = 31u - __clz(mw);
+    mw ^= 1u << ra;
+    const bool two = mw != 0u;
+    const unsigned rb = two ? 31u - __clz(mw) : ra;
+    if (two) mw ^= 1u << rb;
+    const unsigned ea = __shfl_sync(FULL, E, ra), wa = __shfl_sync(FULL, wbase, ra);
+    const unsigned eb = __shfl_sync(FULL, E, rb), wbb = __shfl_sync(FULL, wbase, rb);
+    const unsigned la = lds_u32(stage + 256u * ra + (l8 ^ (16u * (ra & 7u))));
+    const unsigned lb = lds_u32(stage + 256u * rb + (l8 ^ (16u * (rb & 7u))));
+    const bool acta = (ea >> lane) & 1u, actb = two && ((eb >> lane) & 1u);
+    const unsigned oa = (la >> 5) - wa, ob = (lb >> 5) - wbb;
+    if (acta) {
+      sts_u8(stag + oa, lane);
+      sts_u8(ltag + (oa >> 2), lane);
+    }
+    if (actb) {
+      sts_u8(stag + 512u + ob, lane);
+      sts_u8(ltag + 128u + (ob >> 2), lane);
+    }
+    __syncwarp();
+    const bool fsa = acta && lds_u8(stag + oa) == lane, fla = acta && lds_u8(ltag + (oa >> 2)) == lane;
+    const bool fsb = actb && lds_u8(stag + 512u + ob) == lane, flb = actb && lds_u8(ltag + 128u + (ob >> 2)) == lane;
+    const unsigned sa = __popc(__ballot_sync(FULL, fsa)), lxa = __popc(__ballot_sync(FULL, fla));
+    const unsigned sb2 = __popc(__ballot_sync(FULL, fsb)), lxb = __popc(__ballot_sync(FULL, flb));
+    S = lane == ra ? sa : (two && lane == rb) ? sb2 : S;
+    L = lane == ra ? lxa : (two && lane == rb) ? lxb : L;
+    __syncwarp();                                  // reads done before the next rows' stores
+  }
+  while (mwide) {
+    const unsigned src = 31u - __clz(mwide);
+    mwide ^= 1u << src;
+    const unsigned es = __shfl_sync(FULL, E, src);
+    unsigned long long a;
+    asm volatile("ld.shared.u64 %0, [%1];" : "=l"(a) : "r"(stage + 256u * src + (l8 ^ (16u * (src & 7u)))) : "memory");
+    const bool act = (es >> lane) & 1u;
+    const unsigned long long line = a >> 7;
+    const unsigned x0 = (unsigned)line, x1 = (unsigned)(line >> 32);
+    bool ok = false;
+#pragma unroll
+    for (int round = 0; round < 3 && !ok; ++round) {   // warp-uniform
+      const unsigned hsh = (x0 * (0x9E3779B1u + 0x6A09E666u * round) ^ x1 * (0x85EBCA77u + 0x3C6EF372u * round)) + round;
+      const unsigned hb = __umulhi(hsh * 0xC2B2AE3Du + (hsh >> 15), 1280u);
+      if (act) sts_u8(stag + hb, lane);
+      __syncwarp();
+      ok = __all_sync(FULL, !act || lds_u8(stag + hb) == lane);
+      __syncwarp();
+    }
+    unsigned sx, lx;
+    if (ok) {
+      sx = lx = __popc(es);
+    } else {                                       // exact: bitonic sort of the sector keys of E
+      unsigned long long k = act ? a >> 5 : kInvalid;
+#pragma unroll
+      for (unsigned kk = 2; kk <= 32; kk <<= 1) {
+#pragma unroll
+        for (unsigned jj = kk >> 1; jj > 0; jj >>= 1) {
+          const unsigned long long o = __shfl_xor_sync(FULL, k, jj);
+          const bool up = (lane & kk) == 0u, lower = (lane & jj) == 0u;
+          k = (lower == up) ? (o < k ? o : k) : (o > k ? o : k);
+        }
+      }
+      const unsigned long long pk = __shfl_up_sync(FULL, k, 1);
+      const bool valid = k != kInvalid;
+      sx = __popc(__ballot_sync(FULL, valid && (lane == 0u || pk != k)));
+      lx = __popc(__ballot_sync(FULL, valid && (lane == 0u || (pk >> 2) != (k >> 2))));
+    }
+    S = lane == src ? sx : S;
+    L = lane == src ? lx : L;
+  }
+#else
+  // one row per iteration, warp-cooperative; lane l reads address l
+  unsigned m0 = cm0, m1 = cm1, m2 = cm2;
+  const unsigned l8 = 8u * lane;
   while (m0) {
     const unsigned src = 31u - __clz(m0);
     m0 ^= 1u << src;
@@ -479,6 +602,7 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
     S = lane == src ? r.x : S;
     L = lane == src ? r.y : L;
   }
+#endif
   red_shared_add_if(own, s_sS + 4u * pc, S);
   red_shared_add_if(own, s_sL + 4u * pc, L);
   red_shared_add_if(own, s_hist + 4u * S, 1u);          // hS[S]
@@ -496,7 +620,7 @@ k_rpB(const unsigned long long* __restrict__ addr, unsigned P, const uint8_t* __
   constexpr unsigned kScr0 = RB_STAGES * (RB_ROWS * 64 + 2 * RB_ROWS);
   for (unsigned i = threadIdx.x; i < RB_NW * RB_WARP_WORDS; i += blockDim.x) {
     const unsigned o = i % RB_WARP_WORDS;
-    sWarpAll[i] = o >= kScr0 ? scratch_init_word(o - kScr0) : 0u;
+    sWarpAll[i] = o >= kScr0 + SCRATCH_WORDS ? 0xffffffffu : o >= kScr0 ? scratch_init_word(o - kScr0) : 0u;
   }
   __syncthreads();
   const unsigned lane = lane_id(), lanebit = 1u << lane;

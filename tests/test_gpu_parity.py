@@ -349,7 +349,9 @@ def test_replay_merge_equals_single(nvbt, staged):
 def _adversarial_stream(n, seed):
     """Handcrafted replay events stressing every sectors_lines() path: monotone runs, 32 KB bitmap window
     edges (incl. keys below the first lane), 32-bit relative sort, 64-bit sort, partial and sparse masks,
-    duplicate sectors, line-boundary straddles, widths 1..16."""
+    duplicate sectors, line-boundary straddles, widths 1..16; wide rows (upper address words differ) with
+    repeated addresses and with lines shared by lane pairs (the hashed all-distinct test must fail them and
+    the exact fallback count them)."""
     rng = np.random.default_rng(seed)
     prog = programs.replay()
     mem_pcs = np.nonzero(programs.is_mem(prog))[0]
@@ -361,19 +363,20 @@ def _adversarial_stream(n, seed):
                  rng.integers(0, 1 << 32, size=n, dtype=np.uint64).astype(np.uint32))
     lane = np.arange(32, dtype=np.int64)[None, :]
     base = (rng.integers(1 << 20, 1 << 40, size=(n, 1)) & ~127).astype(np.int64)
-    kind = rng.integers(0, 9, size=(n, 1))
+    kind = rng.integers(0, 10, size=(n, 1))
     span = rng.choice([32, 1024 * 32 - 1, 1024 * 32, 1024 * 32 + 32, 1 << 20, 1 << 38], size=(n, 1))
     r = rng.integers(0, 1 << 62, size=(n, 32)) % span - span // 2       # symmetric around base
     stride = rng.choice([0, 1, 4, 8, 16, 31, 32, 33, 64, 127, 128, 129, 4096, 1 << 20], size=(n, 1))
     off = rng.integers(0, 4096, size=(n, 1))                            # unaligned progression starts
     hb = ((base >> 32) + 1) << 32                                       # next 4 GB boundary
-    addr = np.select([kind == 0, kind == 1, kind == 2, kind == 3, kind == 4, kind == 5],
+    addr = np.select([kind == 0, kind == 1, kind == 2, kind == 3, kind == 4, kind == 5, kind == 6],
                      [base + off + lane * stride,                         # monotone / arithmetic progression
                       base - lane * stride,                               # decreasing
                       base + (r // 4) * 4,                                # window / wide random
                       base + (lane % 3) * 32 + 124,                       # duplicates straddling lines
                       base + r[:, (lane[0] * 7) % 8],                     # wide random with repeats
-                      hb - 8 * stride + lane * stride],                   # progression across a 4 GB line
+                      hb - 8 * stride + lane * stride,                    # progression across a 4 GB line
+                      base + (lane % 2) * 32 + (lane // 2) * (1 << 33)],  # lines shared by lane pairs, 4 GB apart
                      base + r)
     addr = np.clip(addr, 0, (1 << 62) - 1).astype(np.uint64)
     return pc.astype(np.int64), warp.astype(np.int64), A, P, addr
