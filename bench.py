@@ -537,9 +537,10 @@ def run_c3(args, torch, nb, dr, rank, world, local, steps):
 
 
 # --------------------------------------------------------------------------- C4 stencil + channel
-def run_c4(args, torch, nb, dr, rank, world, local, steps):
+def run_c4(args, torch, nb, dr, rank, world, local, steps, compact=False):
     """C4: 8192^2 5-point stencil x 100 iterations, every executed global LD/ST traced through the pinned
-    host channel (288 B records, EM §5) and digested on the host; a step is the whole traced run. The
+    host channel (288 B records, EM §5; with `compact` the F3 transport of EM §5.1, decoded back to the
+    same records on the host) and digested on the host; a step is the whole traced run. The
     drain runs on a host thread while the iterations are enqueued (N > 1: row slabs with P2P halos, one
     channel per rank). Device time from the first launch to the last kernel's end (the producers wait on
     the host ring, so it includes the transport), max over ranks."""
@@ -550,8 +551,8 @@ def run_c4(args, torch, nb, dr, rank, world, local, steps):
         nb.nvbt_set_partition(ctx, rank, world)
     x0 = torch.from_numpy(uniform_f32((n, n), 4)).cuda()
     buf0, buf1 = x0.clone(), torch.empty_like(x0)
-    ring = torch.empty(nb.nvbt_channel_bytes(args.ring_records), dtype=torch.uint8, pin_memory=True)
-    ch = nb.nvbt_channel_open(ctx, ring)
+    ring = torch.empty(nb.nvbt_channel_bytes(args.ring_records, compact=compact), dtype=torch.uint8, pin_memory=True)
+    ch = nb.nvbt_channel_open(ctx, ring, compact=compact)
     if world > 1:
         run = lambda t, it: dr.run_stencil_dist(ctx, t, buf0, buf1, n, it, rank, world, gather=False)
     else:
@@ -598,12 +599,15 @@ def run_c4(args, torch, nb, dr, rank, world, local, steps):
     expect = iters * (4 * G + 6 * G * (n - 2))                   # SURVEY I-3 closed form
     dropped_all = sum_over_ranks(dropped, world)
     ok = int(recs) == expect and dropped_all == 0
-    gbs = recs * (288 + 4) / t_dev / 1e9 / world                 # records + commit tags per GPU link
+    slot = nb.nvbt_channel_slot_bytes(compact)                     # ring stride per transport slot
+    gbs = recs * (slot + 4) / t_dev / 1e9 / world                  # slots + commit tags per GPU link
     peak = d2h_peak()
     nb.nvbt_channel_close(ch)
     del ring
-    return {"value": recs / t_dev, "unit": "records/s", "steps": steps,
-            "workload": f"C4 stencil {n}^2 x {iters}, tools TRACE, 288 B records to pinned host, digest drain",
+    transport = "compact slots (EM 5.1)" if compact else "288 B records"
+    return {"value": recs / t_dev if ok else None, "unit": "records/s", "steps": steps,
+            "workload": f"C4 stencil {n}^2 x {iters}, tools TRACE, {transport} to pinned host, digest drain",
+            "records_per_s_measured": recs / t_dev, "transport_slot_bytes": slot,
             "records_per_run": int(recs), "records_expected": expect, "dropped": int(dropped_all),
             "slowdown": t_dev / tp, "plain_ms": 1e3 * tp, "traced_s": t_dev, "traced_wall_s": t_wall,
             "ring_slots": args.ring_records,
@@ -611,7 +615,7 @@ def run_c4(args, torch, nb, dr, rank, world, local, steps):
                             f"mismatch: {int(recs)} records, expected {expect}, dropped {int(dropped_all)}",
             "roofline": {"bound": "pcie", "achieved": gbs, "peak": peak, "unit": "GB/s", "frac": gbs / peak,
                          "peak_source": "measured SM-store D2H into pinned memory (profiles/r1_box_peaks.json)",
-                         "algorithmic_bytes_per_record": 292}}
+                         "algorithmic_bytes_per_record": slot + 4}}
 
 
 # --------------------------------------------------------------------------- C5 replay
@@ -880,6 +884,8 @@ def run_ours(args):
             cfg["c3"] = run_c3(args, torch, nb, dr, rank, world, local, min(args.steps, 5))
         elif c == "c4":
             cfg["c4"] = run_c4(args, torch, nb, dr, rank, world, local, args.c4_steps)
+        elif c == "c4_compact":
+            cfg["c4_compact"] = run_c4(args, torch, nb, dr, rank, world, local, args.c4_steps, compact=True)
         elif c == "c5":
             cfg["c5"] = run_c5(args, torch, nb, dr, rank, world, local, args.c5_steps, peaks, peaks_src)
         torch.cuda.empty_cache()
@@ -936,7 +942,7 @@ def main():
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--workload", choices=["c2", "f1", "f2", "f4"], default="c2",
                     help="c2: the headline line with --configs beside it; f1/f2/f4: NEXT-row profiling lines")
-    ap.add_argument("--configs", default="c1,c3,c4,c5", help="configs measured beside C2 ('none' for C2 only)")
+    ap.add_argument("--configs", default="c1,c3,c4,c4_compact,c5", help="configs measured beside C2 ('none' for C2 only)")
     ap.add_argument("--c4-steps", type=int, default=2)
     ap.add_argument("--c5-steps", type=int, default=3)
     ap.add_argument("--fft-n", type=int, default=1 << 24, help="F4: transforms per launch")

@@ -314,6 +314,11 @@ class Channel:
         self.handle, self.ctx, self.ring = handle, ctx, ring
 
 
+def nvbt_channel_slot_bytes(compact=False):
+    """Ring stride of one transport slot (288, or 192 for the 176 B compact slots, EM §5.1)."""
+    return 192 if compact else RECORD_BYTES
+
+
 def nvbt_channel_bytes(slots, compact=False, on_device=False):
     """Ring size (bytes) that holds `slots` slots: 64 + slots * (record + 4-byte tag) for host rings."""
     rb = COMPACT_RECORD_BYTES if compact else RECORD_BYTES
