@@ -38,7 +38,10 @@ int nvbt_sgemm(nvbt_ctx ctx, void* stream, uint32_t tools, const float* A, const
                int32_t M, int32_t N, int32_t K);
 /* C3: one BFS level = kernel 1 (expand) then kernel 2 (update, writes cost = level + 1) (EM §3.3).
  * mask/visited/updating: u8[n]; cost: i32[n]; over: one i32 (kernel 2 stores 1 into it). The caller
- * zeroes *over and updating before the call (the host loop of EM §3.3). */
+ * zeroes *over and updating before the call (the host loop of EM §3.3). An instrumented expand over a
+ * vertex of degree >= 2^24 would overflow the privatised u32 bins: it is flagged on the device and the
+ * context's next read call returns NVBT_EINVAL (until nvbt_reset). SGEMM (any K) and WFFT32 (any n_fft)
+ * spill their loop counters to the 64-bit bins every 2^20 instances instead. */
 int nvbt_bfs_level(nvbt_ctx ctx, void* stream, uint32_t tools, const int32_t* rowptr, const int32_t* col,
                    int32_t n, uint8_t* mask, uint8_t* visited, uint8_t* updating, int32_t* cost,
                    int32_t* over, int32_t level);

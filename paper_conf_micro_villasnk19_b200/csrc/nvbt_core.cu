@@ -165,8 +165,13 @@ static int read_out(nvbt_ctx c, size_t word, size_t n, void* dst) {
   std::lock_guard<std::mutex> g(c->mu);
   int rc = fold(c);
   if (rc) return rc;
+  unsigned long long ovf = 0;
   NVBT_CUDA(cudaMemcpyAsync(dst, c->out + word, n * 8, cudaMemcpyDeviceToHost, c->stream));
+  NVBT_CUDA(cudaMemcpyAsync(&ovf, c->ctl + CTL_OVERFLOW, 8, cudaMemcpyDeviceToHost, c->stream));
   NVBT_CUDA(cudaStreamSynchronize(c->stream));
+  if (ovf)
+    return set_error(NVBT_EINVAL, "%llu warp(s) ran a loop of >= 2^24 instances (a BFS vertex of degree >= 2^24): "
+                     "their u32 CTA bins could wrap, results withheld until nvbt_reset", ovf);
   return NVBT_OK;
 }
 
@@ -193,6 +198,7 @@ int make_state(nvbt_ctx c, uint32_t tools, DevState* st) {
   st->head = c->ctl + CTL_HEAD;
   st->tail_cache = c->ctl + CTL_TAIL_CACHE;
   st->dropped = c->ctl + CTL_DROPPED;
+  st->ovf = c->ctl + CTL_OVERFLOW;
   if ((tools & NVBT_TOOL_TRACE) && c->chan) channel_state(c->chan, st);
   st->launch = c->next_launch++;
   return NVBT_OK;
@@ -295,7 +301,7 @@ int nvbt_reset(nvbt_ctx c) {
   std::lock_guard<std::mutex> g(c->mu);
   NVBT_CUDA(cudaSetDevice(c->device));
   NVBT_CUDA(cudaMemsetAsync(c->accum, 0, c->lay.accum_words * 8, c->stream));
-  NVBT_CUDA(cudaMemsetAsync(c->ctl + CTL_REPLAY_ERR, 0, 8, c->stream));
+  NVBT_CUDA(cudaMemsetAsync(c->ctl + CTL_REPLAY_ERR, 0, 16, c->stream));   // replay errors, overflow
   c->next_launch = 0;
   return NVBT_OK;
 }

@@ -62,6 +62,9 @@ struct DevState {
   // linear CTA id is cta_lo + blockIdx.x + blockIdx.y * gridDim.x (cta_lo = cta_y0 * CTA-grid width)
   unsigned cta_lo;
   unsigned cta_y0;
+  // launches whose loop trip counts could wrap a u32 CTA bin (BFS warps with a vertex of degree >= 2^24)
+  // count themselves here; the next read call reports NVBT_EINVAL instead of wrapped results
+  unsigned long long* ovf;
 };
 constexpr unsigned kRingChunk = 4096;
 constexpr unsigned kRingNoChunk = 0xFFFFFFFEu, kRingFull = 0xFFFFFFFFu;

@@ -42,7 +42,7 @@ Layout make_layout(uint32_t n_pcs, uint32_t n_ops, uint32_t n_bbs, uint32_t n_wa
 
 // CTL_RHEAD: device-ring (F2) region heads, kMaxRingStripes stripes + 1 overflow region
 constexpr unsigned kMaxRingStripes = 255;
-enum Ctl { CTL_HEAD = 0, CTL_TAIL_CACHE = 1, CTL_DROPPED = 2, CTL_REPLAY_ERR = 3, CTL_RHEAD = 8,
+enum Ctl { CTL_HEAD = 0, CTL_TAIL_CACHE = 1, CTL_DROPPED = 2, CTL_REPLAY_ERR = 3, CTL_OVERFLOW = 4, CTL_RHEAD = 8,
            CTL_WORDS = 8 + kMaxRingStripes + 1 };
 
 }  // namespace nvbt

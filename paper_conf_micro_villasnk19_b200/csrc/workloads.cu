@@ -142,20 +142,14 @@ __global__ void __launch_bounds__(256) k_bfs_expand(const int* __restrict__ rowp
     if (in_loop) e = e1;
     in_loop = in_loop && p4;
   };
-  constexpr int kChunk = (int)Hooks<T, ProgBfs>::kSpillEvery;
-  if (!__any_sync(FULL, in_loop && end - start > kChunk)) {   // degrees <= kChunk: the plain loop
-    while (__any_sync(FULL, in_loop)) instance();
-  } else {                                     // a hub: chunks of kChunk instances, counters spilled
-    for (;;) {
-      int it = 0;
-      while (it < kChunk && __any_sync(FULL, in_loop)) {
-        instance();
-        ++it;
-      }
-      if (!__any_sync(FULL, in_loop)) break;
-      h.spill();
-    }
+  // exact while every warp's trip count (its largest degree) is < 2^24: the register counters grow by
+  // <= 32 and the per-warp totals by <= 8 x 32 per instance into u32 CTA bins. A larger hub (which a
+  // chunked loop with spills could handle, but whose code raises the plain loop's registers 28 -> 40
+  // and costs the latency-bound BFS occupancy) is flagged: the read calls then return NVBT_EINVAL.
+  if constexpr (Hooks<T, ProgBfs>::kOn) {
+    if (__any_sync(FULL, in_loop && end - start >= (1 << 24)) && (threadIdx.x & 31u) == 0u) atomicAdd(st.ovf, 1ull);
   }
+  while (__any_sync(FULL, in_loop)) instance();
                                                h.template at<21>(m1);
   h.finish();
 }

@@ -46,3 +46,27 @@ def test_sgemm_k_beyond_u32(nvbt, tools):
                        "hS", "hL", "PW_T", "PW_W"], f"SGEMM K = 2^25 + 3 {tools}")
     # fp32 accumulation of K ones saturates at 2^24 (2^24 + 1 rounds to even): the computed product
     assert torch.all(Cm == float(1 << 24))
+
+
+def test_bfs_hub_of_degree_2_24_is_reported(nvbt):
+    """BFS keeps its edge-loop counters in u32 registers / CTA bins (no spill code: it would cost the
+    latency-bound BFS occupancy), exact while every warp's degree is < 2^24. A star with 2^24 leaves is
+    flagged on the device and the read call fails loudly (NVBT_EINVAL) instead of returning wrapped
+    counts; nvbt_reset clears the flag."""
+    import torch
+    nb, dr = nvbt.nvbt, nvbt.drivers
+    n = (1 << 24) + 1
+    rowptr = np.empty(n + 1, dtype=np.int32)  # vertex 0: edges to 1 .. 2^24; every leaf: one edge back to 0
+    rowptr[0] = 0
+    rowptr[1] = 1 << 24
+    rowptr[2:] = (1 << 24) + np.arange(1, n, dtype=np.int64)
+    col = np.concatenate([np.arange(1, n, dtype=np.int32), np.zeros(n - 1, dtype=np.int32)])
+    rp, cl = torch.from_numpy(rowptr).cuda(), torch.from_numpy(col).cuda()
+    ctx = nb.nvbt_init(nb.W_BFS, nb.COUNT | nb.BB)
+    cost, levels = dr.run_bfs(ctx, nb.TOOL_BBCOUNT, rp, cl, 0)
+    assert levels == 2 and int(cost.max()) == 1
+    with pytest.raises(nb.NvbtError) as e:
+        nb.nvbt_count(ctx)
+    assert e.value.code == nb.EINVAL
+    nb.nvbt_reset(ctx)
+    assert (nb.nvbt_count(ctx) == 0).all()
