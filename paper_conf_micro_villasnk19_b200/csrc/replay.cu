@@ -287,6 +287,9 @@ constexpr int RB_NW = 20;     // pass B warps per CTA (warp w of pass B analyses
 #ifndef NVBT_RPB_EXPERIMENT
 #define NVBT_RPB_EXPERIMENT 0   // timing experiments (tools/replay_ab.py), never in a product build
 #endif
+#ifndef NVBT_RPB_WIN
+#define NVBT_RPB_WIN 512       // window rows: sectors per tag window, 1024 / WIN rows per iteration (A/B r2_ab9: 256 and 128 slower)
+#endif
 #ifndef NVBT_RPB_TAGS
 #define NVBT_RPB_TAGS 1        // slow rows by tag arrays (0: round-1 atomics + reductions, for A/B)
 #endif
@@ -404,7 +407,9 @@ __device__ __forceinline__ void inc_if_gt(unsigned& c, unsigned x) {
 __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsigned lane, unsigned lanebit,
                                            unsigned s_scr, unsigned s_sS, unsigned s_sL, unsigned s_hist) {
   const unsigned j = lane & 15u, h = lane >> 4, sw = j & 7u;
-  constexpr unsigned kWin = NVBT_RPB_TAGS ? 512u : 1024u;   // window sectors (tags build: two rows in flight)
+  // window sectors of class 1 (tags build: kWR rows in flight, kWin + kWin / 4 tag bytes each)
+  constexpr unsigned kWin = NVBT_RPB_TAGS ? NVBT_RPB_WIN : 1024u;
+  constexpr int kWR = NVBT_RPB_TAGS ? 1024 / NVBT_RPB_WIN : 1;
   unsigned E, pc;
   lds_v2(meta + 8u * j, E, pc);
   const unsigned Eh = h ? E >> 16 : E & 0xffffu;
@@ -489,9 +494,9 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
   // slot exactly one (the last writer) reads its own id, so the number of distinct slots = popc(ballot(own
   // id read)). Stale tags from earlier rows never matter: every lane that reads a slot wrote it this row.
   //  * rows within one 1 KB word (class 0) are settled from the scan's sector bits above;
-  //  * window rows (all sectors of E in the 512-sector window from wbase, upper words equal; class 1):
-  //    the slot is the sector's offset in the window (512 B of tags) and, for lines, offset >> 2 (128 B):
-  //    S and L exactly; two rows per iteration;
+  //  * window rows (all sectors of E in the kWin-sector window from wbase, upper words equal; class 1):
+  //    the slot is the sector's offset in the window (kWin tag bytes) and, for lines, offset >> 2: S and L
+  //    exactly; 1024 / kWin rows per iteration;
   //  * wide rows (class 2): all lines distinct? slots = a hash of the line into 1280 buckets, up to three
   //    independent hashes; all lanes owning their slot proves every line (hence sector) distinct: S = L =
   //    |E|. Rows that collide three times (~3 %) take an exact bitonic sort of the sector keys.
@@ -499,34 +504,41 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
   const unsigned l8 = 8u * lane;
   const unsigned long long kInvalid = ~0ull;
   unsigned mw = cm0 | cm1, mwide = cm2;
-  // two window rows per iteration (independent chains; 512-sector window and 128 line tags per row)
+  // up to kWR window rows per iteration (independent chains; per row a kWin-sector window of tags and
+  // kWin / 4 line tags)
   while (mw) {
-    const unsigned ra = 31u - __clz(mw);
-    mw ^= 1u << ra;
-    const bool two = mw != 0u;
-    const unsigned rb = two ? 31u - __clz(mw) : ra;
-    if (two) mw ^= 1u << rb;
-    const unsigned ea = __shfl_sync(FULL, E, ra), wa = __shfl_sync(FULL, wbase, ra);
-    const unsigned eb = __shfl_sync(FULL, E, rb), wbb = __shfl_sync(FULL, wbase, rb);
-    const unsigned la = lds_u32(stage + 256u * ra + (l8 ^ (16u * (ra & 7u))));
-    const unsigned lb = lds_u32(stage + 256u * rb + (l8 ^ (16u * (rb & 7u))));
-    const bool acta = (ea >> lane) & 1u, actb = two && ((eb >> lane) & 1u);
-    const unsigned oa = (la >> 5) - wa, ob = (lb >> 5) - wbb;
-    if (acta) {
-      sts_u8(stag + oa, lane);
-      sts_u8(ltag + (oa >> 2), lane);
+    unsigned r[kWR], lo[kWR], off[kWR], ev[kWR], wv[kWR];
+    bool v[kWR], act[kWR];
+#pragma unroll
+    for (int k = 0; k < kWR; ++k) {
+      v[k] = mw != 0u;
+      r[k] = v[k] ? 31u - __clz(mw) : 0u;
+      if (v[k]) mw ^= 1u << r[k];
     }
-    if (actb) {
-      sts_u8(stag + 512u + ob, lane);
-      sts_u8(ltag + 128u + (ob >> 2), lane);
+#pragma unroll
+    for (int k = 0; k < kWR; ++k) {
+      ev[k] = __shfl_sync(FULL, E, r[k]);
+      wv[k] = __shfl_sync(FULL, wbase, r[k]);
+      lo[k] = lds_u32(stage + 256u * r[k] + (l8 ^ (16u * (r[k] & 7u))));
+    }
+#pragma unroll
+    for (int k = 0; k < kWR; ++k) {
+      act[k] = v[k] && ((ev[k] >> lane) & 1u);
+      off[k] = (lo[k] >> 5) - wv[k];
+      if (act[k]) {
+        sts_u8(stag + kWin * k + off[k], lane);
+        sts_u8(ltag + (kWin / 4u) * k + (off[k] >> 2), lane);
+      }
     }
     __syncwarp();
-    const bool fsa = acta && lds_u8(stag + oa) == lane, fla = acta && lds_u8(ltag + (oa >> 2)) == lane;
-    const bool fsb = actb && lds_u8(stag + 512u + ob) == lane, flb = actb && lds_u8(ltag + 128u + (ob >> 2)) == lane;
-    const unsigned sa = __popc(__ballot_sync(FULL, fsa)), lxa = __popc(__ballot_sync(FULL, fla));
-    const unsigned sb2 = __popc(__ballot_sync(FULL, fsb)), lxb = __popc(__ballot_sync(FULL, flb));
-    S = lane == ra ? sa : (two && lane == rb) ? sb2 : S;
-    L = lane == ra ? lxa : (two && lane == rb) ? lxb : L;
+#pragma unroll
+    for (int k = 0; k < kWR; ++k) {
+      const bool fs = act[k] && lds_u8(stag + kWin * k + off[k]) == lane;
+      const bool fl = act[k] && lds_u8(ltag + (kWin / 4u) * k + (off[k] >> 2)) == lane;
+      const unsigned sx = __popc(__ballot_sync(FULL, fs)), lx = __popc(__ballot_sync(FULL, fl));
+      S = (v[k] && lane == r[k]) ? sx : S;
+      L = (v[k] && lane == r[k]) ? lx : L;
+    }
     __syncwarp();                                  // reads done before the next rows' stores
   }
   while (mwide) {
