@@ -287,6 +287,15 @@ constexpr int RB_NW = 20;     // pass B warps per CTA (warp w of pass B analyses
 #ifndef NVBT_RPB_EXPERIMENT
 #define NVBT_RPB_EXPERIMENT 0   // timing experiments (tools/replay_ab.py), never in a product build
 #endif
+#ifndef NVBT_RPB_SBITS
+#define NVBT_RPB_SBITS 0       // 1 KB-word rows settled from sector bits gathered in the scan (A/B r2_ab10:
+                               // the 2 ALU ops per address cost more than the window loop they save)
+#endif
+#ifndef NVBT_RPB_HIRAW
+#define NVBT_RPB_HIRAW 1       // high-word check over all scanned lanes, inactive ones too (no select per
+                               // address; r2_ab10: pass B 1.90 -> 1.84 ms with SBITS 0). A row whose inactive
+                               // lanes differ in the upper word only takes the exact wide path.
+#endif
 #ifndef NVBT_RPB_WIN
 #define NVBT_RPB_WIN 512       // window rows: sectors per tag window, 1024 / WIN rows per iteration (A/B r2_ab9: 256 and 128 slower)
 #endif
@@ -428,15 +437,19 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
     for (int u = 0; u < 2; ++u) {
       const bool act = (Eh >> (2 * q + u)) & 1u;
       const unsigned lo = act ? (u ? v.z : v.x) : prev;
+#if NVBT_RPB_HIRAW   // upper words of every scanned lane (inactive ones too: a row whose inactive lanes
+      hb |= (u ? v.w : v.y) ^ f_hi;   // differ only goes to the exact wide path)
+#else
       const unsigned hi = act ? (u ? v.w : v.y) : f_hi;
       hb |= hi ^ f_hi;
+#endif
       viol |= lo < prev;
       const unsigned x = lo ^ prev;
       inc_if_gt<31>(bs, x);
       inc_if_gt<127>(bl, x);
       mn = min(mn, lo);
       mx = max(mx, lo);
-#if NVBT_RPB_TAGS
+#if NVBT_RPB_TAGS && NVBT_RPB_SBITS
       sbits |= __funnelshift_l(0u, 1u, lo >> 5);   // 1 << ((lo >> 5) & 31): one SHF.L.W
 #endif
       prev = lo;
@@ -450,7 +463,7 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
   const unsigned o_hi = __shfl_xor_sync(FULL, f_hi, 16);
   const unsigned o_mn = __shfl_xor_sync(FULL, mn, 16);
   const unsigned o_mx = __shfl_xor_sync(FULL, mx, 16);
-#if NVBT_RPB_TAGS
+#if NVBT_RPB_TAGS && NVBT_RPB_SBITS
   const unsigned o_sb = __shfl_xor_sync(FULL, sbits, 16);
 #endif
   const bool other = (o_pack >> 18) != 0u;
@@ -475,7 +488,7 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
   // address range (one 1 KB word / a 32 KB window / anything else)
   // (NVBT_RPB_EXPERIMENT bits 1, 4, 8, 16: timing experiments only, wrong results: drop all / class-0 /
   // class-1 / class-2 slow rows)
-#if NVBT_RPB_TAGS
+#if NVBT_RPB_TAGS && NVBT_RPB_SBITS
   if (slow && cls == 0u) {   // one 1 KB word: the scan's sector bits are exact (no loop below)
     const unsigned word = (mine ? sbits : 0u) | (other ? o_sb : 0u);
     const unsigned g = word | (word >> 1) | (word >> 2) | (word >> 3);
@@ -483,6 +496,8 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
     L = __popc(g & 0x11111111u);
   }
   const unsigned cm0 = 0u;
+#elif NVBT_RPB_TAGS
+  const unsigned cm0 = __ballot_sync(FULL, own && slow && cls == 0u);   // window loop takes class 0 too
 #else
   const unsigned cm0 = (NVBT_RPB_EXPERIMENT & 5) ? 0u : __ballot_sync(FULL, own && slow && cls == 0u);
 #endif
