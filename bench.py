@@ -539,8 +539,8 @@ def run_c3(args, torch, nb, dr, rank, world, local, steps):
 # --------------------------------------------------------------------------- C4 stencil + channel
 def run_c4(args, torch, nb, dr, rank, world, local, steps, compact=False):
     """C4: 8192^2 5-point stencil x 100 iterations, every executed global LD/ST traced through the pinned
-    host channel (288 B records, EM §5; with `compact` the F3 transport of EM §5.1, decoded back to the
-    same records on the host) and digested on the host; a step is the whole traced run. The
+    host channel (288 B records, EM §5; with `compact` True / 128 the F3 transports of EM §5.1 / §5.2,
+    decoded back to the same records on the host) and digested on the host; a step is the whole traced run. The
     drain runs on a host thread while the iterations are enqueued (N > 1: row slabs with P2P halos, one
     channel per rank). Device time from the first launch to the last kernel's end (the producers wait on
     the host ring, so it includes the transport), max over ranks."""
@@ -604,7 +604,7 @@ def run_c4(args, torch, nb, dr, rank, world, local, steps, compact=False):
     peak = d2h_peak()
     nb.nvbt_channel_close(ch)
     del ring
-    transport = "compact slots (EM 5.1)" if compact else "288 B records"
+    transport = {False: "288 B records", True: "176 B compact slots (EM 5.1)", 128: "128 B line slots (EM 5.2)"}[compact]
     return {"value": recs / t_dev if ok else None, "unit": "records/s", "steps": steps,
             "workload": f"C4 stencil {n}^2 x {iters}, tools TRACE, {transport} to pinned host, digest drain",
             "records_per_s_measured": recs / t_dev, "transport_slot_bytes": slot,
@@ -886,6 +886,8 @@ def run_ours(args):
             cfg["c4"] = run_c4(args, torch, nb, dr, rank, world, local, args.c4_steps)
         elif c == "c4_compact":
             cfg["c4_compact"] = run_c4(args, torch, nb, dr, rank, world, local, args.c4_steps, compact=True)
+        elif c == "c4_line":
+            cfg["c4_line"] = run_c4(args, torch, nb, dr, rank, world, local, args.c4_steps, compact=128)
         elif c == "c5":
             cfg["c5"] = run_c5(args, torch, nb, dr, rank, world, local, args.c5_steps, peaks, peaks_src)
         torch.cuda.empty_cache()
@@ -942,7 +944,7 @@ def main():
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--workload", choices=["c2", "f1", "f2", "f4"], default="c2",
                     help="c2: the headline line with --configs beside it; f1/f2/f4: NEXT-row profiling lines")
-    ap.add_argument("--configs", default="c1,c3,c4,c4_compact,c5", help="configs measured beside C2 ('none' for C2 only)")
+    ap.add_argument("--configs", default="c1,c3,c4,c4_compact,c4_line,c5", help="configs measured beside C2 ('none' for C2 only)")
     ap.add_argument("--c4-steps", type=int, default=2)
     ap.add_argument("--c5-steps", type=int, default=3)
     ap.add_argument("--fft-n", type=int, default=1 << 24, help="F4: transforms per launch")

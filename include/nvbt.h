@@ -126,20 +126,23 @@ int nvbt_mem_divergence(nvbt_ctx ctx, nvbt_memdiv* per_pc, uint32_t n_pcs, nvbt_
 
 /* ---- trace channel (a6; "sent to the CPU for further processing", P:L187 (§6.1)) ----
  * pinned_ring: caller-owned pinned, device-mapped host memory (cudaHostAlloc / torch pin_memory), at
- * least 64 + 2 * (stride + 4) bytes, 64-byte aligned, where stride = 288 for 288 B records and 192 for
- * 176 B compact slots (padded so that two slots cover three 128 B lines). Its first 64 bytes hold the
- * consumer index the producers read for backpressure; the rest is cap = floor((ring_bytes - 64) /
+ * least H + 3 * (stride + 4) bytes, 64-byte aligned (128 for line-aligned 128 B slots), H = 64 (128 for
+ * 128 B slots), where stride = 288 for 288 B records, 192 for
+ * 176 B compact slots (padded so that two slots cover three 128 B lines) and 128 for 128 B slots. Its first 64 bytes hold the
+ * consumer index the producers read for backpressure; the rest is cap = floor((ring_bytes - H) /
  * (stride + 4)) slots followed by cap 4-byte commit tags (one per slot, written by the producer after its
  * record). A CUDA
  * device buffer instead (F2, on-GPU consumers) has no tag array: cap = floor((ring_bytes - 64) / 288).
  * nvbt_channel_bytes gives the ring_bytes that hold `slots` slots. */
 size_t nvbt_channel_bytes(uint32_t record_bytes, uint64_t slots, int on_device);
 /*
- * record_bytes: NVBT_RECORD_BYTES (288: every slot is an EM §5 record) or NVBT_COMPACT_RECORD_BYTES (176:
- * base + 32-bit deltas, wide address sets as two slots; EM §5.1, F3). Either way the drain delivers EM §5
- * records. One channel per context. */
+ * record_bytes: NVBT_RECORD_BYTES (288: every slot is an EM §5 record), NVBT_COMPACT_RECORD_BYTES (176:
+ * base + 32-bit deltas, wide address sets as two slots; EM §5.1, F3) or NVBT_COMPACT128_RECORD_BYTES (128:
+ * one whole PCIe line per record with base + 16-bit deltas, other records as three slots; EM §5.2). Every
+ * way the drain delivers EM §5 records. One channel per context. */
 #define NVBT_RECORD_BYTES 288
 #define NVBT_COMPACT_RECORD_BYTES 176
+#define NVBT_COMPACT128_RECORD_BYTES 128
 int nvbt_channel_open(nvbt_ctx ctx, void* pinned_ring, size_t ring_bytes, uint32_t record_bytes,
                       nvbt_channel* out);
 /* Called with a batch of n contiguous, fully written records (reserved field zeroed); return 0 to
@@ -189,6 +192,11 @@ int nvbt_digest_records(const void* records, uint64_t n_records, nvbt_digest* ou
 /* Decodes n_slots 176 B transport slots (EM §5.1; tags ignored) into EM §5 records at out (capacity
  * out_cap records); *n_out = records written. EINVAL on an unpaired wide slot or a too-small out. */
 int nvbt_decode_compact(const void* slots, uint64_t n_slots, void* out, uint64_t out_cap, uint64_t* n_out);
+/* The same for either compact transport: record_bytes NVBT_COMPACT_RECORD_BYTES or
+ * NVBT_COMPACT128_RECORD_BYTES, slots packed record_bytes apart (tags ignored). EINVAL on a record whose
+ * continuation slots are missing or a too-small out. */
+int nvbt_decode_slots(const void* slots, uint64_t n_slots, uint32_t record_bytes, void* out, uint64_t out_cap,
+                      uint64_t* n_out);
 
 /* ---- trace-replay mode (a7; EM §3.5) ---- */
 /* Writes events [first, first+n) of the counter-based generator (seed) as 16 B headers at d_hdr[n]

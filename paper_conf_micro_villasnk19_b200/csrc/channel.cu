@@ -35,8 +35,10 @@ struct nvbt_chan_s {
   bool on_device = false;              // F2: ring in device memory, consumed by GPU kernels
   unsigned rstripes = 0;               // device ring: per-SM chunk stripes (see DevState)
   bool open = false;
-  bool have_half = false;              // compact: first half of a wide pair seen at the ring end
-  unsigned char half[176];
+  unsigned fmt = 0;                    // 0: 288 B records; 1: 176 B slots (EM §5.1); 2: 128 B slots (EM §5.2)
+  size_t hdr = 64;                     // bytes before slot 0
+  unsigned part_n = 0;                 // compact: slots of a multi-slot record seen at the ring end ...
+  unsigned char part[3 * 192];         // ... stashed until the rest arrives as slots 0.. of the next lap
   std::vector<unsigned char> scratch;  // compact: decoded records of one batch
   // host rings: a private non-blocking stream for the drain's reads of the ticket counter. The drain never
   // synchronises the context's stream: another thread may be enqueueing producers on it, and waiting for
@@ -49,22 +51,26 @@ struct nvbt_chan_s {
 
 namespace nvbt {
 
-static constexpr size_t HDR = 64;
+static constexpr size_t HDR = 64;      // ring header (consumer index); 128 for 128 B slots so they are line aligned
+static inline size_t hdr_of(uint32_t record_bytes) { return record_bytes == NVBT_COMPACT128_RECORD_BYTES ? 128 : HDR; }
 static constexpr unsigned COMPACT_BYTES = NVBT_COMPACT_RECORD_BYTES;
 // Ring stride of a compact slot: the 176 B slot padded to 192 B (pairs of slots cover 3 whole lines; PCIe
 // D2H of SM stores, tools/peaks/d2h_pattern.cu: 176 B at a 176 B stride 33.0 GB/s of slot bytes, at a 192 B
 // stride 36.5). The pad is never written or read.
 static constexpr unsigned COMPACT_STRIDE = 192;
+static constexpr unsigned SLOT128 = NVBT_COMPACT128_RECORD_BYTES;
 static inline unsigned slot_stride(uint32_t record_bytes) { return record_bytes == COMPACT_BYTES ? COMPACT_STRIDE : record_bytes; }
+static inline unsigned fmt_of(uint32_t record_bytes) { return record_bytes == COMPACT_BYTES ? 1u : record_bytes == SLOT128 ? 2u : 0u; }
 
 void channel_state(nvbt_chan_s* ch, DevState* st) {
-  st->ring = ch->dev + HDR;
+  st->ring = ch->dev + ch->hdr;
   st->tail = reinterpret_cast<const unsigned long long*>(ch->dev);
   st->cap = ch->cap;
-  st->tags = ch->on_device ? nullptr : reinterpret_cast<unsigned*>(ch->dev + HDR + ch->cap * ch->slot);
+  st->tags = ch->on_device ? nullptr : reinterpret_cast<unsigned*>(ch->dev + ch->hdr + ch->cap * ch->slot);
   st->slot_bytes = ch->slot;
-  // compact = 1; 2 forces the wide form for every record (NVBT_COMPACT_FORCE_WIDE=1, tests only)
-  st->compact = ch->slot == COMPACT_STRIDE ? (ch->force_wide ? 2u : 1u) : 0u;
+  // compact = 1 / 3 (176 B / 128 B slots); 2 / 4 force the multi-slot form for every record
+  // (NVBT_COMPACT_FORCE_WIDE=1, tests only)
+  st->compact = ch->fmt == 1u ? (ch->force_wide ? 2u : 1u) : ch->fmt == 2u ? (ch->force_wide ? 4u : 3u) : 0u;
   st->no_wait = ch->on_device ? 1u : 0u;   // nobody frees device-ring slots: drop instead of waiting
   st->rheads = ch->on_device ? ch->ctx->ctl + CTL_RHEAD : nullptr;
   st->rstripes = ch->rstripes;
@@ -233,9 +239,53 @@ static void decode_wide_pair(const unsigned char* s0, const unsigned char* s1, u
   std::memcpy(out + 160, s1 + 32, 128);
 }
 
+// EM §5.2, 128 B slots: short (kind | 0x80): header, base at 32, 32 x i16 deltas at 40; long (kind | 0x40):
+// three slots, lanes 0..11 at 32.. of the first, then per continuation slot (flag 0x20 at byte 27) 3 lanes
+// at 0..23 and 12 lanes at 32..127.
+static void decode_short128(const unsigned char* sl, unsigned char* out) {
+  std::memcpy(out, sl, 28);
+  out[27] = sl[27] & 0x1Fu;
+  std::memset(out + 28, 0, 4);
+  uint32_t A, P;
+  std::memcpy(&A, sl + 16, 4);
+  std::memcpy(&P, sl + 20, 4);
+  const uint32_t E = A & P;
+  uint64_t base;
+  std::memcpy(&base, sl + 32, 8);
+  for (int l = 0; l < 32; ++l) {
+    int16_t d;
+    std::memcpy(&d, sl + 40 + 2 * l, 2);
+    const uint64_t a = ((E >> l) & 1u) ? base + (uint64_t)(int64_t)d : 0ull;
+    std::memcpy(out + 32 + 8 * l, &a, 8);
+  }
+}
+static void decode_long128(const unsigned char* s0, const unsigned char* s1, const unsigned char* s2, unsigned char* out) {
+  std::memcpy(out, s0, 28);
+  out[27] = s0[27] & 0x1Fu;
+  std::memset(out + 28, 0, 4);
+  std::memcpy(out + 32, s0 + 32, 96);             // lanes 0..11
+  std::memcpy(out + 32 + 8 * 12, s1, 24);          // lanes 12..14
+  std::memcpy(out + 32 + 8 * 15, s1 + 32, 96);     // lanes 15..26
+  std::memcpy(out + 32 + 8 * 27, s2, 24);          // lanes 27..29
+  std::memcpy(out + 32 + 8 * 30, s2 + 32, 16);     // lanes 30, 31
+}
+// slots per record starting with flags f (0x80 / none: 1; 0x40: 2 or 3)
+static inline unsigned group_len(unsigned fmt, unsigned f) { return f == 0x40u ? (fmt == 2u ? 3u : 2u) : 1u; }
+// the record whose first slot is s0 (its slots ss bytes apart)
+static void decode_group(unsigned fmt, const unsigned char* s0, unsigned ss, unsigned char* out) {
+  const unsigned f = slot_flags(s0);
+  if (fmt == 2u) {
+    if (f == 0x40u) decode_long128(s0, s0 + ss, s0 + 2 * ss, out);
+    else decode_short128(s0, out);
+  } else {
+    if (f == 0x40u) decode_wide_pair(s0, s0 + ss, out);
+    else decode_compact_slot(s0, out);
+  }
+}
+
 // Decodes slots [0, n) into records; a wide-first at the end must not occur (caller keeps pairs whole).
 // Parallel: count records per part, prefix, decode. Returns the record count.
-static uint64_t decode_batch(const unsigned char* sl, uint64_t n, unsigned char* out, unsigned ss) {
+static uint64_t decode_batch(const unsigned char* sl, uint64_t n, unsigned char* out, unsigned ss, unsigned fmt) {
   Pool& pool = Pool::get();
   std::vector<uint64_t> cnt(pool.size() + 1, 0), lo_of(pool.size(), 0), hi_of(pool.size(), 0);
   auto is_rec = [&](uint64_t i) { return slot_flags(sl + (size_t)i * ss) != 0x20u; };
@@ -253,9 +303,7 @@ static uint64_t decode_batch(const unsigned char* sl, uint64_t n, unsigned char*
       const unsigned char* s0 = sl + (size_t)i * ss;
       const unsigned f = slot_flags(s0);
       if (f == 0x20u) continue;
-      unsigned char* r = out + (size_t)o * RECORD_BYTES;
-      if (f == 0x40u) decode_wide_pair(s0, s0 + ss, r);
-      else decode_compact_slot(s0, r);
+      decode_group(fmt, s0, ss, out + (size_t)o * RECORD_BYTES);
       ++o;
     }
   });
@@ -263,7 +311,7 @@ static uint64_t decode_batch(const unsigned char* sl, uint64_t n, unsigned char*
 }
 
 // Digest of the records encoded in slots [0, n) without materialising them (built-in digest callback).
-static uint64_t digest_compact(const unsigned char* sl, uint64_t n, uint64_t* d1, uint64_t* d2, unsigned ss) {
+static uint64_t digest_compact(const unsigned char* sl, uint64_t n, uint64_t* d1, uint64_t* d2, unsigned ss, unsigned fmt) {
   Pool& pool = Pool::get();
   std::vector<uint64_t> p1(pool.size(), 0), p2(pool.size(), 0), pc(pool.size(), 0);
   pool.parallel_for(n, [&](unsigned id, uint64_t lo, uint64_t hi) {
@@ -273,8 +321,7 @@ static uint64_t digest_compact(const unsigned char* sl, uint64_t n, uint64_t* d1
       const unsigned char* s0 = sl + (size_t)i * ss;
       const unsigned f = slot_flags(s0);
       if (f == 0x20u) continue;
-      if (f == 0x40u) decode_wide_pair(s0, s0 + ss, rec);
-      else decode_compact_slot(s0, rec);
+      decode_group(fmt, s0, ss, rec);
       digest_serial(rec, 1, &s1, &s2);
       ++c;
     }
@@ -298,17 +345,18 @@ int nvbt_drain_discard(const void* records, uint64_t n_records, void* user);
 extern "C" {
 
 size_t nvbt_channel_bytes(uint32_t record_bytes, uint64_t slots, int on_device) {
-  return HDR + slots * (slot_stride(record_bytes) + (on_device ? 0u : 4u));
+  return hdr_of(record_bytes) + slots * (slot_stride(record_bytes) + (on_device ? 0u : 4u));
 }
 
 int nvbt_channel_open(nvbt_ctx c, void* ring, size_t bytes, uint32_t record_bytes, nvbt_channel* out) {
   if (!c || !ring || !out) return set_error(NVBT_EINVAL, "null argument");
   if (!(c->flags & NVBT_TRACE)) return set_error(NVBT_ESTATE, "NVBT_TRACE not enabled at init");
   if (c->chan) return set_error(NVBT_ESTATE, "channel already open on this context");
-  if (record_bytes != RECORD_BYTES && record_bytes != COMPACT_BYTES)
-    return set_error(NVBT_EINVAL, "record_bytes %u is neither 288 nor 176", record_bytes);
+  if (record_bytes != RECORD_BYTES && record_bytes != COMPACT_BYTES && record_bytes != SLOT128)
+    return set_error(NVBT_EINVAL, "record_bytes %u is none of 288, 176, 128", record_bytes);
   if (reinterpret_cast<uintptr_t>(ring) % 64) return set_error(NVBT_EINVAL, "ring not 64-byte aligned");
-  if (bytes < HDR + 2 * (slot_stride(record_bytes) + 4)) return set_error(NVBT_ENOMEM, "ring of %zu bytes holds < 2 slots", bytes);
+  if (bytes < hdr_of(record_bytes) + 3 * (slot_stride(record_bytes) + 4))
+    return set_error(NVBT_ENOMEM, "ring of %zu bytes holds < 3 slots", bytes);
   NVBT_CUDA(cudaSetDevice(c->device));
   cudaPointerAttributes pa{};
   NVBT_CUDA(cudaPointerGetAttributes(&pa, ring));
@@ -323,12 +371,14 @@ int nvbt_channel_open(nvbt_ctx c, void* ring, size_t bytes, uint32_t record_byte
   ch->on_device = on_device;
   ch->host = on_device ? nullptr : static_cast<unsigned char*>(ring);
   ch->dev = static_cast<unsigned char*>(on_device ? ring : pa.devicePointer);
-  ch->slots = on_device ? nullptr : ch->host + HDR;
+  ch->hdr = hdr_of(record_bytes);
+  ch->slots = on_device ? nullptr : ch->host + ch->hdr;
   ch->slot = slot_stride(record_bytes);
+  ch->fmt = fmt_of(record_bytes);
   { const char* e = getenv("NVBT_COMPACT_FORCE_WIDE"); ch->force_wide = e && atoi(e) != 0; }
   // host rings: each slot has a 4 B tag in the array after the slots; device rings carry the tag in-record
-  ch->cap = (bytes - HDR) / (ch->slot + (on_device ? 0u : 4u));
-  ch->tags = on_device ? nullptr : reinterpret_cast<const uint32_t*>(ch->host + HDR + ch->cap * ch->slot);
+  ch->cap = (bytes - ch->hdr) / (ch->slot + (on_device ? 0u : 4u));
+  ch->tags = on_device ? nullptr : reinterpret_cast<const uint32_t*>(ch->host + ch->hdr + ch->cap * ch->slot);
   if (on_device) {
     int sms = 148;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, c->device);
@@ -336,7 +386,7 @@ int nvbt_channel_open(nvbt_ctx c, void* ring, size_t bytes, uint32_t record_byte
   }
   cudaError_t e = cudaSuccess;
   if (on_device) e = cudaMemsetAsync(ring, 0, HDR + ch->cap * record_bytes, c->stream);
-  else std::memset(ch->host, 0, HDR + ch->cap * (ch->slot + 4));
+  else std::memset(ch->host, 0, ch->hdr + ch->cap * (ch->slot + 4));
   if (on_device && e == cudaSuccess) {   // every stripe starts without a chunk; chunk counter 0
     std::vector<unsigned long long> w(ch->rstripes + 1, ((unsigned long long)kRingNoChunk << 32) | kRingChunk);
     w.back() = 0;
@@ -706,37 +756,50 @@ int nvbt_channel_drain(nvbt_channel ch, nvbt_drain_fn fn, void* user, int64_t ti
       if (urc) { rc = set_error(NVBT_ESTATE, "drain callback returned %d", urc); break; }
       continue;
     }
-    if (n) {  // compact transport: decode slots into EM §5 records, keep wide pairs together
+    if (n) {  // compact transports: decode slots into EM §5 records, keep multi-slot records together
       std::atomic_thread_fence(std::memory_order_acquire);
       const unsigned char* base = ch->slots + slot * sb;
       if (ch->scratch.size() < (kBatch + 1) * RECORD_BYTES) ch->scratch.resize((kBatch + 1) * RECORD_BYTES);
       unsigned char* out = ch->scratch.data();
       uint64_t first = 0, end = n, consume = n, o = 0;
-      if (ch->have_half) {
-        if (slot_flags(base) != 0x20u) { rc = set_error(NVBT_ESTATE, "channel: unpaired wide record"); break; }
-        decode_wide_pair(ch->half, base, out);
-        ch->have_half = false;
-        first = 1;
-        o = 1;
-      }
-      if (end > first && slot_flags(base + (end - 1) * sb) == 0x40u) {
-        if (slot + end == ch->cap) {      // partner is slot 0 of the next lap: stash this half
-          std::memcpy(ch->half, base + (end - 1) * sb, COMPACT_BYTES);
-          ch->have_half = true;
-        } else {
-          --consume;                       // partner not ready yet: take the pair next time
+      if (ch->part_n) {   // the rest of a record stashed at the ring end: its continuation slots come first
+        const unsigned g = group_len(ch->fmt, slot_flags(ch->part));
+        const uint64_t k = std::min<uint64_t>(g - ch->part_n, n);
+        bool bad = false;
+        for (uint64_t i = 0; i < k; ++i) bad |= slot_flags(base + i * sb) != 0x20u;
+        if (bad) { rc = set_error(NVBT_ESTATE, "channel: multi-slot record without its continuation"); break; }
+        for (uint64_t i = 0; i < k; ++i) std::memcpy(ch->part + (ch->part_n + i) * sb, base + i * sb, sb);
+        ch->part_n += (unsigned)k;
+        first = k;
+        if (ch->part_n == g) {
+          decode_group(ch->fmt, ch->part, sb, out);
+          ch->part_n = 0;
+          o = 1;
         }
-        --end;
+      }
+      // a record whose slots are not all ready (or continue in the next lap) ends the batch early
+      uint64_t cut = end;
+      const unsigned glong = ch->fmt == 2u ? 3u : 2u;
+      for (uint64_t back = 1; back < glong && back <= end - first; ++back)
+        if (slot_flags(base + (end - back) * sb) == 0x40u) { cut = end - back; break; }
+      if (cut < end) {
+        if (slot + end == ch->cap) {      // continues in slots 0.. of the next lap: stash what is here
+          std::memcpy(ch->part, base + cut * sb, (end - cut) * sb);
+          ch->part_n = (unsigned)(end - cut);
+        } else {
+          consume = cut;                   // the rest is not ready yet: take the record next time
+        }
+        end = cut;
       }
       int urc = 0;
       if (fn == nvbt_drain_digest && user) {   // fused decode + digest, no staging of records
         auto* dg = static_cast<nvbt_digest*>(user);
         if (o) urc = fn(out, o, user);
-        const uint64_t k = digest_compact(base + first * sb, end - first, &dg->d1, &dg->d2, sb);
+        const uint64_t k = digest_compact(base + first * sb, end - first, &dg->d1, &dg->d2, sb, ch->fmt);
         dg->n_rec += k;
         o += k;
       } else {
-        o += decode_batch(base + first * sb, end - first, out + o * RECORD_BYTES, sb);
+        o += decode_batch(base + first * sb, end - first, out + o * RECORD_BYTES, sb, ch->fmt);
         urc = o ? fn(out, o, user) : 0;
       }
       ch->consumed += consume;
@@ -799,30 +862,35 @@ int nvbt_drain_copy(const void* records, uint64_t n, void* user) {
   return 0;
 }
 
-int nvbt_decode_compact(const void* slots, uint64_t n, void* out, uint64_t cap, uint64_t* n_out) {
+int nvbt_decode_slots(const void* slots, uint64_t n, uint32_t record_bytes, void* out, uint64_t cap, uint64_t* n_out) {
   if ((!slots && n) || (!out && cap) || !n_out) return set_error(NVBT_EINVAL, "null argument");
+  const unsigned fmt = fmt_of(record_bytes);
+  if (fmt == 0u) return set_error(NVBT_EINVAL, "record_bytes %u is not a compact transport (176 or 128)", record_bytes);
+  const unsigned ss = record_bytes;   // slots packed back to back (no ring padding)
   const unsigned char* sl = static_cast<const unsigned char*>(slots);
   unsigned char* o = static_cast<unsigned char*>(out);
   uint64_t k = 0;
-  for (uint64_t i = 0; i < n; ++i) {
-    const unsigned char* s0 = sl + i * COMPACT_BYTES;
+  for (uint64_t i = 0; i < n;) {
+    const unsigned char* s0 = sl + i * ss;
     const unsigned f = slot_flags(s0);
-    if (f == 0x20u) return set_error(NVBT_EINVAL, "slot %llu: wide second half without first", (unsigned long long)i);
+    if (f != 0x80u && f != 0x40u)
+      return set_error(NVBT_EINVAL, "slot %llu: not the first slot of a record (flags 0x%x)", (unsigned long long)i, f);
+    const unsigned g = group_len(fmt, f);
+    if (i + g > n) return set_error(NVBT_EINVAL, "slot %llu: record continues past the last slot", (unsigned long long)i);
+    for (unsigned q = 1; q < g; ++q)
+      if (slot_flags(s0 + q * ss) != 0x20u)
+        return set_error(NVBT_EINVAL, "slot %llu: missing continuation slot", (unsigned long long)(i + q));
     if (k >= cap) return set_error(NVBT_EINVAL, "output capacity %llu too small", (unsigned long long)cap);
-    if (f == 0x40u) {
-      if (i + 1 >= n || slot_flags(s0 + COMPACT_BYTES) != 0x20u)
-        return set_error(NVBT_EINVAL, "slot %llu: wide first half without second", (unsigned long long)i);
-      decode_wide_pair(s0, s0 + COMPACT_BYTES, o + k * RECORD_BYTES);
-      ++i;
-    } else if (f == 0x80u) {
-      decode_compact_slot(s0, o + k * RECORD_BYTES);
-    } else {
-      return set_error(NVBT_EINVAL, "slot %llu: not a compact slot (flags 0x%x)", (unsigned long long)i, f);
-    }
+    decode_group(fmt, s0, ss, o + k * RECORD_BYTES);
     ++k;
+    i += g;
   }
   *n_out = k;
   return NVBT_OK;
+}
+
+int nvbt_decode_compact(const void* slots, uint64_t n, void* out, uint64_t cap, uint64_t* n_out) {
+  return nvbt_decode_slots(slots, n, COMPACT_BYTES, out, cap, n_out);
 }
 
 int nvbt_digest_records(const void* records, uint64_t n, nvbt_digest* out) {

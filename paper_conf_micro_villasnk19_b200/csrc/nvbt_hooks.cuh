@@ -50,8 +50,9 @@ struct DevState {
   unsigned n_warps;
   unsigned stripes;                // site/mem/hist repeat `stripes` times, stride stripe_words
   unsigned long long stripe_words;
-  unsigned slot_bytes;             // slot stride: 288, or 192 for compact channels (176 B slots, EM §5.1, padded)
-  unsigned compact;
+  unsigned slot_bytes;             // slot stride: 288, 192 (176 B compact slots, EM §5.1, padded) or 128 (EM §5.2)
+  unsigned compact;                // 0 full records; 1 / 2 176 B slots (2: force wide pairs); 3 / 4 128 B slots
+                                   // (4: force the three-slot form)
   unsigned no_wait;                // device-memory ring (F2): drop when full instead of waiting
   // device ring (F2): slots are handed out in chunks of kRingChunk. Each SM owns a stripe word
   // rheads[smid % rstripes] = (chunk << 32 | used) and takes tickets from its current chunk; the warp whose
@@ -465,6 +466,63 @@ struct Hooks {
     const unsigned E = P;
     const unsigned long long base = __shfl_sync(FULL, addr, __ffs(E) - 1);
     const long long dl = (long long)(addr - base);
+    if (st.compact >= 3u) {
+      // 128 B slots (EM §5.2): one whole PCIe line per record when every lane of E is within +-32 KB of
+      // the first (header, base, 32 x i16 deltas), else three slots of full addresses
+      if (st.compact == 3u && __all_sync(FULL, !act || (dl >= -32768ll && dl <= 32767ll))) {
+        if (reserve(1, t)) {
+          unsigned* tp;
+          unsigned char* rec = slot_ptr(t, tag, tp);
+          // u32 word k of the delta area (bytes 40..103) = delta[2k] | delta[2k + 1] << 16, built on lane 2k
+          const unsigned d16 = act ? ((unsigned)dl & 0xFFFFu) : 0u;
+          const unsigned wp = d16 | (__shfl_down_sync(FULL, d16, 1) << 16);
+          // chunk c = bytes 16c .. 16c + 15: 0, 1 header; 2 base + words 0, 1; 3..5 words 4c - 10 ..; 6 words
+          // 14, 15; 7 zero
+          const int k0 = lane == 2u ? 0 : lane == 6u ? 14 : 4 * (int)lane - 10;
+          const unsigned s0 = (2u * (unsigned)k0) & 31u;
+          const unsigned u0 = __shfl_sync(FULL, wp, s0), u1 = __shfl_sync(FULL, wp, (s0 + 2u) & 31u);
+          const unsigned u2 = __shfl_sync(FULL, wp, (s0 + 4u) & 31u), u3 = __shfl_sync(FULL, wp, (s0 + 6u) & 31u);
+          if (lane < 8) {
+            const uint4 v = lane == 0   ? make_uint4(st.launch, gwarp, seq, (unsigned)PC)
+                            : lane == 1 ? make_uint4(A, P, w2 | 0x80000000u, 0u)
+                            : lane == 2 ? make_uint4((unsigned)base, (unsigned)(base >> 32), u0, u1)
+                            : lane <= 5 ? make_uint4(u0, u1, u2, u3)
+                            : lane == 6 ? make_uint4(u0, u1, 0u, 0u)
+                                        : make_uint4(0u, 0u, 0u, 0u);
+            *reinterpret_cast<uint4*>(rec + 16 * lane) = v;
+          }
+          add_pending(tp, tag);
+        }
+      } else if (reserve(3, t)) {
+        // three slots: slot 0 = header (kind | 0x40) + lanes 0..11; slots 1, 2 carry flag 0x20 at byte 27
+        // and lanes 12..26 (bytes 0..23: 3 lanes, 32..127: 12 lanes) and 27..31
+        unsigned tg[3];
+        unsigned* tps[3];
+        unsigned char* r[3];
+#pragma unroll
+        for (int k = 0; k < 3; ++k) r[k] = slot_ptr(t + k, tg[k], tps[k]);
+        const unsigned sl = lane >> 3, c = lane & 7u;
+        // first lane of the chunk's address pair: slot 0 chunk c >= 2: 2(c-2); slots 1, 2: chunk 0 -> 12 + 15(s-1),
+        // chunk 1 -> 14 + 15(s-1) (one address + the flag word), chunk c >= 2 -> 15 + 15(s-1) + 2(c-2)
+        const unsigned src = sl == 0u ? 2u * (c - 2u) : (15u * (sl - 1u) + (c == 0u ? 12u : c == 1u ? 14u : 15u + 2u * (c - 2u)));
+        const unsigned long long a0 = __shfl_sync(FULL, a, src & 31u), a1 = __shfl_sync(FULL, a, (src + 1u) & 31u);
+        if (lane < 24) {
+          const bool hdr = sl == 0u && c < 2u;
+          const bool flagw = sl != 0u && c == 1u;
+          const bool zero = sl == 2u && c >= 3u;
+          const uint4 v = hdr ? (c == 0u ? make_uint4(st.launch, gwarp, seq, (unsigned)PC) : make_uint4(A, P, w2 | 0x40000000u, 0u))
+                        : flagw ? make_uint4((unsigned)a0, (unsigned)(a0 >> 32), 0x20000000u, 0u)
+                        : zero ? make_uint4(0u, 0u, 0u, 0u)
+                               : make_uint4((unsigned)a0, (unsigned)(a0 >> 32), (unsigned)a1, (unsigned)(a1 >> 32));
+          *reinterpret_cast<uint4*>(r[sl] + 16 * c) = v;
+        }
+        add_pending(tps[0], tg[0]);
+        add_pending(tps[1], tg[1]);
+        add_pending(tps[2], tg[2]);
+      }
+      ++seq;
+      return;
+    }
     if (st.compact == 1u && __all_sync(FULL, !act || (dl >= -0x80000000ll && dl <= 0x7fffffffll))) {
       if (reserve(1, t)) {
         unsigned* tp;

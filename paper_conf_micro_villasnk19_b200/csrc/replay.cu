@@ -427,7 +427,9 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
   unsigned f_lo, f_hi;
   lds_v2(rowb + 16u * ((f >> 1) ^ sw) + 8u * (f & 1u), f_lo, f_hi);
   unsigned prev = f_lo, hb = 0, bs = 0, bl = 0, mn = f_lo, mx = f_lo;
-  unsigned sbits = 0;   // (tags build) the 1 KB-word sector bits of the scanned addresses (bit (a >> 5) & 31)
+#if NVBT_RPB_TAGS && NVBT_RPB_SBITS
+  unsigned sbits = 0;   // the 1 KB-word sector bits of the scanned addresses (bit (a >> 5) & 31)
+#endif
   bool viol = false;
 #pragma unroll
   for (int q = 0; q < ((NVBT_RPB_EXPERIMENT & 2) ? 1 : 8); ++q) {   // (experiment 2: scan 2 addresses only)

@@ -28,6 +28,7 @@ W_VECTORADD, W_SGEMM, W_BFS, W_STENCIL, W_REPLAY, W_WFFT_EMU, W_WFFT_SW = 1, 2, 
 WFFT_PROXY, WFFT_SOFTWARE = 0, 1
 RECORD_BYTES = 288
 COMPACT_RECORD_BYTES = 176
+COMPACT128_RECORD_BYTES = 128
 
 
 class InstrDesc(C.Structure):
@@ -93,6 +94,7 @@ _sigs = {
     "nvbt_channel_dropped": ([_P, C.POINTER(C.c_uint64)], C.c_int),
     "nvbt_digest_records": ([_P, C.c_uint64, C.POINTER(Digest)], C.c_int),
     "nvbt_decode_compact": ([_P, C.c_uint64, _P, C.c_uint64, C.POINTER(C.c_uint64)], C.c_int),
+    "nvbt_decode_slots": ([_P, C.c_uint64, C.c_uint32, _P, C.c_uint64, C.POINTER(C.c_uint64)], C.c_int),
     "nvbt_trace_footprint": ([_P, _P, C.c_uint64, C.c_uint32, C.c_uint32, _P, _P], C.c_int),
     "nvbt_gen_events": ([_P, C.c_uint64, C.c_uint64, C.c_uint64, _P, _P], C.c_int),
     "nvbt_replay": ([_P, _P, _P, C.c_uint64], C.c_int),
@@ -180,13 +182,14 @@ def nvbt_workspace_size(prog_len, n_opcodes, n_bbs, flags, n_warps=0):
     return b.value
 
 
-def nvbt_decode_compact(slots_u8):
-    """Decode a numpy uint8 [n, 176] array of compact transport slots into EM §5 records [m, 288]."""
+def nvbt_decode_compact(slots_u8, record_bytes=COMPACT_RECORD_BYTES):
+    """Decode a numpy uint8 [n, record_bytes] array of compact transport slots (176: EM §5.1, 128: EM §5.2)
+    into EM §5 records [m, 288]."""
     sl = np.ascontiguousarray(slots_u8, dtype=np.uint8)
     out = np.zeros((sl.shape[0], RECORD_BYTES), dtype=np.uint8)
     k = C.c_uint64()
-    _check(_lib.nvbt_decode_compact(sl.ctypes.data_as(C.c_void_p), sl.shape[0], out.ctypes.data_as(C.c_void_p),
-                                    sl.shape[0], C.byref(k)))
+    _check(_lib.nvbt_decode_slots(sl.ctypes.data_as(C.c_void_p), sl.shape[0], record_bytes,
+                                  out.ctypes.data_as(C.c_void_p), sl.shape[0], C.byref(k)))
     return out[:k.value]
 
 
@@ -314,23 +317,35 @@ class Channel:
         self.handle, self.ctx, self.ring = handle, ctx, ring
 
 
+def _record_bytes(compact):
+    """compact: False (288 B records), True or 176 (176 B slots, EM §5.1), 128 (128 B slots, EM §5.2)."""
+    if compact is False or compact is None or compact == 0:
+        return RECORD_BYTES
+    if compact is True or compact == COMPACT_RECORD_BYTES:
+        return COMPACT_RECORD_BYTES
+    if compact == COMPACT128_RECORD_BYTES:
+        return COMPACT128_RECORD_BYTES
+    raise ValueError(f"compact={compact!r}: use False, True / 176 or 128")
+
+
 def nvbt_channel_slot_bytes(compact=False):
-    """Ring stride of one transport slot (288, or 192 for the 176 B compact slots, EM §5.1)."""
-    return 192 if compact else RECORD_BYTES
+    """Ring stride of one transport slot: 288, 192 (176 B slots, EM §5.1, padded) or 128 (EM §5.2)."""
+    rb = _record_bytes(compact)
+    return 192 if rb == COMPACT_RECORD_BYTES else rb
 
 
 def nvbt_channel_bytes(slots, compact=False, on_device=False):
-    """Ring size (bytes) that holds `slots` slots: 64 + slots * (record + 4-byte tag) for host rings."""
-    rb = COMPACT_RECORD_BYTES if compact else RECORD_BYTES
-    return int(_lib.nvbt_channel_bytes(rb, slots, 1 if on_device else 0))
+    """Ring size (bytes) that holds `slots` slots: header + slots * (slot stride + 4-byte tag) for host rings."""
+    return int(_lib.nvbt_channel_bytes(_record_bytes(compact), slots, 1 if on_device else 0))
 
 
 def nvbt_channel_open(ctx, ring, compact=False):
     """ring: pinned uint8 torch tensor (torch.empty(..., pin_memory=True)), or a CUDA uint8 tensor for an
-    on-GPU channel (F2); compact: 176 B transport slots (base + 32-bit deltas, EM §5.1)."""
+    on-GPU channel (F2); compact: False (288 B records), True / 176 (base + 32-bit deltas, EM §5.1) or 128
+    (one 128 B line per record with 16-bit deltas, EM §5.2)."""
     h = C.c_void_p()
-    rb = COMPACT_RECORD_BYTES if compact else RECORD_BYTES
-    _check(_lib.nvbt_channel_open(ctx.handle, C.c_void_p(ring.data_ptr()), ring.numel(), rb, C.byref(h)))
+    _check(_lib.nvbt_channel_open(ctx.handle, C.c_void_p(ring.data_ptr()), ring.numel(), _record_bytes(compact),
+                                  C.byref(h)))
     ch = Channel(h, ctx, ring)
     ctx.channel = ch
     return ch

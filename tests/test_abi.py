@@ -123,6 +123,65 @@ def test_compact_decode_matches_records():
         nb.nvbt_decode_compact(slots[(slots[:, 27] & 0xE0) == 0x20][:1])
 
 
+def _encode_compact128(recs, long_mask):
+    """Test-side encoder of EM §5.2 (written from the spec): record r -> one 128 B short slot (base + 32 x
+    i16 deltas), or three slots of full addresses when long_mask[r] (or a delta does not fit 16 bits)."""
+    import struct
+    out = []
+    for r, rec in enumerate(recs):
+        b = bytes(rec)
+        A, P = struct.unpack_from("<II", b, 16)
+        E = A & P
+        addr = struct.unpack_from("<32Q", b, 32)
+        kind = b[27]
+        lanes = [l for l in range(32) if (E >> l) & 1]
+        base = addr[lanes[0]]
+        fits = all(-32768 <= addr[l] - base <= 32767 for l in lanes)
+        if fits and not long_mask[r]:
+            sl = bytearray(128)
+            sl[0:27] = b[0:27]
+            sl[27] = kind | 0x80
+            struct.pack_into("<Q", sl, 32, base)
+            for l in lanes:
+                struct.pack_into("<h", sl, 40 + 2 * l, addr[l] - base)
+            out.append(sl)
+        else:
+            s0 = bytearray(128)
+            s0[0:27] = b[0:27]
+            s0[27] = kind | 0x40
+            struct.pack_into("<12Q", s0, 32, *addr[0:12])
+            s1, s2 = bytearray(128), bytearray(128)
+            for sl, lo in ((s1, 12), (s2, 27)):
+                sl[27] = 0x20
+                struct.pack_into("<3Q", sl, 0, *addr[lo:lo + 3])
+                rest = addr[lo + 3:min(lo + 15, 32)]
+                struct.pack_into(f"<{len(rest)}Q", sl, 32, *rest)
+            out += [s0, s1, s2]
+    return np.frombuffer(b"".join(out), dtype=np.uint8).reshape(-1, 128)
+
+
+def test_compact128_decode_matches_records():
+    """EM §5.2 slots decode back to the EM §5 records (stencil records as short slots, 30 % forced long, and
+    BFS-like records whose spans need the long form)."""
+    from paper_conf_micro_villasnk19_b200 import nvbt as nb
+    from oracle import events as ev, programs
+    from oracle.models import stencil
+    acc = ev.Accumulator(programs.stencil(), trace=True, keep_records=True)
+    stencil.run(acc, 64, 1 << 32, (1 << 32) + (1 << 24))
+    recs = acc.record_array().copy()
+    words = recs.view("<u8").reshape(-1, 36)
+    hdr = recs.view("<u4").reshape(-1, 72)
+    lane5 = ((hdr[:, 4] & hdr[:, 5]) >> 5) & 1 == 1          # lane 5 executes
+    sel = lane5 & (np.arange(len(recs)) % 7 == 0)
+    words[sel, 4 + 5] += np.uint64(1 << 20)                    # 1 MB away: these need the long form
+    long_mask = np.random.default_rng(1).random(len(recs)) < 0.3
+    slots = _encode_compact128(recs, long_mask)
+    dec = nb.nvbt_decode_compact(slots, record_bytes=128)
+    assert dec.shape == recs.shape and (dec == recs).all()
+    with pytest.raises(nb.NvbtError):          # a long record without its continuation slots is rejected
+        nb.nvbt_decode_compact(slots[(slots[:, 27] & 0xE0) == 0x40][:1], record_bytes=128)
+
+
 def test_channel_bytes_layout():
     """nvbt_channel_bytes follows include/nvbt.h: 64-byte header, then per slot the record (compact: 176 B
     padded to 192) plus a 4-byte commit tag for pinned host rings; device rings (F2) carry no tag array."""
@@ -133,3 +192,4 @@ def test_channel_bytes_layout():
     assert f(176, 7, 0) == 64 + 7 * (192 + 4)      # compact slots padded to a 192 B stride
     assert f(288, 1 << 22, 1) == 64 + 288 * (1 << 22)
     assert f(288, 0, 0) == 64
+    assert f(128, 9, 0) == 128 + 9 * (128 + 4)     # 128 B slots: 128 B header, line-aligned slots

@@ -43,7 +43,7 @@ def test_bench_line_all_configs(nvbt):
         assert k in d, k
     assert d["n_gpus"] == 1 and d["counts_check"] == "ok" and d["gpu_launches"] == 3
     assert d["cpu_baseline"]["matches_gpu"] is True
-    assert set(d["configs"]) == {"c1", "c3", "c4", "c4_compact", "c5"}
+    assert set(d["configs"]) == {"c1", "c3", "c4", "c4_compact", "c4_line", "c5"}
     for name, c in d["configs"].items():
         assert c["counts_check"].startswith("ok"), (name, c["counts_check"])
         assert c["value"] > 0

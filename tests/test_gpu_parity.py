@@ -169,6 +169,53 @@ def test_channel_compact_transport(nvbt, monkeypatch, force_wide, ring):
     _stencil_case(nvbt, 64, 2, ring_records=ring, tools_names=("TRACE", "MEMDIV"), compact=True)
 
 
+@pytest.mark.parametrize("force_long,ring", [("0", 1 << 16), ("0", 5), ("1", 1 << 16), ("1", 7), ("1", 4), ("1", 3)])
+def test_channel_compact128_transport(nvbt, monkeypatch, force_long, ring):
+    """EM §5.2 128 B slots: decoded records equal the oracle's; the forced three-slot form on 3/4/7-slot
+    rings exercises records straddling the ring end (the drain stashes their first slots)."""
+    monkeypatch.setenv("NVBT_COMPACT_FORCE_WIDE", force_long)
+    _stencil_case(nvbt, 64, 2, ring_records=ring, tools_names=("TRACE", "MEMDIV"), compact=128)
+
+
+def test_channel_compact128_bfs(nvbt):
+    """BFS records (gathers across MBs) need the three-slot form of EM §5.2; mixed with one-slot records on
+    a small ring, every record arrives intact (multiset == the oracle's)."""
+    import torch
+    nb, dr = nvbt.nvbt, nvbt.drivers
+    rowptr, col = rmat_csr(10, 16, seed=3)
+    n = len(rowptr) - 1
+    src = bfs_source(rowptr)
+    ctx = nb.nvbt_init(nb.W_BFS, nb.TRACE)
+    rp, cl = cuda(rowptr), cuda(col)
+    bufs = dr.bfs_buffers(n, "cuda")
+    ring = torch.empty(nb.nvbt_channel_bytes(1 << 10, compact=128), dtype=torch.uint8, pin_memory=True)
+    ch = nb.nvbt_channel_open(ctx, ring, compact=128)
+    acc = ev.Accumulator(programs.bfs(), trace=True, keep_records=True)
+    ptr = m_bfs.Ptrs(bufs["mask"].data_ptr(), bufs["visited"].data_ptr(), bufs["updating"].data_ptr(),
+                     bufs["cost"].data_ptr(), bufs["over"].data_ptr(), rp.data_ptr(), cl.data_ptr())
+    m_bfs.run(acc, rowptr, col, src, ptr)
+    exp = acc.record_array()
+    dst = np.zeros((len(exp) + 1024, 288), dtype=np.uint8)
+    got_n = 0
+    import threading
+    done, out = threading.Event(), []
+
+    def drain():   # the ring (1024 slots) is far smaller than the trace: drain while the BFS runs
+        while True:
+            fin = done.is_set()
+            out.append(nb.nvbt_channel_drain_copy(ch, dst[sum(out):], timeout_us=60_000_000))
+            if fin:
+                return
+    th = threading.Thread(target=drain)
+    th.start()
+    dr.run_bfs(ctx, nb.TOOL_TRACE, rp, cl, src, bufs)
+    done.set()
+    th.join()
+    got_n = sum(out)
+    assert nb.nvbt_channel_dropped(ch) == 0 and got_n == len(exp)
+    assert (trace.sort_records(dst[:got_n]) == trace.sort_records(exp)).all()
+
+
 def test_channel_digest_drain(nvbt):
     import torch
     nb, dr = nvbt.nvbt, nvbt.drivers
