@@ -385,6 +385,8 @@ def run_c2(args, torch, nb, dr, rank, world, local, peaks, peaks_src):
                 "d2h_bytes_per_step": d2h},
         "gpu_launches": int(gpu_launches), "clocks": clk.summary(), "peaks_source": peaks_src,
         "merge_ms": merge_ms,
+        "paper_context": ("the paper's opcode-histogram tool (this path's a3): 36.4x average, up to 112x slowdown "
+                          "fully instrumented, 2.3x with kernel sampling; TITAN V (Volta), SpecAccel (P:L278-280)"),
     }
     line["roofline"]["peak_source"] = f"148 SMs x 4 issue/clk x sm_max_mhz ({peaks_src})"
     # the binding resource of this workload is the application's own L1 traffic (the naive row-fastest
@@ -878,6 +880,7 @@ def run_ours(args):
     wanted = [c for c in args.configs.split(",") if c and c != "none"]
     cfg = {}
     for c in wanted:
+        torch.cuda.nvtx.range_push(f"nvbt bench {c}")
         if c == "c1":
             cfg["c1"] = run_c1(args, torch, nb, dr, rank, world, local, args.steps)
         elif c == "c3":
@@ -890,6 +893,7 @@ def run_ours(args):
             cfg["c4_line"] = run_c4(args, torch, nb, dr, rank, world, local, args.c4_steps, compact=128)
         elif c == "c5":
             cfg["c5"] = run_c5(args, torch, nb, dr, rank, world, local, args.c5_steps, peaks, peaks_src)
+        torch.cuda.nvtx.range_pop()
         torch.cuda.empty_cache()
     if cfg:
         line["configs"] = cfg

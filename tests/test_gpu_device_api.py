@@ -29,9 +29,12 @@ COUNT_KEYS = ["counts", "H_t", "H_w", "Ent_w", "Ent_t", "Ins_w", "Ins_t"]
 MEM_KEYS = ["mem_n", "mem_S", "mem_L", "hS", "hL"]
 
 
-def build_ext(out_dir):
+def build_ext(out_dir, check_converged=True):
+    """nvcc against include/ only; with check_converged every hook traps unless the whole warp reached it
+    (NVBT_CHECK_CONVERGED, the converged-hook discipline R-15)."""
     so = os.path.join(out_dir, "libext_gather.so")
     cmd = [NVCC, "-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-std=c++17", "-shared", "-Xcompiler", "-fPIC",
+           *(["-DNVBT_CHECK_CONVERGED"] if check_converged else []),
            "-I", os.path.join(ROOT, "include"), SRC, "-o", so]
     r = subprocess.run(cmd, capture_output=True, text=True)
     assert r.returncode == 0, r.stdout + r.stderr

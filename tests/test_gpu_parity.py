@@ -216,6 +216,36 @@ def test_channel_compact128_bfs(nvbt):
     assert (trace.sort_records(dst[:got_n]) == trace.sort_records(exp)).all()
 
 
+def test_channel_drop_is_reported(nvbt):
+    """A host ring nobody drains while the kernel runs: the producers wait ~2 s for room, then give up; the
+    records they drop are counted (nvbt_channel_dropped) and the drain fails loudly (NVBT_ETIMEDOUT) after
+    delivering what was committed, instead of hanging or passing silently (include/nvbt.h: the channel
+    must then be reopened)."""
+    import torch
+    nb, dr = nvbt.nvbt, nvbt.drivers
+    n = 64
+    ctx = nb.nvbt_init(nb.W_STENCIL, nb.TRACE)
+    x0 = cuda(uniform_f32((n, n), 4))
+    b0, b1 = x0.clone(), torch.zeros_like(x0)
+    ring = torch.empty(nb.nvbt_channel_bytes(8), dtype=torch.uint8, pin_memory=True)
+    ch = nb.nvbt_channel_open(ctx, ring)
+    dr.run_stencil(ctx, nb.TOOL_TRACE, b0, b1, n, 1)
+    torch.cuda.synchronize()                     # no consumer ran: the ring filled up
+    dropped = nb.nvbt_channel_dropped(ch)
+    assert dropped > 0
+    dst = np.zeros((1024, 288), dtype=np.uint8)
+    with pytest.raises(nb.NvbtError) as e:
+        nb.nvbt_channel_drain_copy(ch, dst, timeout_us=30_000_000)
+    assert e.value.code == nb.ETIMEDOUT and "dropped" in str(e.value)
+    nb.nvbt_channel_close(ch)
+    ch = nb.nvbt_channel_open(ctx, ring)          # a reopened channel works again
+    nb.nvbt_reset(ctx)
+    dr.run_stencil(ctx, nb.TOOL_TRACE, b0, b1, n, 1)
+    G = n // 32
+    got = nb.nvbt_channel_drain_copy(ch, dst, timeout_us=30_000_000)   # drains while the kernel runs
+    assert got == 4 * G + 6 * G * (n - 2) and nb.nvbt_channel_dropped(ch) == 0
+
+
 def test_channel_digest_drain(nvbt):
     import torch
     nb, dr = nvbt.nvbt, nvbt.drivers
