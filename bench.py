@@ -54,15 +54,15 @@ def _profile_json(name):
 
 
 def load_traffic(kernel):
-    """DRAM bytes per launch of `kernel` from the committed ncu capture (profiles/r1_traffic.json)."""
-    d = _profile_json("r1_traffic.json")
+    """DRAM bytes per launch of `kernel` from the committed ncu capture (profiles/r2_traffic.json)."""
+    d = _profile_json("r2_traffic.json")
     return None if d is None else d.get(kernel)
 
 
 def load_counters(kernel, keys=("warp_inst_per_unit", "dram_bytes_per_unit", "shared_atomic_wavefronts_per_unit",
                                  "global_atomic_sectors_per_unit", "issue_active_pct")):
-    """ncu counters per unit of work of `kernel` from the committed capture (profiles/r1_ncu_counters.json)."""
-    d = (_profile_json("r1_ncu_counters.json") or {}).get(kernel)
+    """ncu counters per unit of work of `kernel` from the committed capture (profiles/r2_ncu_counters.json)."""
+    d = (_profile_json("r2_ncu_counters.json") or {}).get(kernel)
     return None if d is None else {k: d[k] for k in keys if k in d}
 
 
@@ -316,7 +316,7 @@ class SgemmBench:
         t = load_traffic("k_sgemm<6>")
         return {"bound": "alu", "achieved": ach / 1e9, "peak": peak / 1e9, "unit": "Gwarp-inst/s",
                 "frac": ach / peak, "traffic": t["traffic_bytes_per_launch"] if t else None,
-                "traffic_unit": "DRAM bytes per launch (ncu, profiles/r1_traffic.json)",
+                "traffic_unit": "DRAM bytes per launch (ncu, profiles/r2_traffic.json)",
                 "algorithmic_hook_warp_inst_per_launch": ops,
                 "with_app_instructions_frac": (ops + W * self.per_warp) / t_kernel_s / peak}
 
@@ -393,10 +393,10 @@ def run_c2(args, torch, nb, dr, rank, world, local, peaks, peaks_src):
     # SGEMM is L1-wavefront-bound uninstrumented); the hooks run inside that bound
     line["app_bound"] = {"resource": "L1TEX wavefronts of the uninstrumented SGEMM",
                          "instr_speed_vs_plain": statistics.median(t_plain) / statistics.median(t_instr),
-                         "ncu": "profiles/r1_ncu_summary_c2_c5.txt: l1tex 98.8 % (plain) / 95.2 % (instrumented), "
-                                "issue-active 6.9 % / 85.2 %"}
+                         "ncu": "profiles/r2_ncu_summary_c2.txt: l1tex 98.6 % (plain) / 94.9 % (instrumented), "
+                                "issue-active 7.0 % / 85.0 %"}
     line["ncu_per_event"] = {"instrumented": load_counters("k_sgemm<6>"), "plain": load_counters("k_sgemm<0>"),
-                             "source": "profiles/r1_ncu_counters.json (ncu --set full, tools/prof_step.py c2)"}
+                             "source": "profiles/r2_ncu_counters.json (ncu --set full, tools/prof_step.py c2)"}
     return line, wl
 
 
@@ -853,7 +853,7 @@ def run_f4(args, torch, nb, dr, local):
             "roofline": {"bound": "hbm", "achieved": bytes_launch / t_k / 1e9, "peak": hbm_peak, "unit": "GB/s",
                          "frac": bytes_launch / t_k / 1e9 / hbm_peak,
                          "traffic": (load_traffic("k_wfft<17,0>") or {}).get("traffic_bytes_per_launch"),
-                         "traffic_unit": "DRAM bytes per launch (ncu, profiles/r1_traffic.json)",
+                         "traffic_unit": "DRAM bytes per launch (ncu, profiles/r2_traffic.json)",
                          "algorithmic_bytes_per_launch": bytes_launch, "kernel": "k_wfft<EMU|COUNT, proxy>"},
             "sw_plain_hbm_frac": bytes_launch / med["sw_plain"] / 1e9 / hbm_peak,
             "clocks": clk.summary(), "peaks_source": peaks_src,

@@ -12,7 +12,8 @@ from synth import uniform_f32  # noqa: E402
 
 nb = pkg.nvbt
 n = 8192
-compact = len(sys.argv) > 1 and sys.argv[1] == "compact"
+arg = sys.argv[1] if len(sys.argv) > 1 else ""
+compact = {"compact": True, "line": 128}.get(arg, False)   # 176 B slots (EM 5.1) / 128 B line slots (EM 5.2)
 ctx = nb.nvbt_init(nb.W_STENCIL, nb.COUNT | nb.TRACE)
 x = torch.from_numpy(uniform_f32((n, n), 4)).cuda()
 y = torch.empty_like(x)
