@@ -41,7 +41,8 @@
  *                                             64-bit atomic per non-zero bin (P:L89's per-block counters).
  * Event formation (EM §1): A = ballot(in_flow), P = ballot(in_flow && pred) (P is A's subset), E = A & P
  * ("a false predicate value means that the instrumented instruction is not actually executing").
- * All CTA bins are 64-bit, so no count can wrap. Warp ids for the per-warp arrays are EM §1's
+ * All CTA bins are 64-bit, so no count can wrap. Shared memory: NVBT_DEV_SMEM_BYTES(P, W) = 8 (7 P + 66) +
+ * 768 W bytes (about 7 KB for P = 64 pcs and 8 warps); programs beyond ~3,900 pcs do not fit one CTA. Warp ids for the per-warp arrays are EM §1's
  * linear_cta * warps_per_cta + tid_linear / 32; the CTA must hold a whole number of warps.
  */
 #pragma once

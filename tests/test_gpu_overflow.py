@@ -70,3 +70,28 @@ def test_bfs_hub_of_degree_2_24_is_reported(nvbt):
     assert e.value.code == nb.EINVAL
     nb.nvbt_reset(ctx)
     assert (nb.nvbt_count(ctx) == 0).all()
+
+
+def test_wfft_loop_beyond_spill_chunk(nvbt):
+    """WFFT32's per-warp transform loop runs in chunks of 2^20 instances with the counters spilled to the
+    64-bit bins in between (Hooks::spill): one CTA (8 warps), k_w = 2^20 + 2 transforms per warp. Counts and
+    per-warp arrays equal the EM §3.6 closed form (W_issued = 6 + 8 k_w, W_exec = 4 + 8 k_w per warp for
+    WFFT_EMU), divergence bins too (each load / store: 256 contiguous bytes = 8 sectors, 2 lines)."""
+    import torch
+    nb = nvbt.nvbt
+    ctas, kw = 1, (1 << 20) + 2
+    W = 8 * ctas
+    n_fft = W * kw
+    x = torch.zeros((n_fft, 32, 2), dtype=torch.float32, device="cuda").view(torch.complex64).reshape(n_fft, 32)
+    X = torch.empty_like(x)
+    ctx = nb.nvbt_init(nb.W_WFFT_EMU, nb.COUNT | nb.OPHIST | nb.BB | nb.MEMDIV | nb.PER_WARP, n_warps=W)
+    nb.nvbt_wfft32(ctx, nb.TOOL_EMU | nb.TOOL_COUNT | nb.TOOL_MEMDIV, nb.WFFT_PROXY, x, X, n_fft, ctas)
+    g = read_all(nb, ctx, per_warp=True)
+    wi, we = 6 + 8 * kw, 4 + 8 * kw
+    assert g["counts"].tolist() == [32 * W * wi, 32 * W * we, W * wi, W * we]
+    assert g["PW_T"].tolist() == [32 * we] * W and g["PW_W"].tolist() == [we] * W
+    assert (g["mem_n"][6], g["mem_S"][6], g["mem_L"][6]) == (W * kw, 8 * W * kw, 2 * W * kw)
+    assert (g["mem_n"][9], g["mem_S"][9], g["mem_L"][9]) == (W * kw, 8 * W * kw, 2 * W * kw)
+    assert g["hS"][8] == 2 * W * kw and g["hL"][2] == 2 * W * kw
+    del x, X
+    torch.cuda.empty_cache()
