@@ -5,7 +5,7 @@
   C3  BFS on the R-MAT scale-20 graph, COUNT|MEMDIV|PER_WARP and BBCOUNT
   C4  stencil 8192^2 x 100 with COUNT|MEMDIV|TRACE in ONE run through the pinned-host channel: counts,
       histograms, per-pc divergence and the trace multiset digest (N_rec, D1, D2), plus SURVEY I-3's
-      ΣS = 5,450,035,600 and ΣL = 1,675,776,400
+      ΣS = 5,450,035,600 and ΣL = 1,675,776,400; then the same trace through both compact transports
   C5  all 10^10 generated events through the staged replay in 2^27-event chunks (and the single-pass
       kernel on the same chunks)
 
@@ -122,7 +122,21 @@ def test_c4_stencil_trace_full_size(nvbt):
     assert d.n_rec == 1_258_086_400
     assert int(g["mem_S"].sum()) == 5_450_035_600 and int(g["mem_L"].sum()) == 1_675_776_400
     gpu_invariants(g)
+    nb.nvbt_channel_close(ch)
     del ring
+    # the same 100 launches (launch ids restart at reset, same buffers: the same record multiset) through
+    # the two compact transports (F3, EM §5.1 / §5.2), decoded on the host: identical digests
+    for compact in (True, 128):
+        nb.nvbt_reset(ctx)
+        ring = torch.empty(nb.nvbt_channel_bytes(1 << 22, compact=compact), dtype=torch.uint8, pin_memory=True)
+        ch = nb.nvbt_channel_open(ctx, ring, compact=compact)
+        dr.run_stencil(ctx, nb.TOOL_TRACE, b0, b1, n, iters)
+        dc = nb.nvbt_channel_drain_digest(ch, timeout_us=900_000_000)
+        torch.cuda.synchronize()
+        assert nb.nvbt_channel_dropped(ch) == 0
+        assert (dc.n_rec, dc.d1, dc.d2) == tuple(int(x) for x in r["trace"]), f"C4 compact={compact} digest"
+        nb.nvbt_channel_close(ch)
+        del ring
 
 
 def test_c5_replay_full_size(nvbt):
