@@ -71,7 +71,8 @@ __global__ void __launch_bounds__(256) k_gen(GenConsts G, unsigned long long fir
       const unsigned long long b = __shfl_sync(FULL, base, src);
       const unsigned long long ss = __shfl_sync(FULL, s, src);
       const unsigned long long wd = prog[ps].width;
-      const unsigned long long r = mix64(klane ^ is);
+      // R(i, 64 + lane) only for the two random patterns (pt is warp-uniform: no divergence)
+      const unsigned long long r = (pt == 3u || pt == 4u) ? mix64(klane ^ is) : 0ull;
       unsigned long long a;
       switch (pt) {
         case 0: a = b + lane * wd; break;
