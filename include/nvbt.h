@@ -139,7 +139,11 @@ size_t nvbt_channel_bytes(uint32_t record_bytes, uint64_t slots, int on_device);
  * record_bytes: NVBT_RECORD_BYTES (288: every slot is an EM §5 record), NVBT_COMPACT_RECORD_BYTES (176:
  * base + 32-bit deltas, wide address sets as two slots; EM §5.1, F3) or NVBT_COMPACT128_RECORD_BYTES (128:
  * one whole PCIe line per record with base + 16-bit deltas, other records as three slots; EM §5.2). Every
- * way the drain delivers EM §5 records. One channel per context. */
+ * way the drain delivers EM §5 records. One channel per context. The first open on a device loads every
+ * workload kernel variant (cudaFuncGetAttributes): under CUDA lazy loading a kernel's first launch may
+ * synchronise the context, which would wait for a producer that is itself waiting for the drain. A kernel
+ * instrumented through include/nvbt_dev.cuh that traces must likewise be loaded (launched once, or
+ * cudaFuncGetAttributes) before a producer of the same context can block on a full ring. */
 #define NVBT_RECORD_BYTES 288
 #define NVBT_COMPACT_RECORD_BYTES 176
 #define NVBT_COMPACT128_RECORD_BYTES 128

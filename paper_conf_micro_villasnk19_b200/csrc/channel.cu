@@ -358,6 +358,7 @@ int nvbt_channel_open(nvbt_ctx c, void* ring, size_t bytes, uint32_t record_byte
   if (bytes < hdr_of(record_bytes) + 3 * (slot_stride(record_bytes) + 4))
     return set_error(NVBT_ENOMEM, "ring of %zu bytes holds < 3 slots", bytes);
   NVBT_CUDA(cudaSetDevice(c->device));
+  { const int prc = preload_workload_kernels(c->device); if (prc) return prc; }
   cudaPointerAttributes pa{};
   NVBT_CUDA(cudaPointerGetAttributes(&pa, ring));
   const bool on_device = pa.type == cudaMemoryTypeDevice;

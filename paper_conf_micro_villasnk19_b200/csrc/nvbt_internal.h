@@ -88,4 +88,8 @@ int fold(nvbt_ctx ctx);  // runs the fold kernel and copies the result to host-v
 // once per (function, device), errors reported as NVBT_ECUDA.
 int device_sms(int dev);
 int func_smem(const void* fn, int dev, size_t bytes);
+// Loads every workload kernel variant on `dev` once (cudaFuncGetAttributes), so no first launch lazily loads
+// a module while a trace producer waits on the host consumer: under CUDA_MODULE_LOADING=LAZY, loading a
+// kernel may synchronise the context, i.e. wait for a producer that waits for the drain (nvbt_channel_open).
+int preload_workload_kernels(int dev);
 }  // namespace nvbt

@@ -300,6 +300,11 @@ constexpr int RB_NW = 20;     // pass B warps per CTA (warp w of pass B analyses
 #ifndef NVBT_RPB_WIN
 #define NVBT_RPB_WIN 512       // window rows: sectors per tag window, 1024 / WIN rows per iteration (A/B r2_ab9: 256 and 128 slower)
 #endif
+#ifndef NVBT_RPB_PF
+#define NVBT_RPB_PF 0          // 1: list entries two groups ahead and the group after the staged one
+                               // prefetched into L2 (one 256 B cp.async.bulk.prefetch.L2 per row). A/B r2_ab15:
+                               // pass B 1.84 -> 2.21 ms, not kept
+#endif
 #ifndef NVBT_RPB_TAGS
 #define NVBT_RPB_TAGS 1        // slow rows by tag arrays (0: round-1 atomics + reductions, for A/B)
 #endif
@@ -664,25 +669,28 @@ k_rpB(const unsigned long long* __restrict__ addr, unsigned P, const uint8_t* __
   // group cursor over this warp's regions gw, gw + WB, ...
   unsigned r = blockIdx.x * RB_NW + (threadIdx.x >> 5), off = 0;
   unsigned rcnt = r < n_regions ? counts[r] : 0u;
-  // next group's list entries (row j in lanes j and j + 16), loaded one group ahead
-  unsigned nx_rows = 0, nx_r = 0;
-  uint2 nx_ent = make_uint2(0u, 0u);
-  auto fetch = [&]() {
+  // a group: up to 16 list entries of one region (row j in lanes j and j + 16), loaded ahead of use
+  struct Grp { unsigned rows, r; uint2 ent; };
+  auto fetch = [&](Grp& g) {
     while (r < n_regions && off >= rcnt) {
       r += WB;
       off = 0;
       rcnt = r < n_regions ? counts[r] : 0u;
     }
-    nx_rows = r < n_regions ? min(rcnt - off, (unsigned)RB_ROWS) : 0u;
+    g.rows = r < n_regions ? min(rcnt - off, (unsigned)RB_ROWS) : 0u;
     const unsigned long long p = (unsigned long long)r * region_cap + off + j;
-    nx_ent = j < nx_rows ? l_ent[p] : make_uint2(0u, 0u);   // decoded at issue time (load in flight)
-    nx_r = r;
-    off += nx_rows;
+    g.ent = j < g.rows ? l_ent[p] : make_uint2(0u, 0u);   // decoded at use (load in flight)
+    g.r = r;
+    off += g.rows;
   };
-  // stage the fetched group into stage s (meta + slot copies), then fetch the next group
+  auto slot_of = [&](const Grp& g) -> unsigned {   // event index of row j's slot
+    return (g.r + ((g.ent.y >> 5) & 0x7fffu) * n_regions) * 32u + (g.ent.y & 31u);
+  };
+  Grp g1, g2;   // g1: the next group to stage; g2 (NVBT_RPB_PF): the one after it
+  // stage g1 into stage s (meta + slot copies), prefetch g2's slots into L2, advance
   auto issue = [&](unsigned s) {
-    const unsigned nx_E = nx_ent.x, nx_pc = nx_ent.y >> 20;
-    const unsigned nx_idx = (nx_r + ((nx_ent.y >> 5) & 0x7fffu) * n_regions) * 32u + (nx_ent.y & 31u);
+    const unsigned nx_E = g1.ent.x, nx_pc = g1.ent.y >> 20;
+    const unsigned nx_idx = slot_of(g1);
     if (h == 0u)
       asm volatile("st.shared.v2.u32 [%0], {%1, %2};" ::"r"(s_meta + 128u * s + 8u * j), "r"(nx_E), "r"(nx_pc) : "memory");
     const unsigned stg = s_w + 4096u * s;
@@ -691,20 +699,30 @@ k_rpB(const unsigned long long* __restrict__ addr, unsigned P, const uint8_t* __
     for (int k = 0; k < RB_ROWS / 2; ++k) {
       const unsigned row = 2u * k + h;
       const unsigned ix = __shfl_sync(FULL, nx_idx, row);
-      if (row < nx_rows)
+      if (row < g1.rows)
         asm volatile("cp.async.cg.shared.global [%0], [%1], 16;"
                      ::"r"(stg + 256u * row + 16u * (c ^ (row & 7u))), "l"(addr + (unsigned long long)ix * 32u + 2u * c)
                      : "memory");
     }
     asm volatile("cp.async.commit_group;" ::: "memory");
-    fetch();
+#if NVBT_RPB_PF
+    if (h == 0u && j < g2.rows)
+      asm volatile("cp.async.bulk.prefetch.L2.global [%0], 256;" ::"l"(addr + (unsigned long long)slot_of(g2) * 32u) : "memory");
+    g1 = g2;
+    fetch(g2);
+#else
+    fetch(g1);
+#endif
   };
-  fetch();
-  bool live = nx_rows != 0u;
+  fetch(g1);
+#if NVBT_RPB_PF
+  fetch(g2);
+#endif
+  bool live = g1.rows != 0u;
   unsigned s = 0;
   if (live) issue(0);
   while (live) {
-    live = nx_rows != 0u;
+    live = g1.rows != 0u;
     if (live) {
       issue(s ^ 1u);
     } else {

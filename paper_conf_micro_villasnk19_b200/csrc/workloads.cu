@@ -5,6 +5,7 @@
 // reached by all 32 lanes and A/P are exact ballots (EM §1, reading R-15). Loops whose trip count
 // varies per lane run warp-uniformly to the warp's maximum (SIMT-stack / IPDOM semantics). The
 // template parameter T selects the instrumentation variant; T = 0 is the uninstrumented baseline.
+#include <mutex>
 #include <tuple>
 #include <type_traits>
 
@@ -278,6 +279,39 @@ int nvbt_workload_warps(int w, const int64_t* a, uint32_t na, uint64_t* n) {
   }
   return set_error(NVBT_EINVAL, "bad workload %d or arguments", w);
 }
+
+}  // extern "C"
+
+namespace nvbt {
+int preload_workload_kernels(int dev) {
+  static std::mutex mu;
+  static bool done_dev[64] = {};
+  std::lock_guard<std::mutex> g(mu);
+  if (dev < 0 || dev >= 64 || done_dev[dev]) return NVBT_OK;
+  cudaFuncAttributes a;
+  cudaError_t e = cudaSuccess;
+  auto load = [&](const void* fn) { if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, fn); };
+  for (uint32_t t : {0u, 1u, 2u, 4u, 5u, 6u, 8u, 9u, 10u, 12u, 13u, 14u}) {
+    dispatch(t, [&](auto tag) {
+      constexpr uint32_t T = decltype(tag)::value;
+      load((const void*)k_vectoradd<T>);
+      load((const void*)k_sgemm<T>);
+    });
+    for (bool dev_ring : {false, true})
+      dispatch_trace(t, dev_ring, [&](auto tag) {
+        constexpr uint32_t T = decltype(tag)::value;
+        load((const void*)k_bfs_expand<T>);
+        load((const void*)k_bfs_update<T>);
+        load((const void*)k_stencil<T>);
+      });
+  }
+  if (e != cudaSuccess) return set_error(NVBT_ECUDA, "kernel preload: %s", cudaGetErrorString(e));
+  done_dev[dev] = true;
+  return NVBT_OK;
+}
+}  // namespace nvbt
+
+extern "C" {
 
 int nvbt_vectoradd(nvbt_ctx ctx, void* stream, uint32_t tools, const float* a, const float* b, float* c, int32_t N) {
   if (!a || !b || !c || N < 0) return set_error(NVBT_EINVAL, "bad vectorAdd arguments");
