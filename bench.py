@@ -154,6 +154,9 @@ def spawn_ranks(n):
     return subprocess.call(cmd)
 
 
+HOST_PLACEMENT = None   # set by dist_setup for N > 1: the rank's host CPUs (NUMA-local drain)
+
+
 def dist_setup(args):
     import torch
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -162,6 +165,13 @@ def dist_setup(args):
     if os.environ.get("NVBT_BENCH_SAME_GPU"):   # test hook: all ranks on GPU 0 (with a gloo backend)
         local = 0
     torch.cuda.set_device(local)
+    global HOST_PLACEMENT
+    if world > 1 and not os.environ.get("NVBT_BENCH_SAME_GPU") and os.environ.get("NVBT_BENCH_NUMA", "1") != "0":
+        # the rank's drain threads and pinned ring on its GPU's NUMA node, the node's cores split between
+        # the ranks sharing it (before any pinned allocation and before the drain pool exists)
+        from paper_conf_micro_villasnk19_b200 import drivers
+        cpus = drivers.bind_rank_to_gpu_numa(local)
+        HOST_PLACEMENT = {"numa_local": cpus is not None, "cpus": len(cpus) if cpus else len(os.sched_getaffinity(0))}
     if world > 1:
         import torch.distributed as dist
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
@@ -906,6 +916,8 @@ def run_ours(args):
         line["configs"] = cfg
     if world > 1:
         line["allreduce_latency"] = allreduce_latency(world)
+        if HOST_PLACEMENT is not None:
+            line["host_placement_rank0"] = HOST_PLACEMENT
     if rank == 0:
         print(json.dumps(line), flush=True)
     if world > 1:

@@ -15,6 +15,7 @@
 #include <condition_variable>
 #include <cstring>
 #include <functional>
+#include <sched.h>
 #include <immintrin.h>
 #include <thread>
 
@@ -141,7 +142,12 @@ class Pool {
 
  private:
   Pool() {
+    // one thread per CPU this process may run on (a rank bound to its GPU's NUMA node drains on that node's
+    // cores only: drivers.bind_rank_to_gpu_numa), NVBT_DRAIN_THREADS overrides
     unsigned hw = std::thread::hardware_concurrency();
+    cpu_set_t cs;
+    CPU_ZERO(&cs);
+    if (sched_getaffinity(0, sizeof cs, &cs) == 0 && CPU_COUNT(&cs) > 0) hw = (unsigned)CPU_COUNT(&cs);
     const char* e = getenv("NVBT_DRAIN_THREADS");
     if (e) hw = (unsigned)atoi(e);
     if (hw == 0) hw = 1;

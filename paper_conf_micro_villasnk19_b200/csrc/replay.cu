@@ -12,6 +12,9 @@
 #include <cstdlib>
 #include <cstring>
 
+#include <cuda.h>
+#include <cudaTypedefs.h>
+
 #include "nvbt_internal.h"
 #include "nvbt_workloads.h"
 #include "programs.cuh"
@@ -305,6 +308,23 @@ constexpr int RB_NW = 20;     // pass B warps per CTA (warp w of pass B analyses
                                // prefetched into L2 (one 256 B cp.async.bulk.prefetch.L2 per row). A/B r2_ab15:
                                // pass B 1.84 -> 2.21 ms, not kept
 #endif
+#ifndef NVBT_RPB_TMA
+#define NVBT_RPB_TMA 0         // 1: stages filled by TMA gathers (cp.async.bulk.tensor tile::gather4, 128 B swizzle, one
+                               // mbarrier per stage) instead of 16 B cp.async per lane. A/B r2_ab16: results identical,
+                               // pass B 1.84 -> 2.16 ms, not kept
+#endif
+#ifndef NVBT_RPB_RESOLVE
+#define NVBT_RPB_RESOLVE 1     // wide rows whose first hash round collides are resolved against the bucket owners (one
+                               // more tag round) instead of rehashing twice (A/B r2_ab16: pass B 1.839 -> 1.814 ms)
+#endif
+#ifndef NVBT_RPB_WIDE2
+#define NVBT_RPB_WIDE2 0       // 1: wide rows two per iteration (independent chains), 640 hash buckets each, resolved.
+                               // A/B r2_ab17: pass B 1.813 -> 1.894 ms (more collisions, instruction-bound), not kept
+#endif
+#ifndef NVBT_RPB_C0REDUX
+#define NVBT_RPB_C0REDUX 0     // 1: one-1-KB-word rows by an OR-reduction of their sector bits (own loop). A/B r2_ab16:
+                               // pass B 1.839 -> 1.890 ms, not kept
+#endif
 #ifndef NVBT_RPB_TAGS
 #define NVBT_RPB_TAGS 1        // slow rows by tag arrays (0: round-1 atomics + reductions, for A/B)
 #endif
@@ -416,6 +436,35 @@ __device__ __forceinline__ void inc_if_gt(unsigned& c, unsigned x) {
   asm("{\n\t.reg .pred p;\n\tsetp.gt.u32 p, %1, %2;\n\t@p add.u32 %0, %0, 1;\n\t}" : "+r"(c) : "r"(x), "n"(K));
 }
 
+// Exact S, L of one row by a bitonic sort of the sector keys of its active lanes (key a >> 5 of lane `lane`).
+__device__ __forceinline__ void sl_bitonic(unsigned long long a, bool act, unsigned lane, unsigned& sx, unsigned& lx) {
+  unsigned long long k = act ? a >> 5 : ~0ull;
+#pragma unroll
+  for (unsigned kk = 2; kk <= 32; kk <<= 1) {
+#pragma unroll
+    for (unsigned jj = kk >> 1; jj > 0; jj >>= 1) {
+      const unsigned long long o = __shfl_xor_sync(FULL, k, jj);
+      const bool up = (lane & kk) == 0u, lower = (lane & jj) == 0u;
+      k = (lower == up) ? (o < k ? o : k) : (o > k ? o : k);
+    }
+  }
+  const unsigned long long pk = __shfl_up_sync(FULL, k, 1);
+  const bool valid = k != ~0ull;
+  sx = __popc(__ballot_sync(FULL, valid && (lane == 0u || pk != k)));
+  lx = __popc(__ballot_sync(FULL, valid && (lane == 0u || (pk >> 2) != (k >> 2))));
+}
+
+// Byte offset of address idx (0..31) of stage row r. cp.async stages: row r at 256 r, 16 B chunk c at chunk
+// c ^ (r & 7). TMA stages: the two 128 B halves of every row in separate 2 KB blocks (row r at 128 r), chunks
+// XOR-swizzled by (r & 7) -- the tensor map's 128 B swizzle on a 1024-aligned stage.
+__device__ __forceinline__ unsigned rb_off(unsigned r, unsigned idx) {
+#if NVBT_RPB_TMA
+  return 2048u * (idx >> 4) + 128u * r + ((8u * (idx & 15u)) ^ (16u * (r & 7u)));
+#else
+  return 256u * r + ((8u * idx) ^ (16u * (r & 7u)));
+#endif
+}
+
 // Pass B analysis of one stage (up to 16 slots; meta E = 0 marks an empty row). Lane (j, h) = (lane & 15,
 // lane >> 4) scans addresses 16h .. 16h+15 of row j; 16 B chunk c of row j is stored at chunk c ^ (j & 7),
 // so the 8 lanes of a quarter-warp (consecutive j, same h) read 8 distinct bank groups.
@@ -428,10 +477,9 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
   unsigned E, pc;
   lds_v2(meta + 8u * j, E, pc);
   const unsigned Eh = h ? E >> 16 : E & 0xffffu;
-  const unsigned rowb = stage + 256u * j;
   const unsigned f = (Eh ? (unsigned)__ffs(Eh) - 1u : 0u) + 16u * h;
   unsigned f_lo, f_hi;
-  lds_v2(rowb + 16u * ((f >> 1) ^ sw) + 8u * (f & 1u), f_lo, f_hi);
+  lds_v2(stage + rb_off(j, f), f_lo, f_hi);
   unsigned prev = f_lo, hb = 0, bs = 0, bl = 0, mn = f_lo, mx = f_lo;
 #if NVBT_RPB_TAGS && NVBT_RPB_SBITS
   unsigned sbits = 0;   // the 1 KB-word sector bits of the scanned addresses (bit (a >> 5) & 31)
@@ -440,7 +488,7 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
 #pragma unroll
   for (int q = 0; q < ((NVBT_RPB_EXPERIMENT & 2) ? 1 : 8); ++q) {   // (experiment 2: scan 2 addresses only)
     uint4 v;
-    lds_v4(rowb + 16u * ((8u * h + q) ^ sw), v);
+    lds_v4(stage + rb_off(j, 16u * h + 2u * q), v);
 #pragma unroll
     for (int u = 0; u < 2; ++u) {
       const bool act = (Eh >> (2 * q + u)) & 1u;
@@ -505,7 +553,7 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
   }
   const unsigned cm0 = 0u;
 #elif NVBT_RPB_TAGS
-  const unsigned cm0 = __ballot_sync(FULL, own && slow && cls == 0u);   // window loop takes class 0 too
+  const unsigned cm0 = (NVBT_RPB_EXPERIMENT & 5) ? 0u : __ballot_sync(FULL, own && slow && cls == 0u);   // window loop takes class 0 too
 #else
   const unsigned cm0 = (NVBT_RPB_EXPERIMENT & 5) ? 0u : __ballot_sync(FULL, own && slow && cls == 0u);
 #endif
@@ -526,7 +574,19 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
   const unsigned stag = s_scr, ltag = s_scr + 1024u;
   const unsigned l8 = 8u * lane;
   const unsigned long long kInvalid = ~0ull;
+#if NVBT_RPB_C0REDUX
+  unsigned mw = cm1, mwide = cm2;
+  for (unsigned m0 = cm0; m0;) {   // one 1 KB word: OR of the lanes' sector bits (sl_word)
+    const unsigned src = 31u - __clz(m0);
+    m0 ^= 1u << src;
+    const unsigned es = __shfl_sync(FULL, E, src);
+    const uint2 r = sl_word(lds_u32(stage + rb_off(src, lane)), (es & lanebit) != 0u);
+    S = lane == src ? r.x : S;
+    L = lane == src ? r.y : L;
+  }
+#else
   unsigned mw = cm0 | cm1, mwide = cm2;
+#endif
   // up to kWR window rows per iteration (independent chains; per row a kWin-sector window of tags and
   // kWin / 4 line tags)
   while (mw) {
@@ -542,7 +602,7 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
     for (int k = 0; k < kWR; ++k) {
       ev[k] = __shfl_sync(FULL, E, r[k]);
       wv[k] = __shfl_sync(FULL, wbase, r[k]);
-      lo[k] = lds_u32(stage + 256u * r[k] + (l8 ^ (16u * (r[k] & 7u))));
+      lo[k] = lds_u32(stage + rb_off(r[k], lane));
     }
 #pragma unroll
     for (int k = 0; k < kWR; ++k) {
@@ -564,16 +624,104 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
     }
     __syncwarp();                                  // reads done before the next rows' stores
   }
+#if NVBT_RPB_WIDE2
+  // two wide rows per iteration (independent dependency chains); row k hashes into buckets [640 k, 640 k + 640)
+  // of the tag scratch and is resolved against its bucket owners as in the one-row loop below
+  while (mwide) {
+    unsigned src[2], es[2], x0[2], x1[2], hb[2], own[2];
+    unsigned long long a[2];
+    bool v[2], act[2], lose[2], ok[2];
+#pragma unroll
+    for (int k = 0; k < 2; ++k) {
+      v[k] = mwide != 0u;
+      src[k] = v[k] ? 31u - __clz(mwide) : 0u;
+      if (v[k]) mwide ^= 1u << src[k];
+    }
+#pragma unroll
+    for (int k = 0; k < 2; ++k) {
+      es[k] = __shfl_sync(FULL, E, src[k]);
+      asm volatile("ld.shared.u64 %0, [%1];" : "=l"(a[k]) : "r"(stage + rb_off(src[k], lane)) : "memory");
+    }
+#pragma unroll
+    for (int k = 0; k < 2; ++k) {
+      act[k] = v[k] && ((es[k] >> lane) & 1u);
+      const unsigned long long line = a[k] >> 7;
+      x0[k] = (unsigned)line;
+      x1[k] = (unsigned)(line >> 32);
+      const unsigned hsh = x0[k] * 0x9E3779B1u ^ x1[k] * 0x85EBCA77u;
+      hb[k] = 640u * k + __umulhi(hsh * 0xC2B2AE3Du + (hsh >> 15), 640u);
+      if (act[k]) sts_u8(stag + hb[k], lane);
+    }
+    __syncwarp();
+#pragma unroll
+    for (int k = 0; k < 2; ++k) {
+      own[k] = lds_u8(stag + hb[k]) & 31u;
+      lose[k] = act[k] && own[k] != lane;
+      ok[k] = !__any_sync(FULL, lose[k]);
+    }
+    if (!(ok[0] && ok[1])) {                       // warp-uniform
+      bool same[2];
+#pragma unroll
+      for (int k = 0; k < 2; ++k) {
+        const unsigned o0 = __shfl_sync(FULL, x0[k], own[k]), o1 = __shfl_sync(FULL, x1[k], own[k]);
+        same[k] = lose[k] && o0 == x0[k] && o1 == x1[k];
+        if (lose[k]) sts_u8(stag + hb[k], lane);
+      }
+      __syncwarp();
+#pragma unroll
+      for (int k = 0; k < 2; ++k) {
+        const bool lose2 = lose[k] && lds_u8(stag + hb[k]) != lane;
+        ok[k] = !__any_sync(FULL, same[k] || lose2);
+      }
+    }
+    __syncwarp();
+#pragma unroll
+    for (int k = 0; k < 2; ++k) {
+      unsigned sx, lx;
+      if (ok[k]) {
+        sx = lx = __popc(es[k]);
+      } else {
+        sl_bitonic(a[k], act[k], lane, sx, lx);
+      }
+      S = (v[k] && lane == src[k]) ? sx : S;
+      L = (v[k] && lane == src[k]) ? lx : L;
+    }
+  }
+#endif
   while (mwide) {
     const unsigned src = 31u - __clz(mwide);
     mwide ^= 1u << src;
     const unsigned es = __shfl_sync(FULL, E, src);
     unsigned long long a;
-    asm volatile("ld.shared.u64 %0, [%1];" : "=l"(a) : "r"(stage + 256u * src + (l8 ^ (16u * (src & 7u)))) : "memory");
+    asm volatile("ld.shared.u64 %0, [%1];" : "=l"(a) : "r"(stage + rb_off(src, lane)) : "memory");
     const bool act = (es >> lane) & 1u;
     const unsigned long long line = a >> 7;
     const unsigned x0 = (unsigned)line, x1 = (unsigned)(line >> 32);
     bool ok = false;
+#if NVBT_RPB_RESOLVE
+    {
+      // one hash round; if a lane lost its bucket, every loser compares its line with the bucket's owner (the
+      // last writer) and the losers tag their buckets again: when each loser then owns its bucket, every
+      // bucket holds the owner and at most one loser whose line differs from the owner's, so all lines are
+      // distinct (equal lines always share a bucket). Anything else takes the exact sort below.
+      const unsigned hsh = x0 * 0x9E3779B1u ^ x1 * 0x85EBCA77u;
+      const unsigned hb = __umulhi(hsh * 0xC2B2AE3Du + (hsh >> 15), 1280u);
+      if (act) sts_u8(stag + hb, lane);
+      __syncwarp();
+      const unsigned own = lds_u8(stag + hb) & 31u;
+      const bool lose = act && own != lane;
+      ok = !__any_sync(FULL, lose);
+      if (!ok) {                                   // warp-uniform
+        const unsigned o0 = __shfl_sync(FULL, x0, own), o1 = __shfl_sync(FULL, x1, own);
+        const bool same = lose && o0 == x0 && o1 == x1;
+        if (lose) sts_u8(stag + hb, lane);         // every lane has read its owner (__any_sync above)
+        __syncwarp();
+        const bool lose2 = lose && lds_u8(stag + hb) != lane;
+        ok = !__any_sync(FULL, same || lose2);
+      }
+      __syncwarp();
+    }
+#else
 #pragma unroll
     for (int round = 0; round < 3 && !ok; ++round) {   // warp-uniform
       const unsigned hsh = (x0 * (0x9E3779B1u + 0x6A09E666u * round) ^ x1 * (0x85EBCA77u + 0x3C6EF372u * round)) + round;
@@ -583,6 +731,7 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
       ok = __all_sync(FULL, !act || lds_u8(stag + hb) == lane);
       __syncwarp();
     }
+#endif
     unsigned sx, lx;
     if (ok) {
       sx = lx = __popc(es);
@@ -613,7 +762,7 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
     const unsigned src = 31u - __clz(m0);
     m0 ^= 1u << src;
     const unsigned es = __shfl_sync(FULL, E, src);
-    const unsigned a_lo = lds_u32(stage + 256u * src + (l8 ^ (16u * (src & 7u))));
+    const unsigned a_lo = lds_u32(stage + rb_off(src, lane));
     const uint2 r = sl_word(a_lo, (es & lanebit) != 0u);
     S = lane == src ? r.x : S;
     L = lane == src ? r.y : L;
@@ -622,7 +771,7 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
     const unsigned src = 31u - __clz(m1);
     m1 ^= 1u << src;
     const unsigned es = __shfl_sync(FULL, E, src), wb = __shfl_sync(FULL, wbase, src);
-    const unsigned a_lo = lds_u32(stage + 256u * src + (l8 ^ (16u * (src & 7u))));
+    const unsigned a_lo = lds_u32(stage + rb_off(src, lane));
     const uint2 r = sl_window(a_lo, (es & lanebit) != 0u, lane, s_scr, wb);
     S = lane == src ? r.x : S;
     L = lane == src ? r.y : L;
@@ -632,7 +781,7 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
     m2 ^= 1u << src;
     const unsigned es = __shfl_sync(FULL, E, src);
     unsigned long long a;
-    asm volatile("ld.shared.u64 %0, [%1];" : "=l"(a) : "r"(stage + 256u * src + (l8 ^ (16u * (src & 7u)))) : "memory");
+    asm volatile("ld.shared.u64 %0, [%1];" : "=l"(a) : "r"(stage + rb_off(src, lane)) : "memory");
     const uint2 r = sl_wide(a, es, lanebit, lane, s_scr);
     S = lane == src ? r.x : S;
     L = lane == src ? r.y : L;
@@ -645,24 +794,42 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
   __syncwarp();
 }
 
+// TMA stages (NVBT_RPB_TMA): per warp 2 x 4 KB stages in a 1024-aligned area after the bins, then per warp
+// the tag scratch (1280 B), the stage meta (2 x 128 B) and the two stage mbarriers
+constexpr unsigned RB_X_BYTES = 1280u + 256u + 16u;
+
 __global__ void __launch_bounds__(32 * RB_NW, 1)
 k_rpB(const unsigned long long* __restrict__ addr, unsigned P, const uint8_t* __restrict__ kind, DevState st,
-      const unsigned* __restrict__ counts, unsigned n_regions, const uint2* __restrict__ l_ent, unsigned region_cap) {
+      const unsigned* __restrict__ counts, unsigned n_regions, const uint2* __restrict__ l_ent, unsigned region_cap,
+      const __grid_constant__ CUtensorMap tmap) {
   extern __shared__ __align__(16) unsigned sm[];
   const unsigned PB = (2 * P + 66 + 3) & ~3u;      // sS[P] | sL[P] | hist[66]
-  unsigned* sWarpAll = sm + PB;
   for (unsigned i = threadIdx.x; i < PB; i += blockDim.x) sm[i] = 0;
+  const unsigned lane = lane_id(), lanebit = 1u << lane;
+  const unsigned s_base = (unsigned)__cvta_generic_to_shared(sm);
+#if NVBT_RPB_TMA
+  static_assert(NVBT_RPB_TAGS, "TMA stages assume the tag-array slow paths (no scratch initialisation)");
+  const unsigned warp = threadIdx.x >> 5;
+  const unsigned s_stg0 = (s_base + 4u * PB + 1023u) & ~1023u;
+  const unsigned s_w = s_stg0 + 8192u * warp;                                 // stage s: + 4096 s
+  const unsigned s_x = s_stg0 + 8192u * RB_NW + RB_X_BYTES * warp;
+  const unsigned s_scr = s_x, s_meta = s_x + 1280u, s_bar = s_x + 1536u;      // meta, mbarrier of stage s: + 128 s, + 8 s
+  if (lane < 2) asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(s_bar + 8u * lane) : "memory");
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  __syncthreads();
+  unsigned phase = 0;   // bit s: parity of stage s's next completion
+#else
+  unsigned* sWarpAll = sm + PB;
   constexpr unsigned kScr0 = RB_STAGES * (RB_ROWS * 64 + 2 * RB_ROWS);
   for (unsigned i = threadIdx.x; i < RB_NW * RB_WARP_WORDS; i += blockDim.x) {
     const unsigned o = i % RB_WARP_WORDS;
     sWarpAll[i] = o >= kScr0 + SCRATCH_WORDS ? 0xffffffffu : o >= kScr0 ? scratch_init_word(o - kScr0) : 0u;
   }
   __syncthreads();
-  const unsigned lane = lane_id(), lanebit = 1u << lane;
-  const unsigned s_base = (unsigned)__cvta_generic_to_shared(sm);
   const unsigned s_w = (unsigned)__cvta_generic_to_shared(sWarpAll + (threadIdx.x >> 5) * RB_WARP_WORDS);
   const unsigned s_meta = s_w + 4u * RB_STAGES * RB_ROWS * 64;      // stage s: + 128 s
   const unsigned s_scr = s_w + 4u * kScr0;
+#endif
   const unsigned s_sS = s_base, s_sL = s_base + 4u * P, s_hist = s_base + 8u * P;
   const unsigned WB = gridDim.x * RB_NW;
   const unsigned j = lane & 15u, h = lane >> 4;
@@ -694,6 +861,25 @@ k_rpB(const unsigned long long* __restrict__ addr, unsigned P, const uint8_t* __
     if (h == 0u)
       asm volatile("st.shared.v2.u32 [%0], {%1, %2};" ::"r"(s_meta + 128u * s + 8u * j), "r"(nx_E), "r"(nx_pc) : "memory");
     const unsigned stg = s_w + 4096u * s;
+#if NVBT_RPB_TMA
+    // 2 x ceil(rows / 4) gathers of 4 half-rows (128 B each): lane 2 q + hf loads half hf of rows 4q .. 4q + 3
+    // (rows past the group repeat its last row) to stg + 2048 hf + 512 q
+    const unsigned rows = g1.rows, q4 = (lane >> 1) & 3u, hf = lane & 1u;
+    const unsigned ng = 2u * ((rows + 3u) >> 2);
+    unsigned ri[4];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) ri[i] = __shfl_sync(FULL, nx_idx, min(4u * q4 + (unsigned)i, rows - 1u));
+    const unsigned bar = s_bar + 8u * s;
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // this stage's earlier reads before the async writes
+    if (lane == 0) asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(512u * ng) : "memory");
+    __syncwarp();
+    if (lane < ng)
+      asm volatile("cp.async.bulk.tensor.2d.shared::cluster.global.tile::gather4.mbarrier::complete_tx::bytes"
+                   " [%0], [%1, {%2, %3, %4, %5, %6}], [%7];"
+                   ::"r"(stg + 2048u * hf + 512u * q4), "l"(reinterpret_cast<unsigned long long>(&tmap)), "r"(32u * hf),
+                     "r"(ri[0]), "r"(ri[1]), "r"(ri[2]), "r"(ri[3]), "r"(bar)
+                   : "memory");
+#else
     const unsigned c = lane & 15u;
 #pragma unroll
     for (int k = 0; k < RB_ROWS / 2; ++k) {
@@ -705,6 +891,7 @@ k_rpB(const unsigned long long* __restrict__ addr, unsigned P, const uint8_t* __
                      : "memory");
     }
     asm volatile("cp.async.commit_group;" ::: "memory");
+#endif
 #if NVBT_RPB_PF
     if (h == 0u && j < g2.rows)
       asm volatile("cp.async.bulk.prefetch.L2.global [%0], 256;" ::"l"(addr + (unsigned long long)slot_of(g2) * 32u) : "memory");
@@ -723,12 +910,24 @@ k_rpB(const unsigned long long* __restrict__ addr, unsigned P, const uint8_t* __
   if (live) issue(0);
   while (live) {
     live = g1.rows != 0u;
+#if NVBT_RPB_TMA
+    if (live) issue(s ^ 1u);
+    {
+      const unsigned bar = s_bar + 8u * s, par = (phase >> s) & 1u;
+      unsigned ready = 0;
+      while (!ready)
+        asm volatile("{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}"
+                     : "=r"(ready) : "r"(bar), "r"(par) : "memory");
+      phase ^= 1u << s;
+    }
+#else
     if (live) {
       issue(s ^ 1u);
     } else {
       asm volatile("cp.async.commit_group;" ::: "memory");
     }
     asm volatile("cp.async.wait_group 1;" ::: "memory");
+#endif
     __syncwarp();
     rb_process(s_w + 4096u * s, s_meta + 128u * s, lane, lanebit, s_scr, s_sS, s_sL, s_hist);
     s ^= 1u;
@@ -747,7 +946,35 @@ k_rpB(const unsigned long long* __restrict__ addr, unsigned P, const uint8_t* __
 }
 
 static size_t rpA_smem(unsigned P) { return 16ull * P + ((P + 15ull) & ~15ull) + 512ull * RA_DEPTH * RA_NW; }
-static size_t rpB_smem(unsigned P) { return (((2ull * P + 66 + 3) & ~3ull) + (size_t)RB_NW * RB_WARP_WORDS) * 4; }
+static size_t rpB_smem(unsigned P) {
+#if NVBT_RPB_TMA
+  return ((2ull * P + 66 + 3) & ~3ull) * 4 + 1023 + (8192ull + RB_X_BYTES) * RB_NW;
+#else
+  return (((2ull * P + 66 + 3) & ~3ull) + (size_t)RB_NW * RB_WARP_WORDS) * 4;
+#endif
+}
+
+// Tensor map of the pass's address slots for the TMA stages: a 2D tensor of u32, 64 per event (256 B rows),
+// m rows; boxes of 32 x 1 (one 128 B half-row; tile::gather4 loads four rows), 128 B swizzle.
+static int rpB_tmap(const void* d_addr, unsigned long long m, CUtensorMap* tm) {
+  static PFN_cuTensorMapEncodeTiled_v12000 enc = nullptr;
+  if (!enc) {
+    void* f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) != cudaSuccess || !f)
+      return set_error(NVBT_ECUDA, "cuTensorMapEncodeTiled unavailable");
+    enc = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(f);
+  }
+  std::memset(tm, 0, sizeof *tm);
+  const cuuint64_t dims[2] = {64, m};
+  const cuuint64_t strides[1] = {256};
+  const cuuint32_t box[2] = {32, 1}, es[2] = {1, 1};
+  const CUresult r = enc(tm, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, const_cast<void*>(d_addr), dims, strides, box, es,
+                         CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                         CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return set_error(NVBT_ECUDA, "cuTensorMapEncodeTiled failed (%d)", (int)r);
+  return NVBT_OK;
+}
 
 static int sm_count(int dev) { return device_sms(dev); }
 
@@ -899,9 +1126,15 @@ static int launch_staged(nvbt_ctx c, const void* d_hdr, const void* d_addr, uint
     NVBT_CUDA(cudaGetLastError());
     c->launches++;
     if (!memdiv) continue;
+    CUtensorMap tm;
+#if NVBT_RPB_TMA
+    { const int trc = rpB_tmap(static_cast<const unsigned long long*>(d_addr) + off * 32, m, &tm); if (trc) return trc; }
+#else
+    std::memset(&tm, 0, sizeof tm);
+#endif
     k_rpB<<<blocks_b, 32 * RB_NW, rpB_smem(c->n_pcs), c->stream>>>(
         static_cast<const unsigned long long*>(d_addr) + off * 32, c->n_pcs, c->d_kind, st, counts, warps, l_ent,
-        region_cap);
+        region_cap, tm);
     NVBT_CUDA(cudaGetLastError());
     c->launches++;
   }

@@ -265,3 +265,66 @@ class KernelSampler:
         for key, snap in self.snapshots.items():
             nb.nvbt_accum_axpy(self.ctx, snap, self.launches[key])
         return dict(self.launches)
+
+
+# --------------------------------------------------------------------------- host placement of a rank
+# A traced rank moves its records over its GPU's own PCIe link into a pinned ring that its drain threads
+# scan (C4). On a multi-socket box each GPU hangs off one NUMA node: the ring pages and the drain threads
+# belong on that node, and the ranks sharing a node split its cores instead of all spinning on all of them.
+
+def parse_cpulist(text: str):
+    """'0-3,8,10-11' -> [0, 1, 2, 3, 8, 10, 11] (the sysfs cpulist format)."""
+    cpus = []
+    for part in text.strip().split(","):
+        if not part:
+            continue
+        if "-" in part:
+            lo, hi = part.split("-")
+            cpus.extend(range(int(lo), int(hi) + 1))
+        else:
+            cpus.append(int(part))
+    return cpus
+
+
+def rank_cpu_slice(gpu_cpus, device: int, allowed=None):
+    """CPUs for the rank driving GPU `device`, given gpu_cpus[g] = the CPUs local to visible GPU g: the GPUs
+    with the same local CPU set share it in contiguous equal slices (in GPU order), restricted to `allowed`
+    (the process's affinity). Falls back to the whole local set (or `allowed`) when a slice would be empty."""
+    mine = [c for c in gpu_cpus[device] if allowed is None or c in allowed]
+    peers = [g for g, cs in enumerate(gpu_cpus) if sorted(cs) == sorted(gpu_cpus[device])]
+    k, i = len(peers), peers.index(device)
+    lo, hi = len(mine) * i // k, len(mine) * (i + 1) // k
+    if hi > lo:
+        return mine[lo:hi]
+    return mine or (sorted(allowed) if allowed else [])
+
+
+def gpu_local_cpus(sysfs="/sys/bus/pci/devices"):
+    """Per visible CUDA device, the CPUs of its PCIe device's NUMA node (sysfs local_cpulist); None if the
+    topology cannot be read."""
+    import torch
+    out = []
+    for g in range(torch.cuda.device_count()):
+        p = torch.cuda.get_device_properties(g)
+        dev = f"{p.pci_domain_id:04x}:{p.pci_bus_id:02x}:{p.pci_device_id:02x}.0"
+        try:
+            with open(f"{sysfs}/{dev}/local_cpulist") as f:
+                out.append(parse_cpulist(f.read()))
+        except OSError:
+            return None
+    return out
+
+
+def bind_rank_to_gpu_numa(device: int):
+    """Pins this process to its slice of GPU `device`'s NUMA-local CPUs (call before the pinned ring is
+    allocated and before the first drain creates the drain worker pool, which sizes itself to the affinity).
+    Returns the CPU list, or None when the topology is unknown (nothing changed)."""
+    import os
+    local = gpu_local_cpus()
+    if not local:
+        return None
+    cpus = rank_cpu_slice(local, device, set(os.sched_getaffinity(0)))
+    if not cpus:
+        return None
+    os.sched_setaffinity(0, cpus)
+    return cpus
