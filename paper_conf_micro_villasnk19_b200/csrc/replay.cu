@@ -287,7 +287,20 @@ static size_t replay4_smem(unsigned P) {
 //     to the matching exact warp-cooperative path (1 KB word, 32 KB window, hashed).
 // Extra traffic: 16 B per executed memory event (list write + read), ~5 % of the algorithmic bytes.
 constexpr int RA_NW = 20;     // pass A warps per CTA (one list region per warp)
-constexpr int RB_NW = 20;     // pass B warps per CTA (warp w of pass B analyses region w)
+#ifndef NVBT_RPB_NW
+#define NVBT_RPB_NW 20
+#endif
+#ifndef NVBT_RPB_GBINS
+#define NVBT_RPB_GBINS 0       // 1: per-pc sector / line sums as u64 reductions into the CTA's stripe of the global bins
+                               // (no shared per-pc bins: 32 KB more for resident warps). A/B r2_ab19-20: 20 warps
+                               // 1.817 -> 1.847 ms; 22 / 23 warps 2.16 ms (at most 80 registers: 6 warps on one
+                               // SMSP's 16 K registers; 20 warps capped at 80 registers alone cost 1.847 -> 1.878)
+#endif
+#ifndef NVBT_RPB_DYN
+#define NVBT_RPB_DYN 0         // 1: pass-B warps take pass-A regions from a global counter instead of a fixed stride
+                               // (A/B r2_ab19: 1.817 -> 1.831 ms)
+#endif
+constexpr int RB_NW = NVBT_RPB_NW;     // pass B warps per CTA
 #ifndef NVBT_RPB_EXPERIMENT
 #define NVBT_RPB_EXPERIMENT 0   // timing experiments (tools/replay_ab.py), never in a product build
 #endif
@@ -336,7 +349,8 @@ constexpr int RB_STAGES = 2;
 // A/B build without them (NVBT_RPB_TAGS=0) uses its first SCRATCH_WORDS words as sectors_lines_cls scratch
 constexpr int RB_SCR2 = 128;
 constexpr int RB_WARP_WORDS = RB_STAGES * (RB_ROWS * 64 + 2 * RB_ROWS) + SCRATCH_WORDS + RB_SCR2;
-constexpr size_t RS_COUNTS_BYTES = 65536;   // u32 per pass-A warp (<= 16384 warps)
+constexpr size_t RS_COUNTS_BYTES = 65536;   // u32 per pass-A warp (< 16384 warps), then the region counter
+constexpr unsigned kRegionCtr = 16383;      // counts[kRegionCtr]: regions claimed past the first (NVBT_RPB_DYN)
 static_assert(RB_WARP_WORDS % 4 == 0, "16 B aligned warp areas");
 
 __device__ __forceinline__ void lds_v2(unsigned a, unsigned& x, unsigned& y) {
@@ -410,6 +424,7 @@ k_rpA(const uint4* __restrict__ hdr, unsigned n, unsigned P, const uint8_t* __re
   }
   asm volatile("cp.async.wait_group 0;" ::: "memory");
   if (lane == 0 && counts != nullptr) counts[gw] = cnt;
+  if (NVBT_RPB_DYN && counts != nullptr && gw == 0 && lane == 0) counts[kRegionCtr] = 0u;
   bad = __reduce_add_sync(FULL, bad);
   if (lane == 0 && bad) atomicAdd(err, (unsigned long long)bad);
   __syncthreads();
@@ -469,7 +484,8 @@ __device__ __forceinline__ unsigned rb_off(unsigned r, unsigned idx) {
 // lane >> 4) scans addresses 16h .. 16h+15 of row j; 16 B chunk c of row j is stored at chunk c ^ (j & 7),
 // so the 8 lanes of a quarter-warp (consecutive j, same h) read 8 distinct bank groups.
 __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsigned lane, unsigned lanebit,
-                                           unsigned s_scr, unsigned s_sS, unsigned s_sL, unsigned s_hist) {
+                                           unsigned s_scr, unsigned s_sS, unsigned s_sL, unsigned s_hist,
+                                           unsigned long long* gmem) {
   const unsigned j = lane & 15u, h = lane >> 4, sw = j & 7u;
   // window sectors of class 1 (tags build: kWR rows in flight, kWin + kWin / 4 tag bytes each)
   constexpr unsigned kWin = NVBT_RPB_TAGS ? NVBT_RPB_WIN : 1024u;
@@ -787,8 +803,15 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
     L = lane == src ? r.y : L;
   }
 #endif
+#if NVBT_RPB_GBINS
+  if (own) {
+    asm volatile("red.global.add.u64 [%0], %1;" ::"l"(gmem + 3u * pc + 1u), "l"((unsigned long long)S) : "memory");
+    asm volatile("red.global.add.u64 [%0], %1;" ::"l"(gmem + 3u * pc + 2u), "l"((unsigned long long)L) : "memory");
+  }
+#else
   red_shared_add_if(own, s_sS + 4u * pc, S);
   red_shared_add_if(own, s_sL + 4u * pc, L);
+#endif
   red_shared_add_if(own, s_hist + 4u * S, 1u);          // hS[S]
   red_shared_add_if(own, s_hist + 4u * (33u + L), 1u);  // hL[L]
   __syncwarp();
@@ -798,12 +821,23 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
 // the tag scratch (1280 B), the stage meta (2 x 128 B) and the two stage mbarriers
 constexpr unsigned RB_X_BYTES = 1280u + 256u + 16u;
 
-__global__ void __launch_bounds__(32 * RB_NW, 1)
+#ifdef NVBT_RPB_MAXREG
+#define NVBT_RPB_BOUNDS __maxnreg__(NVBT_RPB_MAXREG)
+#else
+#define NVBT_RPB_BOUNDS __launch_bounds__(32 * RB_NW, 1)
+#endif
+__global__ void NVBT_RPB_BOUNDS
 k_rpB(const unsigned long long* __restrict__ addr, unsigned P, const uint8_t* __restrict__ kind, DevState st,
       const unsigned* __restrict__ counts, unsigned n_regions, const uint2* __restrict__ l_ent, unsigned region_cap,
       const __grid_constant__ CUtensorMap tmap) {
   extern __shared__ __align__(16) unsigned sm[];
+#if NVBT_RPB_GBINS
+  const unsigned PB = 68u;                          // hist[66]
+  unsigned long long* const gmem = st.mem + (unsigned long long)(blockIdx.x & (st.stripes - 1u)) * st.stripe_words;
+#else
   const unsigned PB = (2 * P + 66 + 3) & ~3u;      // sS[P] | sL[P] | hist[66]
+  unsigned long long* const gmem = st.mem;
+#endif
   for (unsigned i = threadIdx.x; i < PB; i += blockDim.x) sm[i] = 0;
   const unsigned lane = lane_id(), lanebit = 1u << lane;
   const unsigned s_base = (unsigned)__cvta_generic_to_shared(sm);
@@ -830,7 +864,11 @@ k_rpB(const unsigned long long* __restrict__ addr, unsigned P, const uint8_t* __
   const unsigned s_meta = s_w + 4u * RB_STAGES * RB_ROWS * 64;      // stage s: + 128 s
   const unsigned s_scr = s_w + 4u * kScr0;
 #endif
+#if NVBT_RPB_GBINS
+  const unsigned s_sS = 0u, s_sL = 0u, s_hist = s_base;
+#else
   const unsigned s_sS = s_base, s_sL = s_base + 4u * P, s_hist = s_base + 8u * P;
+#endif
   const unsigned WB = gridDim.x * RB_NW;
   const unsigned j = lane & 15u, h = lane >> 4;
   // group cursor over this warp's regions gw, gw + WB, ...
@@ -840,7 +878,13 @@ k_rpB(const unsigned long long* __restrict__ addr, unsigned P, const uint8_t* __
   struct Grp { unsigned rows, r; uint2 ent; };
   auto fetch = [&](Grp& g) {
     while (r < n_regions && off >= rcnt) {
+#if NVBT_RPB_DYN
+      unsigned nr = 0;   // the next unclaimed region (the first WB regions were taken statically)
+      if (lane == 0) nr = WB + atomicAdd(const_cast<unsigned*>(counts) + kRegionCtr, 1u);
+      r = __shfl_sync(FULL, nr, 0);
+#else
       r += WB;
+#endif
       off = 0;
       rcnt = r < n_regions ? counts[r] : 0u;
     }
@@ -929,10 +973,14 @@ k_rpB(const unsigned long long* __restrict__ addr, unsigned P, const uint8_t* __
     asm volatile("cp.async.wait_group 1;" ::: "memory");
 #endif
     __syncwarp();
-    rb_process(s_w + 4096u * s, s_meta + 128u * s, lane, lanebit, s_scr, s_sS, s_sL, s_hist);
+    rb_process(s_w + 4096u * s, s_meta + 128u * s, lane, lanebit, s_scr, s_sS, s_sL, s_hist, gmem);
     s ^= 1u;
   }
   __syncthreads();
+#if NVBT_RPB_GBINS
+  for (unsigned i = threadIdx.x; i < 66; i += blockDim.x)
+    if (sm[i]) atomicAdd(st.hist + i, (unsigned long long)sm[i]);
+#else
   const uint8_t* kd = kind;
   for (unsigned pc = threadIdx.x; pc < P; pc += blockDim.x) {
     const unsigned a = sm[pc], b = sm[P + pc];
@@ -943,6 +991,7 @@ k_rpB(const unsigned long long* __restrict__ addr, unsigned P, const uint8_t* __
   }
   for (unsigned i = threadIdx.x; i < 66; i += blockDim.x)
     if (sm[2 * P + i]) atomicAdd(st.hist + i, (unsigned long long)sm[2 * P + i]);
+#endif
 }
 
 static size_t rpA_smem(unsigned P) { return 16ull * P + ((P + 15ull) & ~15ull) + 512ull * RA_DEPTH * RA_NW; }
@@ -950,7 +999,7 @@ static size_t rpB_smem(unsigned P) {
 #if NVBT_RPB_TMA
   return ((2ull * P + 66 + 3) & ~3ull) * 4 + 1023 + (8192ull + RB_X_BYTES) * RB_NW;
 #else
-  return (((2ull * P + 66 + 3) & ~3ull) + (size_t)RB_NW * RB_WARP_WORDS) * 4;
+  return ((NVBT_RPB_GBINS ? 68ull : ((2ull * P + 66 + 3) & ~3ull)) + (size_t)RB_NW * RB_WARP_WORDS) * 4;
 #endif
 }
 
@@ -1098,6 +1147,7 @@ static int launch_staged(nvbt_ctx c, const void* d_hdr, const void* d_addr, uint
   const unsigned long long cap = staged_cap(scratch_bytes);
   const unsigned long long max_warps = (unsigned long long)sms * RA_CTAS_PER_SM * RA_NW;
   unsigned long long pass = 1ull << 30;   // keeps every CTA's u32 bins far from overflow
+  if (max_warps >= kRegionCtr) return set_error(NVBT_EINVAL, "staged replay: %llu pass-A warps", max_warps);
   if (memdiv) {
     if (scratch == nullptr || cap <= 32ull * max_warps)
       return set_error(NVBT_ENOMEM, "staged replay scratch of %zu bytes is too small", scratch_bytes);

@@ -200,19 +200,31 @@ def test_channel_compact128_bfs(nvbt):
     import threading
     done, out = threading.Event(), []
 
+    import os
+    import time
+    log = []
+    t0 = time.perf_counter()
+
     def drain():   # the ring (1024 slots) is far smaller than the trace: drain while the BFS runs
-        while True:
-            fin = done.is_set()
-            out.append(nb.nvbt_channel_drain_copy(ch, dst[sum(out):], timeout_us=60_000_000))
-            if fin:
-                return
+        log.append(("start", time.perf_counter() - t0, sorted(os.sched_getaffinity(0))[:4]))
+        try:
+            while True:
+                fin = done.is_set()
+                a = time.perf_counter() - t0
+                out.append(nb.nvbt_channel_drain_copy(ch, dst[sum(out):], timeout_us=60_000_000))
+                log.append((round(a, 4), round(time.perf_counter() - t0, 4), out[-1]))
+                if fin:
+                    return
+        except Exception as e:  # noqa: BLE001 - reported with the log below
+            log.append(("error", time.perf_counter() - t0, str(e)))
     th = threading.Thread(target=drain)
     th.start()
     dr.run_bfs(ctx, nb.TOOL_TRACE, rp, cl, src, bufs)
+    log.append(("bfs done", time.perf_counter() - t0))
     done.set()
     th.join()
     got_n = sum(out)
-    assert nb.nvbt_channel_dropped(ch) == 0 and got_n == len(exp)
+    assert nb.nvbt_channel_dropped(ch) == 0 and got_n == len(exp), (got_n, len(exp), log[:20], log[-5:], threading.enumerate())
     assert (trace.sort_records(dst[:got_n]) == trace.sort_records(exp)).all()
 
 
