@@ -334,6 +334,10 @@ constexpr int RB_NW = NVBT_RPB_NW;     // pass B warps per CTA
 #define NVBT_RPB_WIDE2 0       // 1: wide rows two per iteration (independent chains), 640 hash buckets each, resolved.
                                // A/B r2_ab17: pass B 1.813 -> 1.894 ms (more collisions, instruction-bound), not kept
 #endif
+#ifndef NVBT_RPB_HASH1
+#define NVBT_RPB_HASH1 1       // wide-row bucket = top bits of the line's multiplicative hash, no finaliser (A/B r2_ab21:
+                               // pass B 1.820 -> 1.806 ms; a bad spread only costs the resolve / exact paths)
+#endif
 #ifndef NVBT_RPB_C0REDUX
 #define NVBT_RPB_C0REDUX 0     // 1: one-1-KB-word rows by an OR-reduction of their sector bits (own loop). A/B r2_ab16:
                                // pass B 1.839 -> 1.890 ms, not kept
@@ -721,7 +725,11 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
       // bucket holds the owner and at most one loser whose line differs from the owner's, so all lines are
       // distinct (equal lines always share a bucket). Anything else takes the exact sort below.
       const unsigned hsh = x0 * 0x9E3779B1u ^ x1 * 0x85EBCA77u;
+#if NVBT_RPB_HASH1
+      const unsigned hb = __umulhi(hsh, 1280u);   // Fibonacci hashing: the product's top bits
+#else
       const unsigned hb = __umulhi(hsh * 0xC2B2AE3Du + (hsh >> 15), 1280u);
+#endif
       if (act) sts_u8(stag + hb, lane);
       __syncwarp();
       const unsigned own = lds_u8(stag + hb) & 31u;
