@@ -157,7 +157,7 @@ typedef int (*nvbt_drain_fn)(const void* records, uint64_t n_records, void* user
  * concurrently with kernels already enqueued; it never synchronises the context's stream, so a drain
  * thread may run while another thread keeps enqueueing producers (it returns whenever it sees the stream
  * idle with everything delivered: call it again until the producer thread is done). *n_drained
- * (nullable) = records delivered by this call. A producer that waits ~2 s on a full ring gives up: its
+ * (nullable) = records delivered by this call. A producer that waits 10 s (NVBT_PRODUCER_WAIT_MS, read at channel open) on a full ring gives up: its
  * record is dropped and counted (nvbt_channel_dropped), the drain then reports NVBT_ETIMEDOUT, and the
  * channel must be closed and reopened (the dropped ticket leaves a hole that is never committed). */
 int nvbt_channel_drain(nvbt_channel ch, nvbt_drain_fn fn, void* user, int64_t timeout_us,
@@ -181,7 +181,7 @@ int nvbt_channel_close(nvbt_channel ch);
 int nvbt_trace_footprint(nvbt_channel ch, void* d_scratch, uint64_t table_slots, uint32_t first_launch,
                          uint32_t n_launches, uint64_t* out, float* kernel_ms);
 
-/* Records the producers dropped after waiting ~2 s on a full ring (0 in a healthy run). */
+/* Records the producers dropped after waiting 10 s (NVBT_PRODUCER_WAIT_MS) on a full ring (0 in a healthy run). */
 int nvbt_channel_dropped(nvbt_channel ch, uint64_t* dropped);
 
 /* Built-in drain callbacks. */

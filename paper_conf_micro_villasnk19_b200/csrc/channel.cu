@@ -33,6 +33,7 @@ struct nvbt_chan_s {
   uint64_t consumed = 0;
   unsigned slot = 288;                 // bytes per ring slot (288 full, 176 compact)
   bool force_wide = false;
+  unsigned long long wait_ns = 10000000000ull;   // a producer gives up after this long without room
   bool on_device = false;              // F2: ring in device memory, consumed by GPU kernels
   unsigned rstripes = 0;               // device ring: per-SM chunk stripes (see DevState)
   bool open = false;
@@ -73,6 +74,7 @@ void channel_state(nvbt_chan_s* ch, DevState* st) {
   // (NVBT_COMPACT_FORCE_WIDE=1, tests only)
   st->compact = ch->fmt == 1u ? (ch->force_wide ? 2u : 1u) : ch->fmt == 2u ? (ch->force_wide ? 4u : 3u) : 0u;
   st->no_wait = ch->on_device ? 1u : 0u;   // nobody frees device-ring slots: drop instead of waiting
+  st->wait_ns = ch->wait_ns;
   st->rheads = ch->on_device ? ch->ctx->ctl + CTL_RHEAD : nullptr;
   st->rstripes = ch->rstripes;
 }
@@ -383,6 +385,7 @@ int nvbt_channel_open(nvbt_ctx c, void* ring, size_t bytes, uint32_t record_byte
   ch->slot = slot_stride(record_bytes);
   ch->fmt = fmt_of(record_bytes);
   { const char* e = getenv("NVBT_COMPACT_FORCE_WIDE"); ch->force_wide = e && atoi(e) != 0; }
+  { const char* e = getenv("NVBT_PRODUCER_WAIT_MS"); if (e && atoll(e) > 0) ch->wait_ns = 1000000ull * (unsigned long long)atoll(e); }
   // host rings: each slot has a 4 B tag in the array after the slots; device rings carry the tag in-record
   ch->cap = (bytes - ch->hdr) / (ch->slot + (on_device ? 0u : 4u));
   ch->tags = on_device ? nullptr : reinterpret_cast<const uint32_t*>(ch->host + ch->hdr + ch->cap * ch->slot);

@@ -54,6 +54,7 @@ struct DevState {
   unsigned compact;                // 0 full records; 1 / 2 176 B slots (2: force wide pairs); 3 / 4 128 B slots
                                    // (4: force the three-slot form)
   unsigned no_wait;                // device-memory ring (F2): drop when full instead of waiting
+  unsigned long long wait_ns;      // host ring: a producer waiting this long for room gives up (drops)
   // device ring (F2): slots are handed out in chunks of kRingChunk. Each SM owns a stripe word
   // rheads[smid % rstripes] = (chunk << 32 | used) and takes tickets from its current chunk; the warp whose
   // ticket is exactly kRingChunk opens the stripe's next chunk from the global counter rheads[rstripes].
@@ -92,17 +93,18 @@ template <class Prog> __host__ __device__ constexpr int mem_left(int pc) {
 // Ring backpressure: ticket t may be written once t < tail + cap. has_room() is the
 // cheap check against the device-side cache of the host's consumer index; reserve() then waits on the host
 // index (PCIe reads, poll_room() in a warp-uniform loop) and gives up if the host never freed a slot within
-// ~2 s or another producer already gave up (the record is then dropped and counted, never hangs the GPU).
+// st.wait_ns (10 s; NVBT_PRODUCER_WAIT_MS at channel open) or another producer already gave up (the record is
+// then dropped and counted, never hangs the GPU).
 __device__ __forceinline__ bool has_room(const DevState& st, unsigned long long t) {
   return t < *(volatile const unsigned long long*)st.tail_cache + st.cap;
 }
 // One poll of the host index for ticket t (waiting since t0): 1 = room (tail cache refreshed), -1 = give up
-// (~2 s without progress, or another producer already gave up), 0 = keep waiting.
+// (st.wait_ns without progress, or another producer already gave up), 0 = keep waiting.
 __device__ __forceinline__ int poll_room(const DevState& st, unsigned long long t, unsigned long long t0) {
   if (*(volatile const unsigned long long*)st.dropped != 0) return -1;
   const unsigned long long tl = *(volatile const unsigned long long*)st.tail;
   if (t < tl + st.cap) { atomicMax(st.tail_cache, tl); return 1; }
-  return globaltimer() - t0 > 2000000000ull ? -1 : 0;
+  return globaltimer() - t0 > st.wait_ns ? -1 : 0;
 }
 
 template <uint32_t T, class Prog>

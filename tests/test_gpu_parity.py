@@ -228,8 +228,9 @@ def test_channel_compact128_bfs(nvbt):
     assert (trace.sort_records(dst[:got_n]) == trace.sort_records(exp)).all()
 
 
-def test_channel_drop_is_reported(nvbt):
-    """A host ring nobody drains while the kernel runs: the producers wait ~2 s for room, then give up; the
+def test_channel_drop_is_reported(nvbt, monkeypatch):
+    """A host ring nobody drains while the kernel runs: the producers wait (here 2 s, NVBT_PRODUCER_WAIT_MS)
+    for room, then give up; the
     records they drop are counted (nvbt_channel_dropped) and the drain fails loudly (NVBT_ETIMEDOUT) after
     delivering what was committed, instead of hanging or passing silently (include/nvbt.h: the channel
     must then be reopened)."""
@@ -240,6 +241,7 @@ def test_channel_drop_is_reported(nvbt):
     x0 = cuda(uniform_f32((n, n), 4))
     b0, b1 = x0.clone(), torch.zeros_like(x0)
     ring = torch.empty(nb.nvbt_channel_bytes(8), dtype=torch.uint8, pin_memory=True)
+    monkeypatch.setenv("NVBT_PRODUCER_WAIT_MS", "2000")
     ch = nb.nvbt_channel_open(ctx, ring)
     dr.run_stencil(ctx, nb.TOOL_TRACE, b0, b1, n, 1)
     torch.cuda.synchronize()                     # no consumer ran: the ring filled up
