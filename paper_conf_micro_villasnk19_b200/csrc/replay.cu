@@ -338,6 +338,14 @@ constexpr int RB_NW = NVBT_RPB_NW;     // pass B warps per CTA
 #define NVBT_RPB_HASH1 1       // wide-row bucket = top bits of the line's multiplicative hash, no finaliser (A/B r2_ab21:
                                // pass B 1.820 -> 1.806 ms; a bad spread only costs the resolve / exact paths)
 #endif
+#ifndef NVBT_RPB_REDSEL
+#define NVBT_RPB_REDSEL 1      // pass B's per-row shared reductions run on every lane (others add 0 to a lane-private
+                               // word) instead of a predicated red that ptxas turns into a branch + reconvergence
+#endif
+#ifndef NVBT_RPB_OFF3
+#define NVBT_RPB_OFF3 1        // cp.async stage offsets as one LOP3 on 34 r (see rb_off); with REDSEL: A/B r2_ab22 pass B
+                               // 1.799 -> 1.762 ms (REDSEL alone 1.796, OFF3 alone 1.775)
+#endif
 #ifndef NVBT_RPB_C0REDUX
 #define NVBT_RPB_C0REDUX 0     // 1: one-1-KB-word rows by an OR-reduction of their sector bits (own loop). A/B r2_ab16:
                                // pass B 1.839 -> 1.890 ms, not kept
@@ -479,6 +487,12 @@ __device__ __forceinline__ void sl_bitonic(unsigned long long a, bool act, unsig
 __device__ __forceinline__ unsigned rb_off(unsigned r, unsigned idx) {
 #if NVBT_RPB_TMA
   return 2048u * (idx >> 4) + 128u * r + ((8u * (idx & 15u)) ^ (16u * (r & 7u)));
+#elif NVBT_RPB_OFF3
+  // 8 (32 r + (idx ^ 2 (r & 7))): with a = 34 r (32 r in bits 5.., 2 r in bits 1..4), the index is
+  // idx ^ (a & c) for c = ~0x11 (bits 5.. of idx are zero; bit 4 of 2 r must not flip idx): one LOP3
+  unsigned x;
+  asm("lop3.b32 %0, %1, %2, %3, 0x6C;" : "=r"(x) : "r"(34u * r), "r"(idx), "r"(0xFFFFFFEEu));   // b ^ (a & c)
+  return 8u * x;
 #else
   return 256u * r + ((8u * idx) ^ (16u * (r & 7u)));
 #endif
@@ -817,11 +831,27 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
     asm volatile("red.global.add.u64 [%0], %1;" ::"l"(gmem + 3u * pc + 2u), "l"((unsigned long long)L) : "memory");
   }
 #else
+#if NVBT_RPB_REDSEL
+  {
+    const unsigned dmy = s_scr + 4u * lane;   // lane-private word: adding 0 changes nothing
+    asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(own ? s_sS + 4u * pc : dmy), "r"(own ? S : 0u) : "memory");
+    asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(own ? s_sL + 4u * pc : dmy), "r"(own ? L : 0u) : "memory");
+  }
+#else
   red_shared_add_if(own, s_sS + 4u * pc, S);
   red_shared_add_if(own, s_sL + 4u * pc, L);
 #endif
+#endif
+#if NVBT_RPB_REDSEL
+  {
+    const unsigned dmy = s_scr + 4u * lane, one = own ? 1u : 0u;
+    asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(own ? s_hist + 4u * S : dmy), "r"(one) : "memory");          // hS[S]
+    asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(own ? s_hist + 4u * (33u + L) : dmy), "r"(one) : "memory");  // hL[L]
+  }
+#else
   red_shared_add_if(own, s_hist + 4u * S, 1u);          // hS[S]
   red_shared_add_if(own, s_hist + 4u * (33u + L), 1u);  // hL[L]
+#endif
   __syncwarp();
 }
 
