@@ -346,6 +346,12 @@ constexpr int RB_NW = NVBT_RPB_NW;     // pass B warps per CTA
 #define NVBT_RPB_OFF3 1        // cp.async stage offsets as one LOP3 on 34 r (see rb_off); with REDSEL: A/B r2_ab22 pass B
                                // 1.799 -> 1.762 ms (REDSEL alone 1.796, OFF3 alone 1.775)
 #endif
+#ifndef NVBT_RPB_STG2
+#define NVBT_RPB_STG2 1        // staging copies row k + 8h in step k (slot indices by width-16 shuffles with immediate
+                               // source lanes, smem offsets by one XOR with an immediate), full groups unpredicated:
+                               // 4 instead of ~12 instructions per step (A/B r2_ab23: pass B 1.764 -> 1.761 ms; the
+                               // staging was off the critical path)
+#endif
 #ifndef NVBT_RPB_C0REDUX
 #define NVBT_RPB_C0REDUX 0     // 1: one-1-KB-word rows by an OR-reduction of their sector bits (own loop). A/B r2_ab16:
                                // pass B 1.839 -> 1.890 ms, not kept
@@ -356,7 +362,12 @@ constexpr int RB_NW = NVBT_RPB_NW;     // pass B warps per CTA
 constexpr int RA_CTAS_PER_SM = 2;   // pass A CTAs per SM
 constexpr int RA_DEPTH = 4;   // pass A header tiles in flight per warp
 constexpr int RB_ROWS = 16;   // slots per stage
-constexpr int RB_STAGES = 2;
+#ifndef NVBT_RPB_STAGES
+#define NVBT_RPB_STAGES 2
+#endif
+constexpr int RB_STAGES = NVBT_RPB_STAGES;   // per-warp shared stages (RB_STAGES - 1 groups in flight ahead). A/B
+                                             // r2_ab24: 3 stages x 13 warps 2.49 ms, 3 x 16 (global bins) 2.26, 2 x 16
+                                             // 2.25, 2 x 20 1.77: the pass needs warps, not depth
 // per-warp scratch, 1280 B: the slow rows' tag arrays (1 KB sector / hash tags + 256 B line tags); the
 // A/B build without them (NVBT_RPB_TAGS=0) uses its first SCRATCH_WORDS words as sectors_lines_cls scratch
 constexpr int RB_SCR2 = 128;
@@ -891,7 +902,9 @@ k_rpB(const unsigned long long* __restrict__ addr, unsigned P, const uint8_t* __
   __syncthreads();
   unsigned phase = 0;   // bit s: parity of stage s's next completion
 #else
-  unsigned* sWarpAll = sm + PB;
+  // warp areas 128-byte aligned (9728 B each): stage chunk offsets can then be XOR-ed into full addresses
+  unsigned* sWarpAll = reinterpret_cast<unsigned*>((reinterpret_cast<uintptr_t>(sm + PB) + 127u) & ~uintptr_t(127));
+  static_assert((RB_WARP_WORDS * 4) % 128 == 0, "128 B aligned warp areas");
   constexpr unsigned kScr0 = RB_STAGES * (RB_ROWS * 64 + 2 * RB_ROWS);
   for (unsigned i = threadIdx.x; i < RB_NW * RB_WARP_WORDS; i += blockDim.x) {
     const unsigned o = i % RB_WARP_WORDS;
@@ -961,6 +974,30 @@ k_rpB(const unsigned long long* __restrict__ addr, unsigned P, const uint8_t* __
                    ::"r"(stg + 2048u * hf + 512u * q4), "l"(reinterpret_cast<unsigned long long>(&tmap)), "r"(32u * hf),
                      "r"(ri[0]), "r"(ri[1]), "r"(ri[2]), "r"(ri[3]), "r"(bar)
                    : "memory");
+#elif NVBT_RPB_STG2
+    // step k: lane (h, c) copies 16 B chunk c of row k + 8h. Row r's chunk c lives at 256 r + 16 (c ^ (r & 7)) =
+    // 256 k + (lane_off ^ 16 k) with lane_off = 2048 h + 16 c (r & 7 == k). The upper half first takes the slot
+    // indices of rows 8..15, so step k's index comes from source lane k of each half (width-16 shuffle).
+    const unsigned idx_st = __shfl_sync(FULL, nx_idx, h ? ((lane + 8u) & 15u) : lane);
+    const unsigned sb = stg + 2048u * h + 16u * (lane & 15u);   // stg is 128-aligned: XOR 16 k stays in the chunk bits
+    const unsigned long long* gl = addr + 2u * (lane & 15u);
+    if (g1.rows == (unsigned)RB_ROWS) {            // warp-uniform: a full group
+#pragma unroll
+      for (int k = 0; k < RB_ROWS / 2; ++k) {
+        const unsigned ix = __shfl_sync(FULL, idx_st, k, 16);
+        asm volatile("cp.async.cg.shared.global [%0], [%1], 16;"
+                     ::"r"((sb ^ (16u * k)) + 256u * k), "l"(gl + (unsigned long long)ix * 32u) : "memory");
+      }
+    } else {
+#pragma unroll
+      for (int k = 0; k < RB_ROWS / 2; ++k) {
+        const unsigned ix = __shfl_sync(FULL, idx_st, k, 16);
+        if ((unsigned)k + 8u * h < g1.rows)
+          asm volatile("cp.async.cg.shared.global [%0], [%1], 16;"
+                       ::"r"((sb ^ (16u * k)) + 256u * k), "l"(gl + (unsigned long long)ix * 32u) : "memory");
+      }
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
 #else
     const unsigned c = lane & 15u;
 #pragma unroll
@@ -987,6 +1024,28 @@ k_rpB(const unsigned long long* __restrict__ addr, unsigned P, const uint8_t* __
 #if NVBT_RPB_PF
   fetch(g2);
 #endif
+#if !NVBT_RPB_TMA
+  // RB_STAGES - 1 groups in flight ahead of the one being analysed; stage (s + RB_STAGES - 1) % RB_STAGES was
+  // analysed in the previous step. Steps without a group to issue commit an empty cp.async group, so
+  // wait_group(RB_STAGES - 1) always retires the oldest issued one.
+  unsigned s = 0, pending = 0;
+#pragma unroll
+  for (int i = 0; i < RB_STAGES - 1; ++i) {
+    if (g1.rows != 0u) { issue((unsigned)i); ++pending; }
+    else asm volatile("cp.async.commit_group;" ::: "memory");
+  }
+  while (pending) {
+    const unsigned sn = s == 0u ? (unsigned)RB_STAGES - 1u : s - 1u;
+    if (g1.rows != 0u) { issue(sn); ++pending; }
+    else asm volatile("cp.async.commit_group;" ::: "memory");
+    asm volatile("cp.async.wait_group %0;" ::"n"(RB_STAGES - 1) : "memory");
+    __syncwarp();
+    rb_process(s_w + 4096u * s, s_meta + 128u * s, lane, lanebit, s_scr, s_sS, s_sL, s_hist, gmem);
+    --pending;
+    s = s + 1u == (unsigned)RB_STAGES ? 0u : s + 1u;
+  }
+#else
+  static_assert(RB_STAGES == 2, "TMA stages: double buffering only");
   bool live = g1.rows != 0u;
   unsigned s = 0;
   if (live) issue(0);
@@ -1014,6 +1073,7 @@ k_rpB(const unsigned long long* __restrict__ addr, unsigned P, const uint8_t* __
     rb_process(s_w + 4096u * s, s_meta + 128u * s, lane, lanebit, s_scr, s_sS, s_sL, s_hist, gmem);
     s ^= 1u;
   }
+#endif
   __syncthreads();
 #if NVBT_RPB_GBINS
   for (unsigned i = threadIdx.x; i < 66; i += blockDim.x)
@@ -1037,7 +1097,7 @@ static size_t rpB_smem(unsigned P) {
 #if NVBT_RPB_TMA
   return ((2ull * P + 66 + 3) & ~3ull) * 4 + 1023 + (8192ull + RB_X_BYTES) * RB_NW;
 #else
-  return ((NVBT_RPB_GBINS ? 68ull : ((2ull * P + 66 + 3) & ~3ull)) + (size_t)RB_NW * RB_WARP_WORDS) * 4;
+  return ((NVBT_RPB_GBINS ? 68ull : ((2ull * P + 66 + 3) & ~3ull)) + (size_t)RB_NW * RB_WARP_WORDS) * 4 + 128;
 #endif
 }
 
