@@ -107,6 +107,9 @@ __device__ __forceinline__ int poll_room(const DevState& st, unsigned long long 
   return globaltimer() - t0 > st.wait_ns ? -1 : 0;
 }
 
+#ifndef NVBT_HOOKS_EXPERIMENT
+#define NVBT_HOOKS_EXPERIMENT 0   // timing experiments only (wrong results): 1 no CTA flush, 2 no bin init, 3 both
+#endif
 template <uint32_t T, class Prog>
 struct Hooks {
   static constexpr int NPC = Prog::N;
@@ -147,7 +150,7 @@ struct Hooks {
     gwarp = (st.cta_lo + blockIdx.x + blockIdx.y * gridDim.x) * ((blockDim.x * blockDim.y) >> 5) + (tid >> 5);  // logical CTA
     scr = (unsigned)__cvta_generic_to_shared(sb + kScratchWord0 + SCRATCH_WORDS * ((tid >> 5) & (kMaxWarps - 1)));
     sbase = (unsigned)__cvta_generic_to_shared(sb);
-    if constexpr (kOn) {
+    if constexpr (kOn && !(NVBT_HOOKS_EXPERIMENT & 2)) {
       // (CTAs of exactly kThreads threads; fixed-stride loops avoid a run-time trip-count division)
       constexpr int kInit = (T & TOOL_MEM) ? kSmemWords : kScratchWord0;   // scratch only for divergence
 #pragma unroll
@@ -734,6 +737,7 @@ struct Hooks {
           atomicAdd(st.pw + st.n_warps + gwarp, (unsigned long long)pwW);
         }
       }
+      if (NVBT_HOOKS_EXPERIMENT & 1) return;
       __syncthreads();
       const int tid = threadIdx.x + threadIdx.y * blockDim.x;
       constexpr int nt = kThreads;
