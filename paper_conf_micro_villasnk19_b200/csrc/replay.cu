@@ -332,7 +332,8 @@ constexpr int RB_NW = NVBT_RPB_NW;     // pass B warps per CTA
 #endif
 #ifndef NVBT_RPB_WIDE2
 #define NVBT_RPB_WIDE2 0       // 1: wide rows two per iteration (independent chains), 640 hash buckets each, resolved.
-                               // A/B r2_ab17: pass B 1.813 -> 1.894 ms (more collisions, instruction-bound), not kept
+                               // A/B r2_ab17: pass B 1.813 -> 1.894 ms (more collisions, instruction-bound), not kept;
+                               // with GBINS, 1280 buckets each (r2_ab25): 1.776 -> 1.843 ms (GBINS alone 1.791)
 #endif
 #ifndef NVBT_RPB_HASH1
 #define NVBT_RPB_HASH1 1       // wide-row bucket = top bits of the line's multiplicative hash, no finaliser (A/B r2_ab21:
@@ -370,7 +371,9 @@ constexpr int RB_STAGES = NVBT_RPB_STAGES;   // per-warp shared stages (RB_STAGE
                                              // 2.25, 2 x 20 1.77: the pass needs warps, not depth
 // per-warp scratch, 1280 B: the slow rows' tag arrays (1 KB sector / hash tags + 256 B line tags); the
 // A/B build without them (NVBT_RPB_TAGS=0) uses its first SCRATCH_WORDS words as sectors_lines_cls scratch
-constexpr int RB_SCR2 = 128;
+// (two wide rows per iteration with the global per-pc bins: 1280 more bytes, one 1280-bucket table per row)
+constexpr int RB_SCR2 = 128 + ((NVBT_RPB_WIDE2 && NVBT_RPB_GBINS) ? 320 : 0);
+constexpr unsigned kWideBuckets = (NVBT_RPB_WIDE2 && NVBT_RPB_GBINS) ? 1280u : 640u;   // per row, WIDE2
 constexpr int RB_WARP_WORDS = RB_STAGES * (RB_ROWS * 64 + 2 * RB_ROWS) + SCRATCH_WORDS + RB_SCR2;
 constexpr size_t RS_COUNTS_BYTES = 65536;   // u32 per pass-A warp (< 16384 warps), then the region counter
 constexpr unsigned kRegionCtr = 16383;      // counts[kRegionCtr]: regions claimed past the first (NVBT_RPB_DYN)
@@ -694,7 +697,11 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
       x0[k] = (unsigned)line;
       x1[k] = (unsigned)(line >> 32);
       const unsigned hsh = x0[k] * 0x9E3779B1u ^ x1[k] * 0x85EBCA77u;
-      hb[k] = 640u * k + __umulhi(hsh * 0xC2B2AE3Du + (hsh >> 15), 640u);
+#if NVBT_RPB_HASH1
+      hb[k] = kWideBuckets * k + __umulhi(hsh, kWideBuckets);
+#else
+      hb[k] = kWideBuckets * k + __umulhi(hsh * 0xC2B2AE3Du + (hsh >> 15), kWideBuckets);
+#endif
       if (act[k]) sts_u8(stag + hb[k], lane);
     }
     __syncwarp();
