@@ -197,8 +197,9 @@ int nvbt_digest_records(const void* records, uint64_t n_records, nvbt_digest* ou
  * out_cap records); *n_out = records written. EINVAL on an unpaired wide slot or a too-small out. */
 int nvbt_decode_compact(const void* slots, uint64_t n_slots, void* out, uint64_t out_cap, uint64_t* n_out);
 /* The same for either compact transport: record_bytes NVBT_COMPACT_RECORD_BYTES or
- * NVBT_COMPACT128_RECORD_BYTES, slots packed record_bytes apart (tags ignored). EINVAL on a record whose
- * continuation slots are missing or a too-small out. */
+ * NVBT_COMPACT128_RECORD_BYTES, slots packed record_bytes apart (tags ignored; 128 B skip slots, 0xC0 at
+ * byte 27, carry no record, EM §5.2). EINVAL on a record whose continuation slots are missing or a too-small
+ * out. */
 int nvbt_decode_slots(const void* slots, uint64_t n_slots, uint32_t record_bytes, void* out, uint64_t out_cap,
                       uint64_t* n_out);
 

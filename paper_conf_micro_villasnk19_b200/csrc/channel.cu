@@ -219,8 +219,11 @@ static uint64_t ready_prefix(const uint32_t* base, uint64_t lim, uint32_t lap) {
   for (uint64_t f : first) stop = std::min(stop, f);
   return n + stop;
 }
-// ---- compact transport (EM §5.1): slot flags in byte 27 (kind | 0x80 compact, 0x40 / 0x20 wide halves)
+// ---- compact transport (EM §5.1): slot flags in byte 27 (kind | 0x80 compact, 0x40 / 0x20 wide halves;
+// 0xC0 a skip slot of the 128 B transport: a ticket the producer's block did not use, EM §5.2)
 static inline unsigned slot_flags(const unsigned char* sl) { return sl[27] & 0xE0u; }
+static constexpr unsigned kSkipFlags = 0xC0u;
+static inline bool starts_record(unsigned f) { return f != 0x20u && f != kSkipFlags; }
 
 static void decode_compact_slot(const unsigned char* sl, unsigned char* out) {
   std::memcpy(out, sl, 28);
@@ -296,7 +299,7 @@ static void decode_group(unsigned fmt, const unsigned char* s0, unsigned ss, uns
 static uint64_t decode_batch(const unsigned char* sl, uint64_t n, unsigned char* out, unsigned ss, unsigned fmt) {
   Pool& pool = Pool::get();
   std::vector<uint64_t> cnt(pool.size() + 1, 0), lo_of(pool.size(), 0), hi_of(pool.size(), 0);
-  auto is_rec = [&](uint64_t i) { return slot_flags(sl + (size_t)i * ss) != 0x20u; };
+  auto is_rec = [&](uint64_t i) { return starts_record(slot_flags(sl + (size_t)i * ss)); };
   pool.parallel_for(n, [&](unsigned id, uint64_t lo, uint64_t hi) {
     uint64_t c = 0;
     for (uint64_t i = lo; i < hi; ++i) c += is_rec(i);
@@ -310,7 +313,7 @@ static uint64_t decode_batch(const unsigned char* sl, uint64_t n, unsigned char*
     for (uint64_t i = lo; i < hi; ++i) {
       const unsigned char* s0 = sl + (size_t)i * ss;
       const unsigned f = slot_flags(s0);
-      if (f == 0x20u) continue;
+      if (!starts_record(f)) continue;
       decode_group(fmt, s0, ss, out + (size_t)o * RECORD_BYTES);
       ++o;
     }
@@ -328,7 +331,7 @@ static uint64_t digest_compact(const unsigned char* sl, uint64_t n, uint64_t* d1
     for (uint64_t i = lo; i < hi; ++i) {
       const unsigned char* s0 = sl + (size_t)i * ss;
       const unsigned f = slot_flags(s0);
-      if (f == 0x20u) continue;
+      if (!starts_record(f)) continue;
       decode_group(fmt, s0, ss, rec);
       digest_serial(rec, 1, &s1, &s2);
       ++c;
@@ -909,6 +912,7 @@ int nvbt_decode_slots(const void* slots, uint64_t n, uint32_t record_bytes, void
   for (uint64_t i = 0; i < n;) {
     const unsigned char* s0 = sl + i * ss;
     const unsigned f = slot_flags(s0);
+    if (fmt == 2u && f == kSkipFlags) { ++i; continue; }   // an unused ticket of a producer's block
     if (f != 0x80u && f != 0x40u)
       return set_error(NVBT_EINVAL, "slot %llu: not the first slot of a record (flags 0x%x)", (unsigned long long)i, f);
     const unsigned g = group_len(fmt, f);

@@ -473,9 +473,28 @@ struct Hooks {
     const long long dl = (long long)(addr - base);
     if (st.compact >= 3u) {
       // 128 B slots (EM §5.2): one whole PCIe line per record when every lane of E is within +-32 KB of
-      // the first (header, base, 32 x i16 deltas), else three slots of full addresses
-      if (st.compact == 3u && __all_sync(FULL, !act || (dl >= -32768ll && dl <= 32767ll))) {
-        if (reserve(1, t)) {
+      // the first (header, base, 32 x i16 deltas), else three slots of full addresses. Slots come from a
+      // block of consecutive tickets the warp reserves for the rest of its basic block (x4 in loops), so
+      // the warp's records and commit tags are contiguous on the link (tools/peaks/d2h_line.cu: 309 ->
+      // 387 M lines/s); slots the block does not use are committed as skip slots (EM §5.2, flags 0xC0).
+      constexpr unsigned K = (unsigned)mem_left<Prog>(PC) * ((PC >= Prog::REG_LO && PC <= Prog::REG_HI) ? 4u : 1u);
+      const bool shortf = st.compact == 3u && __all_sync(FULL, !act || (dl >= -32768ll && dl <= 32767ll));
+      const unsigned need = shortf ? 1u : 3u;
+      bool have = true;
+      if (held < need) {                           // warp-uniform
+        release();
+        const unsigned long long want = (unsigned long long)(K > need ? K : need);
+        const unsigned k = (unsigned)(want < st.cap ? want : st.cap);   // a block never exceeds the ring
+        have = reserve(k, hslot);
+        held = have ? k : 0u;
+      }
+      if (have) {
+        t = hslot;
+        hslot += need;
+        held -= need;
+      }
+      if (have && shortf) {
+        {
           unsigned* tp;
           unsigned char* rec = slot_ptr(t, tag, tp);
           // u32 word k of the delta area (bytes 40..103) = delta[2k] | delta[2k + 1] << 16, built on lane 2k
@@ -498,7 +517,7 @@ struct Hooks {
           }
           add_pending(tp, tag);
         }
-      } else if (reserve(3, t)) {
+      } else if (have) {
         // three slots: slot 0 = header (kind | 0x40) + lanes 0..11; slots 1, 2 carry flag 0x20 at byte 27
         // and lanes 12..26 (bytes 0..23: 3 lanes, 32..127: 12 lanes) and 27..31
         unsigned tg[3];
@@ -567,6 +586,25 @@ struct Hooks {
       add_pending(tp1, tag1);
     }
     ++seq;
+  }
+
+  // 128 B line transport: the unused rest of the warp's ticket block becomes skip slots (header chunk with
+  // flags 0xC0 at byte 27, committed like records) so the consumer can pass them.
+  __device__ __forceinline__ void release() {
+    while (held != 0u) {                           // warp-uniform
+      const unsigned k = held < 32u ? held : 32u;
+      unsigned tag = 0;
+      unsigned* tp = nullptr;
+      unsigned char* rec = slot_ptr(hslot + (lane < k ? lane : 0u), tag, tp);
+      if (lane < k) *reinterpret_cast<uint4*>(rec + 16) = make_uint4(0u, 0u, 0xC0000000u, 0u);
+      for (unsigned i = 0; i < k; ++i) {
+        const unsigned ti = __shfl_sync(FULL, tag, i);
+        unsigned* tpi = reinterpret_cast<unsigned*>(__shfl_sync(FULL, reinterpret_cast<unsigned long long>(tp), i));
+        add_pending(tpi, ti);
+      }
+      hslot += k;
+      held -= k;
+    }
   }
 
   __device__ __forceinline__ void commit() {
@@ -727,7 +765,12 @@ struct Hooks {
   // Must be reached by every thread of the CTA.
   __device__ __forceinline__ void finish() {
     if constexpr (kOn) {
-      if constexpr ((T & TOOL_TRACE) != 0) commit();
+      if constexpr ((T & TOOL_TRACE) != 0 && (T & TOOL_TRACE_DEV) == 0) {
+        if (st.compact >= 3u) release();
+        commit();
+      } else if constexpr ((T & TOOL_TRACE) != 0) {
+        commit();
+      }
       retire<0, NPC - 1>();
       if (hS) atomicAdd(&sb[NPC * SITE_WORDS + 1 + lane], hS);
       if (hL) atomicAdd(&sb[NPC * SITE_WORDS + 34 + lane], hL);
