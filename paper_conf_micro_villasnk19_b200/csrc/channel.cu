@@ -912,7 +912,7 @@ int nvbt_decode_slots(const void* slots, uint64_t n, uint32_t record_bytes, void
   for (uint64_t i = 0; i < n;) {
     const unsigned char* s0 = sl + i * ss;
     const unsigned f = slot_flags(s0);
-    if (fmt == 2u && f == kSkipFlags) { ++i; continue; }   // an unused ticket of a producer's block
+    if (f == kSkipFlags) { ++i; continue; }   // an unused ticket of a producer's block
     if (f != 0x80u && f != 0x40u)
       return set_error(NVBT_EINVAL, "slot %llu: not the first slot of a record (flags 0x%x)", (unsigned long long)i, f);
     const unsigned g = group_len(fmt, f);

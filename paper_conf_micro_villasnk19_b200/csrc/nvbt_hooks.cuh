@@ -547,8 +547,25 @@ struct Hooks {
       ++seq;
       return;
     }
-    if (st.compact == 1u && __all_sync(FULL, !act || (dl >= -0x80000000ll && dl <= 0x7fffffffll))) {
-      if (reserve(1, t)) {
+    // 176 B slots: tickets from the warp's block as for 128 B slots (skip slots for the unused ones)
+    const bool shortc = st.compact == 1u && __all_sync(FULL, !act || (dl >= -0x80000000ll && dl <= 0x7fffffffll));
+    const unsigned needc = shortc ? 1u : 2u;
+    bool havec = true;
+    if (held < needc) {                            // warp-uniform
+      release();
+      constexpr unsigned K = (unsigned)mem_left<Prog>(PC) * ((PC >= Prog::REG_LO && PC <= Prog::REG_HI) ? 4u : 1u);
+      const unsigned long long want = (unsigned long long)(K > needc ? K : needc);
+      const unsigned k = (unsigned)(want < st.cap ? want : st.cap);
+      havec = reserve(k, hslot);
+      held = havec ? k : 0u;
+    }
+    if (havec) {
+      t = hslot;
+      hslot += needc;
+      held -= needc;
+    }
+    if (havec && shortc) {
+      {
         unsigned* tp;
         unsigned char* rec = slot_ptr(t, tag, tp);
         // 11 chunks: header, header (kind | 0x80), base, then 4 deltas per chunk (lanes 4(j-3) .. +3)
@@ -565,7 +582,7 @@ struct Hooks {
         }
         add_pending(tp, tag);
       }
-    } else if (reserve(2, t)) {
+    } else if (havec) {
       // wide pair: slot t = lanes 0-15, slot t+1 = lanes 16-31 (full addresses); lanes 0-9 write the
       // first slot's 10 chunks, lanes 16-25 the second's
       unsigned tag0, tag1;
@@ -766,7 +783,7 @@ struct Hooks {
   __device__ __forceinline__ void finish() {
     if constexpr (kOn) {
       if constexpr ((T & TOOL_TRACE) != 0 && (T & TOOL_TRACE_DEV) == 0) {
-        if (st.compact >= 3u) release();
+        if (st.compact != 0u) release();   // compact host rings take tickets in blocks
         commit();
       } else if constexpr ((T & TOOL_TRACE) != 0) {
         commit();

@@ -121,6 +121,25 @@ def test_compact_decode_matches_records():
     assert dec.shape == recs.shape and (dec == recs).all()
     with pytest.raises(nb.NvbtError):          # an unpaired wide half is rejected
         nb.nvbt_decode_compact(slots[(slots[:, 27] & 0xE0) == 0x20][:1])
+    with_skips = _with_skip_slots(slots, 176, seed=3)
+    assert len(with_skips) > len(slots)
+    assert np.array_equal(nb.nvbt_decode_compact(with_skips), dec)
+
+
+def _with_skip_slots(slots, width, seed):
+    """Inserts 0-2 skip slots (0xC0 at byte 27, other bytes random: unused tickets of a producer's block)
+    after every record of a packed slot array; never inside a multi-slot record."""
+    rng = np.random.default_rng(seed)
+    starts = [i for i in range(len(slots)) if (slots[i, 27] & 0xE0) != 0x20]
+    pieces = []
+    for k, i in enumerate(starts):
+        j = starts[k + 1] if k + 1 < len(starts) else len(slots)
+        pieces.append(slots[i:j])
+        for _ in range(int(rng.integers(0, 3))):
+            junk = rng.integers(0, 256, size=(1, width), dtype=np.uint8)
+            junk[0, 27] = 0xC0 | (junk[0, 27] & 0x1F)
+            pieces.append(junk)
+    return np.concatenate(pieces)
 
 
 def _encode_compact128(recs, long_mask):
@@ -180,19 +199,8 @@ def test_compact128_decode_matches_records():
     assert dec.shape == recs.shape and (dec == recs).all()
     with pytest.raises(nb.NvbtError):          # a long record without its continuation slots is rejected
         nb.nvbt_decode_compact(slots[(slots[:, 27] & 0xE0) == 0x40][:1], record_bytes=128)
-    # skip slots (unused tickets of a producer's block: 0xC0 at byte 27, the rest unspecified) between
-    # records, never inside a long record, decode to nothing
-    rng = np.random.default_rng(7)
-    starts = [i for i in range(len(slots)) if (slots[i, 27] & 0xE0) != 0x20]
-    pieces = []
-    for k, i in enumerate(starts):
-        j = starts[k + 1] if k + 1 < len(starts) else len(slots)
-        pieces.append(slots[i:j])
-        for _ in range(int(rng.integers(0, 3))):
-            junk = rng.integers(0, 256, size=(1, 128), dtype=np.uint8)
-            junk[0, 27] = 0xC0 | (junk[0, 27] & 0x1F)
-            pieces.append(junk)
-    with_skips = np.concatenate(pieces)
+    # skip slots between records (never inside a long record) decode to nothing
+    with_skips = _with_skip_slots(slots, 128, seed=7)
     assert len(with_skips) > len(slots)
     assert np.array_equal(nb.nvbt_decode_compact(with_skips, record_bytes=128), dec)
 
