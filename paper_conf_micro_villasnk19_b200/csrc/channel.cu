@@ -198,8 +198,10 @@ static void digest_range(const unsigned char* rec, uint64_t n, uint64_t* d1, uin
 
 // Length of the prefix of slots [0, lim) whose tag equals `lap` (written and committed). Scans a short
 // window serially and, when that is all ready, the rest of the batch in parallel on the pool.
+// (bit 31 of a tag, kSkipTag, marks a ticket committed without a record: the unused rest of a producer's
+// block of 288 B slots)
 static inline bool slot_ready(const uint32_t* tag, uint32_t lap) {
-  return *reinterpret_cast<volatile const uint32_t*>(tag) == lap;
+  return (*reinterpret_cast<volatile const uint32_t*>(tag) & ~kSkipTag) == lap;
 }
 static uint64_t ready_prefix(const uint32_t* base, uint64_t lim, uint32_t lap) {
   const uint64_t w = std::min<uint64_t>(lim, 2048);
@@ -787,9 +789,20 @@ int nvbt_channel_drain(nvbt_channel ch, nvbt_drain_fn fn, void* user, int64_t ti
     if (n && sb == RECORD_BYTES) {
       std::atomic_thread_fence(std::memory_order_acquire);
       unsigned char* base = ch->slots + slot * RECORD_BYTES;
-      const int urc = fn(base, n, user);
+      // runs of records between skip tickets (tags with kSkipTag carry no record)
+      const uint32_t* tg = ch->tags + slot;
+      int urc = 0;
+      for (uint64_t i = 0; i < n && !urc;) {
+        uint64_t j = i;
+        while (j < n && !(tg[j] & kSkipTag)) ++j;
+        if (j > i) {
+          urc = fn(base + i * RECORD_BYTES, j - i, user);
+          delivered += j - i;
+        }
+        i = j;
+        while (i < n && (tg[i] & kSkipTag)) ++i;
+      }
       ch->consumed += n;
-      delivered += n;
       std::atomic_thread_fence(std::memory_order_release);
       *tail = ch->consumed;
       if (urc) { rc = set_error(NVBT_ESTATE, "drain callback returned %d", urc); break; }

@@ -19,6 +19,7 @@
 // Precondition ("converged-hook discipline"): every hook is called by all 32 lanes of the warp
 // (lanes that have exited or are on another path pass in_flow = false).
 #pragma once
+#include <type_traits>
 #include <cstdint>
 #include "nvbt.h"
 #include "nvbt_dev.cuh"   // public device primitives (event formation helpers, sectors_lines)
@@ -88,6 +89,24 @@ template <class Prog> __host__ __device__ constexpr int mem_left(int pc) {
   for (int p = pc; p < Prog::N && (p == pc || !Prog::t[p].is_leader); ++p) n += is_mem_kind(Prog::t[p].kind) ? 1 : 0;
   return n;
 }
+// tickets a warp reserves at memory pc `pc` (the rest of its basic block, x4 in register-mode loops)
+template <class Prog> __host__ __device__ constexpr unsigned block_at(int pc) {
+  return (unsigned)mem_left<Prog>(pc) * ((pc >= Prog::REG_LO && pc <= Prog::REG_HI) ? 4u : 1u);
+}
+template <class Prog> __host__ __device__ constexpr unsigned max_block() {
+  unsigned m = 1;
+  for (int p = 0; p < Prog::N; ++p) m = block_at<Prog>(p) > m ? block_at<Prog>(p) : m;
+  return m;
+}
+
+// programs may opt out of 288 B trace staging (static constexpr bool kStageTrace = false)
+template <class P, class = void> struct stage_trace { static constexpr bool value = true; };
+template <class P> struct stage_trace<P, std::void_t<decltype(P::kStageTrace)>> { static constexpr bool value = P::kStageTrace; };
+
+#ifndef NVBT_STAGE288
+#define NVBT_STAGE288 1   // 288 B host-ring records staged per warp in shared memory and written per ticket block
+#endif
+constexpr unsigned kSkipTag = 0x80000000u;   // a committed ticket that carries no record (288 B host ring)
 
 
 // Ring backpressure: ticket t may be written once t < tail + cap. has_room() is the
@@ -120,7 +139,14 @@ struct Hooks {
   static constexpr int kMaxWarps = 8;  // workload CTAs have 256 threads
   static constexpr int kThreads = 32 * kMaxWarps;
   static constexpr int kScratchWord0 = (NPC * SITE_WORDS + 66 + 3) & ~3;  // 16-byte aligned
-  static constexpr int kSmemWords = kOn ? kScratchWord0 + SCRATCH_WORDS * kMaxWarps : 1;
+  // 288 B host-ring records (EM §5) are staged per warp (one ticket block of up to kBlock records) and written
+  // to the ring together, so the link sees whole 128 B lines except at the block's two ends
+  // (programs whose largest block would need more than 18 KB of staging keep a ticket per record)
+  static constexpr unsigned kBlock = max_block<Prog>();
+  static constexpr bool kStage = NVBT_STAGE288 && (T & TOOL_TRACE) != 0 && (T & TOOL_TRACE_DEV) == 0 &&
+                                 stage_trace<Prog>::value && kBlock * 288u * kMaxWarps <= 18432u;
+  static constexpr int kStageWord0 = kScratchWord0 + SCRATCH_WORDS * kMaxWarps;
+  static constexpr int kSmemWords = kOn ? kStageWord0 + (kStage ? kMaxWarps * (int)kBlock * 72 : 0) : 1;
   static_assert(!((T & TOOL_COUNT) && (T & TOOL_BB)), "COUNT and BBCOUNT are exclusive");
 
   const DevState& st;
@@ -133,6 +159,8 @@ struct Hooks {
   unsigned long long hslot;   // device ring: next slot this warp holds, `held` slots from there
   unsigned held;
   unsigned char* dptr = nullptr;   // device ring (TOOL_TRACE_DEV): this lane's address word of the next held slot
+  unsigned nst = 0;           // 288 B host ring: records staged in the held block (from hslot on)
+  unsigned stg = 0;           // 288 B host ring: this warp's staging area (shared address)
   unsigned npend = 0;         // uncommitted records of this warp (warp-uniform)
   unsigned pend_val = 0;      // lane k: tag value of the k-th uncommitted record
   unsigned* pend_tag = nullptr;
@@ -149,6 +177,7 @@ struct Hooks {
     const unsigned tid = threadIdx.x + threadIdx.y * blockDim.x;
     gwarp = (st.cta_lo + blockIdx.x + blockIdx.y * gridDim.x) * ((blockDim.x * blockDim.y) >> 5) + (tid >> 5);  // logical CTA
     scr = (unsigned)__cvta_generic_to_shared(sb + kScratchWord0 + SCRATCH_WORDS * ((tid >> 5) & (kMaxWarps - 1)));
+    if constexpr (kStage) stg = (unsigned)__cvta_generic_to_shared(sb + kStageWord0 + 72 * (int)kBlock * ((tid >> 5) & (kMaxWarps - 1)));
     sbase = (unsigned)__cvta_generic_to_shared(sb);
     if constexpr (kOn && !(NVBT_HOOKS_EXPERIMENT & 2)) {
       // (CTAs of exactly kThreads threads; fixed-stride loops avoid a run-time trip-count division)
@@ -436,6 +465,29 @@ struct Hooks {
           --held;
         }
       } else {
+        if constexpr (kStage) {   // host ring: stage into the warp's block, written when the block is full
+          if (held == 0u) {       // warp-uniform; nothing staged
+            constexpr unsigned K = block_at<Prog>(PC);
+            const unsigned k = (unsigned)((unsigned long long)K < st.cap ? K : st.cap);
+            if (reserve(k, hslot)) { held = k; nst = 0; }
+          }
+          if (held != 0u) {
+            const unsigned src = 2u * (lane - 2u);
+            const unsigned long long a0 = __shfl_sync(FULL, a, src & 31u), a1 = __shfl_sync(FULL, a, (src + 1u) & 31u);
+            if (lane < 18) {
+              const uint4 v = lane == 0   ? make_uint4(st.launch, gwarp, seq, (unsigned)PC)
+                              : lane == 1 ? make_uint4(A, P, w2, 0u)
+                                          : make_uint4((unsigned)a0, (unsigned)(a0 >> 32), (unsigned)a1, (unsigned)(a1 >> 32));
+              asm volatile("st.shared.v4.u32 [%0], {%1, %2, %3, %4};" ::"r"(stg + 288u * nst + 16u * lane),
+                           "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w) : "memory");
+            }
+            ++nst;
+            --held;
+            if (held == 0u) flush288();
+          }
+          ++seq;
+          return;
+        }
         have = reserve(1, t);
       }
       if (have) {
@@ -603,6 +655,37 @@ struct Hooks {
       add_pending(tp1, tag1);
     }
     ++seq;
+  }
+
+  // 288 B host ring: writes the staged records of the warp's block (tickets hslot .. hslot + nst - 1) to
+  // the ring, 16 B per lane per step over the whole run of slots (contiguous except where the ring wraps),
+  // and commits their tags; the block's unused tickets (held) are committed with the skip bit (no data).
+  __device__ __forceinline__ void flush288() {
+    if constexpr (kStage) {
+      __syncwarp();
+      const unsigned chunks = 18u * nst;
+      for (unsigned c = lane; c < chunks; c += 32u) {
+        const unsigned r = c / 18u, q = c - 18u * r;
+        unsigned tg;
+        unsigned* tp;
+        unsigned char* rec = slot_ptr(hslot + r, tg, tp);
+        uint4 v;
+        asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
+                     : "r"(stg + 288u * r + 16u * q) : "memory");
+        *reinterpret_cast<uint4*>(rec + 16u * q) = v;
+      }
+      const unsigned total = nst + held;
+      for (unsigned r = 0; r < total; ++r) {     // warp-uniform
+        unsigned tg;
+        unsigned* tp;
+        slot_ptr(hslot + r, tg, tp);
+        add_pending(tp, r < nst ? tg : (tg | kSkipTag));
+      }
+      hslot += total;
+      held = 0;
+      nst = 0;
+      __syncwarp();                               // staging reads done before the next block's stores
+    }
   }
 
   // 128 B line transport: the unused rest of the warp's ticket block becomes skip slots (header chunk with
@@ -784,6 +867,7 @@ struct Hooks {
     if constexpr (kOn) {
       if constexpr ((T & TOOL_TRACE) != 0 && (T & TOOL_TRACE_DEV) == 0) {
         if (st.compact != 0u) release();   // compact host rings take tickets in blocks
+        else if (!st.no_wait && (held != 0u || nst != 0u)) flush288();
         commit();
       } else if constexpr ((T & TOOL_TRACE) != 0) {
         commit();

@@ -78,6 +78,7 @@ struct ProgStencil {  // §3.4
 };
 // §3.6 (F4): the kernel that uses the proxy instruction WFFT32 (Listing 10 analogue)
 struct ProgWfftEmu {
+  static constexpr bool kStageTrace = false;   // k_wfft's own shared memory leaves no room for trace staging
   static constexpr int N = 14;
   static constexpr int REG_LO = 5, REG_HI = 12;
   static constexpr nvbt_instr_desc t[N] = {
@@ -97,6 +98,7 @@ struct ProgWfftEmu {
     NVBT_D(FFMA, ALU, 0, b, 0, 0), NVBT_D(FMUL, ALU, 0, b, 0, 0), NVBT_D(FFMA, ALU, 0, b, 0, 0),              \
     NVBT_D(FMUL, ALU, 0, b, 0, 0), NVBT_D(FFMA, ALU, 0, b, 0, 0)
 struct ProgWfftSw {
+  static constexpr bool kStageTrace = false;   // k_wfft's own shared memory leaves no room for trace staging
   static constexpr int N = 83;
   static constexpr int REG_LO = 39, REG_HI = 81;
   static constexpr nvbt_instr_desc t[N] = {
