@@ -146,6 +146,7 @@ struct Hooks {
   static constexpr bool kStage = NVBT_STAGE288 && (T & TOOL_TRACE) != 0 && (T & TOOL_TRACE_DEV) == 0 &&
                                  stage_trace<Prog>::value && kBlock * 288u * kMaxWarps <= 18432u;
   static constexpr int kStageWord0 = kScratchWord0 + SCRATCH_WORDS * kMaxWarps;
+  static_assert(!kStage || kBlock >= 2, "a staged block must hold a 176 B wide pair (2 x 192 B)");
   static constexpr int kSmemWords = kOn ? kStageWord0 + (kStage ? kMaxWarps * (int)kBlock * 72 : 0) : 1;
   static_assert(!((T & TOOL_COUNT) && (T & TOOL_BB)), "COUNT and BBCOUNT are exclusive");
 
@@ -610,16 +611,26 @@ struct Hooks {
       const unsigned k = (unsigned)(want < st.cap ? want : st.cap);
       havec = reserve(k, hslot);
       held = havec ? k : 0u;
+      nst = 0;
     }
+    // staged (kStage): slots are formed in the warp's shared-memory block and written with the block
+    // (flush_c176), 192 B apart as in the ring; else straight into the ring
+    unsigned idx = 0;
     if (havec) {
-      t = hslot;
-      hslot += needc;
+      if constexpr (kStage) {
+        idx = nst;
+        nst += needc;
+      } else {
+        t = hslot;
+        hslot += needc;
+      }
       held -= needc;
     }
     if (havec && shortc) {
       {
-        unsigned* tp;
-        unsigned char* rec = slot_ptr(t, tag, tp);
+        unsigned* tp = nullptr;
+        unsigned char* rec = nullptr;
+        if constexpr (!kStage) rec = slot_ptr(t, tag, tp);
         // 11 chunks: header, header (kind | 0x80), base, then 4 deltas per chunk (lanes 4(j-3) .. +3)
         const unsigned dd = act ? (unsigned)dl : 0u;
         const unsigned s0 = 4u * (lane - 3u);
@@ -630,17 +641,21 @@ struct Hooks {
                           : lane == 1 ? make_uint4(A, P, w2 | 0x80000000u, 0u)
                           : lane == 2 ? make_uint4((unsigned)base, (unsigned)(base >> 32), 0u, 0u)
                                       : make_uint4(d0, d1, d2, d3);
-          *reinterpret_cast<uint4*>(rec + 16 * lane) = v;
+          if constexpr (kStage) sts_v4(stg + 192u * idx + 16u * lane, v);
+          else *reinterpret_cast<uint4*>(rec + 16 * lane) = v;
         }
-        add_pending(tp, tag);
+        if constexpr (!kStage) add_pending(tp, tag);
       }
     } else if (havec) {
       // wide pair: slot t = lanes 0-15, slot t+1 = lanes 16-31 (full addresses); lanes 0-9 write the
       // first slot's 10 chunks, lanes 16-25 the second's
-      unsigned tag0, tag1;
-      unsigned *tp0, *tp1;
-      unsigned char* r0 = slot_ptr(t, tag0, tp0);
-      unsigned char* r1 = slot_ptr(t + 1, tag1, tp1);
+      unsigned tag0 = 0, tag1 = 0;
+      unsigned *tp0 = nullptr, *tp1 = nullptr;
+      unsigned char *r0 = nullptr, *r1 = nullptr;
+      if constexpr (!kStage) {
+        r0 = slot_ptr(t, tag0, tp0);
+        r1 = slot_ptr(t + 1, tag1, tp1);
+      }
       const unsigned h = lane >> 4, j = lane & 15u;
       const unsigned src = 16u * h + 2u * (j - 2u);
       const unsigned long long a0 = __shfl_sync(FULL, a, src & 31u), a1 = __shfl_sync(FULL, a, (src + 1u) & 31u);
@@ -649,12 +664,54 @@ struct Hooks {
         const uint4 v = j == 0   ? make_uint4(st.launch, gwarp, seq, (unsigned)PC)
                         : j == 1 ? make_uint4(A, P, w2 | flag, 0u)
                                  : make_uint4((unsigned)a0, (unsigned)(a0 >> 32), (unsigned)a1, (unsigned)(a1 >> 32));
-        *reinterpret_cast<uint4*>((h ? r1 : r0) + 16 * j) = v;
+        if constexpr (kStage) sts_v4(stg + 192u * (idx + h) + 16u * j, v);
+        else *reinterpret_cast<uint4*>((h ? r1 : r0) + 16 * j) = v;
       }
-      add_pending(tp0, tag0);
-      add_pending(tp1, tag1);
+      if constexpr (!kStage) {
+        add_pending(tp0, tag0);
+        add_pending(tp1, tag1);
+      }
+    }
+    if constexpr (kStage) {
+      if (havec && held == 0u) flush_c176();
     }
     ++seq;
+  }
+
+  __device__ __forceinline__ void sts_v4(unsigned a, const uint4& v) {
+    asm volatile("st.shared.v4.u32 [%0], {%1, %2, %3, %4};" ::"r"(a), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w) : "memory");
+  }
+
+  // 176 B slots staged (kStage): the block's unused slots become skip slots in shared memory (0xC0 at byte
+  // 27), then all of the block's slots (192 B apart, the pad included) go to the ring together and every
+  // ticket is committed.
+  __device__ __forceinline__ void flush_c176() {
+    if constexpr (kStage) {
+      if (lane < held) sts_v4(stg + 192u * (nst + lane) + 16u, make_uint4(0u, 0u, 0xC0000000u, 0u));
+      nst += held;
+      held = 0;
+      __syncwarp();
+      const unsigned chunks = 12u * nst;
+      for (unsigned c = lane; c < chunks; c += 32u) {
+        const unsigned r = c / 12u, q = c - 12u * r;
+        unsigned tg;
+        unsigned* tp;
+        unsigned char* rec = slot_ptr(hslot + r, tg, tp);
+        uint4 v;
+        asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
+                     : "r"(stg + 192u * r + 16u * q) : "memory");
+        *reinterpret_cast<uint4*>(rec + 16u * q) = v;
+      }
+      for (unsigned r = 0; r < nst; ++r) {       // warp-uniform
+        unsigned tg;
+        unsigned* tp;
+        slot_ptr(hslot + r, tg, tp);
+        add_pending(tp, tg);
+      }
+      hslot += nst;
+      nst = 0;
+      __syncwarp();
+    }
   }
 
   // 288 B host ring: writes the staged records of the warp's block (tickets hslot .. hslot + nst - 1) to
@@ -691,6 +748,12 @@ struct Hooks {
   // 128 B line transport: the unused rest of the warp's ticket block becomes skip slots (header chunk with
   // flags 0xC0 at byte 27, committed like records) so the consumer can pass them.
   __device__ __forceinline__ void release() {
+    if constexpr (kStage) {
+      if (st.compact <= 2u) {                      // 176 B slots, staged
+        if (held != 0u || nst != 0u) flush_c176();
+        return;
+      }
+    }
     while (held != 0u) {                           // warp-uniform
       const unsigned k = held < 32u ? held : 32u;
       unsigned tag = 0;
