@@ -153,7 +153,9 @@ int nvbt_channel_open(nvbt_ctx ctx, void* pinned_ring, size_t ring_bytes, uint32
  * continue, non-zero to stop draining (nvbt_channel_drain then returns NVBT_ESTATE). */
 typedef int (*nvbt_drain_fn)(const void* records, uint64_t n_records, void* user);
 /* Consumes records in ticket order until the context's stream is idle and every reserved record has
- * been delivered, or timeout_us elapses (-1 = no limit; NVBT_ETIMEDOUT). Runs on the calling thread,
+ * been delivered, or timeout_us elapses (-1 = no limit; NVBT_ETIMEDOUT). Producers reserve tickets in
+ * per-warp blocks; tickets a block did not use (skip tag bit 31 for 288 B slots, 0xC0 skip slots for the
+ * compact transports, EM §5) are consumed without being delivered. Runs on the calling thread,
  * concurrently with kernels already enqueued; it never synchronises the context's stream, so a drain
  * thread may run while another thread keeps enqueueing producers (it returns whenever it sees the stream
  * idle with everything delivered: call it again until the producer thread is done). *n_drained
