@@ -227,13 +227,14 @@ using namespace nvbt;
 // Dynamic shared memory that caps k_stencil<T> (256 threads) at 3 CTAs per SM on `dev`: 4 x (dyn + static
 // + per-block reserved) must exceed the SM's shared memory, 3 x must fit. Derived from the kernel's own
 // static size and the device's limits, checked with the occupancy calculator, cached per (kernel, device).
-static int stencil_pad(const void* fn, int dev, size_t* dyn) {
+// Dynamic shared memory that caps a host-channel traced stencil at kC CTAs per SM (see nvbt_stencil).
+static int stencil_pad(const void* fn, int dev, int kC, size_t* dyn) {
   static std::mutex m;
-  static std::vector<std::tuple<const void*, int, size_t>> cache;
+  static std::vector<std::tuple<const void*, int, size_t, int>> cache;
   {
     std::lock_guard<std::mutex> g(m);
     for (auto& c : cache)
-      if (std::get<0>(c) == fn && std::get<1>(c) == dev) { *dyn = std::get<2>(c); return NVBT_OK; }
+      if (std::get<0>(c) == fn && std::get<1>(c) == dev && std::get<3>(c) == kC) { *dyn = std::get<2>(c); return NVBT_OK; }
   }
   cudaFuncAttributes fa{};
   int per_sm = 0, reserved = 0;
@@ -241,17 +242,17 @@ static int stencil_pad(const void* fn, int dev, size_t* dyn) {
   NVBT_CUDA(cudaDeviceGetAttribute(&per_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, dev));
   NVBT_CUDA(cudaDeviceGetAttribute(&reserved, cudaDevAttrReservedSharedMemoryPerBlock, dev));
   const size_t used = fa.sharedSizeBytes + (size_t)reserved;
-  const size_t quarter = (size_t)per_sm / 4 + 128;              // 4 CTAs of this size exceed the SM
-  const size_t d = quarter > used ? ((quarter - used + 127) & ~size_t(127)) : 0;
-  if (3 * (d + used) > (size_t)per_sm) return set_error(NVBT_ECUDA, "stencil pad: 3 CTAs do not fit (%zu B)", d);
+  const size_t part = (size_t)per_sm / (kC + 1) + 128;        // kC + 1 CTAs of this size exceed the SM
+  const size_t d = part > used ? ((part - used + 127) & ~size_t(127)) : 0;
+  if (kC * (d + used) > (size_t)per_sm) return set_error(NVBT_ECUDA, "stencil pad: %d CTAs do not fit (%zu B)", kC, d);
   int rc = func_smem(fn, dev, d);
   if (rc) return rc;
   int blocks = 0;
   NVBT_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks, fn, 256, d));
-  if (blocks > 3 || blocks < 1)
-    return set_error(NVBT_ECUDA, "stencil pad %zu B gives %d CTAs per SM, expected <= 3", d, blocks);
+  if (blocks > kC || blocks < 1)
+    return set_error(NVBT_ECUDA, "stencil pad %zu B gives %d CTAs per SM, expected <= %d", d, blocks, kC);
   std::lock_guard<std::mutex> g(m);
-  cache.emplace_back(fn, dev, d);
+  cache.emplace_back(fn, dev, d, kC);
   *dyn = d;
   return NVBT_OK;
 }
@@ -394,12 +395,13 @@ int nvbt_stencil(nvbt_ctx ctx, void* stream, uint32_t tools, const float* in, fl
     constexpr uint32_t T = decltype(tag)::value;
     size_t dyn = 0;
     if constexpr ((T & TOOL_TRACE) && !(T & TOOL_TRACE_DEV)) {
-      // Host-channel producer: at most 3 CTAs (24 warps) per SM, enforced by padding dynamic shared memory
-      // just past a quarter of the SM's shared memory (so 4 CTAs never fit, and as much as possible stays
-      // L1). The PCIe link is saturated; fewer warps fencing and writing partial lines at once move more
-      // records (C4 measured in round 1: uncapped 147 M records/s, 3 CTAs 151, 2 CTAs 154 / compact 205,
-      // 214, 199-221; 6 CTAs per SM 134 / 182).
-      pad_rc = stencil_pad((const void*)k_stencil<T>, ctx->device, &dyn);
+      // Host-channel producer: at most 3 CTAs (24 warps) per SM, 6 for 128 B line slots, enforced by padding
+      // dynamic shared memory just past 1/4 (1/7) of the SM's shared memory. The PCIe link is saturated;
+      // fewer warps fencing at once move more records (round 1, per-record tickets: uncapped 147 M
+      // records/s, 3 CTAs 151, 2 CTAs 154; round 2, staged blocks (profiles/r2_c4_ctas_ab.txt): 288 B
+      // 2 / 3 / 4 / 6 CTAs 149 / 161 / 162 / 161 M, 176 B 226 / 242 / 242 / 238 M, 128 B lines 313 / 325-332 /
+      // 326 / 345 M).
+      pad_rc = stencil_pad((const void*)k_stencil<T>, ctx->device, lc.st.compact >= 3u ? 6 : 3, &dyn);
       if (pad_rc) return;
     }
     k_stencil<T><<<lc.grid, block, dyn, lc.stream>>>(in, out, n, lc.st);
