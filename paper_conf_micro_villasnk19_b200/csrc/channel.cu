@@ -558,12 +558,7 @@ __global__ void __launch_bounds__(256) k_fp_count(const unsigned long long* __re
 // written (the unused tail of each SM's last chunk, slots a warp reserved but did not use) have tag 0 and
 // are skipped. Each warp takes a contiguous range of slots, 32 at a time: lane i reads record i's
 // header, then the warp walks the 32 records 8 at a time, 4 lanes per record (quad pass).
-#ifndef NVBT_FP_PIPE
-#define NVBT_FP_PIPE 0   // 1: each quad pass's 4 x 16 B address loads are issued during the previous quad pass (80
-                         // registers, 3 CTAs per SM): consumer 8.82 -> 10.35 ms per 125.8 M records, not kept
-                         // (profiles/r2_f2_pipe_ab.txt)
-#endif
-__global__ void __launch_bounds__(256, NVBT_FP_PIPE ? 3 : 4) k_footprint(const unsigned char* __restrict__ ring,
+__global__ void __launch_bounds__(256, 4) k_footprint(const unsigned char* __restrict__ ring,
                                                     const unsigned long long* __restrict__ chunks,
                                                     unsigned long long cap,
                                                     unsigned long long* __restrict__ keys, unsigned* __restrict__ pool,
@@ -625,24 +620,7 @@ __global__ void __launch_bounds__(256, NVBT_FP_PIPE ? 3 : 4) k_footprint(const u
     // the record's sector bits with one atomic (common: a warp access covers <= 1 KB). Records spanning
     // several words take the warp-cooperative fp_record().
     const unsigned qb = lane >> 2, qq = lane & 3u;
-#if NVBT_FP_PIPE
-    uint4 vn[4];   // the next quad pass's addresses, in flight while the current one is analysed
-    auto qload = [&](unsigned j, uint4* v) {
-      const unsigned jj = j + qb;
-      if ((live >> jj) & 1u) {
-        const uint4* src = reinterpret_cast<const uint4*>(ring + 64 + (base + jj) * RECORD_BYTES + 32 + 64 * qq);
-#pragma unroll
-        for (int k = 0; k < 4; ++k) v[k] = __ldcs(src + k);
-      }
-    };
-    qload(0, vn);
-#pragma unroll
-#endif
     for (unsigned j = 0; j < 32; j += 8) {
-#if NVBT_FP_PIPE
-      uint4 vc[4] = {vn[0], vn[1], vn[2], vn[3]};
-      if (j + 8 < 32) qload(j + 8, vn);
-#endif
       if (((live >> j) & 0xFFu) == 0u) continue;   // uniform
       const unsigned jj = j + qb;
       const bool qlive = (live >> jj) & 1u;
@@ -653,14 +631,10 @@ __global__ void __launch_bounds__(256, NVBT_FP_PIPE ? 3 : 4) k_footprint(const u
       unsigned ref_lo = 0, ref_hi = 0, nd = 0, bits = 0;
       bool have = false;
       if (qlive) {
-#if NVBT_FP_PIPE
-        const uint4* va = vc;
-#else
         const uint4* src = reinterpret_cast<const uint4*>(ring + 64 + (base + jj) * RECORD_BYTES + 32 + 64 * qq);
         uint4 va[4];
 #pragma unroll
         for (int k = 0; k < 4; ++k) va[k] = __ldcs(src + k);
-#endif
 #pragma unroll
         for (int k = 0; k < 4; ++k) {
 #pragma unroll

@@ -12,8 +12,6 @@
 #include <cstdlib>
 #include <cstring>
 
-#include <cuda.h>
-#include <cudaTypedefs.h>
 
 #include "nvbt_internal.h"
 #include "nvbt_workloads.h"
@@ -290,17 +288,13 @@ constexpr int RA_NW = 20;     // pass A warps per CTA (one list region per warp)
 #ifndef NVBT_RPB_NW
 #define NVBT_RPB_NW 20
 #endif
-#ifndef NVBT_RPB_GBINS
-#define NVBT_RPB_GBINS 0       // 1: per-pc sector / line sums as u64 reductions into the CTA's stripe of the global bins
-                               // (no shared per-pc bins: 32 KB more for resident warps). A/B r2_ab19-20: 20 warps
-                               // 1.817 -> 1.847 ms; 22 / 23 warps 2.16 ms (at most 80 registers: 6 warps on one
-                               // SMSP's 16 K registers; 20 warps capped at 80 registers alone cost 1.847 -> 1.878)
-#endif
-#ifndef NVBT_RPB_DYN
-#define NVBT_RPB_DYN 0         // 1: pass-B warps take pass-A regions from a global counter instead of a fixed stride
-                               // (A/B r2_ab19: 1.817 -> 1.831 ms)
-#endif
 constexpr int RB_NW = NVBT_RPB_NW;     // pass B warps per CTA
+// Pass-B variants measured in round 2 and removed (code in commit 834b1ce; profiles/r2_replay_ab.txt, identical
+// results in each): TMA tile::gather4 stages with mbarriers (r2_ab16, slower), an L2 prefetch of the next
+// group (r2_ab15), global per-pc bins with 20-23 warps and dynamic regions (r2_ab19-20), two wide rows per
+// iteration (r2_ab17, r2_ab25), class-0 rows by REDUX.OR (r2_ab16), an 80-register cap (r2_ab20). Kept:
+// the wide-row owner resolve (r2_ab16), the multiplicative-hash bucket (r2_ab21), unpredicated per-row
+// reductions and LOP3 stage offsets (r2_ab22), the row k + 8h staging (r2_ab23).
 #ifndef NVBT_RPB_EXPERIMENT
 #define NVBT_RPB_EXPERIMENT 0   // timing experiments (tools/replay_ab.py), never in a product build
 #endif
@@ -316,47 +310,6 @@ constexpr int RB_NW = NVBT_RPB_NW;     // pass B warps per CTA
 #ifndef NVBT_RPB_WIN
 #define NVBT_RPB_WIN 512       // window rows: sectors per tag window, 1024 / WIN rows per iteration (A/B r2_ab9: 256 and 128 slower)
 #endif
-#ifndef NVBT_RPB_PF
-#define NVBT_RPB_PF 0          // 1: list entries two groups ahead and the group after the staged one
-                               // prefetched into L2 (one 256 B cp.async.bulk.prefetch.L2 per row). A/B r2_ab15:
-                               // pass B 1.84 -> 2.21 ms, not kept
-#endif
-#ifndef NVBT_RPB_TMA
-#define NVBT_RPB_TMA 0         // 1: stages filled by TMA gathers (cp.async.bulk.tensor tile::gather4, 128 B swizzle, one
-                               // mbarrier per stage) instead of 16 B cp.async per lane. A/B r2_ab16: results identical,
-                               // pass B 1.84 -> 2.16 ms, not kept
-#endif
-#ifndef NVBT_RPB_RESOLVE
-#define NVBT_RPB_RESOLVE 1     // wide rows whose first hash round collides are resolved against the bucket owners (one
-                               // more tag round) instead of rehashing twice (A/B r2_ab16: pass B 1.839 -> 1.814 ms)
-#endif
-#ifndef NVBT_RPB_WIDE2
-#define NVBT_RPB_WIDE2 0       // 1: wide rows two per iteration (independent chains), 640 hash buckets each, resolved.
-                               // A/B r2_ab17: pass B 1.813 -> 1.894 ms (more collisions, instruction-bound), not kept;
-                               // with GBINS, 1280 buckets each (r2_ab25): 1.776 -> 1.843 ms (GBINS alone 1.791)
-#endif
-#ifndef NVBT_RPB_HASH1
-#define NVBT_RPB_HASH1 1       // wide-row bucket = top bits of the line's multiplicative hash, no finaliser (A/B r2_ab21:
-                               // pass B 1.820 -> 1.806 ms; a bad spread only costs the resolve / exact paths)
-#endif
-#ifndef NVBT_RPB_REDSEL
-#define NVBT_RPB_REDSEL 1      // pass B's per-row shared reductions run on every lane (others add 0 to a lane-private
-                               // word) instead of a predicated red that ptxas turns into a branch + reconvergence
-#endif
-#ifndef NVBT_RPB_OFF3
-#define NVBT_RPB_OFF3 1        // cp.async stage offsets as one LOP3 on 34 r (see rb_off); with REDSEL: A/B r2_ab22 pass B
-                               // 1.799 -> 1.762 ms (REDSEL alone 1.796, OFF3 alone 1.775)
-#endif
-#ifndef NVBT_RPB_STG2
-#define NVBT_RPB_STG2 1        // staging copies row k + 8h in step k (slot indices by width-16 shuffles with immediate
-                               // source lanes, smem offsets by one XOR with an immediate), full groups unpredicated:
-                               // 4 instead of ~12 instructions per step (A/B r2_ab23: pass B 1.764 -> 1.761 ms; the
-                               // staging was off the critical path)
-#endif
-#ifndef NVBT_RPB_C0REDUX
-#define NVBT_RPB_C0REDUX 0     // 1: one-1-KB-word rows by an OR-reduction of their sector bits (own loop). A/B r2_ab16:
-                               // pass B 1.839 -> 1.890 ms, not kept
-#endif
 #ifndef NVBT_RPB_TAGS
 #define NVBT_RPB_TAGS 1        // slow rows by tag arrays (0: round-1 atomics + reductions, for A/B)
 #endif
@@ -371,12 +324,9 @@ constexpr int RB_STAGES = NVBT_RPB_STAGES;   // per-warp shared stages (RB_STAGE
                                              // 2.25, 2 x 20 1.77: the pass needs warps, not depth
 // per-warp scratch, 1280 B: the slow rows' tag arrays (1 KB sector / hash tags + 256 B line tags); the
 // A/B build without them (NVBT_RPB_TAGS=0) uses its first SCRATCH_WORDS words as sectors_lines_cls scratch
-// (two wide rows per iteration with the global per-pc bins: 1280 more bytes, one 1280-bucket table per row)
-constexpr int RB_SCR2 = 128 + ((NVBT_RPB_WIDE2 && NVBT_RPB_GBINS) ? 320 : 0);
-constexpr unsigned kWideBuckets = (NVBT_RPB_WIDE2 && NVBT_RPB_GBINS) ? 1280u : 640u;   // per row, WIDE2
+constexpr int RB_SCR2 = 128;
 constexpr int RB_WARP_WORDS = RB_STAGES * (RB_ROWS * 64 + 2 * RB_ROWS) + SCRATCH_WORDS + RB_SCR2;
-constexpr size_t RS_COUNTS_BYTES = 65536;   // u32 per pass-A warp (< 16384 warps), then the region counter
-constexpr unsigned kRegionCtr = 16383;      // counts[kRegionCtr]: regions claimed past the first (NVBT_RPB_DYN)
+constexpr size_t RS_COUNTS_BYTES = 65536;   // u32 per pass-A warp (<= 16384 warps)
 static_assert(RB_WARP_WORDS % 4 == 0, "16 B aligned warp areas");
 
 __device__ __forceinline__ void lds_v2(unsigned a, unsigned& x, unsigned& y) {
@@ -450,7 +400,6 @@ k_rpA(const uint4* __restrict__ hdr, unsigned n, unsigned P, const uint8_t* __re
   }
   asm volatile("cp.async.wait_group 0;" ::: "memory");
   if (lane == 0 && counts != nullptr) counts[gw] = cnt;
-  if (NVBT_RPB_DYN && counts != nullptr && gw == 0 && lane == 0) counts[kRegionCtr] = 0u;
   bad = __reduce_add_sync(FULL, bad);
   if (lane == 0 && bad) atomicAdd(err, (unsigned long long)bad);
   __syncthreads();
@@ -499,26 +448,19 @@ __device__ __forceinline__ void sl_bitonic(unsigned long long a, bool act, unsig
 // c ^ (r & 7). TMA stages: the two 128 B halves of every row in separate 2 KB blocks (row r at 128 r), chunks
 // XOR-swizzled by (r & 7) -- the tensor map's 128 B swizzle on a 1024-aligned stage.
 __device__ __forceinline__ unsigned rb_off(unsigned r, unsigned idx) {
-#if NVBT_RPB_TMA
-  return 2048u * (idx >> 4) + 128u * r + ((8u * (idx & 15u)) ^ (16u * (r & 7u)));
-#elif NVBT_RPB_OFF3
   // 8 (32 r + (idx ^ 2 (r & 7))): with a = 34 r (32 r in bits 5.., 2 r in bits 1..4), the index is
   // idx ^ (a & c) for c = ~0x11 (bits 5.. of idx are zero; bit 4 of 2 r must not flip idx): one LOP3
   unsigned x;
   asm("lop3.b32 %0, %1, %2, %3, 0x6C;" : "=r"(x) : "r"(34u * r), "r"(idx), "r"(0xFFFFFFEEu));   // b ^ (a & c)
   return 8u * x;
-#else
-  return 256u * r + ((8u * idx) ^ (16u * (r & 7u)));
-#endif
 }
 
 // Pass B analysis of one stage (up to 16 slots; meta E = 0 marks an empty row). Lane (j, h) = (lane & 15,
 // lane >> 4) scans addresses 16h .. 16h+15 of row j; 16 B chunk c of row j is stored at chunk c ^ (j & 7),
 // so the 8 lanes of a quarter-warp (consecutive j, same h) read 8 distinct bank groups.
 __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsigned lane, unsigned lanebit,
-                                           unsigned s_scr, unsigned s_sS, unsigned s_sL, unsigned s_hist,
-                                           unsigned long long* gmem) {
-  const unsigned j = lane & 15u, h = lane >> 4, sw = j & 7u;
+                                           unsigned s_scr, unsigned s_sS, unsigned s_sL, unsigned s_hist) {
+  const unsigned j = lane & 15u, h = lane >> 4;
   // window sectors of class 1 (tags build: kWR rows in flight, kWin + kWin / 4 tag bytes each)
   constexpr unsigned kWin = NVBT_RPB_TAGS ? NVBT_RPB_WIN : 1024u;
   constexpr int kWR = NVBT_RPB_TAGS ? 1024 / NVBT_RPB_WIN : 1;
@@ -616,25 +558,12 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
   //  * window rows (all sectors of E in the kWin-sector window from wbase, upper words equal; class 1):
   //    the slot is the sector's offset in the window (kWin tag bytes) and, for lines, offset >> 2: S and L
   //    exactly; 1024 / kWin rows per iteration;
-  //  * wide rows (class 2): all lines distinct? slots = a hash of the line into 1280 buckets, up to three
-  //    independent hashes; all lanes owning their slot proves every line (hence sector) distinct: S = L =
-  //    |E|. Rows that collide three times (~3 %) take an exact bitonic sort of the sector keys.
+  //  * wide rows (class 2): all lines distinct? slots = a hash of the line into 1280 buckets; all lanes
+  //    owning their slot proves every line (hence sector) distinct: S = L = |E|; collisions are resolved
+  //    against the bucket owners (below). Rows with a three-way collision or a repeated line (~0.3 %) take
+  //    an exact bitonic sort of the sector keys.
   const unsigned stag = s_scr, ltag = s_scr + 1024u;
-  const unsigned l8 = 8u * lane;
-  const unsigned long long kInvalid = ~0ull;
-#if NVBT_RPB_C0REDUX
-  unsigned mw = cm1, mwide = cm2;
-  for (unsigned m0 = cm0; m0;) {   // one 1 KB word: OR of the lanes' sector bits (sl_word)
-    const unsigned src = 31u - __clz(m0);
-    m0 ^= 1u << src;
-    const unsigned es = __shfl_sync(FULL, E, src);
-    const uint2 r = sl_word(lds_u32(stage + rb_off(src, lane)), (es & lanebit) != 0u);
-    S = lane == src ? r.x : S;
-    L = lane == src ? r.y : L;
-  }
-#else
   unsigned mw = cm0 | cm1, mwide = cm2;
-#endif
   // up to kWR window rows per iteration (independent chains; per row a kWin-sector window of tags and
   // kWin / 4 line tags)
   while (mw) {
@@ -672,74 +601,6 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
     }
     __syncwarp();                                  // reads done before the next rows' stores
   }
-#if NVBT_RPB_WIDE2
-  // two wide rows per iteration (independent dependency chains); row k hashes into buckets [640 k, 640 k + 640)
-  // of the tag scratch and is resolved against its bucket owners as in the one-row loop below
-  while (mwide) {
-    unsigned src[2], es[2], x0[2], x1[2], hb[2], own[2];
-    unsigned long long a[2];
-    bool v[2], act[2], lose[2], ok[2];
-#pragma unroll
-    for (int k = 0; k < 2; ++k) {
-      v[k] = mwide != 0u;
-      src[k] = v[k] ? 31u - __clz(mwide) : 0u;
-      if (v[k]) mwide ^= 1u << src[k];
-    }
-#pragma unroll
-    for (int k = 0; k < 2; ++k) {
-      es[k] = __shfl_sync(FULL, E, src[k]);
-      asm volatile("ld.shared.u64 %0, [%1];" : "=l"(a[k]) : "r"(stage + rb_off(src[k], lane)) : "memory");
-    }
-#pragma unroll
-    for (int k = 0; k < 2; ++k) {
-      act[k] = v[k] && ((es[k] >> lane) & 1u);
-      const unsigned long long line = a[k] >> 7;
-      x0[k] = (unsigned)line;
-      x1[k] = (unsigned)(line >> 32);
-      const unsigned hsh = x0[k] * 0x9E3779B1u ^ x1[k] * 0x85EBCA77u;
-#if NVBT_RPB_HASH1
-      hb[k] = kWideBuckets * k + __umulhi(hsh, kWideBuckets);
-#else
-      hb[k] = kWideBuckets * k + __umulhi(hsh * 0xC2B2AE3Du + (hsh >> 15), kWideBuckets);
-#endif
-      if (act[k]) sts_u8(stag + hb[k], lane);
-    }
-    __syncwarp();
-#pragma unroll
-    for (int k = 0; k < 2; ++k) {
-      own[k] = lds_u8(stag + hb[k]) & 31u;
-      lose[k] = act[k] && own[k] != lane;
-      ok[k] = !__any_sync(FULL, lose[k]);
-    }
-    if (!(ok[0] && ok[1])) {                       // warp-uniform
-      bool same[2];
-#pragma unroll
-      for (int k = 0; k < 2; ++k) {
-        const unsigned o0 = __shfl_sync(FULL, x0[k], own[k]), o1 = __shfl_sync(FULL, x1[k], own[k]);
-        same[k] = lose[k] && o0 == x0[k] && o1 == x1[k];
-        if (lose[k]) sts_u8(stag + hb[k], lane);
-      }
-      __syncwarp();
-#pragma unroll
-      for (int k = 0; k < 2; ++k) {
-        const bool lose2 = lose[k] && lds_u8(stag + hb[k]) != lane;
-        ok[k] = !__any_sync(FULL, same[k] || lose2);
-      }
-    }
-    __syncwarp();
-#pragma unroll
-    for (int k = 0; k < 2; ++k) {
-      unsigned sx, lx;
-      if (ok[k]) {
-        sx = lx = __popc(es[k]);
-      } else {
-        sl_bitonic(a[k], act[k], lane, sx, lx);
-      }
-      S = (v[k] && lane == src[k]) ? sx : S;
-      L = (v[k] && lane == src[k]) ? lx : L;
-    }
-  }
-#endif
   while (mwide) {
     const unsigned src = 31u - __clz(mwide);
     mwide ^= 1u << src;
@@ -749,19 +610,14 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
     const bool act = (es >> lane) & 1u;
     const unsigned long long line = a >> 7;
     const unsigned x0 = (unsigned)line, x1 = (unsigned)(line >> 32);
-    bool ok = false;
-#if NVBT_RPB_RESOLVE
+    bool ok;
     {
       // one hash round; if a lane lost its bucket, every loser compares its line with the bucket's owner (the
       // last writer) and the losers tag their buckets again: when each loser then owns its bucket, every
       // bucket holds the owner and at most one loser whose line differs from the owner's, so all lines are
       // distinct (equal lines always share a bucket). Anything else takes the exact sort below.
       const unsigned hsh = x0 * 0x9E3779B1u ^ x1 * 0x85EBCA77u;
-#if NVBT_RPB_HASH1
       const unsigned hb = __umulhi(hsh, 1280u);   // Fibonacci hashing: the product's top bits
-#else
-      const unsigned hb = __umulhi(hsh * 0xC2B2AE3Du + (hsh >> 15), 1280u);
-#endif
       if (act) sts_u8(stag + hb, lane);
       __syncwarp();
       const unsigned own = lds_u8(stag + hb) & 31u;
@@ -777,35 +633,11 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
       }
       __syncwarp();
     }
-#else
-#pragma unroll
-    for (int round = 0; round < 3 && !ok; ++round) {   // warp-uniform
-      const unsigned hsh = (x0 * (0x9E3779B1u + 0x6A09E666u * round) ^ x1 * (0x85EBCA77u + 0x3C6EF372u * round)) + round;
-      const unsigned hb = __umulhi(hsh * 0xC2B2AE3Du + (hsh >> 15), 1280u);
-      if (act) sts_u8(stag + hb, lane);
-      __syncwarp();
-      ok = __all_sync(FULL, !act || lds_u8(stag + hb) == lane);
-      __syncwarp();
-    }
-#endif
     unsigned sx, lx;
     if (ok) {
       sx = lx = __popc(es);
     } else {                                       // exact: bitonic sort of the sector keys of E
-      unsigned long long k = act ? a >> 5 : kInvalid;
-#pragma unroll
-      for (unsigned kk = 2; kk <= 32; kk <<= 1) {
-#pragma unroll
-        for (unsigned jj = kk >> 1; jj > 0; jj >>= 1) {
-          const unsigned long long o = __shfl_xor_sync(FULL, k, jj);
-          const bool up = (lane & kk) == 0u, lower = (lane & jj) == 0u;
-          k = (lower == up) ? (o < k ? o : k) : (o > k ? o : k);
-        }
-      }
-      const unsigned long long pk = __shfl_up_sync(FULL, k, 1);
-      const bool valid = k != kInvalid;
-      sx = __popc(__ballot_sync(FULL, valid && (lane == 0u || pk != k)));
-      lx = __popc(__ballot_sync(FULL, valid && (lane == 0u || (pk >> 2) != (k >> 2))));
+      sl_bitonic(a, act, lane, sx, lx);
     }
     S = lane == src ? sx : S;
     L = lane == src ? lx : L;
@@ -843,72 +675,27 @@ __device__ __forceinline__ void rb_process(unsigned stage, unsigned meta, unsign
     L = lane == src ? r.y : L;
   }
 #endif
-#if NVBT_RPB_GBINS
-  if (own) {
-    asm volatile("red.global.add.u64 [%0], %1;" ::"l"(gmem + 3u * pc + 1u), "l"((unsigned long long)S) : "memory");
-    asm volatile("red.global.add.u64 [%0], %1;" ::"l"(gmem + 3u * pc + 2u), "l"((unsigned long long)L) : "memory");
-  }
-#else
-#if NVBT_RPB_REDSEL
   {
     const unsigned dmy = s_scr + 4u * lane;   // lane-private word: adding 0 changes nothing
     asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(own ? s_sS + 4u * pc : dmy), "r"(own ? S : 0u) : "memory");
     asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(own ? s_sL + 4u * pc : dmy), "r"(own ? L : 0u) : "memory");
   }
-#else
-  red_shared_add_if(own, s_sS + 4u * pc, S);
-  red_shared_add_if(own, s_sL + 4u * pc, L);
-#endif
-#endif
-#if NVBT_RPB_REDSEL
   {
     const unsigned dmy = s_scr + 4u * lane, one = own ? 1u : 0u;
     asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(own ? s_hist + 4u * S : dmy), "r"(one) : "memory");          // hS[S]
     asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(own ? s_hist + 4u * (33u + L) : dmy), "r"(one) : "memory");  // hL[L]
   }
-#else
-  red_shared_add_if(own, s_hist + 4u * S, 1u);          // hS[S]
-  red_shared_add_if(own, s_hist + 4u * (33u + L), 1u);  // hL[L]
-#endif
   __syncwarp();
 }
 
-// TMA stages (NVBT_RPB_TMA): per warp 2 x 4 KB stages in a 1024-aligned area after the bins, then per warp
-// the tag scratch (1280 B), the stage meta (2 x 128 B) and the two stage mbarriers
-constexpr unsigned RB_X_BYTES = 1280u + 256u + 16u;
-
-#ifdef NVBT_RPB_MAXREG
-#define NVBT_RPB_BOUNDS __maxnreg__(NVBT_RPB_MAXREG)
-#else
-#define NVBT_RPB_BOUNDS __launch_bounds__(32 * RB_NW, 1)
-#endif
-__global__ void NVBT_RPB_BOUNDS
+__global__ void __launch_bounds__(32 * RB_NW, 1)
 k_rpB(const unsigned long long* __restrict__ addr, unsigned P, const uint8_t* __restrict__ kind, DevState st,
-      const unsigned* __restrict__ counts, unsigned n_regions, const uint2* __restrict__ l_ent, unsigned region_cap,
-      const __grid_constant__ CUtensorMap tmap) {
+      const unsigned* __restrict__ counts, unsigned n_regions, const uint2* __restrict__ l_ent, unsigned region_cap) {
   extern __shared__ __align__(16) unsigned sm[];
-#if NVBT_RPB_GBINS
-  const unsigned PB = 68u;                          // hist[66]
-  unsigned long long* const gmem = st.mem + (unsigned long long)(blockIdx.x & (st.stripes - 1u)) * st.stripe_words;
-#else
   const unsigned PB = (2 * P + 66 + 3) & ~3u;      // sS[P] | sL[P] | hist[66]
-  unsigned long long* const gmem = st.mem;
-#endif
   for (unsigned i = threadIdx.x; i < PB; i += blockDim.x) sm[i] = 0;
   const unsigned lane = lane_id(), lanebit = 1u << lane;
   const unsigned s_base = (unsigned)__cvta_generic_to_shared(sm);
-#if NVBT_RPB_TMA
-  static_assert(NVBT_RPB_TAGS, "TMA stages assume the tag-array slow paths (no scratch initialisation)");
-  const unsigned warp = threadIdx.x >> 5;
-  const unsigned s_stg0 = (s_base + 4u * PB + 1023u) & ~1023u;
-  const unsigned s_w = s_stg0 + 8192u * warp;                                 // stage s: + 4096 s
-  const unsigned s_x = s_stg0 + 8192u * RB_NW + RB_X_BYTES * warp;
-  const unsigned s_scr = s_x, s_meta = s_x + 1280u, s_bar = s_x + 1536u;      // meta, mbarrier of stage s: + 128 s, + 8 s
-  if (lane < 2) asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(s_bar + 8u * lane) : "memory");
-  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-  __syncthreads();
-  unsigned phase = 0;   // bit s: parity of stage s's next completion
-#else
   // warp areas 128-byte aligned (9728 B each): stage chunk offsets can then be XOR-ed into full addresses
   unsigned* sWarpAll = reinterpret_cast<unsigned*>((reinterpret_cast<uintptr_t>(sm + PB) + 127u) & ~uintptr_t(127));
   static_assert((RB_WARP_WORDS * 4) % 128 == 0, "128 B aligned warp areas");
@@ -921,12 +708,7 @@ k_rpB(const unsigned long long* __restrict__ addr, unsigned P, const uint8_t* __
   const unsigned s_w = (unsigned)__cvta_generic_to_shared(sWarpAll + (threadIdx.x >> 5) * RB_WARP_WORDS);
   const unsigned s_meta = s_w + 4u * RB_STAGES * RB_ROWS * 64;      // stage s: + 128 s
   const unsigned s_scr = s_w + 4u * kScr0;
-#endif
-#if NVBT_RPB_GBINS
-  const unsigned s_sS = 0u, s_sL = 0u, s_hist = s_base;
-#else
   const unsigned s_sS = s_base, s_sL = s_base + 4u * P, s_hist = s_base + 8u * P;
-#endif
   const unsigned WB = gridDim.x * RB_NW;
   const unsigned j = lane & 15u, h = lane >> 4;
   // group cursor over this warp's regions gw, gw + WB, ...
@@ -936,13 +718,7 @@ k_rpB(const unsigned long long* __restrict__ addr, unsigned P, const uint8_t* __
   struct Grp { unsigned rows, r; uint2 ent; };
   auto fetch = [&](Grp& g) {
     while (r < n_regions && off >= rcnt) {
-#if NVBT_RPB_DYN
-      unsigned nr = 0;   // the next unclaimed region (the first WB regions were taken statically)
-      if (lane == 0) nr = WB + atomicAdd(const_cast<unsigned*>(counts) + kRegionCtr, 1u);
-      r = __shfl_sync(FULL, nr, 0);
-#else
       r += WB;
-#endif
       off = 0;
       rcnt = r < n_regions ? counts[r] : 0u;
     }
@@ -955,33 +731,14 @@ k_rpB(const unsigned long long* __restrict__ addr, unsigned P, const uint8_t* __
   auto slot_of = [&](const Grp& g) -> unsigned {   // event index of row j's slot
     return (g.r + ((g.ent.y >> 5) & 0x7fffu) * n_regions) * 32u + (g.ent.y & 31u);
   };
-  Grp g1, g2;   // g1: the next group to stage; g2 (NVBT_RPB_PF): the one after it
-  // stage g1 into stage s (meta + slot copies), prefetch g2's slots into L2, advance
+  Grp g1{};   // the next group to stage
+  // stage g1 into stage s (meta + slot copies), then fetch the next group
   auto issue = [&](unsigned s) {
     const unsigned nx_E = g1.ent.x, nx_pc = g1.ent.y >> 20;
     const unsigned nx_idx = slot_of(g1);
     if (h == 0u)
       asm volatile("st.shared.v2.u32 [%0], {%1, %2};" ::"r"(s_meta + 128u * s + 8u * j), "r"(nx_E), "r"(nx_pc) : "memory");
     const unsigned stg = s_w + 4096u * s;
-#if NVBT_RPB_TMA
-    // 2 x ceil(rows / 4) gathers of 4 half-rows (128 B each): lane 2 q + hf loads half hf of rows 4q .. 4q + 3
-    // (rows past the group repeat its last row) to stg + 2048 hf + 512 q
-    const unsigned rows = g1.rows, q4 = (lane >> 1) & 3u, hf = lane & 1u;
-    const unsigned ng = 2u * ((rows + 3u) >> 2);
-    unsigned ri[4];
-#pragma unroll
-    for (int i = 0; i < 4; ++i) ri[i] = __shfl_sync(FULL, nx_idx, min(4u * q4 + (unsigned)i, rows - 1u));
-    const unsigned bar = s_bar + 8u * s;
-    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // this stage's earlier reads before the async writes
-    if (lane == 0) asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(512u * ng) : "memory");
-    __syncwarp();
-    if (lane < ng)
-      asm volatile("cp.async.bulk.tensor.2d.shared::cluster.global.tile::gather4.mbarrier::complete_tx::bytes"
-                   " [%0], [%1, {%2, %3, %4, %5, %6}], [%7];"
-                   ::"r"(stg + 2048u * hf + 512u * q4), "l"(reinterpret_cast<unsigned long long>(&tmap)), "r"(32u * hf),
-                     "r"(ri[0]), "r"(ri[1]), "r"(ri[2]), "r"(ri[3]), "r"(bar)
-                   : "memory");
-#elif NVBT_RPB_STG2
     // step k: lane (h, c) copies 16 B chunk c of row k + 8h. Row r's chunk c lives at 256 r + 16 (c ^ (r & 7)) =
     // 256 k + (lane_off ^ 16 k) with lane_off = 2048 h + 16 c (r & 7 == k). The upper half first takes the slot
     // indices of rows 8..15, so step k's index comes from source lane k of each half (width-16 shuffle).
@@ -1005,33 +762,9 @@ k_rpB(const unsigned long long* __restrict__ addr, unsigned P, const uint8_t* __
       }
     }
     asm volatile("cp.async.commit_group;" ::: "memory");
-#else
-    const unsigned c = lane & 15u;
-#pragma unroll
-    for (int k = 0; k < RB_ROWS / 2; ++k) {
-      const unsigned row = 2u * k + h;
-      const unsigned ix = __shfl_sync(FULL, nx_idx, row);
-      if (row < g1.rows)
-        asm volatile("cp.async.cg.shared.global [%0], [%1], 16;"
-                     ::"r"(stg + 256u * row + 16u * (c ^ (row & 7u))), "l"(addr + (unsigned long long)ix * 32u + 2u * c)
-                     : "memory");
-    }
-    asm volatile("cp.async.commit_group;" ::: "memory");
-#endif
-#if NVBT_RPB_PF
-    if (h == 0u && j < g2.rows)
-      asm volatile("cp.async.bulk.prefetch.L2.global [%0], 256;" ::"l"(addr + (unsigned long long)slot_of(g2) * 32u) : "memory");
-    g1 = g2;
-    fetch(g2);
-#else
     fetch(g1);
-#endif
   };
   fetch(g1);
-#if NVBT_RPB_PF
-  fetch(g2);
-#endif
-#if !NVBT_RPB_TMA
   // RB_STAGES - 1 groups in flight ahead of the one being analysed; stage (s + RB_STAGES - 1) % RB_STAGES was
   // analysed in the previous step. Steps without a group to issue commit an empty cp.async group, so
   // wait_group(RB_STAGES - 1) always retires the oldest issued one.
@@ -1047,45 +780,11 @@ k_rpB(const unsigned long long* __restrict__ addr, unsigned P, const uint8_t* __
     else asm volatile("cp.async.commit_group;" ::: "memory");
     asm volatile("cp.async.wait_group %0;" ::"n"(RB_STAGES - 1) : "memory");
     __syncwarp();
-    rb_process(s_w + 4096u * s, s_meta + 128u * s, lane, lanebit, s_scr, s_sS, s_sL, s_hist, gmem);
+    rb_process(s_w + 4096u * s, s_meta + 128u * s, lane, lanebit, s_scr, s_sS, s_sL, s_hist);
     --pending;
     s = s + 1u == (unsigned)RB_STAGES ? 0u : s + 1u;
   }
-#else
-  static_assert(RB_STAGES == 2, "TMA stages: double buffering only");
-  bool live = g1.rows != 0u;
-  unsigned s = 0;
-  if (live) issue(0);
-  while (live) {
-    live = g1.rows != 0u;
-#if NVBT_RPB_TMA
-    if (live) issue(s ^ 1u);
-    {
-      const unsigned bar = s_bar + 8u * s, par = (phase >> s) & 1u;
-      unsigned ready = 0;
-      while (!ready)
-        asm volatile("{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}"
-                     : "=r"(ready) : "r"(bar), "r"(par) : "memory");
-      phase ^= 1u << s;
-    }
-#else
-    if (live) {
-      issue(s ^ 1u);
-    } else {
-      asm volatile("cp.async.commit_group;" ::: "memory");
-    }
-    asm volatile("cp.async.wait_group 1;" ::: "memory");
-#endif
-    __syncwarp();
-    rb_process(s_w + 4096u * s, s_meta + 128u * s, lane, lanebit, s_scr, s_sS, s_sL, s_hist, gmem);
-    s ^= 1u;
-  }
-#endif
   __syncthreads();
-#if NVBT_RPB_GBINS
-  for (unsigned i = threadIdx.x; i < 66; i += blockDim.x)
-    if (sm[i]) atomicAdd(st.hist + i, (unsigned long long)sm[i]);
-#else
   const uint8_t* kd = kind;
   for (unsigned pc = threadIdx.x; pc < P; pc += blockDim.x) {
     const unsigned a = sm[pc], b = sm[P + pc];
@@ -1096,38 +795,11 @@ k_rpB(const unsigned long long* __restrict__ addr, unsigned P, const uint8_t* __
   }
   for (unsigned i = threadIdx.x; i < 66; i += blockDim.x)
     if (sm[2 * P + i]) atomicAdd(st.hist + i, (unsigned long long)sm[2 * P + i]);
-#endif
 }
 
 static size_t rpA_smem(unsigned P) { return 16ull * P + ((P + 15ull) & ~15ull) + 512ull * RA_DEPTH * RA_NW; }
 static size_t rpB_smem(unsigned P) {
-#if NVBT_RPB_TMA
-  return ((2ull * P + 66 + 3) & ~3ull) * 4 + 1023 + (8192ull + RB_X_BYTES) * RB_NW;
-#else
-  return ((NVBT_RPB_GBINS ? 68ull : ((2ull * P + 66 + 3) & ~3ull)) + (size_t)RB_NW * RB_WARP_WORDS) * 4 + 128;
-#endif
-}
-
-// Tensor map of the pass's address slots for the TMA stages: a 2D tensor of u32, 64 per event (256 B rows),
-// m rows; boxes of 32 x 1 (one 128 B half-row; tile::gather4 loads four rows), 128 B swizzle.
-static int rpB_tmap(const void* d_addr, unsigned long long m, CUtensorMap* tm) {
-  static PFN_cuTensorMapEncodeTiled_v12000 enc = nullptr;
-  if (!enc) {
-    void* f = nullptr;
-    cudaDriverEntryPointQueryResult q;
-    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) != cudaSuccess || !f)
-      return set_error(NVBT_ECUDA, "cuTensorMapEncodeTiled unavailable");
-    enc = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(f);
-  }
-  std::memset(tm, 0, sizeof *tm);
-  const cuuint64_t dims[2] = {64, m};
-  const cuuint64_t strides[1] = {256};
-  const cuuint32_t box[2] = {32, 1}, es[2] = {1, 1};
-  const CUresult r = enc(tm, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, const_cast<void*>(d_addr), dims, strides, box, es,
-                         CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-                         CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-  if (r != CUDA_SUCCESS) return set_error(NVBT_ECUDA, "cuTensorMapEncodeTiled failed (%d)", (int)r);
-  return NVBT_OK;
+  return (((2ull * P + 66 + 3) & ~3ull) + (size_t)RB_NW * RB_WARP_WORDS) * 4 + 128;
 }
 
 static int sm_count(int dev) { return device_sms(dev); }
@@ -1252,7 +924,7 @@ static int launch_staged(nvbt_ctx c, const void* d_hdr, const void* d_addr, uint
   const unsigned long long cap = staged_cap(scratch_bytes);
   const unsigned long long max_warps = (unsigned long long)sms * RA_CTAS_PER_SM * RA_NW;
   unsigned long long pass = 1ull << 30;   // keeps every CTA's u32 bins far from overflow
-  if (max_warps >= kRegionCtr) return set_error(NVBT_EINVAL, "staged replay: %llu pass-A warps", max_warps);
+  if (max_warps > RS_COUNTS_BYTES / 4) return set_error(NVBT_EINVAL, "staged replay: %llu pass-A warps", max_warps);
   if (memdiv) {
     if (scratch == nullptr || cap <= 32ull * max_warps)
       return set_error(NVBT_ENOMEM, "staged replay scratch of %zu bytes is too small", scratch_bytes);
@@ -1281,15 +953,9 @@ static int launch_staged(nvbt_ctx c, const void* d_hdr, const void* d_addr, uint
     NVBT_CUDA(cudaGetLastError());
     c->launches++;
     if (!memdiv) continue;
-    CUtensorMap tm;
-#if NVBT_RPB_TMA
-    { const int trc = rpB_tmap(static_cast<const unsigned long long*>(d_addr) + off * 32, m, &tm); if (trc) return trc; }
-#else
-    std::memset(&tm, 0, sizeof tm);
-#endif
     k_rpB<<<blocks_b, 32 * RB_NW, rpB_smem(c->n_pcs), c->stream>>>(
         static_cast<const unsigned long long*>(d_addr) + off * 32, c->n_pcs, c->d_kind, st, counts, warps, l_ent,
-        region_cap, tm);
+        region_cap);
     NVBT_CUDA(cudaGetLastError());
     c->launches++;
   }
