@@ -682,67 +682,49 @@ struct Hooks {
     asm volatile("st.shared.v4.u32 [%0], {%1, %2, %3, %4};" ::"r"(a), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w) : "memory");
   }
 
-  // 176 B slots staged (kStage): the block's unused slots become skip slots in shared memory (0xC0 at byte
-  // 27), then all of the block's slots (192 B apart, the pad included) go to the ring together and every
-  // ticket is committed.
+  // Staged ticket blocks (kStage): writes the warp's n_data staged slots (stride bytes apart in shared memory
+  // and in the ring; Q 16 B chunks each) to ring tickets hslot .. hslot + n_data - 1, 16 B per lane per step
+  // over the whole run (contiguous except where the ring wraps), then commits tickets hslot .. + n_tags - 1:
+  // those past n_data with the skip bit (no record).
+  template <unsigned Q>
+  __device__ __forceinline__ void write_block(unsigned n_data, unsigned n_tags, unsigned stride) {
+    __syncwarp();
+    for (unsigned c = lane; c < Q * n_data; c += 32u) {
+      const unsigned r = c / Q, q = c - Q * r;
+      unsigned tg;
+      unsigned* tp;
+      unsigned char* rec = slot_ptr(hslot + r, tg, tp);
+      uint4 v;
+      asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
+                   : "r"(stg + stride * r + 16u * q) : "memory");
+      *reinterpret_cast<uint4*>(rec + 16u * q) = v;
+    }
+    for (unsigned r = 0; r < n_tags; ++r) {       // warp-uniform
+      unsigned tg;
+      unsigned* tp;
+      slot_ptr(hslot + r, tg, tp);
+      add_pending(tp, r < n_data ? tg : (tg | kSkipTag));
+    }
+    hslot += n_tags;
+    held = 0;
+    nst = 0;
+    __syncwarp();                                 // staging reads done before the next block's stores
+  }
+
+  // 176 B slots: the block's unused slots become skip slots in shared memory (0xC0 at byte 27), and all of
+  // them go out with the block (192 B apart, the pad included; two slots = three whole lines).
   __device__ __forceinline__ void flush_c176() {
     if constexpr (kStage) {
       if (lane < held) sts_v4(stg + 192u * (nst + lane) + 16u, make_uint4(0u, 0u, 0xC0000000u, 0u));
-      nst += held;
-      held = 0;
-      __syncwarp();
-      const unsigned chunks = 12u * nst;
-      for (unsigned c = lane; c < chunks; c += 32u) {
-        const unsigned r = c / 12u, q = c - 12u * r;
-        unsigned tg;
-        unsigned* tp;
-        unsigned char* rec = slot_ptr(hslot + r, tg, tp);
-        uint4 v;
-        asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
-                     : "r"(stg + 192u * r + 16u * q) : "memory");
-        *reinterpret_cast<uint4*>(rec + 16u * q) = v;
-      }
-      for (unsigned r = 0; r < nst; ++r) {       // warp-uniform
-        unsigned tg;
-        unsigned* tp;
-        slot_ptr(hslot + r, tg, tp);
-        add_pending(tp, tg);
-      }
-      hslot += nst;
-      nst = 0;
-      __syncwarp();
+      const unsigned n = nst + held;
+      write_block<12>(n, n, 192u);
     }
   }
 
-  // 288 B host ring: writes the staged records of the warp's block (tickets hslot .. hslot + nst - 1) to
-  // the ring, 16 B per lane per step over the whole run of slots (contiguous except where the ring wraps),
-  // and commits their tags; the block's unused tickets (held) are committed with the skip bit (no data).
+  // 288 B records: the staged records go out with the block; its unused tickets are committed with the skip
+  // bit in their tags, no data.
   __device__ __forceinline__ void flush288() {
-    if constexpr (kStage) {
-      __syncwarp();
-      const unsigned chunks = 18u * nst;
-      for (unsigned c = lane; c < chunks; c += 32u) {
-        const unsigned r = c / 18u, q = c - 18u * r;
-        unsigned tg;
-        unsigned* tp;
-        unsigned char* rec = slot_ptr(hslot + r, tg, tp);
-        uint4 v;
-        asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
-                     : "r"(stg + 288u * r + 16u * q) : "memory");
-        *reinterpret_cast<uint4*>(rec + 16u * q) = v;
-      }
-      const unsigned total = nst + held;
-      for (unsigned r = 0; r < total; ++r) {     // warp-uniform
-        unsigned tg;
-        unsigned* tp;
-        slot_ptr(hslot + r, tg, tp);
-        add_pending(tp, r < nst ? tg : (tg | kSkipTag));
-      }
-      hslot += total;
-      held = 0;
-      nst = 0;
-      __syncwarp();                               // staging reads done before the next block's stores
-    }
+    if constexpr (kStage) write_block<18>(nst, nst + held, 288u);
   }
 
   // 128 B line transport: the unused rest of the warp's ticket block becomes skip slots (header chunk with
