@@ -540,16 +540,25 @@ struct Hooks {
         const unsigned k = (unsigned)(want < st.cap ? want : st.cap);   // a block never exceeds the ring
         have = reserve(k, hslot);
         held = have ? k : 0u;
+        nst = 0;
       }
+      // staged (kStage): the block's lines are formed in shared memory and written together (flush_line)
+      unsigned lidx = 0;
       if (have) {
-        t = hslot;
-        hslot += need;
+        if constexpr (kStage) {
+          lidx = nst;
+          nst += need;
+        } else {
+          t = hslot;
+          hslot += need;
+        }
         held -= need;
       }
       if (have && shortf) {
         {
-          unsigned* tp;
-          unsigned char* rec = slot_ptr(t, tag, tp);
+          unsigned* tp = nullptr;
+          unsigned char* rec = nullptr;
+          if constexpr (!kStage) rec = slot_ptr(t, tag, tp);
           // u32 word k of the delta area (bytes 40..103) = delta[2k] | delta[2k + 1] << 16, built on lane 2k
           const unsigned d16 = act ? ((unsigned)dl & 0xFFFFu) : 0u;
           const unsigned wp = d16 | (__shfl_down_sync(FULL, d16, 1) << 16);
@@ -566,18 +575,21 @@ struct Hooks {
                             : lane <= 5 ? make_uint4(u0, u1, u2, u3)
                             : lane == 6 ? make_uint4(u0, u1, 0u, 0u)
                                         : make_uint4(0u, 0u, 0u, 0u);
-            *reinterpret_cast<uint4*>(rec + 16 * lane) = v;
+            if constexpr (kStage) sts_v4(stg + 128u * lidx + 16u * lane, v);
+            else *reinterpret_cast<uint4*>(rec + 16 * lane) = v;
           }
-          add_pending(tp, tag);
+          if constexpr (!kStage) add_pending(tp, tag);
         }
       } else if (have) {
         // three slots: slot 0 = header (kind | 0x40) + lanes 0..11; slots 1, 2 carry flag 0x20 at byte 27
         // and lanes 12..26 (bytes 0..23: 3 lanes, 32..127: 12 lanes) and 27..31
-        unsigned tg[3];
-        unsigned* tps[3];
-        unsigned char* r[3];
+        unsigned tg[3] = {0u, 0u, 0u};
+        unsigned* tps[3] = {nullptr, nullptr, nullptr};
+        unsigned char* r[3] = {nullptr, nullptr, nullptr};
+        if constexpr (!kStage) {
 #pragma unroll
-        for (int k = 0; k < 3; ++k) r[k] = slot_ptr(t + k, tg[k], tps[k]);
+          for (int k = 0; k < 3; ++k) r[k] = slot_ptr(t + k, tg[k], tps[k]);
+        }
         const unsigned sl = lane >> 3, c = lane & 7u;
         // first lane of the chunk's address pair: slot 0 chunk c >= 2: 2(c-2); slots 1, 2: chunk 0 -> 12 + 15(s-1),
         // chunk 1 -> 14 + 15(s-1) (one address + the flag word), chunk c >= 2 -> 15 + 15(s-1) + 2(c-2)
@@ -591,11 +603,17 @@ struct Hooks {
                         : flagw ? make_uint4((unsigned)a0, (unsigned)(a0 >> 32), 0x20000000u, 0u)
                         : zero ? make_uint4(0u, 0u, 0u, 0u)
                                : make_uint4((unsigned)a0, (unsigned)(a0 >> 32), (unsigned)a1, (unsigned)(a1 >> 32));
-          *reinterpret_cast<uint4*>(r[sl] + 16 * c) = v;
+          if constexpr (kStage) sts_v4(stg + 128u * (lidx + sl) + 16u * c, v);
+          else *reinterpret_cast<uint4*>(r[sl] + 16 * c) = v;
         }
-        add_pending(tps[0], tg[0]);
-        add_pending(tps[1], tg[1]);
-        add_pending(tps[2], tg[2]);
+        if constexpr (!kStage) {
+          add_pending(tps[0], tg[0]);
+          add_pending(tps[1], tg[1]);
+          add_pending(tps[2], tg[2]);
+        }
+      }
+      if constexpr (kStage) {
+        if (have && held == 0u) flush_line();
       }
       ++seq;
       return;
@@ -721,21 +739,35 @@ struct Hooks {
     }
   }
 
+  // 128 B line slots: as for 176 B slots, 128 B apart (each slot one whole line)
+  __device__ __forceinline__ void flush_line() {
+    if constexpr (kStage) {
+      if (lane < held) sts_v4(stg + 128u * (nst + lane) + 16u, make_uint4(0u, 0u, 0xC0000000u, 0u));
+      const unsigned n = nst + held;
+      write_block<8>(n, n, 128u);
+    }
+  }
+
   // 288 B records: the staged records go out with the block; its unused tickets are committed with the skip
   // bit in their tags, no data.
   __device__ __forceinline__ void flush288() {
     if constexpr (kStage) write_block<18>(nst, nst + held, 288u);
   }
 
-  // 128 B line transport: the unused rest of the warp's ticket block becomes skip slots (header chunk with
-  // flags 0xC0 at byte 27, committed like records) so the consumer can pass them.
+  // Compact transports: the rest of the warp's ticket block goes out now, its unused tickets as skip slots
+  // (header chunk with flags 0xC0 at byte 27, committed like records) so the consumer can pass them.
+  // Kernels without staging write the skip headers straight into the ring.
   __device__ __forceinline__ void release() {
     if constexpr (kStage) {
-      if (st.compact <= 2u) {                      // 176 B slots, staged
-        if (held != 0u || nst != 0u) flush_c176();
-        return;
+      if (held != 0u || nst != 0u) {
+        if (st.compact <= 2u) flush_c176();        // 176 B slots, staged
+        else flush_line();                         // 128 B line slots, staged
       }
+    } else {
+      release_unstaged();
     }
+  }
+  __device__ __forceinline__ void release_unstaged() {
     while (held != 0u) {                           // warp-uniform
       const unsigned k = held < 32u ? held : 32u;
       unsigned tag = 0;
